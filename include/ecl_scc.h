@@ -1,0 +1,160 @@
+/*
+ * ecl_scc.h -- C ABI of the B200-native ECL-SCC hot path (libeclscc.so).
+ *
+ * Citation key: P:n = line n of the paper's text (Alabandi, Sands, Biros, Burtscher,
+ * "A GPU Algorithm for Detecting Strongly Connected Components", SC'23).
+ *
+ * WHAT IS COMPUTED.  Input: "a directed graph G = (V, E) with unique vertex IDs" (P:116,
+ * Alg. 1 "Input"); vertex IDs are CSR row indices 0..n-1 (reading 8).
+ * Output: "for all v: v_in (and v_out) denotes to which SCC vertex v belongs" (P:156,
+ * Alg. 1 "Output"); the signature of an SCC is its highest vertex ID (Sec. 3.2.1),
+ * so labels_out[v] = max{ w : v and w are mutually reachable } -- a unique, schedule
+ * independent answer, bit-exact against Tarjan.
+ *
+ * WHERE.  The graph is already on the GPU and the result is needed on the GPU;
+ * every graph pointer below is a DEVICE pointer on the calling thread's current CUDA
+ * device, unless marked "host".
+ *
+ * CONVENTIONS (all entry points).
+ *  - Ownership: the caller owns every input and output buffer.  Inputs are never
+ *    modified (the library compacts its own working copies).  The library owns its
+ *    plan/workspace; passing a plan makes repeated calls allocation-free.
+ *  - Errors: every call returns an ecl_scc_status and never aborts.  On error labels_out
+ *    is unspecified; ecl_scc_last_error() returns a thread-local message.
+ *      n == 0                                      -> ECL_SCC_OK, nothing written
+ *      nnz == 0                                    -> labels[v] = v
+ *      n < 0, nnz < 0, NULL pointer with n > 0     -> ECL_SCC_EINVAL
+ *      row_ptr[0] != 0, row_ptr[n] != nnz, decreasing offsets, col_idx outside [0,n)
+ *                                                  -> ECL_SCC_ERANGE (device validation
+ *                                                     pass; skipped with ECL_SCC_NO_VALIDATE)
+ *      nnz >= 2^31                                 -> ECL_SCC_EUNSUPPORTED (int32 offsets)
+ *      workspace allocation failure                -> ECL_SCC_ENOMEM
+ *      any CUDA runtime error                      -> ECL_SCC_ECUDA
+ *  - Graph contents: self-loops and duplicate edges are accepted; they change no SCC
+ *    (reading 9).
+ *  - Synchrony: ecl_scc() returns after labels_out is written.  The _async form enqueues
+ *    on `stream`; it waits on that stream only for the outer-loop convergence decision
+ *    (one small device->host read per outer iteration), never on other streams.
+ *  - Thread safety: distinct plans may be used concurrently from different host threads;
+ *    a plan must not be used by two calls at once.
+ */
+#ifndef ECL_SCC_H
+#define ECL_SCC_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* ecl_scc_stream_t; /* == cudaStream_t; NULL = legacy default */
+
+typedef enum {
+    ECL_SCC_OK = 0,
+    ECL_SCC_EINVAL = 1,
+    ECL_SCC_ERANGE = 2,
+    ECL_SCC_ENOMEM = 3,
+    ECL_SCC_ECUDA = 4,
+    ECL_SCC_ENCCL = 5,
+    ECL_SCC_EUNSUPPORTED = 6
+} ecl_scc_status;
+
+/* plan flags (DESIGN.md "Readings" and "Kernels") */
+#define ECL_SCC_NO_TRIM 0x1u      /* disable the Trim-1 round run with every edge removal */
+#define ECL_SCC_COMPRESS 0x2u     /* path compression: pull in[in[u]], out[out[w]] */
+#define ECL_SCC_NO_VALIDATE 0x4u  /* skip the device validation pass over row_ptr/col_idx */
+#define ECL_SCC_SYNC_PASSES 0x8u  /* ablation: no block-local iteration, one Jacobi-like
+                                     relaxation per global pass ("separate kernels") */
+
+#define ECL_SCC_TRACE_MAX 64
+
+/* Per-run statistics (host struct, optional).  Index k = outer iteration k+1. */
+typedef struct {
+    int32_t iterations;                      /* outer iterations that ran Phase 2        */
+    int32_t trace_len;                       /* min(iterations, ECL_SCC_TRACE_MAX)       */
+    int64_t passes;                          /* global Phase-2 passes, all iterations    */
+    int64_t edges_in[ECL_SCC_TRACE_MAX];     /* live edges entering Phase 2 (after trim) */
+    int64_t vertices_in[ECL_SCC_TRACE_MAX];  /* vertices with a live edge in Phase 2     */
+    int64_t edges_kept[ECL_SCC_TRACE_MAX];   /* edges kept by Phase 3 (before next trim) */
+    int64_t passes_iter[ECL_SCC_TRACE_MAX];  /* global passes of Phase 2, per iteration  */
+    int64_t prop_bytes;                      /* algorithmic bytes of all Phase-2 passes
+                                                (SURVEY 8(d) accounting)      */
+} ecl_scc_stats;
+
+typedef struct ecl_scc_plan_s* ecl_scc_plan_t;
+
+/* Workspace for graphs with n <= n_max, nnz <= nnz_max on the current device.
+ * flags: ECL_SCC_* above.  Allocates device memory (about 24*n_max + 12*nnz_max bytes). */
+int ecl_scc_plan_create(int32_t n_max, int64_t nnz_max, uint32_t flags, ecl_scc_plan_t* out);
+int ecl_scc_plan_destroy(ecl_scc_plan_t plan);
+
+/* Single graph, synchronous.  row_ptr: n+1 int32 offsets; col_idx: nnz int32 IDs;
+ * labels_out: n int32 (written).  Uses a temporary plan with default flags. */
+int ecl_scc(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx,
+            int32_t* labels_out);
+
+/* Single graph, on `stream`, with an optional plan (NULL: temporary) and optional host
+ * stats (NULL: none).  Same arguments and layout as ecl_scc(). */
+int ecl_scc_async(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx,
+                  int32_t* labels_out, ecl_scc_stream_t stream, ecl_scc_plan_t plan,
+                  ecl_scc_stats* stats);
+
+/* Test/diagnostic entry: run until Phase 2 of outer iteration `stop_iter` (>= 1) has
+ * reached its fixed point and write that iteration's signatures v_in -> sig_in[n] and
+ * v_out -> sig_out[n] (device).  If the run terminates before stop_iter, both receive
+ * the final labels.  Used for per-iteration parity against the oracle (DESIGN.md
+ * reading 12: the state after each Phase 2 is schedule independent). */
+int ecl_scc_debug_run(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx,
+                      uint32_t flags, int32_t stop_iter, int32_t* sig_in, int32_t* sig_out,
+                      ecl_scc_stream_t stream, ecl_scc_stats* stats);
+
+/* Batch of G independent graphs on one GPU (one discrete ordinate each).
+ * n, nnz: host arrays [G]; row_ptr, col_idx, labels_out: host arrays [G] of device
+ * pointers.  Labels are per-graph LOCAL IDs (max local ID of the SCC).  The graphs are
+ * solved together as one disjoint union (clusters never interact); a plan sized
+ * for sum(n), sum(nnz) may be passed (NULL: temporary). */
+int ecl_scc_batched(int32_t G, const int32_t* n, const int64_t* nnz,
+                    const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                    int32_t* const* labels_out, ecl_scc_stream_t stream, ecl_scc_plan_t plan,
+                    ecl_scc_stats* stats);
+
+/* ---- multi-GPU: one large graph, edge-partitioned by source rows (SPMD) ---------- */
+typedef struct ecl_scc_comm_s* ecl_scc_comm_t;
+
+/* 128-byte NCCL unique id (rank 0 creates it; broadcast it out of band, e.g. over the
+ * torch.distributed process group). */
+int ecl_scc_get_unique_id(uint8_t id[128]);
+/* Collective: every rank calls with the same id; binds to the current device. */
+int ecl_scc_comm_create(int32_t nranks, int32_t rank, const uint8_t id[128], ecl_scc_comm_t* out);
+int ecl_scc_comm_destroy(ecl_scc_comm_t comm);
+
+/* Collective over comm.  This rank owns source rows [row_begin, row_end) of the global
+ * graph (n vertices): local_row_ptr has row_end-row_begin+1 offsets starting at 0,
+ * local_col_idx holds local_nnz GLOBAL destination IDs.  Signatures are replicated and
+ * combined with ncclAllReduce(MAX) after every local fixed point; degrees for trim with
+ * ncclAllReduce(SUM).  labels_out: n int32 on every rank (replicated result). */
+int ecl_scc_partitioned(ecl_scc_comm_t comm, int32_t n, int32_t row_begin, int32_t row_end,
+                        int64_t local_nnz, const int32_t* local_row_ptr,
+                        const int32_t* local_col_idx, int32_t* labels_out,
+                        ecl_scc_stream_t stream, ecl_scc_stats* stats);
+
+/* Single-process emulation of the partitioned algorithm with P partitions on the
+ * current device (the all-reduce replaced by an element-wise max over P replicas).
+ * Same arithmetic as ecl_scc_partitioned at P ranks; used to test the partitioned path
+ * on one GPU.  Inputs as ecl_scc(); row ranges are chosen balanced by edge count. */
+int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_t* row_ptr,
+                                 const int32_t* col_idx, int32_t* labels_out,
+                                 ecl_scc_stream_t stream, ecl_scc_stats* stats);
+
+/* Host helper: split rows [0,n) into P contiguous ranges of about equal edge count
+ * (binary search on the host row_ptr[n+1]); bounds_out[P+1] (host). */
+int ecl_scc_partition_rows(int32_t P, int32_t n, const int32_t* row_ptr_host, int32_t* bounds_out);
+
+const char* ecl_scc_status_string(int status);
+const char* ecl_scc_last_error(void); /* thread-local, "" if none */
+int ecl_scc_version(void);            /* 100 * major + minor */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ECL_SCC_H */

@@ -1,0 +1,463 @@
+// driver.cu -- plan/workspace, the outer loop of Alg. 1, and the C ABI (include/ecl_scc.h).
+//
+// Outer loop (Alg. 1 l.2-21) as run here, rule R2 (reading 1):
+//   ingest:  v_in = v_out = v (l.3-6); CSC transpose of the input CSR
+//   repeat:  edge removal + Trim-1 + compaction  (Phase 3 of the previous iteration,
+//            l.15-19 and P:186), then Phase 1 for the unfinished (l.3-6),
+//            stop if no live edge is left (reading 2), else
+//            Phase 2 to its fixed point (l.7-14).
+// labels_out doubles as the v_in array, so the final signatures need no copy.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "../../include/ecl_scc.h"
+#include "common.cuh"
+#include "kernels.cuh"
+#include "scan.cuh"
+#include "driver.h"
+
+namespace eclscc {
+
+static thread_local char g_err[512] = "";
+
+int fail(int status, const char* fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return status;
+}
+void clear_err() { g_err[0] = 0; }
+const char* last_err() { return g_err; }
+
+#define CK(call)                                                                                      \
+    do {                                                                                              \
+        cudaError_t _e = (call);                                                                      \
+        if (_e != cudaSuccess)                                                                        \
+            return fail(ECL_SCC_ECUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(_e)); \
+    } while (0)
+
+static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+static inline unsigned grid_for(int64_t work, int threads) {
+    int64_t g = cdiv(work, threads);
+    if (g < 1) g = 1;
+    return (unsigned)std::min<int64_t>(g, 0x7FFFFFFF);
+}
+
+constexpr int TPB = 256;
+
+// --------------------------------------------------------------------------- plan
+int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
+    p->n_cap = std::max<int32_t>(n_max, 1);
+    p->m_cap = std::max<int64_t>(m_max, 1);
+    const size_t n1 = (size_t)p->n_cap + 1;
+    const size_t m = (size_t)p->m_cap;
+    p->nw_cap = cdiv(p->n_cap, TPB) * (TPB / WARP) + 1;
+    p->bsum_cap = cdiv(std::max<int64_t>(n1, p->nw_cap), SCAN_TILE) + 1;
+    auto A = [&](void** ptr, size_t bytes) -> cudaError_t { return cudaMalloc(ptr, bytes); };
+    cudaError_t e = cudaSuccess;
+    e = e ? e : A((void**)&p->sig_in, n1 * 4);
+    e = e ? e : A((void**)&p->sig_out, n1 * 4);
+    e = e ? e : A((void**)&p->kin, n1 * 4);
+    e = e ? e : A((void**)&p->kout, n1 * 4);
+    for (int b = 0; b < 2; b++) {
+        e = e ? e : A((void**)&p->act[b], n1 * 4);
+        e = e ? e : A((void**)&p->optr[b], n1 * 4);
+        e = e ? e : A((void**)&p->iptr[b], n1 * 4);
+        e = e ? e : A((void**)&p->oadj[b], m * 4);
+        e = e ? e : A((void**)&p->iadj[b], m * 4);
+    }
+    e = e ? e : A((void**)&p->wsum, (size_t)p->nw_cap * sizeof(int4));
+    e = e ? e : A((void**)&p->wscan, (size_t)p->nw_cap * sizeof(int4));
+    e = e ? e : A((void**)&p->bsum, (size_t)p->bsum_cap * sizeof(int4));
+    e = e ? e : A((void**)&p->dc, sizeof(DevCounters));
+    if (e == cudaSuccess) e = cudaMallocHost((void**)&p->hc, sizeof(DevCounters));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ECL_SCC_ENOMEM, "plan allocation (n=%d, nnz=%lld): %s", n_max, (long long)m_max,
+                    cudaGetErrorString(e));
+    }
+    return ECL_SCC_OK;
+}
+
+void plan_free(Plan* p) {
+    cudaFree(p->sig_in); cudaFree(p->sig_out); cudaFree(p->kin); cudaFree(p->kout);
+    for (int b = 0; b < 2; b++) {
+        cudaFree(p->act[b]); cudaFree(p->optr[b]); cudaFree(p->iptr[b]);
+        cudaFree(p->oadj[b]); cudaFree(p->iadj[b]);
+    }
+    cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->dc);
+    cudaFree(p->u_rp); cudaFree(p->u_ci);
+    if (p->hc) cudaFreeHost(p->hc);
+    memset(p, 0, sizeof(*p));
+}
+
+// --------------------------------------------------------------------------- scans
+template <typename T>
+static int scan_excl(const T* in, int64_t N, T* out, T* grand, void* bsum, int write_total, cudaStream_t s) {
+    const int64_t nb = std::max<int64_t>(cdiv(N, SCAN_TILE), 1);
+    k_scan_reduce<T><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, N, (T*)bsum);
+    k_scan_top<T><<<1, SCAN_THREADS, 0, s>>>((T*)bsum, nb, grand);
+    k_scan_apply<T><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, N, (T*)bsum, out, grand, write_total);
+    CK(cudaGetLastError());
+    return ECL_SCC_OK;
+}
+
+// --------------------------------------------------------------------------- steps
+// a1: CSC of the input graph into buffer 0 (in-degree histogram, scan, scatter)
+static int build_csc(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, cudaStream_t s) {
+    CK(cudaMemsetAsync(p->kin, 0, sizeof(int32_t) * (size_t)(n + 1), s));
+    k_indeg<<<grid_for(nnz, TPB), TPB, 0, s>>>(nnz, ci, p->kin);
+    int r = scan_excl<I1>((const I1*)p->kin, n, (I1*)p->iptr[0], (I1*)&p->dc->grand1, p->bsum, 1, s);
+    if (r) return r;
+    CK(cudaMemsetAsync(p->kout, 0, sizeof(int32_t) * (size_t)n, s));
+    k_csc_scatter<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, ci, p->iptr[0], p->kout, p->iadj[0]);
+    CK(cudaGetLastError());
+    return ECL_SCC_OK;
+}
+
+// a2/a7/a3: Phase 3 + Trim-1 + compaction into buffer `ob`, then Phase 1 reset
+template <bool FIRST, bool TRIM>
+static int remove_and_compact(Plan* p, const WGraph& g, int ob, int32_t* vin, int32_t* vout, cudaStream_t s) {
+    const unsigned grid = grid_for(g.na, TPB);
+    const int64_t nw = (int64_t)grid * (TPB / WARP);
+    CK(cudaMemsetAsync(&p->dc->kept, 0, sizeof(unsigned long long), s));
+    k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, vin, vout, p->kin, p->kout, &p->dc->kept);
+    k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, vin, vout, p->kin, p->kout, p->wsum);
+    int r = scan_excl<I3>((const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
+    if (r) return r;
+    k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, vin, vout, p->kin, p->kout, p->wscan, &p->dc->totals,
+                                                          p->act[ob], p->optr[ob], p->oadj[ob], p->iptr[ob],
+                                                          p->iadj[ob]);
+    if (!FIRST) k_reset<<<grid, TPB, 0, s>>>(g, vin, vout);
+    CK(cudaGetLastError());
+    return ECL_SCC_OK;
+}
+
+// a4-a6: Phase 2 to its fixed point.  Passes are enqueued in growing batches; a pass
+// whose predecessor changed nothing exits at once, so over-enqueueing costs only a launch.
+static int propagate(Plan* p, const WGraph& g, int32_t* vin, int32_t* vout, cudaStream_t s, int64_t* passes_out) {
+    CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
+    CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
+    const unsigned grid = grid_for(g.na, TPB);
+    const bool compress = (p->flags & ECL_SCC_COMPRESS) != 0;
+    int pass = 0;
+    int batch = 2;
+    for (;;) {
+        for (int k = 0; k < batch; k++, pass++) {
+            if (compress) k_prop<true><<<grid, TPB, 0, s>>>(g, vin, vout, p->dc, pass);
+            else k_prop<false><<<grid, TPB, 0, s>>>(g, vin, vout, p->dc, pass);
+        }
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (p->hc->changed[(pass - 1) & (RING - 1)] == 0) break;
+        batch = std::min(batch * 2, RING / 2);
+    }
+    *passes_out = (int64_t)p->hc->passes;
+    return ECL_SCC_OK;
+}
+
+// the whole path for one (possibly union) graph
+int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, int32_t* vin,
+              cudaStream_t s, ecl_scc_stats* st, int stop_iter, int32_t* dbg_in, int32_t* dbg_out) {
+    int32_t* vout = p->sig_out;
+    if (st) memset(st, 0, sizeof(*st));
+    k_init_sig<<<grid_for(n, TPB), TPB, 0, s>>>(n, vin, vout);
+    CK(cudaGetLastError());
+    if (!(p->flags & ECL_SCC_NO_VALIDATE) && n > 0) {
+        CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
+        k_validate<<<std::min<unsigned>(grid_for(std::max<int64_t>(n, nnz), TPB), 148 * 16), TPB, 0, s>>>(n, nnz, rp, ci, &p->dc->err);
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (p->hc->err) return fail(ECL_SCC_ERANGE, "invalid CSR: offsets not monotone from 0 to nnz, or column outside [0,n)");
+    }
+    const bool trim = !(p->flags & ECL_SCC_NO_TRIM);
+    int iters = 0;
+    if (nnz > 0) {
+        int r = build_csc(p, n, nnz, rp, ci, s);
+        if (r) return r;
+        WGraph g{nullptr, rp, ci, p->iptr[0], p->iadj[0], n};
+        int ob = 1;
+        for (int iter = 1;; iter++) {
+            if (iter == 1) r = trim ? remove_and_compact<true, true>(p, g, ob, vin, vout, s)
+                                    : remove_and_compact<true, false>(p, g, ob, vin, vout, s);
+            else r = trim ? remove_and_compact<false, true>(p, g, ob, vin, vout, s)
+                          : remove_and_compact<false, false>(p, g, ob, vin, vout, s);
+            if (r) return r;
+            CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));
+            const int4 t = p->hc->totals;
+            if (st && iter >= 2 && iter - 2 < ECL_SCC_TRACE_MAX) st->edges_kept[iter - 2] = (int64_t)p->hc->kept;
+            if (t.y != t.z) return fail(ECL_SCC_ECUDA, "internal: CSR/CSC survivor mismatch %d vs %d", t.y, t.z);
+            g = WGraph{p->act[ob], p->optr[ob], p->oadj[ob], p->iptr[ob], p->iadj[ob], t.x};
+            if (t.y == 0) break;
+            int64_t passes = 0;
+            r = propagate(p, g, vin, vout, s, &passes);
+            if (r) return r;
+            iters = iter;
+            if (st) {
+                if (iter - 1 < ECL_SCC_TRACE_MAX) {
+                    st->edges_in[iter - 1] = t.y;
+                    st->vertices_in[iter - 1] = t.x;
+                    st->passes_iter[iter - 1] = passes;
+                }
+                st->passes += passes;
+                // 4(n_p+1) offsets + 12 B/edge + 16 B/vertex (+8 B/vertex compressed)
+                const int64_t per = 4 * ((int64_t)t.x + 1) + 12 * (int64_t)t.y + 16 * (int64_t)t.x +
+                                    ((p->flags & ECL_SCC_COMPRESS) ? 8 * (int64_t)t.x : 0);
+                st->prop_bytes += per * passes;
+            }
+            if (stop_iter == iter) {
+                CK(cudaMemcpyAsync(dbg_in, vin, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+                CK(cudaMemcpyAsync(dbg_out, vout, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+                CK(cudaStreamSynchronize(s));
+                if (st) { st->iterations = iters; st->trace_len = std::min(iters, ECL_SCC_TRACE_MAX); }
+                return ECL_SCC_OK;
+            }
+            ob ^= 1;
+        }
+    }
+    if (stop_iter > 0) {
+        CK(cudaMemcpyAsync(dbg_in, vin, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+        CK(cudaMemcpyAsync(dbg_out, vin, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+    }
+    if (st) { st->iterations = iters; st->trace_len = std::min(iters, ECL_SCC_TRACE_MAX); }
+    CK(cudaStreamSynchronize(s));
+    return ECL_SCC_OK;
+}
+
+// --------------------------------------------------------------------------- batched union
+__global__ void k_set1(int32_t* p, int32_t v) { *p = v; }
+__global__ void k_union_rows(int32_t n, const int32_t* __restrict__ rp, int32_t voff, int32_t eoff,
+                             int32_t* __restrict__ urp) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        urp[voff + v] = rp[v] + eoff;
+}
+__global__ void k_union_cols(int64_t m, const int32_t* __restrict__ ci, int32_t voff, int32_t* __restrict__ uci) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x)
+        uci[e] = ci[e] + voff;
+}
+__global__ void k_split_labels(int32_t n, const int32_t* __restrict__ ul, int32_t voff, int32_t* __restrict__ out) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        out[v] = ul[voff + v] - voff;
+}
+
+int run_batched(Plan* p, int32_t G, const int32_t* n, const int64_t* nnz, const int32_t* const* rp,
+                const int32_t* const* ci, int32_t* const* labels, cudaStream_t s, ecl_scc_stats* st) {
+    int64_t N = 0, M = 0;
+    for (int g = 0; g < G; g++) { N += n[g]; M += nnz[g]; }
+    if (!p->u_rp || p->u_n_cap < N) {
+        cudaFree(p->u_rp);
+        p->u_rp = nullptr;
+        if (cudaMalloc((void**)&p->u_rp, sizeof(int32_t) * (size_t)(N + 1)) != cudaSuccess) {
+            cudaGetLastError();
+            return fail(ECL_SCC_ENOMEM, "batched union offsets (%lld vertices)", (long long)N);
+        }
+        p->u_n_cap = N;
+    }
+    if (!p->u_ci || p->u_m_cap < M) {
+        cudaFree(p->u_ci);
+        p->u_ci = nullptr;
+        if (cudaMalloc((void**)&p->u_ci, sizeof(int32_t) * (size_t)std::max<int64_t>(M, 1)) != cudaSuccess) {
+            cudaGetLastError();
+            return fail(ECL_SCC_ENOMEM, "batched union columns (%lld edges)", (long long)M);
+        }
+        p->u_m_cap = M;
+    }
+    // validate each graph individually first (offsets are rebased below)
+    if (!(p->flags & ECL_SCC_NO_VALIDATE)) {
+        CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
+        for (int g = 0; g < G; g++)
+            if (n[g] > 0)
+                k_validate<<<std::min<unsigned>(grid_for(std::max<int64_t>(n[g], nnz[g]), TPB), 148 * 16), TPB, 0, s>>>(
+                    n[g], nnz[g], rp[g], ci[g], &p->dc->err);
+        CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (p->hc->err) return fail(ECL_SCC_ERANGE, "invalid CSR in batch");
+    }
+    int64_t vo = 0, eo = 0;
+    for (int g = 0; g < G; g++) {
+        if (n[g] > 0) k_union_rows<<<grid_for(n[g], TPB), TPB, 0, s>>>(n[g], rp[g], (int32_t)vo, (int32_t)eo, p->u_rp);
+        if (nnz[g] > 0) k_union_cols<<<grid_for(nnz[g], TPB), TPB, 0, s>>>(nnz[g], ci[g], (int32_t)vo, p->u_ci + eo);
+        vo += n[g];
+        eo += nnz[g];
+    }
+    k_set1<<<1, 1, 0, s>>>(p->u_rp + N, (int32_t)M);
+    CK(cudaGetLastError());
+    const uint32_t saved = p->flags;
+    p->flags |= ECL_SCC_NO_VALIDATE;
+    int r = run_graph(p, (int32_t)N, M, p->u_rp, p->u_ci, p->sig_in, s, st, 0, nullptr, nullptr);
+    p->flags = saved;
+    if (r) return r;
+    vo = 0;
+    for (int g = 0; g < G; g++) {
+        if (n[g] > 0) k_split_labels<<<grid_for(n[g], TPB), TPB, 0, s>>>(n[g], p->sig_in, (int32_t)vo, labels[g]);
+        vo += n[g];
+    }
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(s));
+    return ECL_SCC_OK;
+}
+
+}  // namespace eclscc
+
+// =========================================================================== C ABI
+using namespace eclscc;
+
+struct ecl_scc_plan_s {
+    Plan p;
+};
+
+static int check_graph_args(int32_t n, int64_t nnz, const void* rp, const void* ci, const void* out) {
+    if (n < 0 || nnz < 0) return fail(ECL_SCC_EINVAL, "negative size (n=%d, nnz=%lld)", n, (long long)nnz);
+    if (n > 0 && (!rp || !out)) return fail(ECL_SCC_EINVAL, "NULL row_ptr or labels_out");
+    if (nnz > 0 && !ci) return fail(ECL_SCC_EINVAL, "NULL col_idx");
+    if (nnz >= (int64_t)INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "nnz >= 2^31 needs 64-bit offsets");
+    if (n == INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "n must be < 2^31 - 1");
+    return ECL_SCC_OK;
+}
+
+extern "C" {
+
+int ecl_scc_version(void) { return 100; }
+
+const char* ecl_scc_status_string(int s) {
+    switch (s) {
+        case ECL_SCC_OK: return "ok";
+        case ECL_SCC_EINVAL: return "invalid argument";
+        case ECL_SCC_ERANGE: return "malformed graph (offsets or column out of range)";
+        case ECL_SCC_ENOMEM: return "out of device memory";
+        case ECL_SCC_ECUDA: return "CUDA error";
+        case ECL_SCC_ENCCL: return "NCCL error";
+        case ECL_SCC_EUNSUPPORTED: return "unsupported";
+        default: return "unknown status";
+    }
+}
+
+const char* ecl_scc_last_error(void) { return last_err(); }
+
+int ecl_scc_plan_create(int32_t n_max, int64_t nnz_max, uint32_t flags, ecl_scc_plan_t* out) {
+    clear_err();
+    if (!out || n_max < 0 || nnz_max < 0) return fail(ECL_SCC_EINVAL, "plan_create: bad arguments");
+    if (nnz_max >= (int64_t)INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "nnz_max >= 2^31");
+    ecl_scc_plan_s* h = (ecl_scc_plan_s*)calloc(1, sizeof(ecl_scc_plan_s));
+    if (!h) return fail(ECL_SCC_ENOMEM, "host allocation");
+    h->p.flags = flags;
+    int r = plan_alloc(&h->p, n_max, nnz_max);
+    if (r) {
+        plan_free(&h->p);
+        free(h);
+        return r;
+    }
+    *out = h;
+    return ECL_SCC_OK;
+}
+
+int ecl_scc_plan_destroy(ecl_scc_plan_t plan) {
+    clear_err();
+    if (!plan) return ECL_SCC_OK;
+    plan_free(&plan->p);
+    free(plan);
+    return ECL_SCC_OK;
+}
+
+int ecl_scc_async(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx, int32_t* labels_out,
+                  ecl_scc_stream_t stream, ecl_scc_plan_t plan, ecl_scc_stats* stats) {
+    clear_err();
+    int r = check_graph_args(n, nnz, row_ptr, col_idx, labels_out);
+    if (r) return r;
+    if (stats) memset(stats, 0, sizeof(*stats));
+    if (n == 0) return ECL_SCC_OK;
+    if (plan && (plan->p.n_cap < n || plan->p.m_cap < nnz))
+        return fail(ECL_SCC_EINVAL, "plan too small (n_max=%d, nnz_max=%lld)", plan->p.n_cap, (long long)plan->p.m_cap);
+    ecl_scc_plan_t tmp = nullptr;
+    if (!plan) {
+        r = ecl_scc_plan_create(n, nnz, 0, &tmp);
+        if (r) return r;
+        plan = tmp;
+    }
+    r = run_graph(&plan->p, n, nnz, row_ptr, col_idx, labels_out, (cudaStream_t)stream, stats, 0, nullptr, nullptr);
+    if (tmp) ecl_scc_plan_destroy(tmp);
+    return r;
+}
+
+int ecl_scc(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx, int32_t* labels_out) {
+    return ecl_scc_async(n, nnz, row_ptr, col_idx, labels_out, nullptr, nullptr, nullptr);
+}
+
+int ecl_scc_debug_run(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx, uint32_t flags,
+                      int32_t stop_iter, int32_t* sig_in, int32_t* sig_out, ecl_scc_stream_t stream,
+                      ecl_scc_stats* stats) {
+    clear_err();
+    int r = check_graph_args(n, nnz, row_ptr, col_idx, sig_in);
+    if (r) return r;
+    if (stop_iter < 1 || (n > 0 && !sig_out)) return fail(ECL_SCC_EINVAL, "debug_run: stop_iter >= 1 and sig_out required");
+    if (n == 0) return ECL_SCC_OK;
+    ecl_scc_plan_t tmp = nullptr;
+    r = ecl_scc_plan_create(n, nnz, flags, &tmp);
+    if (r) return r;
+    r = run_graph(&tmp->p, n, nnz, row_ptr, col_idx, tmp->p.sig_in, (cudaStream_t)stream, stats, stop_iter, sig_in,
+                  sig_out);
+    cudaStreamSynchronize((cudaStream_t)stream);
+    ecl_scc_plan_destroy(tmp);
+    return r;
+}
+
+int ecl_scc_batched(int32_t G, const int32_t* n, const int64_t* nnz, const int32_t* const* row_ptr,
+                    const int32_t* const* col_idx, int32_t* const* labels_out, ecl_scc_stream_t stream,
+                    ecl_scc_plan_t plan, ecl_scc_stats* stats) {
+    clear_err();
+    if (G < 0 || (G > 0 && (!n || !nnz || !row_ptr || !col_idx || !labels_out)))
+        return fail(ECL_SCC_EINVAL, "batched: bad arguments");
+    int64_t N = 0, M = 0;
+    for (int g = 0; g < G; g++) {
+        int r = check_graph_args(n[g], nnz[g], row_ptr[g], col_idx[g], labels_out[g]);
+        if (r) return r;
+        N += n[g];
+        M += nnz[g];
+    }
+    if (stats) memset(stats, 0, sizeof(*stats));
+    if (N == 0) return ECL_SCC_OK;
+    if (N >= INT32_MAX || M >= INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "batch union exceeds 2^31 vertices or edges");
+    if (plan && (plan->p.n_cap < N || plan->p.m_cap < M))
+        return fail(ECL_SCC_EINVAL, "plan too small for the batch union");
+    ecl_scc_plan_t tmp = nullptr;
+    if (!plan) {
+        int r = ecl_scc_plan_create((int32_t)N, M, 0, &tmp);
+        if (r) return r;
+        plan = tmp;
+    }
+    int r = run_batched(&plan->p, G, n, nnz, row_ptr, col_idx, labels_out, (cudaStream_t)stream, stats);
+    if (tmp) ecl_scc_plan_destroy(tmp);
+    return r;
+}
+
+int ecl_scc_partition_rows(int32_t P, int32_t n, const int32_t* rp, int32_t* bounds) {
+    clear_err();
+    if (P < 1 || n < 0 || !rp || !bounds) return fail(ECL_SCC_EINVAL, "partition_rows: bad arguments");
+    const int64_t m = rp[n];
+    bounds[0] = 0;
+    for (int r = 1; r < P; r++) {
+        // first row whose start offset reaches r*m/P
+        const int64_t target = (m * r + P - 1) / P;
+        int32_t lo = bounds[r - 1], hi = n;
+        while (lo < hi) {
+            const int32_t mid = lo + (hi - lo) / 2;
+            if ((int64_t)rp[mid] < target) lo = mid + 1; else hi = mid;
+        }
+        bounds[r] = lo;
+    }
+    bounds[P] = n;
+    return ECL_SCC_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,206 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Labels are integers with a unique definition, so every comparison is
+bit-exact.  Per-iteration states (live edge counts, signatures after each Phase 2) are
+schedule independent (reading 12) and compared exactly against O2 with the same
+trim rule.  Pass counts are schedule dependent and never compared.
+"""
+import json
+import os
+import random
+
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+import paper_conf_sc_alabandisbb23_b200 as E
+
+pytestmark = pytest.mark.gpu
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def dev(g):
+    return (torch.from_numpy(np.ascontiguousarray(g.row_ptr, dtype=np.int32)).cuda(),
+            torch.from_numpy(np.ascontiguousarray(g.col_idx, dtype=np.int32)).cuda())
+
+
+def gpu_labels(g, flags=0, plan=None):
+    rp, ci = dev(g)
+    if flags and plan is None:
+        plan = E.Plan(g.n, g.nnz, flags)
+    lab, st = E.ecl_scc(rp, ci, plan=plan, stats=True)
+    torch.cuda.synchronize()
+    return lab.cpu().numpy(), st
+
+
+def check_trace(g, trim, flags=0, max_iters=None):
+    """GPU per-iteration edge counts and signatures == O2's (same trim rule)."""
+    tr = oracle.ecl_scc(g.row_ptr, g.col_idx, trim=trim)
+    fl = flags | (0 if trim else E.NO_TRIM)
+    rp, ci = dev(g)
+    _, st = gpu_labels(g, fl)
+    k = tr.iterations
+    assert st["iterations"] == k
+    assert st["edges_in"] == tr.edges_in[:64]
+    assert st["edges_kept"] == tr.edges_kept[:max(min(k, 64) - 1, 0)]
+    for it in range(1, (k if max_iters is None else min(k, max_iters)) + 1):
+        s = oracle.ecl_scc(g.row_ptr, g.col_idx, trim=trim, snap_iter=it)
+        gi, go, _ = E.ecl_scc_debug_run(rp, ci, it, flags=fl)
+        np.testing.assert_array_equal(gi.cpu().numpy(), s.snap_in, err_msg=f"in, iteration {it}")
+        np.testing.assert_array_equal(go.cpu().numpy(), s.snap_out, err_msg=f"out, iteration {it}")
+
+
+# ----------------------------------------------------------------- C1: worked example
+@pytest.mark.parametrize("flags", [0, E.COMPRESS, E.SYNC_PASSES])
+def test_appendix_a(flags):
+    gold = json.load(open(os.path.join(GOLDEN, "appendix_a.json")))
+    g = gen.appendix_a()
+    for trim, key in ((False, "r2_no_trim"), (True, "r2_trim1")):
+        fl = flags | (0 if trim else E.NO_TRIM)
+        lab, st = gpu_labels(g, fl)
+        np.testing.assert_array_equal(lab, gold["labels"])
+        exp = gold[key]
+        assert st["edges_in"] == exp["edges_in"]
+        assert st["edges_kept"] == exp["edges_kept"][:-1]
+        rp, ci = dev(g)
+        for it in range(1, len(exp["in"]) + 1):
+            gi, go, _ = E.ecl_scc_debug_run(rp, ci, it, flags=fl)
+            np.testing.assert_array_equal(gi.cpu().numpy(), exp["in"][it - 1])
+            np.testing.assert_array_equal(go.cpu().numpy(), exp["out"][it - 1])
+
+
+def test_random_small_graphs_labels_and_traces():
+    rng = random.Random(77)
+    for trial in range(150):
+        n = rng.randrange(1, 300)
+        m = rng.randrange(0, 4 * n)
+        edges = [(rng.randrange(n), rng.randrange(n)) for _ in range(m)]
+        g = gen.from_edges(n, edges)
+        truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+        for flags in (0, E.NO_TRIM, E.COMPRESS):
+            lab, _ = gpu_labels(g, flags)
+            np.testing.assert_array_equal(lab, truth, err_msg=f"trial {trial} flags {flags}")
+        if trial % 10 == 0:
+            check_trace(g, trim=True)
+            check_trace(g, trim=False)
+
+
+def test_c1_gnm_2000_8000():
+    g = gen.config("c1")
+    truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+    for flags in (0, E.COMPRESS, E.NO_TRIM, E.SYNC_PASSES):
+        lab, _ = gpu_labels(g, flags)
+        np.testing.assert_array_equal(lab, truth)
+    check_trace(g, trim=True)
+    check_trace(g, trim=False)
+
+
+# ----------------------------------------------------------------- edge cases
+def test_edge_cases():
+    # empty graph
+    rp = torch.zeros(1, dtype=torch.int32, device="cuda")
+    ci = torch.zeros(0, dtype=torch.int32, device="cuda")
+    assert E.ecl_scc(rp, ci).numel() == 0
+    # no edges
+    g = gen.from_edges(7, [])
+    np.testing.assert_array_equal(gpu_labels(g)[0], np.arange(7))
+    # self-loops and duplicates only
+    g = gen.from_edges(5, [(1, 1), (2, 3), (2, 3), (4, 4)])
+    np.testing.assert_array_equal(gpu_labels(g)[0], np.arange(5))
+    # one directed cycle in random ID order -> one SCC named n-1 (P:247 twist-hex-like)
+    n = 100_000
+    perm = np.random.default_rng(1).permutation(n)
+    g = gen.from_edges(n, np.stack([perm, np.roll(perm, -1)], 1))
+    for flags in (0, E.COMPRESS):
+        assert (gpu_labels(g, flags)[0] == n - 1).all()
+    # long path (deep DAG): identity
+    g = gen.from_edges(n, np.stack([perm[:-1], perm[1:]], 1))
+    np.testing.assert_array_equal(gpu_labels(g)[0], np.arange(n))
+    # disjoint k-cycles on consecutive IDs
+    k = 5
+    e = [(b * k + i, b * k + (i + 1) % k) for b in range(1000) for i in range(k)]
+    g = gen.from_edges(5000, e)
+    v = np.arange(5000)
+    np.testing.assert_array_equal(gpu_labels(g)[0], (v // k) * k + k - 1)
+
+
+def test_heavy_vertices():
+    """Hubs far above the warp-cooperation threshold in both directions."""
+    rng = np.random.default_rng(5)
+    n = 50_000
+    hub = 123
+    src = np.concatenate([np.full(20_000, hub), rng.integers(0, n, 30_000), rng.integers(0, n, 20_000)])
+    dst = np.concatenate([rng.integers(0, n, 20_000), np.full(30_000, 777), rng.integers(0, n, 20_000)])
+    g = gen.from_edges(n, np.stack([src, dst], 1))
+    truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+    for flags in (0, E.NO_TRIM, E.COMPRESS):
+        np.testing.assert_array_equal(gpu_labels(g, flags)[0], truth)
+    check_trace(g, trim=True, max_iters=3)
+
+
+def test_invalid_input_reports_erange():
+    rp = torch.tensor([0, 2, 1, 3], dtype=torch.int32, device="cuda")      # decreasing offsets
+    ci = torch.tensor([1, 2, 0], dtype=torch.int32, device="cuda")
+    with pytest.raises(E.EclSccError) as ex:
+        E.ecl_scc(rp, ci)
+    assert ex.value.status == E.ERANGE
+    rp = torch.tensor([0, 1, 2, 3], dtype=torch.int32, device="cuda")
+    ci = torch.tensor([1, 5, 0], dtype=torch.int32, device="cuda")         # column out of range
+    with pytest.raises(E.EclSccError) as ex:
+        E.ecl_scc(rp, ci)
+    assert ex.value.status == E.ERANGE
+    plan = E.Plan(2, 2)
+    with pytest.raises(E.EclSccError) as ex:                               # plan too small
+        E.ecl_scc(rp, torch.tensor([1, 2, 0], dtype=torch.int32, device="cuda"), plan=plan)
+    assert ex.value.status == E.EINVAL
+
+
+def test_plan_reuse_and_stream():
+    g1, g2 = gen.config("c1"), gen.mesh(12, gen.ordinate(7), kappa=0.2, seed=9)
+    plan = E.Plan(max(g1.n, g2.n), max(g1.nnz, g2.nnz))
+    s = torch.cuda.Stream()
+    for g in (g1, g2, g1):
+        rp, ci = dev(g)
+        torch.cuda.synchronize()
+        with torch.cuda.stream(s):
+            lab = E.ecl_scc(rp, ci, plan=plan)
+        s.synchronize()
+        np.testing.assert_array_equal(lab.cpu().numpy(), oracle.tarjan_labels(g.row_ptr, g.col_idx))
+
+
+# ----------------------------------------------------------------- C2..C5
+@pytest.mark.parametrize("order", ["lex", "blocked8"])
+def test_c2_mesh_1m(order):
+    g = gen.config("c2", order=order)
+    truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+    lab, st = gpu_labels(g)
+    np.testing.assert_array_equal(lab, truth)
+    tr = oracle.ecl_scc(g.row_ptr, g.col_idx, trim=True)
+    assert st["edges_in"] == tr.edges_in[:64] and st["iterations"] == tr.iterations
+    lab, _ = gpu_labels(g, E.COMPRESS)
+    np.testing.assert_array_equal(lab, truth)
+
+
+def test_c3_rmat_scale22():
+    g = gen.config("c3")
+    truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+    lab, st = gpu_labels(g)
+    np.testing.assert_array_equal(lab, truth)
+
+
+def test_c4_mesh_16m():
+    g = gen.config("c4")
+    truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+    lab, _ = gpu_labels(g)
+    np.testing.assert_array_equal(lab, truth)
+
+
+def test_c5_batched_meshes():
+    graphs = [gen.config("c5one", d=d) for d in range(0, 64, 4)]   # 16 of the 64 ordinates
+    dg = [dev(g) for g in graphs]
+    labs, st = E.ecl_scc_batched(dg, stats=True)
+    torch.cuda.synchronize()
+    for g, lab in zip(graphs, labs):
+        np.testing.assert_array_equal(lab.cpu().numpy(), oracle.tarjan_labels(g.row_ptr, g.col_idx))

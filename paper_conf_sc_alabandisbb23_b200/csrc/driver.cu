@@ -159,6 +159,9 @@ static int propagate(Plan* p, const WGraph& g, int32_t* vin, int32_t* vout, cuda
         CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         if (p->hc->changed[(pass - 1) & (RING - 1)] == 0) break;
+        // a monotone max over int32 IDs cannot take more passes than this
+        if ((int64_t)pass > 4 * (int64_t)g.na + 1024)
+            return fail(ECL_SCC_ECUDA, "internal: Phase 2 did not converge after %d passes", pass);
         batch = std::min(batch * 2, RING / 2);
     }
     *passes_out = (int64_t)p->hc->passes;
@@ -188,6 +191,7 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         WGraph g{nullptr, rp, ci, p->iptr[0], p->iadj[0], n};
         int ob = 1;
         for (int iter = 1;; iter++) {
+            if (iter > n + 2) return fail(ECL_SCC_ECUDA, "internal: outer loop exceeded n+2 iterations");
             if (iter == 1) r = trim ? remove_and_compact<true, true>(p, g, ob, vin, vout, s)
                                     : remove_and_compact<true, false>(p, g, ob, vin, vout, s);
             else r = trim ? remove_and_compact<false, true>(p, g, ob, vin, vout, s)

@@ -289,16 +289,16 @@ __global__ void k_reset(WGraph g, int32_t* __restrict__ vin, int32_t* __restrict
 // new value, both valid ancestors/descendants (monotone).  A pass that changes
 // nothing observed a consistent snapshot, so it certifies the fixed point.
 //
-// Pass protocol: pass p returns at once if pass p-1 changed nothing; otherwise it clears
-// changed[p+1] and sets changed[p] if it wrote anything.
+// Pass protocol: pass p clears changed[p+1]; it returns at once if pass p-1 changed
+// nothing; otherwise it sets changed[p] if it wrote anything.
 template <bool COMPRESS>
 __global__ void __launch_bounds__(256) k_prop(WGraph g, int32_t* __restrict__ vin, int32_t* __restrict__ vout,
                                               DevCounters* __restrict__ dc, int pass) {
+    // every pass (also a skipped one) clears its successor's word, so changed[p] is 0
+    // unless pass p itself ran and changed something
+    if (blockIdx.x == 0 && threadIdx.x == 0) dc->changed[(pass + 1) & (RING - 1)] = 0;
     if (pass > 0 && ld_vol(&dc->changed[(pass - 1) & (RING - 1)]) == 0) return;
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        dc->changed[(pass + 1) & (RING - 1)] = 0;
-        atomicAdd(&dc->passes, 1ull);
-    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(&dc->passes, 1ull);
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const bool valid = i < g.na;

@@ -11,10 +11,10 @@ constexpr int HEAVY = 32;      // rows longer than this are processed by a whole
 constexpr int RING = 64;       // ring of per-pass "changed" words (Phase-2 driver)
 
 // Working graph after an edge removal (the surviving edges, here as a compacted
-// CSR + CSC pair over the ACTIVE vertices -- those that still have a live edge).
-//   active index i in [0, na) -> vertex act[i] (act == nullptr: identity, first pass)
-//   out-edges of act[i]: oadj[optr[i] .. optr[i+1])  (global destination IDs)
-//   in-edges  of act[i]: iadj[iptr[i] .. iptr[i+1])  (global source IDs)
+// CSR + CSC pair over the ACTIVE vertices -- those that still have a live edge), in local
+// numbering: local i in [0, na) is vertex act[i] (act == nullptr: identity, the input)
+//   out-edges of i: oadj[optr[i] .. optr[i+1])  (local destination indices)
+//   in-edges  of i: iadj[iptr[i] .. iptr[i+1])  (local source indices)
 struct WGraph {
     const int32_t* act;
     const int32_t* optr;
@@ -29,6 +29,7 @@ struct DevCounters {
     int4 totals;                     // after a compaction scan: (na', m_out', m_in', 0)
     unsigned long long kept;         // edges kept by Phase 3 (before trim)
     unsigned long long passes;       // Phase-2 passes that did work
+    int nchunks;                     // heavy-row chunks of the current working graph
     int err;                         // validation error
     int grand1;                      // scratch total of an int32 scan
     int changed[RING];               // per-pass changed words

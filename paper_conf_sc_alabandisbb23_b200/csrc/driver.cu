@@ -61,22 +61,26 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     const size_t m = (size_t)p->m_cap;
     p->nw_cap = cdiv(p->n_cap, TPB) * (TPB / WARP) + 1;
     p->bsum_cap = cdiv(std::max<int64_t>(n1, p->nw_cap), SCAN_TILE) + 1;
+    p->chunk_cap = 2 * (int64_t)m / HEAVY_T + 16;
     auto A = [&](void** ptr, size_t bytes) -> cudaError_t { return cudaMalloc(ptr, bytes); };
     cudaError_t e = cudaSuccess;
-    e = e ? e : A((void**)&p->sig_in, n1 * 4);
-    e = e ? e : A((void**)&p->sig_out, n1 * 4);
-    e = e ? e : A((void**)&p->kin, n1 * 4);
-    e = e ? e : A((void**)&p->kout, n1 * 4);
     for (int b = 0; b < 2; b++) {
         e = e ? e : A((void**)&p->act[b], n1 * 4);
+        e = e ? e : A((void**)&p->cin[b], n1 * 4);
+        e = e ? e : A((void**)&p->cout[b], n1 * 4);
         e = e ? e : A((void**)&p->optr[b], n1 * 4);
         e = e ? e : A((void**)&p->iptr[b], n1 * 4);
         e = e ? e : A((void**)&p->oadj[b], m * 4);
         e = e ? e : A((void**)&p->iadj[b], m * 4);
     }
+    e = e ? e : A((void**)&p->kin, n1 * 4);
+    e = e ? e : A((void**)&p->kout, n1 * 4);
+    e = e ? e : A((void**)&p->newidx, n1 * 4);
+    e = e ? e : A((void**)&p->cnt, n1 * sizeof(int2));
     e = e ? e : A((void**)&p->wsum, (size_t)p->nw_cap * sizeof(int4));
     e = e ? e : A((void**)&p->wscan, (size_t)p->nw_cap * sizeof(int4));
     e = e ? e : A((void**)&p->bsum, (size_t)p->bsum_cap * sizeof(int4));
+    e = e ? e : A((void**)&p->chunks, (size_t)p->chunk_cap * sizeof(Chunk));
     e = e ? e : A((void**)&p->dc, sizeof(DevCounters));
     if (e == cudaSuccess) e = cudaMallocHost((void**)&p->hc, sizeof(DevCounters));
     if (e != cudaSuccess) {
@@ -88,13 +92,13 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
 }
 
 void plan_free(Plan* p) {
-    cudaFree(p->sig_in); cudaFree(p->sig_out); cudaFree(p->kin); cudaFree(p->kout);
     for (int b = 0; b < 2; b++) {
-        cudaFree(p->act[b]); cudaFree(p->optr[b]); cudaFree(p->iptr[b]);
-        cudaFree(p->oadj[b]); cudaFree(p->iadj[b]);
+        cudaFree(p->act[b]); cudaFree(p->cin[b]); cudaFree(p->cout[b]);
+        cudaFree(p->optr[b]); cudaFree(p->iptr[b]); cudaFree(p->oadj[b]); cudaFree(p->iadj[b]);
     }
-    cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->dc);
-    cudaFree(p->u_rp); cudaFree(p->u_ci);
+    cudaFree(p->kin); cudaFree(p->kout); cudaFree(p->newidx); cudaFree(p->cnt);
+    cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
+    cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
     if (p->hc) cudaFreeHost(p->hc);
     memset(p, 0, sizeof(*p));
 }
@@ -110,6 +114,19 @@ static int scan_excl(const T* in, int64_t N, T* out, T* grand, void* bsum, int w
     return ECL_SCC_OK;
 }
 
+__global__ void k_iota(int32_t n, int32_t* __restrict__ out) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        out[v] = (int32_t)v;
+}
+// debug snapshot: signatures of the active vertices over the labels of the others
+__global__ void k_scatter_sigs(int32_t na, const int32_t* __restrict__ act, const int32_t* __restrict__ cin,
+                               const int32_t* __restrict__ cout, int32_t* __restrict__ din, int32_t* __restrict__ dout) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= na) return;
+    din[act[i]] = cin[i];
+    dout[act[i]] = cout[i];
+}
+
 // --------------------------------------------------------------------------- steps
 // a1: CSC of the input graph into buffer 0 (in-degree histogram, scan, scatter)
 static int build_csc(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, cudaStream_t s) {
@@ -123,37 +140,44 @@ static int build_csc(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const i
     return ECL_SCC_OK;
 }
 
-// a2/a7/a3: Phase 3 + Trim-1 + compaction into buffer `ob`, then Phase 1 reset
+// a7 + a2 + a3 + a8: Phase 3 edge removal, Trim-1, compaction into buffer `ob` with the
+// Phase-1 reset of the survivors and the final labels of the vertices that leave
 template <bool FIRST, bool TRIM>
-static int remove_and_compact(Plan* p, const WGraph& g, int ob, int32_t* vin, int32_t* vout, cudaStream_t s) {
+static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, const int32_t* cout, int ob,
+                              int32_t* labels, cudaStream_t s) {
     const unsigned grid = grid_for(g.na, TPB);
     const int64_t nw = (int64_t)grid * (TPB / WARP);
     CK(cudaMemsetAsync(&p->dc->kept, 0, sizeof(unsigned long long), s));
-    k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, vin, vout, p->kin, p->kout, &p->dc->kept);
-    k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, vin, vout, p->kin, p->kout, p->wsum);
+    CK(cudaMemsetAsync(&p->dc->nchunks, 0, sizeof(int), s));
+    k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, &p->dc->kept);
+    k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->cnt, p->wsum);
     int r = scan_excl<I3>((const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
     if (r) return r;
-    k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, vin, vout, p->kin, p->kout, p->wscan, &p->dc->totals,
-                                                          p->act[ob], p->optr[ob], p->oadj[ob], p->iptr[ob],
-                                                          p->iadj[ob]);
-    if (!FIRST) k_reset<<<grid, TPB, 0, s>>>(g, vin, vout);
+    k_compact_map<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
+                                              p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
+                                              (Chunk*)p->chunks, &p->dc->nchunks, (int)p->chunk_cap);
+    k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->newidx, p->optr[ob],
+                                                          p->iptr[ob], p->oadj[ob], p->iadj[ob]);
     CK(cudaGetLastError());
     return ECL_SCC_OK;
 }
 
 // a4-a6: Phase 2 to its fixed point.  Passes are enqueued in growing batches; a pass
 // whose predecessor changed nothing exits at once, so over-enqueueing costs only a launch.
-static int propagate(Plan* p, const WGraph& g, int32_t* vin, int32_t* vout, cudaStream_t s, int64_t* passes_out) {
+static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int nchunks, cudaStream_t s,
+                     int64_t* passes_out) {
     CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
     CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
-    const unsigned grid = grid_for(g.na, TPB);
-    const bool compress = (p->flags & ECL_SCC_COMPRESS) != 0;
+    const unsigned ntiles = (unsigned)cdiv(g.na, TILE);
+    const unsigned hgrid = (unsigned)std::min<int64_t>(cdiv(std::max(nchunks, 1), TPB / WARP), 148 * 8);
+    const bool sync = (p->flags & ECL_SCC_SYNC_PASSES) != 0;
     int pass = 0;
     int batch = 2;
     for (;;) {
         for (int k = 0; k < batch; k++, pass++) {
-            if (compress) k_prop<true><<<grid, TPB, 0, s>>>(g, vin, vout, p->dc, pass);
-            else k_prop<false><<<grid, TPB, 0, s>>>(g, vin, vout, p->dc, pass);
+            if (nchunks) k_prop_heavy<<<hgrid, TPB, 0, s>>>((const Chunk*)p->chunks, nchunks, g, cin, cout, p->dc, pass);
+            if (sync) k_prop_tile<true><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0);
+            else k_prop_tile<false><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0);
         }
         CK(cudaGetLastError());
         CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
@@ -168,13 +192,10 @@ static int propagate(Plan* p, const WGraph& g, int32_t* vin, int32_t* vout, cuda
     return ECL_SCC_OK;
 }
 
-// the whole path for one (possibly union) graph
-int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, int32_t* vin,
+// the whole path for one (possibly union) graph; labels_out receives the result
+int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, int32_t* labels,
               cudaStream_t s, ecl_scc_stats* st, int stop_iter, int32_t* dbg_in, int32_t* dbg_out) {
-    int32_t* vout = p->sig_out;
     if (st) memset(st, 0, sizeof(*st));
-    k_init_sig<<<grid_for(n, TPB), TPB, 0, s>>>(n, vin, vout);
-    CK(cudaGetLastError());
     if (!(p->flags & ECL_SCC_NO_VALIDATE) && n > 0) {
         CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
         k_validate<<<std::min<unsigned>(grid_for(std::max<int64_t>(n, nnz), TPB), 148 * 16), TPB, 0, s>>>(n, nnz, rp, ci, &p->dc->err);
@@ -185,27 +206,36 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
     }
     const bool trim = !(p->flags & ECL_SCC_NO_TRIM);
     int iters = 0;
-    if (nnz > 0) {
+    bool stopped = false;
+    if (nnz == 0) {
+        k_iota<<<grid_for(n, TPB), TPB, 0, s>>>(n, labels);      // Alg. 1 l.3-6, nothing to remove
+        CK(cudaGetLastError());
+    } else {
         int r = build_csc(p, n, nnz, rp, ci, s);
         if (r) return r;
         WGraph g{nullptr, rp, ci, p->iptr[0], p->iadj[0], n};
+        const int32_t *cin = nullptr, *cout = nullptr;          // identity (l.3-6) in the input
         int ob = 1;
         for (int iter = 1;; iter++) {
             if (iter > n + 2) return fail(ECL_SCC_ECUDA, "internal: outer loop exceeded n+2 iterations");
-            if (iter == 1) r = trim ? remove_and_compact<true, true>(p, g, ob, vin, vout, s)
-                                    : remove_and_compact<true, false>(p, g, ob, vin, vout, s);
-            else r = trim ? remove_and_compact<false, true>(p, g, ob, vin, vout, s)
-                          : remove_and_compact<false, false>(p, g, ob, vin, vout, s);
+            if (iter == 1) r = trim ? remove_and_compact<true, true>(p, g, cin, cout, ob, labels, s)
+                                    : remove_and_compact<true, false>(p, g, cin, cout, ob, labels, s);
+            else r = trim ? remove_and_compact<false, true>(p, g, cin, cout, ob, labels, s)
+                          : remove_and_compact<false, false>(p, g, cin, cout, ob, labels, s);
             if (r) return r;
             CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
             CK(cudaStreamSynchronize(s));
             const int4 t = p->hc->totals;
+            const int nchunks = p->hc->nchunks;
             if (st && iter >= 2 && iter - 2 < ECL_SCC_TRACE_MAX) st->edges_kept[iter - 2] = (int64_t)p->hc->kept;
             if (t.y != t.z) return fail(ECL_SCC_ECUDA, "internal: CSR/CSC survivor mismatch %d vs %d", t.y, t.z);
+            if (nchunks > p->chunk_cap) return fail(ECL_SCC_ECUDA, "internal: heavy chunk list overflow");
             g = WGraph{p->act[ob], p->optr[ob], p->oadj[ob], p->iptr[ob], p->iadj[ob], t.x};
-            if (t.y == 0) break;
+            cin = p->cin[ob];
+            cout = p->cout[ob];
+            if (t.y == 0) break;                                   // no live edge: done
             int64_t passes = 0;
-            r = propagate(p, g, vin, vout, s, &passes);
+            r = propagate(p, g, p->cin[ob], p->cout[ob], nchunks, s, &passes);
             if (r) return r;
             iters = iter;
             if (st) {
@@ -215,24 +245,23 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
                     st->passes_iter[iter - 1] = passes;
                 }
                 st->passes += passes;
-                // 4(n_p+1) offsets + 12 B/edge + 16 B/vertex (+8 B/vertex compressed)
-                const int64_t per = 4 * ((int64_t)t.x + 1) + 12 * (int64_t)t.y + 16 * (int64_t)t.x +
-                                    ((p->flags & ECL_SCC_COMPRESS) ? 8 * (int64_t)t.x : 0);
-                st->prop_bytes += per * passes;
+                // 4(n_p+1) offsets + 12 B/edge + 16 B/vertex
+                st->prop_bytes += (4 * ((int64_t)t.x + 1) + 12 * (int64_t)t.y + 16 * (int64_t)t.x) * passes;
             }
             if (stop_iter == iter) {
-                CK(cudaMemcpyAsync(dbg_in, vin, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
-                CK(cudaMemcpyAsync(dbg_out, vout, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
-                CK(cudaStreamSynchronize(s));
-                if (st) { st->iterations = iters; st->trace_len = std::min(iters, ECL_SCC_TRACE_MAX); }
-                return ECL_SCC_OK;
+                CK(cudaMemcpyAsync(dbg_in, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+                CK(cudaMemcpyAsync(dbg_out, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+                k_scatter_sigs<<<grid_for(t.x, TPB), TPB, 0, s>>>(t.x, g.act, cin, cout, dbg_in, dbg_out);
+                CK(cudaGetLastError());
+                stopped = true;
+                break;
             }
             ob ^= 1;
         }
     }
-    if (stop_iter > 0) {
-        CK(cudaMemcpyAsync(dbg_in, vin, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
-        CK(cudaMemcpyAsync(dbg_out, vin, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+    if (stop_iter > 0 && !stopped) {
+        CK(cudaMemcpyAsync(dbg_in, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+        CK(cudaMemcpyAsync(dbg_out, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
     }
     if (st) { st->iterations = iters; st->trace_len = std::min(iters, ECL_SCC_TRACE_MAX); }
     CK(cudaStreamSynchronize(s));
@@ -261,8 +290,10 @@ int run_batched(Plan* p, int32_t G, const int32_t* n, const int64_t* nnz, const 
     for (int g = 0; g < G; g++) { N += n[g]; M += nnz[g]; }
     if (!p->u_rp || p->u_n_cap < N) {
         cudaFree(p->u_rp);
-        p->u_rp = nullptr;
-        if (cudaMalloc((void**)&p->u_rp, sizeof(int32_t) * (size_t)(N + 1)) != cudaSuccess) {
+        cudaFree(p->u_lab);
+        p->u_rp = p->u_lab = nullptr;
+        if (cudaMalloc((void**)&p->u_rp, sizeof(int32_t) * (size_t)(N + 1)) != cudaSuccess ||
+            cudaMalloc((void**)&p->u_lab, sizeof(int32_t) * (size_t)(N + 1)) != cudaSuccess) {
             cudaGetLastError();
             return fail(ECL_SCC_ENOMEM, "batched union offsets (%lld vertices)", (long long)N);
         }
@@ -299,12 +330,12 @@ int run_batched(Plan* p, int32_t G, const int32_t* n, const int64_t* nnz, const 
     CK(cudaGetLastError());
     const uint32_t saved = p->flags;
     p->flags |= ECL_SCC_NO_VALIDATE;
-    int r = run_graph(p, (int32_t)N, M, p->u_rp, p->u_ci, p->sig_in, s, st, 0, nullptr, nullptr);
+    int r = run_graph(p, (int32_t)N, M, p->u_rp, p->u_ci, p->u_lab, s, st, 0, nullptr, nullptr);
     p->flags = saved;
     if (r) return r;
     vo = 0;
     for (int g = 0; g < G; g++) {
-        if (n[g] > 0) k_split_labels<<<grid_for(n[g], TPB), TPB, 0, s>>>(n[g], p->sig_in, (int32_t)vo, labels[g]);
+        if (n[g] > 0) k_split_labels<<<grid_for(n[g], TPB), TPB, 0, s>>>(n[g], p->u_lab, (int32_t)vo, labels[g]);
         vo += n[g];
     }
     CK(cudaGetLastError());
@@ -409,8 +440,15 @@ int ecl_scc_debug_run(int32_t n, int64_t nnz, const int32_t* row_ptr, const int3
     ecl_scc_plan_t tmp = nullptr;
     r = ecl_scc_plan_create(n, nnz, flags, &tmp);
     if (r) return r;
-    r = run_graph(&tmp->p, n, nnz, row_ptr, col_idx, tmp->p.sig_in, (cudaStream_t)stream, stats, stop_iter, sig_in,
-                  sig_out);
+    int32_t* lab = nullptr;
+    if (cudaMalloc((void**)&lab, sizeof(int32_t) * (size_t)n) != cudaSuccess) {
+        cudaGetLastError();
+        ecl_scc_plan_destroy(tmp);
+        return fail(ECL_SCC_ENOMEM, "debug_run labels");
+    }
+    r = run_graph(&tmp->p, n, nnz, row_ptr, col_idx, lab, (cudaStream_t)stream, stats, stop_iter, sig_in, sig_out);
+    cudaStreamSynchronize((cudaStream_t)stream);
+    cudaFree(lab);
     cudaStreamSynchronize((cudaStream_t)stream);
     ecl_scc_plan_destroy(tmp);
     return r;

@@ -13,17 +13,23 @@ struct Plan {
     uint32_t flags;
     int32_t n_cap;
     int64_t m_cap;
-    int64_t nw_cap, bsum_cap;
-    int32_t *sig_in, *sig_out;          // v_in / v_out (v_in may be the caller's labels_out)
-    int32_t *kin, *kout;                // kept in/out degree (global-indexed), CSC cursor
-    int32_t *act[2], *optr[2], *iptr[2];// double-buffered compacted working graph
-    int32_t *oadj[2], *iadj[2];
-    int4 *wsum, *wscan;                 // per-warp compaction counts and their prefix
-    void* bsum;                         // scan block totals
-    DevCounters* dc;                    // device counters
-    DevCounters* hc;                    // pinned host mirror
-    int32_t* u_rp;                      // batched: union CSR
+    int64_t nw_cap, bsum_cap, chunk_cap;
+    // double-buffered working graph in local numbering (kernels.cuh "Layout")
+    int32_t *act[2], *cin[2], *cout[2];  // vertex IDs and signatures v_in / v_out
+    int32_t *optr[2], *iptr[2];          // CSR / CSC offsets
+    int32_t *oadj[2], *iadj[2];          // CSR / CSC adjacency
+    int32_t *kin, *kout;                 // kept in/out degree; CSC build cursor
+    int32_t* newidx;                     // old local -> new local (-1: leaves)
+    int2* cnt;                           // per-vertex surviving (out, in) degree
+    int4 *wsum, *wscan;                  // per-warp compaction counts and their prefix
+    void* bsum;                          // scan block totals
+    void* chunks;                        // heavy-row chunks (Chunk[chunk_cap])
+    int32_t *dbg_tmp;                    // unused placeholder
+    DevCounters* dc;                     // device counters
+    DevCounters* hc;                     // pinned host mirror
+    int32_t* u_rp;                       // batched: union CSR and union labels
     int32_t* u_ci;
+    int32_t* u_lab;
     int64_t u_n_cap, u_m_cap;
 };
 
@@ -32,7 +38,7 @@ void clear_err();
 const char* last_err();
 int plan_alloc(Plan* p, int32_t n_max, int64_t m_max);
 void plan_free(Plan* p);
-int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, int32_t* vin,
+int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, int32_t* labels,
               cudaStream_t s, ecl_scc_stats* st, int stop_iter, int32_t* dbg_in, int32_t* dbg_out);
 
 }  // namespace eclscc

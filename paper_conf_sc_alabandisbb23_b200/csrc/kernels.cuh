@@ -1,27 +1,39 @@
 // kernels.cuh -- sm_100a kernels of the ECL-SCC hot path.
 //
 // Citation key: P:n = PAPER.md line n.  Steps:
-//   a1 k_validate, k_indeg, k_csc_scatter       CSR -> CSC transpose of the input
-//   a2/a7 k_keep_count, k_compact_count, k_compact_scatter
-//                                               Phase 3 edge removal
-//                                               fused with one Trim-1 round and the
+//   a1    k_validate, k_indeg, k_csc_scatter    CSR -> CSC transpose of the input
+//   a2/a7 k_keep_count, k_compact_count,        Phase 3 edge removal
+//         k_compact_map, k_compact_scatter      fused with one Trim-1 round and the
 //                                               compaction of CSR and CSC
-//   a3 k_reset                                  Phase 1 for the next iteration
-//   a4-a6 k_prop                                Phase 2 max propagation
+//   a3    (inside k_compact_map)                Phase 1 of the next iteration
+//   a4-a6 k_prop_tile, k_prop_heavy             Phase 2 max propagation with
+//                                               block-local fixed points
+//   a8    (inside k_compact_map)                final labels
+//
+// Layout: after every compaction the working graph is renumbered
+// to LOCAL indices 0..na-1 (stable, so local order = vertex-ID order).  act[i] is the
+// vertex ID of local i, cin[i]/cout[i] its signatures (values are vertex IDs), and
+// optr/oadj (out-edges, CSR) and iptr/iadj (in-edges, CSC) hold local indices.  Later
+// iterations therefore touch small, dense arrays.
 #pragma once
 #include "common.cuh"
 
 namespace eclscc {
 
-// ------------------------------------------------------------------ init / validation
-__global__ void k_init_sig(int32_t n, int32_t* __restrict__ vin, int32_t* __restrict__ vout) {
-    // Alg. 1 l.3-6: v_in <- v_id, v_out <- v_id
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-        vin[v] = (int32_t)v;
-        vout[v] = (int32_t)v;
-    }
-}
+constexpr int TILE = 2048;          // vertices per block-local fixed point
+constexpr int TILE_THREADS = 512;   // threads per tile CTA
+constexpr int VPT = TILE / TILE_THREADS;
+constexpr int HEAVY_T = 64;         // rows longer than this are reduced by k_prop_heavy
+constexpr int CHUNK = 512;          // edges per heavy-row chunk (one warp)
 
+// Heavy-row chunk (a piece of one long adjacency row, one warp each)
+struct Chunk {
+    int32_t i;      // local vertex
+    int32_t dir;    // 0: out-row (pull cout), 1: in-row (pull cin)
+    int32_t beg, end;
+};
+
+// ------------------------------------------------------------------ init / validation
 __global__ void k_validate(int32_t n, int64_t nnz, const int32_t* __restrict__ rp,
                            const int32_t* __restrict__ ci, int* __restrict__ err) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -74,177 +86,136 @@ __global__ void k_csc_scatter(int32_t n, const int32_t* __restrict__ rp, const i
 }
 
 // ------------------------------------------------------------------ Phase 3 predicates
-// keep(u->w) in iteration k >= 2 (P:147 negated): both endpoints carry the same
-// (in, out) pair and that pair is unfinished (in != out).  Evaluated from either end: the
-// row owner's pair (a, b) is passed in, the other endpoint's pair is gathered.
-// In the first removal (FIRST) every edge except a self-loop is kept (DESIGN reading 9).
+// keep(i->k) in iteration >= 2 (P:147 negated): both endpoints carry the same
+// (in, out) pair and that pair is unfinished (in != out; checked once per row via `live`).
+// Evaluated from either end: the row owner's pair (a, b) is passed in, the other
+// endpoint's pair is gathered.  In the first removal (FIRST) every edge except a
+// self-loop is kept (DESIGN reading 9).
 template <bool FIRST>
-__device__ __forceinline__ bool keep_edge(int owner, int a, int other, const int32_t* __restrict__ vin,
-                                          const int32_t* __restrict__ vout, int b) {
+__device__ __forceinline__ bool keep_edge(int owner, int a, int b, int other, const int32_t* __restrict__ cin,
+                                          const int32_t* __restrict__ cout) {
     if (FIRST) return other != owner;
-    return ld_cg(vin + other) == a && ld_cg(vout + other) == b;
+    return __ldg(cin + other) == a && __ldg(cout + other) == b;
 }
-// Trim-1 on the kept graph: a vertex without a kept in-edge or out-edge
+// Trim-1 on the kept graph: no kept in-edge or no kept out-edge
 __device__ __forceinline__ bool trimmed(const int32_t* __restrict__ kin, const int32_t* __restrict__ kout, int x) {
-    return ld_cg(kin + x) == 0 || ld_cg(kout + x) == 0;
+    return __ldg(kin + x) == 0 || __ldg(kout + x) == 0;
 }
 
 struct RowCtx {
-    int v, ob, oe, ib, ie, a, b;
+    int ob, oe, ib, ie, a, b;
     bool valid, live;
 };
 
 template <bool FIRST>
-__device__ __forceinline__ RowCtx load_row(const WGraph& g, int64_t i, const int32_t* __restrict__ vin,
-                                           const int32_t* __restrict__ vout) {
+__device__ __forceinline__ RowCtx load_row(const WGraph& g, int64_t i, const int32_t* __restrict__ cin,
+                                           const int32_t* __restrict__ cout) {
     RowCtx r{};
     r.valid = i < g.na;
     if (r.valid) {
-        r.v = g.act ? g.act[i] : (int)i;
         r.ob = g.optr[i]; r.oe = g.optr[i + 1];
         r.ib = g.iptr[i]; r.ie = g.iptr[i + 1];
-        if (!FIRST) { r.a = ld_cg(vin + r.v); r.b = ld_cg(vout + r.v); }
+        if (!FIRST) { r.a = cin[i]; r.b = cout[i]; }
     }
     r.live = r.valid && (FIRST || r.a != r.b);
     return r;
 }
 
-// kept in/out degree per vertex (global-indexed), plus the number of kept edges
-template <bool FIRST>
-__global__ void k_keep_count(WGraph g, const int32_t* __restrict__ vin, const int32_t* __restrict__ vout,
-                             int32_t* __restrict__ kin, int32_t* __restrict__ kout,
-                             unsigned long long* __restrict__ kept) {
-    const int lane = threadIdx.x & 31;
-    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const RowCtx r = load_row<FIRST>(g, i, vin, vout);
-    int co = 0, ci = 0;
-    if (r.live && r.oe - r.ob <= HEAVY)
-        for (int e = r.ob; e < r.oe; e++) co += keep_edge<FIRST>(r.v, r.a, g.oadj[e], vin, vout, r.b);
-    if (r.live && r.ie - r.ib <= HEAVY)
-        for (int e = r.ib; e < r.ie; e++) ci += keep_edge<FIRST>(r.v, r.a, g.iadj[e], vin, vout, r.b);
-    for (int dir = 0; dir < 2; dir++) {
-        const int rb = dir ? r.ib : r.ob, re = dir ? r.ie : r.oe;
-        const int32_t* adj = dir ? g.iadj : g.oadj;
-        unsigned hm = __ballot_sync(FULL, r.live && re - rb > HEAVY);
-        while (hm) {
-            const int src = __ffs(hm) - 1;
-            hm &= hm - 1;
-            const int sb = __shfl_sync(FULL, rb, src), se = __shfl_sync(FULL, re, src);
-            const int sv = __shfl_sync(FULL, r.v, src), sa = __shfl_sync(FULL, r.a, src);
-            const int sbb = __shfl_sync(FULL, r.b, src);
-            int c = 0;
-            for (int e = sb + lane; e < se; e += WARP) c += keep_edge<FIRST>(sv, sa, adj[e], vin, vout, sbb);
-            c = warp_sum(c);
-            if (lane == src) { if (dir) ci = c; else co = c; }
-        }
-    }
-    if (r.valid) { kin[r.v] = ci; kout[r.v] = co; }
-    const int s = warp_sum(co);
-    if (lane == 0 && s) atomicAdd(kept, (unsigned long long)s);
-}
-
-// surviving (kept and not trimmed) degree of one row; light rows by the lane, heavy rows
-// by the warp
-template <bool FIRST, bool TRIM>
-__device__ __forceinline__ void survivor_counts(const WGraph& g, const RowCtx& r, bool vtrim,
-                                                const int32_t* __restrict__ vin, const int32_t* __restrict__ vout,
-                                                const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
-                                                int lane, int& nout, int& nin) {
-    nout = 0; nin = 0;
-    const bool go = r.live && !vtrim;
-    if (!TRIM) {
-        if (go) { nout = ld_cg(kout + r.v); nin = ld_cg(kin + r.v); }
-        return;
-    }
-    if (go && r.oe - r.ob <= HEAVY)
-        for (int e = r.ob; e < r.oe; e++) {
-            const int w = g.oadj[e];
-            nout += keep_edge<FIRST>(r.v, r.a, w, vin, vout, r.b) && !trimmed(kin, kout, w);
-        }
-    if (go && r.ie - r.ib <= HEAVY)
-        for (int e = r.ib; e < r.ie; e++) {
-            const int u = g.iadj[e];
-            nin += keep_edge<FIRST>(r.v, r.a, u, vin, vout, r.b) && !trimmed(kin, kout, u);
-        }
-    for (int dir = 0; dir < 2; dir++) {
-        const int rb = dir ? r.ib : r.ob, re = dir ? r.ie : r.oe;
-        const int32_t* adj = dir ? g.iadj : g.oadj;
-        unsigned hm = __ballot_sync(FULL, go && re - rb > HEAVY);
-        while (hm) {
-            const int src = __ffs(hm) - 1;
-            hm &= hm - 1;
-            const int sb = __shfl_sync(FULL, rb, src), se = __shfl_sync(FULL, re, src);
-            const int sv = __shfl_sync(FULL, r.v, src), sa = __shfl_sync(FULL, r.a, src);
-            const int sbb = __shfl_sync(FULL, r.b, src);
-            int c = 0;
-            for (int e = sb + lane; e < se; e += WARP) {
-                const int x = adj[e];
-                c += keep_edge<FIRST>(sv, sa, x, vin, vout, sbb) && !trimmed(kin, kout, x);
-            }
-            c = warp_sum(c);
-            if (lane == src) { if (dir) nin = c; else nout = c; }
-        }
-    }
-}
-
-// per-warp totals (alive vertices, surviving out-edges, surviving in-edges)
-template <bool FIRST, bool TRIM>
-__global__ void k_compact_count(WGraph g, const int32_t* __restrict__ vin, const int32_t* __restrict__ vout,
-                                const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
-                                int4* __restrict__ wsum) {
-    const int lane = threadIdx.x & 31;
-    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const RowCtx r = load_row<FIRST>(g, i, vin, vout);
-    const bool vtrim = TRIM && r.live && trimmed(kin, kout, r.v);
-    int nout, nin;
-    survivor_counts<FIRST, TRIM>(g, r, vtrim, vin, vout, kin, kout, lane, nout, nin);
-    const int alive = (nout + nin) > 0;
-    const int sa = warp_sum(alive), so = warp_sum(nout), si = warp_sum(nin);
-    if (lane == 0) wsum[i >> 5] = make_int4(sa, so, si, 0);
-}
-
-// write one row's survivors starting at dst[pos]; light rows by the lane, heavy by the warp
-template <bool FIRST, bool TRIM>
-__device__ __forceinline__ void emit_rows(const int32_t* __restrict__ adj, int rb, int re, bool go, int pos,
-                                          const RowCtx& r, const int32_t* __restrict__ vin,
-                                          const int32_t* __restrict__ vout, const int32_t* __restrict__ kin,
-                                          const int32_t* __restrict__ kout, int32_t* __restrict__ dst, int lane) {
-    if (go && re - rb <= HEAVY) {
-        for (int e = rb; e < re; e++) {
-            const int x = adj[e];
-            if (keep_edge<FIRST>(r.v, r.a, x, vin, vout, r.b) && !(TRIM && trimmed(kin, kout, x))) dst[pos++] = x;
-        }
-    }
+// count edges of one row (light: by the lane, heavy: by the whole warp) that satisfy P
+template <typename P>
+__device__ __forceinline__ int count_row(const int32_t* __restrict__ adj, int rb, int re, bool go, int lane, P pred) {
+    int c = 0;
+    if (go && re - rb <= HEAVY)
+        for (int e = rb; e < re; e++) c += pred(__ldg(adj + e));
     unsigned hm = __ballot_sync(FULL, go && re - rb > HEAVY);
     while (hm) {
         const int src = __ffs(hm) - 1;
         hm &= hm - 1;
         const int sb = __shfl_sync(FULL, rb, src), se = __shfl_sync(FULL, re, src);
-        const int sv = __shfl_sync(FULL, r.v, src), sa = __shfl_sync(FULL, r.a, src);
-        const int sbb = __shfl_sync(FULL, r.b, src);
-        int spos = __shfl_sync(FULL, pos, src);
-        for (int base = sb; base < se; base += WARP) {
-            const int e = base + lane;
-            bool k = false;
-            int x = 0;
-            if (e < se) {
-                x = adj[e];
-                k = keep_edge<FIRST>(sv, sa, x, vin, vout, sbb) && !(TRIM && trimmed(kin, kout, x));
-            }
-            const unsigned bm = __ballot_sync(FULL, k);
-            if (k) dst[spos + __popc(bm & ((1u << lane) - 1))] = x;
-            spos += __popc(bm);
-        }
+        const P bp = pred.bcast(src);
+        int cc = 0;
+        for (int e = sb + lane; e < se; e += WARP) cc += bp(__ldg(adj + e));
+        cc = warp_sum(cc);
+        if (lane == src) c = cc;
     }
+    return c;
 }
 
-// stable compaction: new active list, new CSR/CSC offsets and adjacency
+// predicate objects: evaluated for the row owner's lane; bcast(src) gives lane src's
+// predicate to the whole warp (all lanes must call it)
+template <bool FIRST>
+struct KeepPred {
+    int i, a, b;
+    const int32_t *cin, *cout;
+    __device__ __forceinline__ bool operator()(int k) const { return keep_edge<FIRST>(i, a, b, k, cin, cout); }
+    __device__ __forceinline__ KeepPred bcast(int src) const {
+        KeepPred p = *this;
+        p.i = __shfl_sync(FULL, i, src); p.a = __shfl_sync(FULL, a, src); p.b = __shfl_sync(FULL, b, src);
+        return p;
+    }
+};
 template <bool FIRST, bool TRIM>
-__global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ vin, const int32_t* __restrict__ vout,
-                                  const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
-                                  const int4* __restrict__ wscan, const int4* __restrict__ totals,
-                                  int32_t* __restrict__ act2, int32_t* __restrict__ optr2, int32_t* __restrict__ oadj2,
-                                  int32_t* __restrict__ iptr2, int32_t* __restrict__ iadj2) {
+struct SurvivePred {
+    int i, a, b;
+    const int32_t *cin, *cout, *kin, *kout;
+    __device__ __forceinline__ bool operator()(int k) const {
+        return keep_edge<FIRST>(i, a, b, k, cin, cout) && !(TRIM && trimmed(kin, kout, k));
+    }
+    __device__ __forceinline__ SurvivePred bcast(int src) const {
+        SurvivePred p = *this;
+        p.i = __shfl_sync(FULL, i, src); p.a = __shfl_sync(FULL, a, src); p.b = __shfl_sync(FULL, b, src);
+        return p;
+    }
+};
+
+// kept in/out degree per local vertex, plus the number of kept edges
+template <bool FIRST>
+__global__ void k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+                             int32_t* __restrict__ kin, int32_t* __restrict__ kout,
+                             unsigned long long* __restrict__ kept) {
+    const int lane = threadIdx.x & 31;
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const RowCtx r = load_row<FIRST>(g, i, cin, cout);
+    KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout};
+    const int co = count_row(g.oadj, r.ob, r.oe, r.live, lane, pred);
+    const int ci = count_row(g.iadj, r.ib, r.ie, r.live, lane, pred);
+    if (r.valid) { kin[i] = ci; kout[i] = co; }
+    const int s = warp_sum(co);
+    if (lane == 0 && s) atomicAdd(kept, (unsigned long long)s);
+}
+
+// per-vertex surviving (kept, not trimmed) degrees and per-warp totals (alive, out, in)
+template <bool FIRST, bool TRIM>
+__global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+                                const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
+                                int2* __restrict__ cnt, int4* __restrict__ wsum) {
+    const int lane = threadIdx.x & 31;
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const RowCtx r = load_row<FIRST>(g, i, cin, cout);
+    int nout = 0, nin = 0;
+    if (!TRIM) {
+        if (r.live) { nout = kout[i]; nin = kin[i]; }
+    } else {
+        const bool go = r.live && !trimmed(kin, kout, (int)i);
+        SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
+        nout = count_row(g.oadj, r.ob, r.oe, go, lane, pred);
+        nin = count_row(g.iadj, r.ib, r.ie, go, lane, pred);
+    }
+    if (r.valid) cnt[i] = make_int2(nout, nin);
+    const int alive = (nout + nin) > 0;
+    const int sa = warp_sum(alive), so = warp_sum(nout), si = warp_sum(nin);
+    if (lane == 0) wsum[i >> 5] = make_int4(sa, so, si, 0);
+}
+
+// New numbering, Phase 1 reset of the survivors (rule R2), final labels of
+// the vertices that leave, new offsets, heavy-row chunk list.
+template <bool FIRST>
+__global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+                              const int2* __restrict__ cnt, const int4* __restrict__ wscan,
+                              const int4* __restrict__ totals, int32_t* __restrict__ newidx,
+                              int32_t* __restrict__ act2, int32_t* __restrict__ cin2, int32_t* __restrict__ cout2,
+                              int32_t* __restrict__ optr2, int32_t* __restrict__ iptr2, int32_t* __restrict__ labels,
+                              Chunk* __restrict__ chunks, int* __restrict__ nchunks, int chunk_cap) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i == 0) {
@@ -252,111 +223,219 @@ __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ vin, con
         optr2[t.x] = t.y;
         iptr2[t.x] = t.z;
     }
-    const RowCtx r = load_row<FIRST>(g, i, vin, vout);
-    const bool vtrim = TRIM && r.live && trimmed(kin, kout, r.v);
-    int nout, nin;
-    survivor_counts<FIRST, TRIM>(g, r, vtrim, vin, vout, kin, kout, lane, nout, nin);
-    const int alive = (nout + nin) > 0;
+    const bool valid = i < g.na;
+    int2 c = valid ? cnt[i] : make_int2(0, 0);
+    const int alive = (c.x + c.y) > 0;
     const int4 base = wscan[i >> 5];
-    const int pa = warp_incl_scan(alive, lane) - alive + base.x;
-    const int po = warp_incl_scan(nout, lane) - nout + base.y;
-    const int pi = warp_incl_scan(nin, lane) - nin + base.z;
+    const int j = warp_incl_scan(alive, lane) - alive + base.x;
+    const int po = warp_incl_scan(c.x, lane) - c.x + base.y;
+    const int pi = warp_incl_scan(c.y, lane) - c.y + base.z;
+    if (!valid) return;
+    const int v = g.act ? g.act[i] : (int)i;
     if (alive) {
-        act2[pa] = r.v;
-        optr2[pa] = po;
-        iptr2[pa] = pi;
+        newidx[i] = j;
+        act2[j] = v;
+        cin2[j] = v;        // Phase 1: v_in <- v_id, v_out <- v_id for the unfinished
+        cout2[j] = v;
+        optr2[j] = po;
+        iptr2[j] = pi;
+        for (int dir = 0; dir < 2; dir++) {
+            const int deg = dir ? c.y : c.x, beg = dir ? pi : po;
+            if (deg > HEAVY_T) {
+                const int nc = (deg + CHUNK - 1) / CHUNK;
+                const int at = atomicAdd(nchunks, nc);
+                for (int k = 0; k < nc && at + k < chunk_cap; k++)
+                    chunks[at + k] = Chunk{j, dir, beg + k * CHUNK, min(beg + (k + 1) * CHUNK, beg + deg)};
+            }
+        }
+    } else {
+        newidx[i] = -1;
+        // leaves the working graph: a finished vertex keeps its signature (the SCC's max
+        // ID), an unfinished one is a singleton (its own ID)
+        int lab = v;
+        if (!FIRST) {
+            const int a = cin[i], b = cout[i];
+            if (a == b) lab = a;
+        }
+        labels[v] = lab;
     }
-    const bool go = r.live && !vtrim;
-    emit_rows<FIRST, TRIM>(g.oadj, r.ob, r.oe, go, po, r, vin, vout, kin, kout, oadj2, lane);
-    emit_rows<FIRST, TRIM>(g.iadj, r.ib, r.ie, go, pi, r, vin, vout, kin, kout, iadj2, lane);
 }
 
-// Phase 1 of the next iteration (R2, DESIGN reading 1): unfinished vertices restart from
-// their own ID; this also finalises vertices that just lost their last edge.
-__global__ void k_reset(WGraph g, int32_t* __restrict__ vin, int32_t* __restrict__ vout) {
+// write one row's survivors (as new local indices) starting at dst[pos]
+template <typename P>
+__device__ __forceinline__ void emit_row(const int32_t* __restrict__ adj, int rb, int re, bool go, int pos,
+                                         const int32_t* __restrict__ newidx, int32_t* __restrict__ dst, int lane,
+                                         P pred) {
+    if (go && re - rb <= HEAVY) {
+        for (int e = rb; e < re; e++) {
+            const int x = __ldg(adj + e);
+            if (pred(x)) dst[pos++] = __ldg(newidx + x);
+        }
+    }
+    unsigned hm = __ballot_sync(FULL, go && re - rb > HEAVY);
+    while (hm) {
+        const int src = __ffs(hm) - 1;
+        hm &= hm - 1;
+        const int sb = __shfl_sync(FULL, rb, src), se = __shfl_sync(FULL, re, src);
+        int spos = __shfl_sync(FULL, pos, src);
+        const P bp = pred.bcast(src);
+        for (int base = sb; base < se; base += WARP) {
+            const int e = base + lane;
+            int x = 0;
+            if (e < se) x = __ldg(adj + e);
+            const bool k = (e < se) && bp(x);
+            const unsigned bm = __ballot_sync(FULL, k);
+            if (k) dst[spos + __popc(bm & ((1u << lane) - 1))] = __ldg(newidx + x);
+            spos += __popc(bm);
+        }
+    }
+}
+
+template <bool FIRST, bool TRIM>
+__global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+                                  const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
+                                  const int32_t* __restrict__ newidx, const int32_t* __restrict__ optr2,
+                                  const int32_t* __restrict__ iptr2, int32_t* __restrict__ oadj2,
+                                  int32_t* __restrict__ iadj2) {
+    const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= g.na) return;
-    const int v = g.act ? g.act[i] : (int)i;
-    if (vin[v] != vout[v]) { vin[v] = v; vout[v] = v; }
+    const RowCtx r = load_row<FIRST>(g, i, cin, cout);
+    const int j = r.valid ? newidx[i] : -1;
+    const bool go = j >= 0;
+    int po = 0, pi = 0;
+    if (go) { po = optr2[j]; pi = iptr2[j]; }
+    SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
+    emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred);
+    emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred);
 }
 
 // ------------------------------------------------------------------ Phase 2
-// One global relaxation pass (Alg. 1 l.9-11), pull form: the owner of v gathers
-//   in[v]  <- max(in[v],  in[u])   over live in-edges  u->v   (l.11)
-//   out[v] <- max(out[v], out[w])  over live out-edges v->w   (l.10)
-// With COMPRESS the gathered value is in[in[u]] / out[out[w]].  Values are
-// written in place (owner writes, so no atomics); concurrent readers see the old or the
-// new value, both valid ancestors/descendants (monotone).  A pass that changes
-// nothing observed a consistent snapshot, so it certifies the fixed point.
-//
-// Pass protocol: pass p clears changed[p+1]; it returns at once if pass p-1 changed
-// nothing; otherwise it sets changed[p] if it wrote anything.
-template <bool COMPRESS>
-__global__ void __launch_bounds__(256) k_prop(WGraph g, int32_t* __restrict__ vin, int32_t* __restrict__ vout,
-                                              DevCounters* __restrict__ dc, int pass) {
-    // every pass (also a skipped one) clears its successor's word, so changed[p] is 0
-    // unless pass p itself ran and changed something
-    if (blockIdx.x == 0 && threadIdx.x == 0) dc->changed[(pass + 1) & (RING - 1)] = 0;
-    if (pass > 0 && ld_vol(&dc->changed[(pass - 1) & (RING - 1)]) == 0) return;
-    if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(&dc->passes, 1ull);
+// Pass protocol (shared by the kernels of one pass; `first` marks the first kernel of
+// the pass): pass p clears changed[p+1]; all kernels of pass p return at once if pass
+// p-1 changed nothing; a kernel sets changed[p] if it raised any signature.  A pass that
+// changes nothing observed a consistent snapshot and so certifies the fixed point.
+__device__ __forceinline__ bool pass_begin(DevCounters* dc, int pass, bool first) {
+    if (first && blockIdx.x == 0 && threadIdx.x == 0) dc->changed[(pass + 1) & (RING - 1)] = 0;
+    if (pass > 0 && ld_vol(&dc->changed[(pass - 1) & (RING - 1)]) == 0) return false;
+    if (first && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(&dc->passes, 1ull);
+    return true;
+}
+
+// Heavy rows: one warp per chunk of a long row; the chunk max is folded in with
+// atomicMax (monotone, so concurrent chunks of one row commute).
+__global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ chunks, int nchunks, WGraph g,
+                                                    int32_t* __restrict__ cin, int32_t* __restrict__ cout,
+                                                    DevCounters* __restrict__ dc, int pass) {
+    if (!pass_begin(dc, pass, true)) return;
     const int lane = threadIdx.x & 31;
-    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const bool valid = i < g.na;
-    int v = 0, ob = 0, oe = 0, ib = 0, ie = 0, x0 = 0, y0 = 0;
-    if (valid) {
-        v = g.act ? g.act[i] : (int)i;
-        ob = g.optr[i]; oe = g.optr[i + 1];
-        ib = g.iptr[i]; ie = g.iptr[i + 1];
-        x0 = ld_cg(vin + v);
-        y0 = ld_cg(vout + v);
-    }
-    int x = x0, y = y0;
-    if (valid && ie - ib <= HEAVY)
-        for (int e = ib; e < ie; e++) {
-            int t = ld_cg(vin + g.iadj[e]);
-            if (COMPRESS) t = ld_cg(vin + t);
-            x = max(x, t);
-        }
-    if (valid && oe - ob <= HEAVY)
-        for (int e = ob; e < oe; e++) {
-            int t = ld_cg(vout + g.oadj[e]);
-            if (COMPRESS) t = ld_cg(vout + t);
-            y = max(y, t);
-        }
-    {
-        unsigned hm = __ballot_sync(FULL, valid && ie - ib > HEAVY);
-        while (hm) {
-            const int src = __ffs(hm) - 1;
-            hm &= hm - 1;
-            const int sb = __shfl_sync(FULL, ib, src), se = __shfl_sync(FULL, ie, src);
-            int acc = 0;
-            for (int e = sb + lane; e < se; e += WARP) {
-                int t = ld_cg(vin + g.iadj[e]);
-                if (COMPRESS) t = ld_cg(vin + t);
-                acc = max(acc, t);
-            }
-            acc = warp_max(acc);
-            if (lane == src) x = max(x, acc);
-        }
-        hm = __ballot_sync(FULL, valid && oe - ob > HEAVY);
-        while (hm) {
-            const int src = __ffs(hm) - 1;
-            hm &= hm - 1;
-            const int sb = __shfl_sync(FULL, ob, src), se = __shfl_sync(FULL, oe, src);
-            int acc = 0;
-            for (int e = sb + lane; e < se; e += WARP) {
-                int t = ld_cg(vout + g.oadj[e]);
-                if (COMPRESS) t = ld_cg(vout + t);
-                acc = max(acc, t);
-            }
-            acc = warp_max(acc);
-            if (lane == src) y = max(y, acc);
-        }
-    }
+    const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     bool ch = false;
-    if (x > x0) { vin[v] = x; ch = true; }
-    if (y > y0) { vout[v] = y; ch = true; }
+    for (int64_t c = wid; c < nchunks; c += nw) {
+        const Chunk k = chunks[c];
+        const int32_t* adj = k.dir ? g.iadj : g.oadj;
+        int32_t* sig = k.dir ? cin : cout;
+        int acc = 0;
+        for (int e = k.beg + lane; e < k.end; e += WARP) acc = max(acc, ld_cg(sig + __ldg(adj + e)));
+        acc = warp_max(acc);
+        if (lane == 0 && acc > ld_cg(sig + k.i)) {
+            if (atomicMax(sig + k.i, acc) < acc) ch = true;
+        }
+    }
     if (__any_sync(FULL, ch) && lane == 0) dc->changed[pass & (RING - 1)] = 1;
+}
+
+// Block-local fixed point ("every thread block internally iterates until none of
+// the edges assigned to it propagate any more values").  CTA = tile of TILE consecutive
+// local vertices; its signatures live in shared memory.  Each visit:
+//   1. gather the tile's out-of-tile neighbours from global memory (Alg. 1 l.10-11, pull:
+//      in[v] <- max in[u] over in-edges, out[v] <- max out[w] over out-edges);
+//   2. iterate the intra-tile edges in shared memory until nothing changes;
+//   3. write raised signatures back.
+// Rows longer than HEAVY_T are skipped here (k_prop_heavy folds them in).  Tile order
+// alternates with the pass parity so values can ride the block schedule both ways.
+// SYNC = ablation: no step 2 (one relaxation per pass, "separate kernels").
+template <bool SYNC>
+__global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t* __restrict__ cin,
+                                                            int32_t* __restrict__ cout, DevCounters* __restrict__ dc,
+                                                            int pass, int first) {
+    __shared__ int s_in[TILE], s_out[TILE];
+    if (!pass_begin(dc, pass, first)) return;
+    const int ntiles = (g.na + TILE - 1) / TILE;
+    const int tile = (pass & 1) ? (ntiles - 1 - (int)blockIdx.x) : (int)blockIdx.x;
+    const int base = tile * TILE;
+    const int cnt = min(TILE, g.na - base);
+    const int tid = threadIdx.x;
+
+    int ob[VPT], oe[VPT], ib[VPT], ie[VPT], o_in[VPT], o_out[VPT];
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int v = tid + k * TILE_THREADS;
+        ob[k] = oe[k] = ib[k] = ie[k] = 0;
+        o_in[k] = o_out[k] = 0;
+        if (v < cnt) {
+            const int gi = base + v;
+            ob[k] = __ldg(g.optr + gi); oe[k] = __ldg(g.optr + gi + 1);
+            ib[k] = __ldg(g.iptr + gi); ie[k] = __ldg(g.iptr + gi + 1);
+            o_in[k] = ld_cg(cin + gi);
+            o_out[k] = ld_cg(cout + gi);
+            if (oe[k] - ob[k] > HEAVY_T) { ob[k] = oe[k]; }   // heavy: reduced elsewhere
+            if (ie[k] - ib[k] > HEAVY_T) { ib[k] = ie[k]; }
+        }
+    }
+    // step 1: out-of-tile neighbours (global, L2-coherent loads)
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int v = tid + k * TILE_THREADS;
+        if (v >= cnt) continue;
+        int x = o_in[k], y = o_out[k];
+        for (int e = ib[k]; e < ie[k]; e++) {
+            const int u = __ldg(g.iadj + e);
+            if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) x = max(x, ld_cg(cin + u));
+        }
+        for (int e = ob[k]; e < oe[k]; e++) {
+            const int w = __ldg(g.oadj + e);
+            if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) y = max(y, ld_cg(cout + w));
+        }
+        s_in[v] = x;
+        s_out[v] = y;
+    }
+    __syncthreads();
+    // step 2: intra-tile fixed point in shared memory (owner writes, no atomics)
+    if (!SYNC) {
+        for (;;) {
+            int changed = 0;
+#pragma unroll
+            for (int k = 0; k < VPT; k++) {
+                const int v = tid + k * TILE_THREADS;
+                if (v >= cnt) continue;
+                int x = s_in[v], y = s_out[v];
+                const int x0 = x, y0 = y;
+                for (int e = ib[k]; e < ie[k]; e++) {
+                    const int u = __ldg(g.iadj + e) - base;
+                    if ((unsigned)u < (unsigned)cnt) x = max(x, s_in[u]);
+                }
+                for (int e = ob[k]; e < oe[k]; e++) {
+                    const int w = __ldg(g.oadj + e) - base;
+                    if ((unsigned)w < (unsigned)cnt) y = max(y, s_out[w]);
+                }
+                if (x > x0) { s_in[v] = x; changed = 1; }
+                if (y > y0) { s_out[v] = y; changed = 1; }
+            }
+            if (!__syncthreads_or(changed)) break;
+        }
+    }
+    // step 3: write back
+    int ch = 0;
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int v = tid + k * TILE_THREADS;
+        if (v >= cnt) continue;
+        const int x = s_in[v], y = s_out[v];
+        if (x > o_in[k]) { atomicMax(cin + base + v, x); ch = 1; }
+        if (y > o_out[k]) { atomicMax(cout + base + v, y); ch = 1; }
+    }
+    if (__syncthreads_or(ch) && tid == 0) dc->changed[pass & (RING - 1)] = 1;
 }
 
 }  // namespace eclscc

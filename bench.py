@@ -1,0 +1,341 @@
+"""bench.py -- SCC detection throughput of the B200-native ECL-SCC path.
+
+Contract (driver): ``python bench.py --gpus N --steps K --warmup W`` prints ONE JSON line.
+A "step" is one whole ECL-SCC run (CSC build, trim, every outer iteration, labels) over
+the BASELINE.json workload: at N=1 the 16M-vertex directed mesh sweep graph (configs[3],
+"large directed mesh, 16M vertices"), inputs resident in HBM.  Metric: SCC detection
+Medges/s = nnz / device time / 1e6 (BASELINE.json), plus Mvertices/s (the paper's unit,
+P:208).  For N>1 (torchrun) the same graph is edge-partitioned over the ranks
+(ecl_scc_partitioned, NCCL all-reduce MAX), strong scaling.
+
+``--impl reference`` times the CPU oracle (iterative Tarjan + max relabel, oracle/) on the
+same graph on the host -- the reference arm of this tier (there is no installable
+reference implementation: the paper ships no code).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    "c4": "large directed mesh, 16M vertices, single graph edge-partitioned across 1/2/4/8 GPUs",
+    "c2": "directed 3-D tetrahedral-style mesh sweep graph, 1M vertices, degree~4, many small SCCs",
+    "c3": "R-MAT power-law graph scale 22 (4M vertices, 64M edges), one giant SCC",
+}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="c4", choices=sorted(CONFIGS))
+    ap.add_argument("--order", default="blocked8", choices=["lex", "blocked8"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+def load_graph(args):
+    import gen
+    if args.config in ("c2", "c4"):
+        return gen.config(args.config, order=args.order)
+    return gen.config(args.config)
+
+
+def workload(args, g):
+    w = {"workload": CONFIGS[args.config], "config": args.config, "n": g.n, "nnz": g.nnz,
+         "generator": g.name, "seed": {"c2": 2, "c3": 3, "c4": 4}[args.config]}
+    if args.config in ("c2", "c4"):
+        w["element_order"] = args.order
+    return w
+
+
+# ------------------------------------------------------------------ clocks sampler
+class Clocks:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index, self.samples, self.proc = index, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.samples.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        self.thread.join(timeout=2)
+        sm = [float(s[0]) for s in self.samples if len(s) >= 8 and s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if len(s) >= 8 and s[1].replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for s in self.samples:
+            if len(s) < 8:
+                continue
+            for k, nm in enumerate(names):
+                if s[4 + k].lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------ CPU oracle baseline
+def cpu_oracle_time(g, reps: int = 3):
+    import oracle
+    ts = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        oracle.tarjan_labels(g.row_ptr, g.col_idx)
+        ts.append(time.perf_counter() - t0)
+    return statistics.median(ts)
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def reference_arm(args):
+    """Reference arm: the oracle (O1, iterative Tarjan + max relabel, 1 thread) on the
+    same graph, each step = one full SCC decomposition on the host."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    g = load_graph(args)
+    import oracle
+    oracle.build()
+    for _ in range(args.warmup):
+        oracle.tarjan_labels(g.row_ptr, g.col_idx)
+    ts = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.tarjan_labels(g.row_ptr, g.col_idx)
+        ts.append(time.perf_counter() - t0)
+    t = sum(ts) / len(ts)
+    v = g.nnz / t / 1e6
+    line = {"impl": "reference", "metric": "SCC detection Medges/s", "value": round(v, 3), "unit": "Medges/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+            "data": "synthetic", "config": workload(args, g),
+            "cpu_baseline": {"value": round(v, 3), "unit": "Medges/s", "cores": 1, "kind": "oracle",
+                             "sample": f"full graph ({g.n} vertices, {g.nnz} edges), O1 Tarjan+max-relabel, "
+                                       f"1 of {os.cpu_count()} host threads ({cpu_model()})"},
+            "e2e": {"value": round(v, 3), "unit": "Medges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ our arm
+def roofline_traffic(kernel: str):
+    """dram bytes per launch of the dominant kernel from the committed ncu capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        d = json.load(open(p))
+        return d.get("kernels", {}).get(kernel, {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+def measured_peak():
+    try:
+        d = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def flush_l2(buf):
+    buf.add_(1)     # writes 256 MiB > 126 MB L2
+
+
+def ours(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_alabandisbb23_b200 as E
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    g = load_graph(args)
+    dev = torch.device("cuda", local)
+    flush = torch.zeros(64 * 1024 * 1024, dtype=torch.int32, device=dev)
+
+    if world == 1:
+        rp = torch.from_numpy(g.row_ptr).to(dev)
+        ci = torch.from_numpy(g.col_idx).to(dev)
+        lab = torch.empty(g.n, dtype=torch.int32, device=dev)
+        plan = E.Plan(g.n, g.nnz, E.NO_VALIDATE)
+        plan_t = E.Plan(g.n, g.nnz, E.NO_VALIDATE | E.TIME_STAGES)
+        stream = torch.cuda.current_stream()
+
+        def step(p=plan):
+            return E.ecl_scc(rp, ci, lab, plan=p, stats=True)[1]
+    else:
+        bounds = E.ecl_scc_partition_rows(world, g.row_ptr)
+        rb, re_ = bounds[rank], bounds[rank + 1]
+        lrp = torch.from_numpy((g.row_ptr[rb:re_ + 1] - g.row_ptr[rb]).astype(np.int32)).to(dev)
+        lci = torch.from_numpy(g.col_idx[g.row_ptr[rb]:g.row_ptr[re_]]).to(dev)
+        lab = torch.empty(g.n, dtype=torch.int32, device=dev)
+        uid = [E.get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        comm = E.Comm(world, rank, uid[0])
+        plan_t = None
+
+        def step(p=None):
+            return E.ecl_scc_partitioned(comm, g.n, rb, re_, lrp, lci, lab, stats=True)[1]
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    # correctness guard on the measured configuration: sampled labels vs closed form
+    # (full parity lives in tests/; here: label >= v and label[label] == label)
+    L = lab.cpu().numpy()
+    assert (L >= np.arange(g.n)).all() and (L[L] == L).all(), "bench: invalid labels"
+
+    clocks = Clocks(local)
+    clocks.start()
+    times, stats = [], None
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for _ in range(args.steps):
+        flush_l2(flush)
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record()
+        stats = step()
+        b.record()
+        b.synchronize()
+        times.append(a.elapsed_time(b))
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    # stage breakdown + roofline figures, same workload, stage events on
+    rstats = []
+    if plan_t is not None:
+        for _ in range(max(3, min(args.steps, 5))):
+            flush_l2(flush)
+            rstats.append(step(plan_t))
+    ck = clocks.stop()
+    t_ms = sum(times) / len(times)
+    if world > 1:
+        tt = torch.tensor([t_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_ms = float(tt.item())
+
+    # ---- end to end through the public API with host buffers (pinned H2D + D2H)
+    e2e = None
+    if not args.no_e2e and world == 1:
+        hrp = torch.from_numpy(g.row_ptr).pin_memory()
+        hci = torch.from_numpy(g.col_idx).pin_memory()
+        hlab = torch.empty(g.n, dtype=torch.int32).pin_memory()
+        et = []
+        for k in range(args.warmup + args.steps):
+            flush_l2(flush)
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record()
+            rp.copy_(hrp, non_blocking=True)
+            ci.copy_(hci, non_blocking=True)
+            E.ecl_scc(rp, ci, lab, plan=plan)
+            hlab.copy_(lab, non_blocking=True)
+            b.record()
+            b.synchronize()
+            if k >= args.warmup:
+                et.append(a.elapsed_time(b))
+        te = sum(et) / len(et)
+        e2e = {"value": round(g.nnz / te / 1e3, 3), "unit": "Medges/s", "ms_per_step": round(te, 3),
+               "h2d_bytes_per_step": int(hrp.numel() * 4 + hci.numel() * 4),
+               "d2h_bytes_per_step": int(hlab.numel() * 4)}
+
+    if rank != 0:
+        dist.destroy_process_group() if world > 1 else None
+        return 0
+
+    value = g.nnz / t_ms / 1e3      # one graph (all ranks together), Medges/s
+    peak, peak_src = measured_peak()
+    roof = None
+    if rstats:
+        pb = sum(s["prop_bytes"] for s in rstats) / len(rstats)
+        pms = sum(s["ms_prop"] for s in rstats) / len(rstats)
+        launches = sum(s["passes"] for s in rstats) / len(rstats)
+        achieved = pb / (pms * 1e-3) / 1e9 if pms > 0 else None
+        traffic = roofline_traffic("k_prop_tile")
+        roof = {"bound": "hbm", "kernel": "Phase 2 (k_prop_tile + k_prop_heavy)",
+                "achieved": round(achieved, 1) if achieved else None, "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4) if achieved else None,
+                "traffic": traffic, "peak_source": peak_src,
+                "algorithmic_bytes_per_step": int(pb), "prop_ms_per_step": round(pms, 3),
+                "passes_per_step": launches,
+                "stage_ms": {k: round(sum(s[k] for s in rstats) / len(rstats), 3)
+                             for k in ("ms_ingest", "ms_compact", "ms_prop")}}
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        tc = cpu_oracle_time(g, reps=3)
+        cpu = {"value": round(g.nnz / tc / 1e6, 3), "unit": "Medges/s", "cores": 1, "kind": "oracle",
+               "sample": f"full graph ({g.n} vertices, {g.nnz} edges), O1 iterative Tarjan + max relabel, "
+                         f"median of 3, 1 of {os.cpu_count()} host threads ({cpu_model()})"}
+    line = {
+        "metric": "SCC detection Medges/s", "value": round(value, 3), "unit": "Medges/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t_ms, 4),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "int32", "data": "synthetic",
+        "config": {**workload(args, g), "parallelism": f"edge-partitioned x{world}" if world > 1 else "single GPU",
+                   "l2": "flushed between steps (256 MiB write)", "mvertices_per_s": round(g.n / t_ms / 1e3, 3)},
+        "gpu_launches": int(stats["kernel_launches"]) * args.steps if stats else None,
+        "iterations": stats["iterations"] if stats else None, "passes": stats["passes"] if stats else None,
+        "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": ck,
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return reference_arm(args)
+    return ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

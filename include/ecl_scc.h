@@ -65,6 +65,7 @@ typedef enum {
 #define ECL_SCC_NO_VALIDATE 0x4u  /* skip the device validation pass over row_ptr/col_idx */
 #define ECL_SCC_SYNC_PASSES 0x8u  /* ablation: no block-local iteration, one Jacobi-like
                                      relaxation per global pass ("separate kernels") */
+#define ECL_SCC_TIME_STAGES 0x10u /* record CUDA events around the stages (stats->ms_*) */
 
 #define ECL_SCC_TRACE_MAX 64
 
@@ -79,6 +80,12 @@ typedef struct {
     int64_t passes_iter[ECL_SCC_TRACE_MAX];  /* global passes of Phase 2, per iteration  */
     int64_t prop_bytes;                      /* algorithmic bytes of all Phase-2 passes
                                                 (SURVEY 8(d) accounting)      */
+    int64_t kernel_launches;                 /* kernels this call launched                */
+    /* device time per stage (CUDA events on the call's stream), only with
+       ECL_SCC_TIME_STAGES; 0 otherwise */
+    double ms_ingest;                        /* validation + CSC build                    */
+    double ms_compact;                       /* Phase 3 + trim + compaction + Phase 1     */
+    double ms_prop;                          /* Phase 2 (all passes)                      */
 } ecl_scc_stats;
 
 typedef struct ecl_scc_plan_s* ecl_scc_plan_t;

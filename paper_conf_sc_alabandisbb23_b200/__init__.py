@@ -18,7 +18,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "libeclscc.so")
 
 OK, EINVAL, ERANGE, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED = range(7)
-NO_TRIM, COMPRESS, NO_VALIDATE, SYNC_PASSES = 0x1, 0x2, 0x4, 0x8
+NO_TRIM, COMPRESS, NO_VALIDATE, SYNC_PASSES, TIME_STAGES = 0x1, 0x2, 0x4, 0x8, 0x10
 TRACE_MAX = 64
 
 _lib = None
@@ -35,11 +35,14 @@ class Stats(ctypes.Structure):
                 ("passes", ctypes.c_int64),
                 ("edges_in", ctypes.c_int64 * TRACE_MAX), ("vertices_in", ctypes.c_int64 * TRACE_MAX),
                 ("edges_kept", ctypes.c_int64 * TRACE_MAX), ("passes_iter", ctypes.c_int64 * TRACE_MAX),
-                ("prop_bytes", ctypes.c_int64)]
+                ("prop_bytes", ctypes.c_int64), ("kernel_launches", ctypes.c_int64),
+                ("ms_ingest", ctypes.c_double), ("ms_compact", ctypes.c_double), ("ms_prop", ctypes.c_double)]
 
     def as_dict(self) -> dict:
         k = self.trace_len
         return dict(iterations=self.iterations, passes=self.passes, prop_bytes=self.prop_bytes,
+                    kernel_launches=self.kernel_launches, ms_ingest=self.ms_ingest,
+                    ms_compact=self.ms_compact, ms_prop=self.ms_prop,
                     edges_in=list(self.edges_in[:k]), vertices_in=list(self.vertices_in[:k]),
                     edges_kept=list(self.edges_kept[:max(k - 1, 0)]),
                     passes_iter=list(self.passes_iter[:k]))

@@ -100,16 +100,18 @@ void plan_free(Plan* p) {
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
     cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
     if (p->hc) cudaFreeHost(p->hc);
+    if (p->ev_ok)
+        for (int k = 0; k < 6; k++) cudaEventDestroy(p->ev[k]);
     memset(p, 0, sizeof(*p));
 }
 
 // --------------------------------------------------------------------------- scans
 template <typename T>
-static int scan_excl(const T* in, int64_t N, T* out, T* grand, void* bsum, int write_total, cudaStream_t s) {
+static int scan_excl(Plan* p, const T* in, int64_t N, T* out, T* grand, void* bsum, int write_total, cudaStream_t s) {
     const int64_t nb = std::max<int64_t>(cdiv(N, SCAN_TILE), 1);
-    k_scan_reduce<T><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, N, (T*)bsum);
-    k_scan_top<T><<<1, SCAN_THREADS, 0, s>>>((T*)bsum, nb, grand);
-    k_scan_apply<T><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, N, (T*)bsum, out, grand, write_total);
+    p->launches++; k_scan_reduce<T><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, N, (T*)bsum);
+    p->launches++; k_scan_top<T><<<1, SCAN_THREADS, 0, s>>>((T*)bsum, nb, grand);
+    p->launches++; k_scan_apply<T><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, N, (T*)bsum, out, grand, write_total);
     CK(cudaGetLastError());
     return ECL_SCC_OK;
 }
@@ -131,11 +133,11 @@ __global__ void k_scatter_sigs(int32_t na, const int32_t* __restrict__ act, cons
 // a1: CSC of the input graph into buffer 0 (in-degree histogram, scan, scatter)
 static int build_csc(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, cudaStream_t s) {
     CK(cudaMemsetAsync(p->kin, 0, sizeof(int32_t) * (size_t)(n + 1), s));
-    k_indeg<<<grid_for(nnz, TPB), TPB, 0, s>>>(nnz, ci, p->kin);
-    int r = scan_excl<I1>((const I1*)p->kin, n, (I1*)p->iptr[0], (I1*)&p->dc->grand1, p->bsum, 1, s);
+    p->launches++; k_indeg<<<grid_for(nnz, TPB), TPB, 0, s>>>(nnz, ci, p->kin);
+    int r = scan_excl<I1>(p, (const I1*)p->kin, n, (I1*)p->iptr[0], (I1*)&p->dc->grand1, p->bsum, 1, s);
     if (r) return r;
     CK(cudaMemsetAsync(p->kout, 0, sizeof(int32_t) * (size_t)n, s));
-    k_csc_scatter<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, ci, p->iptr[0], p->kout, p->iadj[0]);
+    p->launches++; k_csc_scatter<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, ci, p->iptr[0], p->kout, p->iadj[0]);
     CK(cudaGetLastError());
     return ECL_SCC_OK;
 }
@@ -149,14 +151,14 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     const int64_t nw = (int64_t)grid * (TPB / WARP);
     CK(cudaMemsetAsync(&p->dc->kept, 0, sizeof(unsigned long long), s));
     CK(cudaMemsetAsync(&p->dc->nchunks, 0, sizeof(int), s));
-    k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, &p->dc->kept);
-    k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->cnt, p->wsum);
-    int r = scan_excl<I3>((const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
+    p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, &p->dc->kept);
+    p->launches++; k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->cnt, p->wsum);
+    int r = scan_excl<I3>(p, (const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
     if (r) return r;
-    k_compact_map<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
+    p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
                                               (Chunk*)p->chunks, &p->dc->nchunks, (int)p->chunk_cap);
-    k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->newidx, p->optr[ob],
+    p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob]);
     CK(cudaGetLastError());
     return ECL_SCC_OK;
@@ -175,9 +177,9 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     int batch = 2;
     for (;;) {
         for (int k = 0; k < batch; k++, pass++) {
-            if (nchunks) k_prop_heavy<<<hgrid, TPB, 0, s>>>((const Chunk*)p->chunks, nchunks, g, cin, cout, p->dc, pass);
-            if (sync) k_prop_tile<true><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0);
-            else k_prop_tile<false><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0);
+            if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>((const Chunk*)p->chunks, nchunks, g, cin, cout, p->dc, pass); }
+            if (sync) { p->launches++; k_prop_tile<true><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0); }
+            else { p->launches++; k_prop_tile<false><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0); }
         }
         CK(cudaGetLastError());
         CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
@@ -192,13 +194,30 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     return ECL_SCC_OK;
 }
 
+// stage timing: events 2k/2k+1 bracket stage k (0 ingest, 1 compaction, 2 Phase 2)
+static void stage_mark(Plan* p, int ev, cudaStream_t s) {
+    if (!(p->flags & ECL_SCC_TIME_STAGES)) return;
+    if (!p->ev_ok) {
+        for (int k = 0; k < 6; k++) cudaEventCreate(&p->ev[k]);
+        p->ev_ok = true;
+    }
+    cudaEventRecord(p->ev[ev], s);
+}
+static double stage_ms(Plan* p, int k) {   // call after a stream sync
+    if (!(p->flags & ECL_SCC_TIME_STAGES) || !p->ev_ok) return 0.0;
+    float ms = 0.f;
+    if (cudaEventElapsedTime(&ms, p->ev[2 * k], p->ev[2 * k + 1]) != cudaSuccess) { cudaGetLastError(); return 0.0; }
+    return (double)ms;
+}
+
 // the whole path for one (possibly union) graph; labels_out receives the result
 int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, int32_t* labels,
               cudaStream_t s, ecl_scc_stats* st, int stop_iter, int32_t* dbg_in, int32_t* dbg_out) {
     if (st) memset(st, 0, sizeof(*st));
+    stage_mark(p, 0, s);
     if (!(p->flags & ECL_SCC_NO_VALIDATE) && n > 0) {
         CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
-        k_validate<<<std::min<unsigned>(grid_for(std::max<int64_t>(n, nnz), TPB), 148 * 16), TPB, 0, s>>>(n, nnz, rp, ci, &p->dc->err);
+        p->launches++; k_validate<<<std::min<unsigned>(grid_for(std::max<int64_t>(n, nnz), TPB), 148 * 16), TPB, 0, s>>>(n, nnz, rp, ci, &p->dc->err);
         CK(cudaGetLastError());
         CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
@@ -208,23 +227,30 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
     int iters = 0;
     bool stopped = false;
     if (nnz == 0) {
-        k_iota<<<grid_for(n, TPB), TPB, 0, s>>>(n, labels);      // Alg. 1 l.3-6, nothing to remove
+        p->launches++; k_iota<<<grid_for(n, TPB), TPB, 0, s>>>(n, labels);      // Alg. 1 l.3-6, nothing to remove
         CK(cudaGetLastError());
     } else {
         int r = build_csc(p, n, nnz, rp, ci, s);
         if (r) return r;
+        stage_mark(p, 1, s);
         WGraph g{nullptr, rp, ci, p->iptr[0], p->iadj[0], n};
         const int32_t *cin = nullptr, *cout = nullptr;          // identity (l.3-6) in the input
         int ob = 1;
         for (int iter = 1;; iter++) {
             if (iter > n + 2) return fail(ECL_SCC_ECUDA, "internal: outer loop exceeded n+2 iterations");
+            stage_mark(p, 2, s);
             if (iter == 1) r = trim ? remove_and_compact<true, true>(p, g, cin, cout, ob, labels, s)
                                     : remove_and_compact<true, false>(p, g, cin, cout, ob, labels, s);
             else r = trim ? remove_and_compact<false, true>(p, g, cin, cout, ob, labels, s)
                           : remove_and_compact<false, false>(p, g, cin, cout, ob, labels, s);
             if (r) return r;
+            stage_mark(p, 3, s);
             CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
             CK(cudaStreamSynchronize(s));
+            if (st) {
+                if (iter == 1) st->ms_ingest += stage_ms(p, 0);
+                st->ms_compact += stage_ms(p, 1);
+            }
             const int4 t = p->hc->totals;
             const int nchunks = p->hc->nchunks;
             if (st && iter >= 2 && iter - 2 < ECL_SCC_TRACE_MAX) st->edges_kept[iter - 2] = (int64_t)p->hc->kept;
@@ -235,8 +261,14 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             cout = p->cout[ob];
             if (t.y == 0) break;                                   // no live edge: done
             int64_t passes = 0;
+            stage_mark(p, 4, s);
             r = propagate(p, g, p->cin[ob], p->cout[ob], nchunks, s, &passes);
             if (r) return r;
+            stage_mark(p, 5, s);
+            if (st && (p->flags & ECL_SCC_TIME_STAGES)) {
+                CK(cudaEventSynchronize(p->ev[5]));
+                st->ms_prop += stage_ms(p, 2);
+            }
             iters = iter;
             if (st) {
                 if (iter - 1 < ECL_SCC_TRACE_MAX) {
@@ -251,7 +283,7 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             if (stop_iter == iter) {
                 CK(cudaMemcpyAsync(dbg_in, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
                 CK(cudaMemcpyAsync(dbg_out, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
-                k_scatter_sigs<<<grid_for(t.x, TPB), TPB, 0, s>>>(t.x, g.act, cin, cout, dbg_in, dbg_out);
+                p->launches++; k_scatter_sigs<<<grid_for(t.x, TPB), TPB, 0, s>>>(t.x, g.act, cin, cout, dbg_in, dbg_out);
                 CK(cudaGetLastError());
                 stopped = true;
                 break;
@@ -263,7 +295,11 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         CK(cudaMemcpyAsync(dbg_in, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
         CK(cudaMemcpyAsync(dbg_out, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
     }
-    if (st) { st->iterations = iters; st->trace_len = std::min(iters, ECL_SCC_TRACE_MAX); }
+    if (st) {
+        st->iterations = iters;
+        st->trace_len = std::min(iters, ECL_SCC_TRACE_MAX);
+        st->kernel_launches = p->launches;
+    }
     CK(cudaStreamSynchronize(s));
     return ECL_SCC_OK;
 }
@@ -288,6 +324,7 @@ int run_batched(Plan* p, int32_t G, const int32_t* n, const int64_t* nnz, const 
                 const int32_t* const* ci, int32_t* const* labels, cudaStream_t s, ecl_scc_stats* st) {
     int64_t N = 0, M = 0;
     for (int g = 0; g < G; g++) { N += n[g]; M += nnz[g]; }
+    p->launches = 0;
     if (!p->u_rp || p->u_n_cap < N) {
         cudaFree(p->u_rp);
         cudaFree(p->u_lab);
@@ -312,34 +349,39 @@ int run_batched(Plan* p, int32_t G, const int32_t* n, const int64_t* nnz, const 
     if (!(p->flags & ECL_SCC_NO_VALIDATE)) {
         CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
         for (int g = 0; g < G; g++)
-            if (n[g] > 0)
+            if (n[g] > 0) {
+                p->launches++;
                 k_validate<<<std::min<unsigned>(grid_for(std::max<int64_t>(n[g], nnz[g]), TPB), 148 * 16), TPB, 0, s>>>(
                     n[g], nnz[g], rp[g], ci[g], &p->dc->err);
+            }
         CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         if (p->hc->err) return fail(ECL_SCC_ERANGE, "invalid CSR in batch");
     }
     int64_t vo = 0, eo = 0;
     for (int g = 0; g < G; g++) {
-        if (n[g] > 0) k_union_rows<<<grid_for(n[g], TPB), TPB, 0, s>>>(n[g], rp[g], (int32_t)vo, (int32_t)eo, p->u_rp);
-        if (nnz[g] > 0) k_union_cols<<<grid_for(nnz[g], TPB), TPB, 0, s>>>(nnz[g], ci[g], (int32_t)vo, p->u_ci + eo);
+        if (n[g] > 0) { p->launches++; k_union_rows<<<grid_for(n[g], TPB), TPB, 0, s>>>(n[g], rp[g], (int32_t)vo, (int32_t)eo, p->u_rp); }
+        if (nnz[g] > 0) { p->launches++; k_union_cols<<<grid_for(nnz[g], TPB), TPB, 0, s>>>(nnz[g], ci[g], (int32_t)vo, p->u_ci + eo); }
         vo += n[g];
         eo += nnz[g];
     }
-    k_set1<<<1, 1, 0, s>>>(p->u_rp + N, (int32_t)M);
+    p->launches++; k_set1<<<1, 1, 0, s>>>(p->u_rp + N, (int32_t)M);
     CK(cudaGetLastError());
     const uint32_t saved = p->flags;
     p->flags |= ECL_SCC_NO_VALIDATE;
     int r = run_graph(p, (int32_t)N, M, p->u_rp, p->u_ci, p->u_lab, s, st, 0, nullptr, nullptr);
     p->flags = saved;
     if (r) return r;
+    const int64_t l0 = p->launches;
     vo = 0;
     for (int g = 0; g < G; g++) {
-        if (n[g] > 0) k_split_labels<<<grid_for(n[g], TPB), TPB, 0, s>>>(n[g], p->u_lab, (int32_t)vo, labels[g]);
+        if (n[g] > 0) { p->launches++; k_split_labels<<<grid_for(n[g], TPB), TPB, 0, s>>>(n[g], p->u_lab, (int32_t)vo, labels[g]); }
         vo += n[g];
     }
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(s));
+    if (st) st->kernel_launches = p->launches;
+    (void)l0;
     return ECL_SCC_OK;
 }
 
@@ -420,6 +462,7 @@ int ecl_scc_async(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t*
         if (r) return r;
         plan = tmp;
     }
+    plan->p.launches = 0;
     r = run_graph(&plan->p, n, nnz, row_ptr, col_idx, labels_out, (cudaStream_t)stream, stats, 0, nullptr, nullptr);
     if (tmp) ecl_scc_plan_destroy(tmp);
     return r;

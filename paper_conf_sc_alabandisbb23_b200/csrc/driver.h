@@ -31,6 +31,9 @@ struct Plan {
     int32_t* u_ci;
     int32_t* u_lab;
     int64_t u_n_cap, u_m_cap;
+    int64_t launches;                    // kernels launched by the current call
+    cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
+    bool ev_ok;
 };
 
 int fail(int status, const char* fmt, ...);

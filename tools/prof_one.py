@@ -1,0 +1,20 @@
+"""One ecl_scc run between cudaProfilerStart/Stop (for ncu --profile-from-start off)."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import gen
+import paper_conf_sc_alabandisbb23_b200 as E
+
+cfg = sys.argv[1] if len(sys.argv) > 1 else "c4"
+order = sys.argv[2] if len(sys.argv) > 2 else "blocked8"
+g = gen.config(cfg, order=order) if cfg in ("c2", "c4") else gen.config(cfg)
+rp = torch.from_numpy(g.row_ptr).cuda(); ci = torch.from_numpy(g.col_idx).cuda()
+lab = torch.empty(g.n, dtype=torch.int32, device="cuda")
+plan = E.Plan(g.n, g.nnz, E.NO_VALIDATE)
+_, st = E.ecl_scc(rp, ci, lab, plan=plan, stats=True)
+torch.cuda.synchronize()
+torch.cuda.cudart().cudaProfilerStart()
+_, st = E.ecl_scc(rp, ci, lab, plan=plan, stats=True)
+torch.cuda.synchronize()
+torch.cuda.cudart().cudaProfilerStop()
+print({k: v for k, v in st.items() if k not in ("edges_kept",)})

@@ -61,11 +61,15 @@ typedef enum {
 
 /* plan flags (DESIGN.md "Readings" and "Kernels") */
 #define ECL_SCC_NO_TRIM 0x1u      /* disable the Trim-1 round run with every edge removal */
-#define ECL_SCC_COMPRESS 0x2u     /* path compression: pull in[in[u]], out[out[w]] */
+/* 0x2u is reserved for path compression, not in this build */
 #define ECL_SCC_NO_VALIDATE 0x4u  /* skip the device validation pass over row_ptr/col_idx */
 #define ECL_SCC_SYNC_PASSES 0x8u  /* ablation: no block-local iteration, one Jacobi-like
                                      relaxation per global pass ("separate kernels") */
 #define ECL_SCC_TIME_STAGES 0x10u /* record CUDA events around the stages (stats->ms_*) */
+#define ECL_SCC_IDENTITY_IDS 0x20u /* propagate the raw vertex IDs instead of the internal
+                                      priorities pi(v) (reading 16); labels are
+                                      identical either way */
+#define ECL_SCC_NO_DIRTY 0x40u    /* ablation: visit every tile in every Phase-2 pass */
 
 #define ECL_SCC_TRACE_MAX 64
 

@@ -18,7 +18,8 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.path.join(_HERE, "libeclscc.so")
 
 OK, EINVAL, ERANGE, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED = range(7)
-NO_TRIM, COMPRESS, NO_VALIDATE, SYNC_PASSES, TIME_STAGES = 0x1, 0x2, 0x4, 0x8, 0x10
+NO_TRIM, NO_VALIDATE, SYNC_PASSES, TIME_STAGES = 0x1, 0x4, 0x8, 0x10
+IDENTITY_IDS, NO_DIRTY = 0x20, 0x40
 TRACE_MAX = 64
 
 _lib = None

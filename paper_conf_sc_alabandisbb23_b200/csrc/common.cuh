@@ -35,6 +35,48 @@ struct DevCounters {
     int changed[RING];               // per-pass changed words
 };
 
+// Internal vertex priorities (reading 16).  The signatures propagate
+// pi(v), a keyed bijection of [0, n): a 4-round Feistel network on 2*half >= log2(n) bits
+// with cycle walking.  With ids == false pi is the identity (the paper's raw IDs).
+struct Prio {
+    uint32_t n, half, mask, ids;
+    uint32_t key[4];
+};
+__host__ __device__ __forceinline__ uint32_t prio_hash(uint32_t x) {
+    x *= 0x9E3779B1u;
+    x ^= x >> 15;
+    x *= 0x85EBCA77u;
+    x ^= x >> 13;
+    return x;
+}
+__host__ __device__ __forceinline__ uint32_t prio_of(const Prio& P, uint32_t v) {
+    if (P.ids) return v;
+    uint32_t x = v;
+    do {
+        uint32_t L = x >> P.half, R = x & P.mask;
+#pragma unroll
+        for (int r = 0; r < 4; r++) {
+            const uint32_t nl = R;
+            R = L ^ (prio_hash(R ^ P.key[r]) & P.mask);
+            L = nl;
+        }
+        x = (L << P.half) | R;
+    } while (x >= P.n);
+    return x;
+}
+inline Prio make_prio(uint32_t n, bool ids) {
+    Prio P{};
+    P.n = n;
+    P.ids = ids ? 1u : 0u;
+    uint32_t bits = 1;
+    while (bits < 32 && (1ull << bits) < (unsigned long long)n) bits++;
+    P.half = (bits + 1) / 2;
+    P.mask = (1u << P.half) - 1u;
+    const uint32_t keys[4] = {0x3C6EF372u, 0xA54FF53Au, 0x510E527Fu, 0x9B05688Cu};
+    for (int r = 0; r < 4; r++) P.key[r] = keys[r];
+    return P;
+}
+
 __device__ __forceinline__ int ld_cg(const int32_t* p) { return __ldcg(p); }
 __device__ __forceinline__ int ld_vol(const int* p) { return *(volatile const int*)p; }
 

@@ -62,6 +62,7 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     p->nw_cap = cdiv(p->n_cap, TPB) * (TPB / WARP) + 1;
     p->bsum_cap = cdiv(std::max<int64_t>(n1, p->nw_cap), SCAN_TILE) + 1;
     p->chunk_cap = 2 * (int64_t)m / HEAVY_T + 16;
+    p->dirty_cap = cdiv(p->n_cap, TILE) + 1;
     auto A = [&](void** ptr, size_t bytes) -> cudaError_t { return cudaMalloc(ptr, bytes); };
     cudaError_t e = cudaSuccess;
     for (int b = 0; b < 2; b++) {
@@ -81,6 +82,7 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     e = e ? e : A((void**)&p->wscan, (size_t)p->nw_cap * sizeof(int4));
     e = e ? e : A((void**)&p->bsum, (size_t)p->bsum_cap * sizeof(int4));
     e = e ? e : A((void**)&p->chunks, (size_t)p->chunk_cap * sizeof(Chunk));
+    e = e ? e : A((void**)&p->dirty, 2 * (size_t)p->dirty_cap);
     e = e ? e : A((void**)&p->dc, sizeof(DevCounters));
     if (e == cudaSuccess) e = cudaMallocHost((void**)&p->hc, sizeof(DevCounters));
     if (e != cudaSuccess) {
@@ -98,6 +100,7 @@ void plan_free(Plan* p) {
     }
     cudaFree(p->kin); cudaFree(p->kout); cudaFree(p->newidx); cudaFree(p->cnt);
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
+    cudaFree(p->dirty);
     cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
     if (p->hc) cudaFreeHost(p->hc);
     if (p->ev_ok)
@@ -146,7 +149,7 @@ static int build_csc(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const i
 // Phase-1 reset of the survivors and the final labels of the vertices that leave
 template <bool FIRST, bool TRIM>
 static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, const int32_t* cout, int ob,
-                              int32_t* labels, cudaStream_t s) {
+                              int32_t* labels, const Prio& P, cudaStream_t s) {
     const unsigned grid = grid_for(g.na, TPB);
     const int64_t nw = (int64_t)grid * (TPB / WARP);
     CK(cudaMemsetAsync(&p->dc->kept, 0, sizeof(unsigned long long), s));
@@ -157,7 +160,7 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     if (r) return r;
     p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
-                                              (Chunk*)p->chunks, &p->dc->nchunks, (int)p->chunk_cap);
+                                              (Chunk*)p->chunks, &p->dc->nchunks, (int)p->chunk_cap, P);
     p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob]);
     CK(cudaGetLastError());
@@ -173,13 +176,23 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     const unsigned ntiles = (unsigned)cdiv(g.na, TILE);
     const unsigned hgrid = (unsigned)std::min<int64_t>(cdiv(std::max(nchunks, 1), TPB / WARP), 148 * 8);
     const bool sync = (p->flags & ECL_SCC_SYNC_PASSES) != 0;
+    // dirty-tile skipping needs every raise to be seen by the tile kernel (no heavy rows)
+    // and a local fixed point per visit (not the SYNC ablation)
+    const bool use_dirty = nchunks == 0 && !sync && !(p->flags & ECL_SCC_NO_DIRTY);
+    uint8_t* D[2] = {p->dirty, p->dirty + p->dirty_cap};
+    if (use_dirty) {
+        CK(cudaMemsetAsync(D[0], 1, ntiles, s));
+        CK(cudaMemsetAsync(D[1], 0, ntiles, s));
+    }
     int pass = 0;
     int batch = 2;
     for (;;) {
         for (int k = 0; k < batch; k++, pass++) {
+            uint8_t* dc_ = use_dirty ? D[pass & 1] : nullptr;
+            uint8_t* dn_ = use_dirty ? D[(pass + 1) & 1] : nullptr;
             if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>((const Chunk*)p->chunks, nchunks, g, cin, cout, p->dc, pass); }
-            if (sync) { p->launches++; k_prop_tile<true><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0); }
-            else { p->launches++; k_prop_tile<false><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0); }
+            if (sync) { p->launches++; k_prop_tile<true><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0, nullptr, nullptr); }
+            else { p->launches++; k_prop_tile<false><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0, dc_, dn_); }
         }
         CK(cudaGetLastError());
         CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
@@ -224,12 +237,15 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         if (p->hc->err) return fail(ECL_SCC_ERANGE, "invalid CSR: offsets not monotone from 0 to nnz, or column outside [0,n)");
     }
     const bool trim = !(p->flags & ECL_SCC_NO_TRIM);
+    const Prio P = make_prio((uint32_t)n, (p->flags & ECL_SCC_IDENTITY_IDS) != 0);
     int iters = 0;
     bool stopped = false;
     if (nnz == 0) {
         p->launches++; k_iota<<<grid_for(n, TPB), TPB, 0, s>>>(n, labels);      // Alg. 1 l.3-6, nothing to remove
         CK(cudaGetLastError());
     } else {
+        // the debug snapshot reads every label slot; start from a defined value
+        if (stop_iter > 0) CK(cudaMemsetAsync(labels, 0, sizeof(int32_t) * (size_t)n, s));
         int r = build_csc(p, n, nnz, rp, ci, s);
         if (r) return r;
         stage_mark(p, 1, s);
@@ -239,10 +255,10 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         for (int iter = 1;; iter++) {
             if (iter > n + 2) return fail(ECL_SCC_ECUDA, "internal: outer loop exceeded n+2 iterations");
             stage_mark(p, 2, s);
-            if (iter == 1) r = trim ? remove_and_compact<true, true>(p, g, cin, cout, ob, labels, s)
-                                    : remove_and_compact<true, false>(p, g, cin, cout, ob, labels, s);
-            else r = trim ? remove_and_compact<false, true>(p, g, cin, cout, ob, labels, s)
-                          : remove_and_compact<false, false>(p, g, cin, cout, ob, labels, s);
+            if (iter == 1) r = trim ? remove_and_compact<true, true>(p, g, cin, cout, ob, labels, P, s)
+                                    : remove_and_compact<true, false>(p, g, cin, cout, ob, labels, P, s);
+            else r = trim ? remove_and_compact<false, true>(p, g, cin, cout, ob, labels, P, s)
+                          : remove_and_compact<false, false>(p, g, cin, cout, ob, labels, P, s);
             if (r) return r;
             stage_mark(p, 3, s);
             CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
@@ -281,14 +297,21 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
                 st->prop_bytes += (4 * ((int64_t)t.x + 1) + 12 * (int64_t)t.y + 16 * (int64_t)t.x) * passes;
             }
             if (stop_iter == iter) {
-                CK(cudaMemcpyAsync(dbg_in, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
-                CK(cudaMemcpyAsync(dbg_out, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+                p->launches++; k_snapshot_left<<<grid_for(n, TPB), TPB, 0, s>>>(n, labels, dbg_in, dbg_out, P);
                 p->launches++; k_scatter_sigs<<<grid_for(t.x, TPB), TPB, 0, s>>>(t.x, g.act, cin, cout, dbg_in, dbg_out);
                 CK(cudaGetLastError());
                 stopped = true;
                 break;
             }
             ob ^= 1;
+        }
+        if (!P.ids && !stopped) {
+            // labels of finished vertices are still max priorities: map to max vertex IDs
+            const unsigned gr = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
+            p->launches++; k_relabel_rep<<<gr, TPB, 0, s>>>(n, labels, p->kin, P);
+            p->launches++; k_relabel_max<<<gr, TPB, 0, s>>>(n, labels, p->kin, P);
+            p->launches++; k_relabel_apply<<<gr, TPB, 0, s>>>(n, labels, p->kin);
+            CK(cudaGetLastError());
         }
     }
     if (stop_iter > 0 && !stopped) {

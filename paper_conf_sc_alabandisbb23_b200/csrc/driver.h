@@ -31,6 +31,8 @@ struct Plan {
     int32_t* u_ci;
     int32_t* u_lab;
     int64_t u_n_cap, u_m_cap;
+    uint8_t* dirty;                      // 2 x dirty_cap tile flags (Phase-2 skipping)
+    int64_t dirty_cap;
     int64_t launches;                    // kernels launched by the current call
     cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
     bool ev_ok;

@@ -209,13 +209,16 @@ __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const
 
 // New numbering, Phase 1 reset of the survivors (rule R2), final labels of
 // the vertices that leave, new offsets, heavy-row chunk list.
+// Survivors restart from their priority pi(v) (reading 16).  A finished vertex leaves
+// with its signature s = max priority of its SCC; with raw IDs that is the label itself,
+// otherwise it is stored as -(s+1) and k_relabel_* turn it into the SCC's max vertex ID.
 template <bool FIRST>
 __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                               const int2* __restrict__ cnt, const int4* __restrict__ wscan,
                               const int4* __restrict__ totals, int32_t* __restrict__ newidx,
                               int32_t* __restrict__ act2, int32_t* __restrict__ cin2, int32_t* __restrict__ cout2,
                               int32_t* __restrict__ optr2, int32_t* __restrict__ iptr2, int32_t* __restrict__ labels,
-                              Chunk* __restrict__ chunks, int* __restrict__ nchunks, int chunk_cap) {
+                              Chunk* __restrict__ chunks, int* __restrict__ nchunks, int chunk_cap, Prio P) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i == 0) {
@@ -235,8 +238,9 @@ __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, const i
     if (alive) {
         newidx[i] = j;
         act2[j] = v;
-        cin2[j] = v;        // Phase 1: v_in <- v_id, v_out <- v_id for the unfinished
-        cout2[j] = v;
+        const int pv = (int)prio_of(P, (uint32_t)v);
+        cin2[j] = pv;       // Phase 1: v_in <- v_id, v_out <- v_id for the unfinished
+        cout2[j] = pv;
         optr2[j] = po;
         iptr2[j] = pi;
         for (int dir = 0; dir < 2; dir++) {
@@ -250,14 +254,44 @@ __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, const i
         }
     } else {
         newidx[i] = -1;
-        // leaves the working graph: a finished vertex keeps its signature (the SCC's max
-        // ID), an unfinished one is a singleton (its own ID)
-        int lab = v;
+        int lab = v;    // unfinished (or trimmed) and edgeless: a singleton SCC
         if (!FIRST) {
             const int a = cin[i], b = cout[i];
-            if (a == b) lab = a;
+            if (a == b) lab = P.ids ? a : -(a + 1);
         }
         labels[v] = lab;
+    }
+}
+
+// Final labels under priorities: an SCC is named by s = max priority; its label is the
+// largest vertex ID with signature s.  rep: the member with pi(v) == s seeds the slot;
+// max: the others fold in with atomicMax; apply: write the label.
+__global__ void k_relabel_rep(int32_t n, int32_t* __restrict__ labels, int32_t* __restrict__ slot, Prio P) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const int l = labels[v];
+        if (l < 0 && (int)prio_of(P, (uint32_t)v) == -l - 1) slot[-l - 1] = (int)v;
+    }
+}
+__global__ void k_relabel_max(int32_t n, const int32_t* __restrict__ labels, int32_t* __restrict__ slot, Prio P) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const int l = labels[v];
+        if (l < 0 && (int)prio_of(P, (uint32_t)v) != -l - 1) atomicMax(slot - l - 1, (int)v);
+    }
+}
+__global__ void k_relabel_apply(int32_t n, int32_t* __restrict__ labels, const int32_t* __restrict__ slot) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const int l = labels[v];
+        if (l < 0) labels[v] = slot[-l - 1];
+    }
+}
+// debug snapshot of the vertices that already left: their (in, out) in priority space
+__global__ void k_snapshot_left(int32_t n, const int32_t* __restrict__ labels, int32_t* __restrict__ din,
+                                int32_t* __restrict__ dout, Prio P) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const int l = labels[v];
+        const int s = l < 0 ? -l - 1 : (int)prio_of(P, (uint32_t)l);
+        din[v] = s;
+        dout[v] = s;
     }
 }
 
@@ -357,15 +391,28 @@ __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ ch
 // SYNC = ablation: no step 2 (one relaxation per pass, "separate kernels").
 template <bool SYNC>
 __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t* __restrict__ cin,
-                                                            int32_t* __restrict__ cout, DevCounters* __restrict__ dc,
-                                                            int pass, int first) {
+                                                               int32_t* __restrict__ cout, DevCounters* __restrict__ dc,
+                                                               int pass, int first, uint8_t* __restrict__ dirty_cur,
+                                                               uint8_t* __restrict__ dirty_next) {
     __shared__ int s_in[TILE], s_out[TILE];
+    __shared__ int s_dirty;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + TILE - 1) / TILE;
     const int tile = (pass & 1) ? (ntiles - 1 - (int)blockIdx.x) : (int)blockIdx.x;
+    const int tid = threadIdx.x;
+    // dirty-tile skipping: a tile whose inputs did not change since its last visit is at
+    // its local fixed point already.  The read flag is cleared here, so after pass p the
+    // buffer read in pass p is all zero and pass p+1 can fill it for pass p+2.
+    if (dirty_cur) {
+        if (tid == 0) {
+            s_dirty = dirty_cur[tile];
+            dirty_cur[tile] = 0;
+        }
+        __syncthreads();
+        if (!s_dirty) return;
+    }
     const int base = tile * TILE;
     const int cnt = min(TILE, g.na - base);
-    const int tid = threadIdx.x;
 
     int ob[VPT], oe[VPT], ib[VPT], ie[VPT], o_in[VPT], o_out[VPT];
 #pragma unroll
@@ -425,15 +472,32 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
             if (!__syncthreads_or(changed)) break;
         }
     }
-    // step 3: write back
+    // step 3: write back; a raised v_in must reach the out-neighbours' tiles, a raised
+    // v_out the in-neighbours' tiles (next pass)
     int ch = 0;
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int v = tid + k * TILE_THREADS;
         if (v >= cnt) continue;
         const int x = s_in[v], y = s_out[v];
-        if (x > o_in[k]) { atomicMax(cin + base + v, x); ch = 1; }
-        if (y > o_out[k]) { atomicMax(cout + base + v, y); ch = 1; }
+        if (x > o_in[k]) {
+            atomicMax(cin + base + v, x);
+            ch = 1;
+            if (dirty_next)
+                for (int e = ob[k]; e < oe[k]; e++) {
+                    const int w = __ldg(g.oadj + e);
+                    if ((unsigned)(w - base) >= (unsigned)cnt) dirty_next[w / TILE] = 1;
+                }
+        }
+        if (y > o_out[k]) {
+            atomicMax(cout + base + v, y);
+            ch = 1;
+            if (dirty_next)
+                for (int e = ib[k]; e < ie[k]; e++) {
+                    const int u = __ldg(g.iadj + e);
+                    if ((unsigned)(u - base) >= (unsigned)cnt) dirty_next[u / TILE] = 1;
+                }
+        }
     }
     if (__syncthreads_or(ch) && tid == 0) dc->changed[pass & (RING - 1)] = 1;
 }

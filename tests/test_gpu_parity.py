@@ -16,6 +16,7 @@ import torch
 import gen
 import oracle
 import paper_conf_sc_alabandisbb23_b200 as E
+from prio_ref import prio
 
 pytestmark = pytest.mark.gpu
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
@@ -35,10 +36,23 @@ def gpu_labels(g, flags=0, plan=None):
     return lab.cpu().numpy(), st
 
 
+def relabel(g, pi):
+    """The same graph with vertex v renamed pi[v] (rows permuted accordingly)."""
+    src = np.repeat(np.arange(g.n), np.diff(g.row_ptr))
+    return gen.from_edges(g.n, np.stack([pi[src], pi[g.col_idx]], 1))
+
+
 def check_trace(g, trim, flags=0, max_iters=None):
-    """GPU per-iteration edge counts and signatures == O2's (same trim rule)."""
-    tr = oracle.ecl_scc(g.row_ptr, g.col_idx, trim=trim)
+    """GPU per-iteration edge counts and signatures == O2's (same trim rule).
+
+    With raw IDs (IDENTITY_IDS) O2 runs on the graph itself.  By default the GPU
+    propagates priorities pi(v) (reading 16), which is Alg. 1 on the graph
+    relabelled by pi: O2 runs on that graph and vertex v is compared at pi(v)."""
     fl = flags | (0 if trim else E.NO_TRIM)
+    ids = bool(fl & E.IDENTITY_IDS)
+    pi = np.arange(g.n) if ids else prio(g.n)
+    og = g if ids else relabel(g, pi)
+    tr = oracle.ecl_scc(og.row_ptr, og.col_idx, trim=trim)
     rp, ci = dev(g)
     _, st = gpu_labels(g, fl)
     k = tr.iterations
@@ -46,19 +60,20 @@ def check_trace(g, trim, flags=0, max_iters=None):
     assert st["edges_in"] == tr.edges_in[:64]
     assert st["edges_kept"] == tr.edges_kept[:max(min(k, 64) - 1, 0)]
     for it in range(1, (k if max_iters is None else min(k, max_iters)) + 1):
-        s = oracle.ecl_scc(g.row_ptr, g.col_idx, trim=trim, snap_iter=it)
+        s = oracle.ecl_scc(og.row_ptr, og.col_idx, trim=trim, snap_iter=it)
         gi, go, _ = E.ecl_scc_debug_run(rp, ci, it, flags=fl)
-        np.testing.assert_array_equal(gi.cpu().numpy(), s.snap_in, err_msg=f"in, iteration {it}")
-        np.testing.assert_array_equal(go.cpu().numpy(), s.snap_out, err_msg=f"out, iteration {it}")
+        np.testing.assert_array_equal(gi.cpu().numpy(), s.snap_in[pi], err_msg=f"in, iteration {it}")
+        np.testing.assert_array_equal(go.cpu().numpy(), s.snap_out[pi], err_msg=f"out, iteration {it}")
 
 
 # ----------------------------------------------------------------- C1: worked example
-@pytest.mark.parametrize("flags", [0, E.COMPRESS, E.SYNC_PASSES])
+@pytest.mark.parametrize("flags", [0, E.SYNC_PASSES, E.NO_DIRTY])
 def test_appendix_a(flags):
+    """The hand-derived worked example (raw IDs, so the golden signatures apply as is)."""
     gold = json.load(open(os.path.join(GOLDEN, "appendix_a.json")))
     g = gen.appendix_a()
     for trim, key in ((False, "r2_no_trim"), (True, "r2_trim1")):
-        fl = flags | (0 if trim else E.NO_TRIM)
+        fl = flags | E.IDENTITY_IDS | (0 if trim else E.NO_TRIM)
         lab, st = gpu_labels(g, fl)
         np.testing.assert_array_equal(lab, gold["labels"])
         exp = gold[key]
@@ -79,22 +94,24 @@ def test_random_small_graphs_labels_and_traces():
         edges = [(rng.randrange(n), rng.randrange(n)) for _ in range(m)]
         g = gen.from_edges(n, edges)
         truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-        for flags in (0, E.NO_TRIM, E.COMPRESS):
+        for flags in (0, E.NO_TRIM, E.IDENTITY_IDS, E.SYNC_PASSES, E.NO_DIRTY):
             lab, _ = gpu_labels(g, flags)
             np.testing.assert_array_equal(lab, truth, err_msg=f"trial {trial} flags {flags}")
         if trial % 10 == 0:
             check_trace(g, trim=True)
             check_trace(g, trim=False)
+            check_trace(g, trim=True, flags=E.IDENTITY_IDS)
 
 
 def test_c1_gnm_2000_8000():
     g = gen.config("c1")
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-    for flags in (0, E.COMPRESS, E.NO_TRIM, E.SYNC_PASSES):
+    for flags in (0, E.IDENTITY_IDS, E.NO_TRIM, E.SYNC_PASSES, E.NO_DIRTY):
         lab, _ = gpu_labels(g, flags)
         np.testing.assert_array_equal(lab, truth)
     check_trace(g, trim=True)
     check_trace(g, trim=False)
+    check_trace(g, trim=True, flags=E.IDENTITY_IDS)
 
 
 # ----------------------------------------------------------------- edge cases
@@ -113,7 +130,7 @@ def test_edge_cases():
     n = 100_000
     perm = np.random.default_rng(1).permutation(n)
     g = gen.from_edges(n, np.stack([perm, np.roll(perm, -1)], 1))
-    for flags in (0, E.COMPRESS):
+    for flags in (0, E.IDENTITY_IDS):
         assert (gpu_labels(g, flags)[0] == n - 1).all()
     # long path (deep DAG): identity
     g = gen.from_edges(n, np.stack([perm[:-1], perm[1:]], 1))
@@ -135,7 +152,7 @@ def test_heavy_vertices():
     dst = np.concatenate([rng.integers(0, n, 20_000), np.full(30_000, 777), rng.integers(0, n, 20_000)])
     g = gen.from_edges(n, np.stack([src, dst], 1))
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-    for flags in (0, E.NO_TRIM, E.COMPRESS):
+    for flags in (0, E.NO_TRIM, E.IDENTITY_IDS):
         np.testing.assert_array_equal(gpu_labels(g, flags)[0], truth)
     check_trace(g, trim=True, max_iters=3)
 
@@ -177,10 +194,13 @@ def test_c2_mesh_1m(order):
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
     lab, st = gpu_labels(g)
     np.testing.assert_array_equal(lab, truth)
+    pi = prio(g.n)
+    tr = oracle.ecl_scc(*(lambda h: (h.row_ptr, h.col_idx))(relabel(g, pi)), trim=True)
+    assert st["edges_in"] == tr.edges_in[:64] and st["iterations"] == tr.iterations
+    lab, st = gpu_labels(g, E.IDENTITY_IDS)
+    np.testing.assert_array_equal(lab, truth)
     tr = oracle.ecl_scc(g.row_ptr, g.col_idx, trim=True)
     assert st["edges_in"] == tr.edges_in[:64] and st["iterations"] == tr.iterations
-    lab, _ = gpu_labels(g, E.COMPRESS)
-    np.testing.assert_array_equal(lab, truth)
 
 
 def test_c3_rmat_scale22():
@@ -190,8 +210,9 @@ def test_c3_rmat_scale22():
     np.testing.assert_array_equal(lab, truth)
 
 
-def test_c4_mesh_16m():
-    g = gen.config("c4")
+@pytest.mark.parametrize("order", ["lex", "blocked8"])
+def test_c4_mesh_16m(order):
+    g = gen.config("c4", order=order)
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
     lab, _ = gpu_labels(g)
     np.testing.assert_array_equal(lab, truth)

@@ -18,19 +18,21 @@ def run(name, g, flags=0, reps=5):
     t = float(np.median(ts))
     print(f"{name:28s} flags={flags} n={g.n} m={g.nnz} t={t:.3f} ms  {g.nnz/t/1e3:.1f} Me/s  iters={st['iterations']} passes={st['passes']} per-iter={st['passes_iter'][:8]} ein={st['edges_in'][:6]}", flush=True)
 
+FLAGS = [0, E.IDENTITY_IDS, E.NO_DIRTY, E.IDENTITY_IDS | E.NO_DIRTY]
+
 if __name__ == "__main__":
     which = sys.argv[1:] or ["c2", "c4", "c3"]
     for w in which:
         if w == "c2":
             for order in ("lex", "blocked8"):
                 g = gen.config("c2", order=order)
-                for fl in (0, E.COMPRESS): run(f"c2 {order}", g, fl)
+                for fl in FLAGS: run(f"c2 {order}", g, fl)
         elif w == "c4":
             for order in ("lex", "blocked8"):
                 g = gen.config("c4", order=order)
-                for fl in (0, E.COMPRESS): run(f"c4 {order}", g, fl)
+                for fl in FLAGS: run(f"c4 {order}", g, fl, reps=3)
         elif w == "c3":
             g = gen.config("c3")
-            for fl in (0, E.COMPRESS): run("c3 rmat22", g, fl)
+            for fl in (0, E.IDENTITY_IDS): run("c3 rmat22", g, fl)
         elif w == "c1":
             run("c1", gen.config("c1"))

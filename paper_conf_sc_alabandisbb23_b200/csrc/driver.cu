@@ -169,8 +169,18 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
 
 // a4-a6: Phase 2 to its fixed point.  Passes are enqueued in growing batches; a pass
 // whose predecessor changed nothing exits at once, so over-enqueueing costs only a launch.
+static int set_kernel_attrs() {
+    static int done = 0;
+    if (done) return ECL_SCC_OK;
+    CK(cudaFuncSetAttribute(k_prop_tile<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TILE_DYN_SMEM));
+    CK(cudaFuncSetAttribute(k_prop_tile<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TILE_DYN_SMEM));
+    done = 1;
+    return ECL_SCC_OK;
+}
+
 static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int nchunks, cudaStream_t s,
                      int64_t* passes_out) {
+    if (int r = set_kernel_attrs()) return r;
     CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
     CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
     const unsigned ntiles = (unsigned)cdiv(g.na, TILE);
@@ -191,8 +201,9 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             uint8_t* dc_ = use_dirty ? D[pass & 1] : nullptr;
             uint8_t* dn_ = use_dirty ? D[(pass + 1) & 1] : nullptr;
             if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>((const Chunk*)p->chunks, nchunks, g, cin, cout, p->dc, pass); }
-            if (sync) { p->launches++; k_prop_tile<true><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0, nullptr, nullptr); }
-            else { p->launches++; k_prop_tile<false><<<ntiles, TILE_THREADS, 0, s>>>(g, cin, cout, p->dc, pass, nchunks == 0, dc_, dn_); }
+            const int full = (pass == 0 || nchunks > 0);
+            if (sync) { p->launches++; k_prop_tile<true><<<ntiles, TILE_THREADS, TILE_DYN_SMEM, s>>>(g, cin, cout, p->dc, pass, nchunks == 0, nullptr, nullptr, 1); }
+            else { p->launches++; k_prop_tile<false><<<ntiles, TILE_THREADS, TILE_DYN_SMEM, s>>>(g, cin, cout, p->dc, pass, nchunks == 0, dc_, dn_, full); }
         }
         CK(cudaGetLastError());
         CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));

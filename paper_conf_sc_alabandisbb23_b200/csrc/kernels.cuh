@@ -381,20 +381,50 @@ __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ ch
 
 // Block-local fixed point ("every thread block internally iterates until none of
 // the edges assigned to it propagate any more values").  CTA = tile of TILE consecutive
-// local vertices; its signatures live in shared memory.  Each visit:
-//   1. gather the tile's out-of-tile neighbours from global memory (Alg. 1 l.10-11, pull:
-//      in[v] <- max in[u] over in-edges, out[v] <- max out[w] over out-edges);
-//   2. iterate the intra-tile edges in shared memory until nothing changes;
-//   3. write raised signatures back.
+// local vertices; thread t owns vertices 4t..4t+3 of the tile.  Each visit:
+//   1. gather the out-of-tile neighbours from global memory (Alg. 1 l.10-11, pull:
+//      in[v] <- max in[u] over in-edges, out[v] <- max out[w] over out-edges) and cache
+//      the intra-tile neighbours as 16-bit slots in shared memory;
+//   2. frontier rounds in shared memory: a vertex whose value rose pushes it to its
+//      intra-tile dependents (in along out-edges, out along in-edges) with shared-memory
+//      atomicMax; a dependent that rose is flagged for the next round.  Work is
+//      proportional to the number of raises, not to rounds x tile size;
+//   3. write raised signatures back and flag the out-of-tile dependents' tiles dirty.
 // Rows longer than HEAVY_T are skipped here (k_prop_heavy folds them in).  Tile order
 // alternates with the pass parity so values can ride the block schedule both ways.
+// full: every vertex starts flagged (first visit of a phase, or heavy rows present).
 // SYNC = ablation: no step 2 (one relaxation per pass, "separate kernels").
+constexpr int SLOTS = 4;                 // cached intra-tile neighbours per vertex and direction
+constexpr uint16_t NOSLOT = 0xFFFF;
+constexpr size_t TILE_DYN_SMEM = TILE * (4 + 4 + 8 + 8);   // values + slots: 48 KiB (+ 8 KiB static flags)
+
+// slots are packed 4 x 16 bit in a 64-bit word (NOSLOT = empty)
+__device__ __forceinline__ void push_slots(unsigned long long nb, int val, int* __restrict__ sig,
+                                           uint8_t* __restrict__ fnext, int& any) {
+#pragma unroll
+    for (int q = 0; q < SLOTS; q++) {
+        const unsigned w = (unsigned)(nb >> (16 * q)) & 0xFFFFu;
+        if (w == NOSLOT) break;
+        if (sig[w] < val && atomicMax(sig + w, val) < val) { fnext[w] = 1; any = 1; }
+    }
+}
+__device__ __forceinline__ void add_slot(unsigned long long& pk, int& ns, unsigned idx) {
+    pk &= ~(0xFFFFull << (16 * ns));
+    pk |= (unsigned long long)idx << (16 * ns);
+    ns++;
+}
+
 template <bool SYNC>
 __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t* __restrict__ cin,
                                                                int32_t* __restrict__ cout, DevCounters* __restrict__ dc,
                                                                int pass, int first, uint8_t* __restrict__ dirty_cur,
-                                                               uint8_t* __restrict__ dirty_next) {
-    __shared__ int s_in[TILE], s_out[TILE];
+                                                               uint8_t* __restrict__ dirty_next, int full) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    int* s_in = (int*)smem_raw;                              // [TILE]
+    int* s_out = s_in + TILE;                                // [TILE]
+    unsigned long long* s_nin = (unsigned long long*)(s_out + TILE);   // [TILE] intra in-neighbours
+    unsigned long long* s_nout = s_nin + TILE;                         // [TILE] intra out-neighbours
+    __shared__ __align__(16) uint8_t s_flag[4][TILE];         // round flags: in x2, out x2
     __shared__ int s_dirty;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + TILE - 1) / TILE;
@@ -415,61 +445,96 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
     const int cnt = min(TILE, g.na - base);
 
     int ob[VPT], oe[VPT], ib[VPT], ie[VPT], o_in[VPT], o_out[VPT];
+    unsigned slow = 0;       // bit k: in-row of vertex k has > SLOTS intra neighbours; bit 4+k: out-row
+    unsigned fin = 0, fout = 0;
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
-        const int v = tid + k * TILE_THREADS;
+        const int v = tid * VPT + k;
         ob[k] = oe[k] = ib[k] = ie[k] = 0;
         o_in[k] = o_out[k] = 0;
+        int x = 0, y = 0;
+        unsigned long long ni = ~0ull, no = ~0ull;
         if (v < cnt) {
             const int gi = base + v;
             ob[k] = __ldg(g.optr + gi); oe[k] = __ldg(g.optr + gi + 1);
             ib[k] = __ldg(g.iptr + gi); ie[k] = __ldg(g.iptr + gi + 1);
+            if (oe[k] - ob[k] > HEAVY_T) ob[k] = oe[k];       // heavy: reduced elsewhere
+            if (ie[k] - ib[k] > HEAVY_T) ib[k] = ie[k];
             o_in[k] = ld_cg(cin + gi);
             o_out[k] = ld_cg(cout + gi);
-            if (oe[k] - ob[k] > HEAVY_T) { ob[k] = oe[k]; }   // heavy: reduced elsewhere
-            if (ie[k] - ib[k] > HEAVY_T) { ib[k] = ie[k]; }
-        }
-    }
-    // step 1: out-of-tile neighbours (global, L2-coherent loads)
-#pragma unroll
-    for (int k = 0; k < VPT; k++) {
-        const int v = tid + k * TILE_THREADS;
-        if (v >= cnt) continue;
-        int x = o_in[k], y = o_out[k];
-        for (int e = ib[k]; e < ie[k]; e++) {
-            const int u = __ldg(g.iadj + e);
-            if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) x = max(x, ld_cg(cin + u));
-        }
-        for (int e = ob[k]; e < oe[k]; e++) {
-            const int w = __ldg(g.oadj + e);
-            if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) y = max(y, ld_cg(cout + w));
-        }
-        s_in[v] = x;
-        s_out[v] = y;
-    }
-    __syncthreads();
-    // step 2: intra-tile fixed point in shared memory (owner writes, no atomics)
-    if (!SYNC) {
-        for (;;) {
-            int changed = 0;
-#pragma unroll
-            for (int k = 0; k < VPT; k++) {
-                const int v = tid + k * TILE_THREADS;
-                if (v >= cnt) continue;
-                int x = s_in[v], y = s_out[v];
-                const int x0 = x, y0 = y;
-                for (int e = ib[k]; e < ie[k]; e++) {
-                    const int u = __ldg(g.iadj + e) - base;
-                    if ((unsigned)u < (unsigned)cnt) x = max(x, s_in[u]);
-                }
-                for (int e = ob[k]; e < oe[k]; e++) {
-                    const int w = __ldg(g.oadj + e) - base;
-                    if ((unsigned)w < (unsigned)cnt) y = max(y, s_out[w]);
-                }
-                if (x > x0) { s_in[v] = x; changed = 1; }
-                if (y > y0) { s_out[v] = y; changed = 1; }
+            x = o_in[k];
+            y = o_out[k];
+            // step 1: out-of-tile neighbours from global memory, intra-tile ones cached
+            int ns = 0;
+            for (int e = ib[k]; e < ie[k]; e++) {
+                const int u = __ldg(g.iadj + e);
+                if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) x = max(x, ld_cg(cin + u));
+                else if (ns < SLOTS) add_slot(ni, ns, (unsigned)(u - base));
+                else slow |= 1u << k;
             }
-            if (!__syncthreads_or(changed)) break;
+            ns = 0;
+            for (int e = ob[k]; e < oe[k]; e++) {
+                const int w = __ldg(g.oadj + e);
+                if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) y = max(y, ld_cg(cout + w));
+                else if (ns < SLOTS) add_slot(no, ns, (unsigned)(w - base));
+                else slow |= 1u << (4 + k);
+            }
+            if (full || x > o_in[k]) fin |= 1u << (8 * k);
+            if (full || y > o_out[k]) fout |= 1u << (8 * k);
+        }
+        if (v < TILE) {
+            s_in[v] = x;
+            s_out[v] = y;
+            s_nin[v] = ni;
+            s_nout[v] = no;
+        }
+    }
+    // round-0 flags: this thread's four vertices in one word per direction
+    ((unsigned*)s_flag[0])[tid] = fin;
+    ((unsigned*)s_flag[2])[tid] = fout;
+    ((unsigned*)s_flag[1])[tid] = 0;
+    ((unsigned*)s_flag[3])[tid] = 0;
+    __syncthreads();
+    // step 2: frontier rounds in shared memory
+    if (!SYNC) {
+        int cur = 0;
+        for (;;) {
+            int any = 0;
+            const unsigned wi = ((unsigned*)s_flag[cur])[tid], wo = ((unsigned*)s_flag[2 + cur])[tid];
+            if (wi | wo) {
+                ((unsigned*)s_flag[cur])[tid] = 0;
+                ((unsigned*)s_flag[2 + cur])[tid] = 0;
+                uint8_t* ni_ = s_flag[cur ^ 1];
+                uint8_t* no_ = s_flag[2 + (cur ^ 1)];
+#pragma unroll
+                for (int k = 0; k < VPT; k++) {
+                    const int v = tid * VPT + k;
+                    if ((wi >> (8 * k)) & 0xFF) {            // v_in rose: push along out-edges
+                        const int val = s_in[v];
+                        push_slots(s_nout[v], val, s_in, ni_, any);
+                        if (slow & (1u << (4 + k)))
+                            for (int e = ob[k]; e < oe[k]; e++) {
+                                const int w = __ldg(g.oadj + e) - base;
+                                if ((unsigned)w < (unsigned)cnt && s_in[w] < val && atomicMax(s_in + w, val) < val) {
+                                    ni_[w] = 1; any = 1;
+                                }
+                            }
+                    }
+                    if ((wo >> (8 * k)) & 0xFF) {            // v_out rose: push along in-edges
+                        const int val = s_out[v];
+                        push_slots(s_nin[v], val, s_out, no_, any);
+                        if (slow & (1u << k))
+                            for (int e = ib[k]; e < ie[k]; e++) {
+                                const int u = __ldg(g.iadj + e) - base;
+                                if ((unsigned)u < (unsigned)cnt && s_out[u] < val && atomicMax(s_out + u, val) < val) {
+                                    no_[u] = 1; any = 1;
+                                }
+                            }
+                    }
+                }
+            }
+            if (!__syncthreads_or(any)) break;
+            cur ^= 1;
         }
     }
     // step 3: write back; a raised v_in must reach the out-neighbours' tiles, a raised
@@ -477,11 +542,11 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
     int ch = 0;
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
-        const int v = tid + k * TILE_THREADS;
+        const int v = tid * VPT + k;
         if (v >= cnt) continue;
         const int x = s_in[v], y = s_out[v];
         if (x > o_in[k]) {
-            atomicMax(cin + base + v, x);
+            cin[base + v] = x;
             ch = 1;
             if (dirty_next)
                 for (int e = ob[k]; e < oe[k]; e++) {
@@ -490,7 +555,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
                 }
         }
         if (y > o_out[k]) {
-            atomicMax(cout + base + v, y);
+            cout[base + v] = y;
             ch = 1;
             if (dirty_next)
                 for (int e = ib[k]; e < ie[k]; e++) {

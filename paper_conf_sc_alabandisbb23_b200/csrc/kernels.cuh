@@ -392,7 +392,9 @@ __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ ch
 //   3. write raised signatures back and flag the out-of-tile dependents' tiles dirty.
 // Rows longer than HEAVY_T are skipped here (k_prop_heavy folds them in).  Tile order
 // alternates with the pass parity so values can ride the block schedule both ways.
-// full: every vertex starts flagged (first visit of a phase, or heavy rows present).
+// full: every vertex starts flagged and step 1 also pulls the intra-tile neighbours'
+// values (first visit of a phase, and every visit when heavy rows exist: an intra-tile
+// edge whose source row is heavy is not in any push list, so it is covered by the pull).
 // SYNC = ablation: no step 2 (one relaxation per pass, "separate kernels").
 constexpr int SLOTS = 4;                 // cached intra-tile neighbours per vertex and direction
 constexpr uint16_t NOSLOT = 0xFFFF;
@@ -468,15 +470,17 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
             int ns = 0;
             for (int e = ib[k]; e < ie[k]; e++) {
                 const int u = __ldg(g.iadj + e);
-                if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) x = max(x, ld_cg(cin + u));
-                else if (ns < SLOTS) add_slot(ni, ns, (unsigned)(u - base));
+                if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) { x = max(x, ld_cg(cin + u)); continue; }
+                if (full) x = max(x, ld_cg(cin + u));   // see "full" above: heavy rows do not push
+                if (ns < SLOTS) add_slot(ni, ns, (unsigned)(u - base));
                 else slow |= 1u << k;
             }
             ns = 0;
             for (int e = ob[k]; e < oe[k]; e++) {
                 const int w = __ldg(g.oadj + e);
-                if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) y = max(y, ld_cg(cout + w));
-                else if (ns < SLOTS) add_slot(no, ns, (unsigned)(w - base));
+                if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) { y = max(y, ld_cg(cout + w)); continue; }
+                if (full) y = max(y, ld_cg(cout + w));
+                if (ns < SLOTS) add_slot(no, ns, (unsigned)(w - base));
                 else slow |= 1u << (4 + k);
             }
             if (full || x > o_in[k]) fin |= 1u << (8 * k);

@@ -385,10 +385,12 @@ __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ ch
 //   1. gather the out-of-tile neighbours from global memory (Alg. 1 l.10-11, pull:
 //      in[v] <- max in[u] over in-edges, out[v] <- max out[w] over out-edges) and cache
 //      the intra-tile neighbours as 16-bit slots in shared memory;
-//   2. frontier rounds in shared memory: a vertex whose value rose pushes it to its
+//   2. frontier propagation in shared memory: a vertex whose value rose pushes it to its
 //      intra-tile dependents (in along out-edges, out along in-edges) with shared-memory
-//      atomicMax; a dependent that rose is flagged for the next round.  Work is
-//      proportional to the number of raises, not to rounds x tile size;
+//      atomicMax, and a dependent that rose is flagged.  Each warp keeps draining the
+//      flags of its own 128 vertices (atomic fetch-and-clear) so chains inside a warp's
+//      region need no block barrier; block rounds repeat until a round does no work.
+//      Work is proportional to the number of raises, not to rounds x tile size;
 //   3. write raised signatures back and flag the out-of-tile dependents' tiles dirty.
 // Rows longer than HEAVY_T are skipped here (k_prop_heavy folds them in).  Tile order
 // alternates with the pass parity so values can ride the block schedule both ways.
@@ -400,14 +402,18 @@ constexpr int SLOTS = 4;                 // cached intra-tile neighbours per ver
 constexpr uint16_t NOSLOT = 0xFFFF;
 constexpr size_t TILE_DYN_SMEM = TILE * (4 + 4 + 8 + 8);   // values + slots: 48 KiB (+ 8 KiB static flags)
 
-// slots are packed 4 x 16 bit in a 64-bit word (NOSLOT = empty)
+// slots are packed 4 x 16 bit in a 64-bit word (NOSLOT = empty).  A raised target w is
+// flagged in its owner's flag word (thread w/4 owns byte w%4).
+__device__ __forceinline__ void flag_set(unsigned* __restrict__ fw, unsigned w) {
+    atomicOr(fw + (w >> 2), 1u << (8 * (w & 3)));
+}
 __device__ __forceinline__ void push_slots(unsigned long long nb, int val, int* __restrict__ sig,
-                                           uint8_t* __restrict__ fnext, int& any) {
+                                           unsigned* __restrict__ fw, int& any) {
 #pragma unroll
     for (int q = 0; q < SLOTS; q++) {
         const unsigned w = (unsigned)(nb >> (16 * q)) & 0xFFFFu;
         if (w == NOSLOT) break;
-        if (sig[w] < val && atomicMax(sig + w, val) < val) { fnext[w] = 1; any = 1; }
+        if (sig[w] < val && atomicMax(sig + w, val) < val) { flag_set(fw, w); any = 1; }
     }
 }
 __device__ __forceinline__ void add_slot(unsigned long long& pk, int& ns, unsigned idx) {
@@ -426,7 +432,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
     int* s_out = s_in + TILE;                                // [TILE]
     unsigned long long* s_nin = (unsigned long long*)(s_out + TILE);   // [TILE] intra in-neighbours
     unsigned long long* s_nout = s_nin + TILE;                         // [TILE] intra out-neighbours
-    __shared__ __align__(16) uint8_t s_flag[4][TILE];         // round flags: in x2, out x2
+    __shared__ unsigned s_fin[TILE_THREADS], s_fout[TILE_THREADS];   // raise flags, byte k = vertex 4t+k
     __shared__ int s_dirty;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + TILE - 1) / TILE;
@@ -493,52 +499,51 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
             s_nout[v] = no;
         }
     }
-    // round-0 flags: this thread's four vertices in one word per direction
-    ((unsigned*)s_flag[0])[tid] = fin;
-    ((unsigned*)s_flag[2])[tid] = fout;
-    ((unsigned*)s_flag[1])[tid] = 0;
-    ((unsigned*)s_flag[3])[tid] = 0;
+    // initial flags: this thread's four vertices in one word per direction
+    s_fin[tid] = fin;
+    s_fout[tid] = fout;
     __syncthreads();
-    // step 2: frontier rounds in shared memory
+    // step 2: frontier propagation in shared memory
     if (!SYNC) {
-        int cur = 0;
         for (;;) {
-            int any = 0;
-            const unsigned wi = ((unsigned*)s_flag[cur])[tid], wo = ((unsigned*)s_flag[2 + cur])[tid];
-            if (wi | wo) {
-                ((unsigned*)s_flag[cur])[tid] = 0;
-                ((unsigned*)s_flag[2 + cur])[tid] = 0;
-                uint8_t* ni_ = s_flag[cur ^ 1];
-                uint8_t* no_ = s_flag[2 + (cur ^ 1)];
+            int worked = 0;
+            for (;;) {                                       // drain this warp's flags
+                const unsigned wi = atomicExch(s_fin + tid, 0u), wo = atomicExch(s_fout + tid, 0u);
+                int any = 0;
+                if (wi | wo) {
+                    worked = 1;
 #pragma unroll
-                for (int k = 0; k < VPT; k++) {
-                    const int v = tid * VPT + k;
-                    if ((wi >> (8 * k)) & 0xFF) {            // v_in rose: push along out-edges
-                        const int val = s_in[v];
-                        push_slots(s_nout[v], val, s_in, ni_, any);
-                        if (slow & (1u << (4 + k)))
-                            for (int e = ob[k]; e < oe[k]; e++) {
-                                const int w = __ldg(g.oadj + e) - base;
-                                if ((unsigned)w < (unsigned)cnt && s_in[w] < val && atomicMax(s_in + w, val) < val) {
-                                    ni_[w] = 1; any = 1;
+                    for (int k = 0; k < VPT; k++) {
+                        const int v = tid * VPT + k;
+                        if ((wi >> (8 * k)) & 0xFF) {        // v_in rose: push along out-edges
+                            const int val = s_in[v];
+                            push_slots(s_nout[v], val, s_in, s_fin, any);
+                            if (slow & (1u << (4 + k)))
+                                for (int e = ob[k]; e < oe[k]; e++) {
+                                    const int w = __ldg(g.oadj + e) - base;
+                                    if ((unsigned)w < (unsigned)cnt && s_in[w] < val && atomicMax(s_in + w, val) < val) {
+                                        flag_set(s_fin, w); any = 1;
+                                    }
                                 }
-                            }
-                    }
-                    if ((wo >> (8 * k)) & 0xFF) {            // v_out rose: push along in-edges
-                        const int val = s_out[v];
-                        push_slots(s_nin[v], val, s_out, no_, any);
-                        if (slow & (1u << k))
-                            for (int e = ib[k]; e < ie[k]; e++) {
-                                const int u = __ldg(g.iadj + e) - base;
-                                if ((unsigned)u < (unsigned)cnt && s_out[u] < val && atomicMax(s_out + u, val) < val) {
-                                    no_[u] = 1; any = 1;
+                        }
+                        if ((wo >> (8 * k)) & 0xFF) {        // v_out rose: push along in-edges
+                            const int val = s_out[v];
+                            push_slots(s_nin[v], val, s_out, s_fout, any);
+                            if (slow & (1u << k))
+                                for (int e = ib[k]; e < ie[k]; e++) {
+                                    const int u = __ldg(g.iadj + e) - base;
+                                    if ((unsigned)u < (unsigned)cnt && s_out[u] < val && atomicMax(s_out + u, val) < val) {
+                                        flag_set(s_fout, u); any = 1;
+                                    }
                                 }
-                            }
+                        }
                     }
                 }
+                __syncwarp();
+                // another pass while this warp raised something (possibly its own vertices)
+                if (!__any_sync(FULL, any)) break;
             }
-            if (!__syncthreads_or(any)) break;
-            cur ^= 1;
+            if (!__syncthreads_or(worked)) break;            // a round with no work: done
         }
     }
     // step 3: write back; a raised v_in must reach the out-neighbours' tiles, a raised

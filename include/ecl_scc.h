@@ -161,6 +161,11 @@ int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_
  * (binary search on the host row_ptr[n+1]); bounds_out[P+1] (host). */
 int ecl_scc_partition_rows(int32_t P, int32_t n, const int32_t* row_ptr_host, int32_t* bounds_out);
 
+/* Diagnostics: kernel event counters of the plan's last run (tile visits, block rounds,
+ * warp drain iterations, vertex pushes, ...); all zero unless the library was built
+ * with -DECL_PROF.  out: 8 host uint64. */
+int ecl_scc_plan_counters(ecl_scc_plan_t plan, uint64_t out[8]);
+
 const char* ecl_scc_status_string(int status);
 const char* ecl_scc_last_error(void); /* thread-local, "" if none */
 int ecl_scc_version(void);            /* 100 * major + minor */

@@ -75,6 +75,7 @@ def lib() -> ctypes.CDLL:
         "ecl_scc_status_string": [ctypes.c_int],
         "ecl_scc_last_error": [],
         "ecl_scc_version": [],
+        "ecl_scc_plan_counters": [vp, vp],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -91,7 +92,7 @@ ABI_SYMBOLS = ("ecl_scc", "ecl_scc_async", "ecl_scc_debug_run", "ecl_scc_plan_cr
                "ecl_scc_plan_destroy", "ecl_scc_batched", "ecl_scc_get_unique_id",
                "ecl_scc_comm_create", "ecl_scc_comm_destroy", "ecl_scc_partitioned",
                "ecl_scc_partitioned_emulated", "ecl_scc_partition_rows", "ecl_scc_status_string",
-               "ecl_scc_last_error", "ecl_scc_version")
+               "ecl_scc_last_error", "ecl_scc_version", "ecl_scc_plan_counters")
 
 
 def status_string(s: int) -> str:
@@ -124,6 +125,12 @@ class Plan:
         h = ctypes.c_void_p()
         _check(lib().ecl_scc_plan_create(n_max, nnz_max, flags, ctypes.byref(h)), "ecl_scc_plan_create")
         self.handle, self.n_max, self.nnz_max, self.flags = h, n_max, nnz_max, flags
+
+    def counters(self) -> list[int]:
+        """Kernel event counters of the last run (non-zero only in -DECL_PROF builds)."""
+        out = (ctypes.c_uint64 * 8)()
+        _check(lib().ecl_scc_plan_counters(self.handle, out), "ecl_scc_plan_counters")
+        return list(out)
 
     def close(self):
         if self.handle:

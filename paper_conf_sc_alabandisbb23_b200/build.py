@@ -32,13 +32,16 @@ def deps() -> list[str]:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    if os.environ.get("ECL_PROF") == "1":
+        force = True
     if not force and os.path.exists(LIB):
         t = os.path.getmtime(LIB)
         if all(os.path.getmtime(d) <= t for d in deps()):
             return LIB
     inc, lib = nccl_dirs()
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC", "-shared",
+    extra = ["-DECL_PROF"] if os.environ.get("ECL_PROF") == "1" else []
+    cmd = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", *extra, "-Xcompiler", "-fPIC", "-shared",
            "-I", os.path.join(ROOT, "include"), "-I", inc, "-o", tmp, *sources(),
            "-L", lib, "-l:libnccl.so.2", f"-Xlinker", f"-rpath={lib}"]
     if verbose:

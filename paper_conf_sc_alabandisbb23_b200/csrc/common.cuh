@@ -33,6 +33,7 @@ struct DevCounters {
     int err;                         // validation error
     int grand1;                      // scratch total of an int32 scan
     int changed[RING];               // per-pass changed words
+    unsigned long long prof[8];      // ECL_PROF builds only: kernel event counters
 };
 
 // Internal vertex priorities (reading 16).  The signatures propagate

@@ -62,7 +62,12 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     p->nw_cap = cdiv(p->n_cap, TPB) * (TPB / WARP) + 1;
     p->bsum_cap = cdiv(std::max<int64_t>(n1, p->nw_cap), SCAN_TILE) + 1;
     p->chunk_cap = 2 * (int64_t)m / HEAVY_T + 16;
-    p->dirty_cap = cdiv(p->n_cap, TILE) + 1;
+    p->dirty_cap = cdiv(p->n_cap, 512) + 1;
+    p->tile = TILE;
+    if (const char* t = getenv("ECL_SCC_TILE")) {      // tuning knob: 512, 1024, 2048, 4096
+        const int v = atoi(t);
+        if (v == 512 || v == 1024 || v == 2048 || v == 4096) p->tile = v;
+    }
     auto A = [&](void** ptr, size_t bytes) -> cudaError_t { return cudaMalloc(ptr, bytes); };
     cudaError_t e = cudaSuccess;
     for (int b = 0; b < 2; b++) {
@@ -169,21 +174,32 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
 
 // a4-a6: Phase 2 to its fixed point.  Passes are enqueued in growing batches; a pass
 // whose predecessor changed nothing exits at once, so over-enqueueing costs only a launch.
-static int set_kernel_attrs() {
+template <int TT>
+static int set_tile_attrs() {
     static int done = 0;
     if (done) return ECL_SCC_OK;
-    CK(cudaFuncSetAttribute(k_prop_tile<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TILE_DYN_SMEM));
-    CK(cudaFuncSetAttribute(k_prop_tile<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)TILE_DYN_SMEM));
+    CK(cudaFuncSetAttribute(k_prop_tile<false, TT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tile_dyn_smem<TT>()));
+    CK(cudaFuncSetAttribute(k_prop_tile<true, TT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tile_dyn_smem<TT>()));
     done = 1;
+    return ECL_SCC_OK;
+}
+
+template <int TT>
+static int launch_tile(Plan* p, bool sync, const WGraph& g, int32_t* cin, int32_t* cout, int pass, int first,
+                       uint8_t* dcur, uint8_t* dnext, int full, cudaStream_t s) {
+    if (int r = set_tile_attrs<TT>()) return r;
+    const unsigned ntiles = (unsigned)cdiv(g.na, TT);
+    p->launches++;
+    if (sync) k_prop_tile<true, TT><<<ntiles, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, nullptr, nullptr, 1);
+    else k_prop_tile<false, TT><<<ntiles, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, dcur, dnext, full);
     return ECL_SCC_OK;
 }
 
 static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int nchunks, cudaStream_t s,
                      int64_t* passes_out) {
-    if (int r = set_kernel_attrs()) return r;
     CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
     CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
-    const unsigned ntiles = (unsigned)cdiv(g.na, TILE);
+    const unsigned ntiles = (unsigned)cdiv(g.na, p->tile);
     const unsigned hgrid = (unsigned)std::min<int64_t>(cdiv(std::max(nchunks, 1), TPB / WARP), 148 * 8);
     const bool sync = (p->flags & ECL_SCC_SYNC_PASSES) != 0;
     // dirty-tile skipping needs every raise to be seen by the tile kernel (no heavy rows)
@@ -202,8 +218,14 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             uint8_t* dn_ = use_dirty ? D[(pass + 1) & 1] : nullptr;
             if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>((const Chunk*)p->chunks, nchunks, g, cin, cout, p->dc, pass); }
             const int full = (pass == 0 || nchunks > 0);
-            if (sync) { p->launches++; k_prop_tile<true><<<ntiles, TILE_THREADS, TILE_DYN_SMEM, s>>>(g, cin, cout, p->dc, pass, nchunks == 0, nullptr, nullptr, 1); }
-            else { p->launches++; k_prop_tile<false><<<ntiles, TILE_THREADS, TILE_DYN_SMEM, s>>>(g, cin, cout, p->dc, pass, nchunks == 0, dc_, dn_, full); }
+            int r = ECL_SCC_OK;
+            switch (p->tile) {
+                case 512: r = launch_tile<512>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, s); break;
+                case 1024: r = launch_tile<1024>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, s); break;
+                case 4096: r = launch_tile<4096>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, s); break;
+                default: r = launch_tile<2048>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, s); break;
+            }
+            if (r) return r;
         }
         CK(cudaGetLastError());
         CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
@@ -238,6 +260,7 @@ static double stage_ms(Plan* p, int k) {   // call after a stream sync
 int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, int32_t* labels,
               cudaStream_t s, ecl_scc_stats* st, int stop_iter, int32_t* dbg_in, int32_t* dbg_out) {
     if (st) memset(st, 0, sizeof(*st));
+    CK(cudaMemsetAsync(p->dc->prof, 0, sizeof(p->dc->prof), s));
     stage_mark(p, 0, s);
     if (!(p->flags & ECL_SCC_NO_VALIDATE) && n > 0) {
         CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
@@ -470,6 +493,13 @@ int ecl_scc_plan_create(int32_t n_max, int64_t nnz_max, uint32_t flags, ecl_scc_
         return r;
     }
     *out = h;
+    return ECL_SCC_OK;
+}
+
+int ecl_scc_plan_counters(ecl_scc_plan_t plan, uint64_t out[8]) {
+    clear_err();
+    if (!plan || !out) return fail(ECL_SCC_EINVAL, "plan_counters: bad arguments");
+    CK(cudaMemcpy(out, plan->p.dc->prof, sizeof(plan->p.dc->prof), cudaMemcpyDeviceToHost));
     return ECL_SCC_OK;
 }
 

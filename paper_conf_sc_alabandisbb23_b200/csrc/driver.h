@@ -33,6 +33,7 @@ struct Plan {
     int64_t u_n_cap, u_m_cap;
     uint8_t* dirty;                      // 2 x dirty_cap tile flags (Phase-2 skipping)
     int64_t dirty_cap;
+    int tile;                            // Phase-2 tile size (vertices per CTA)
     int64_t launches;                    // kernels launched by the current call
     cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
     bool ev_ok;

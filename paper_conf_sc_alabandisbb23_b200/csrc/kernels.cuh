@@ -398,9 +398,15 @@ __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ ch
 // values (first visit of a phase, and every visit when heavy rows exist: an intra-tile
 // edge whose source row is heavy is not in any push list, so it is covered by the pull).
 // SYNC = ablation: no step 2 (one relaxation per pass, "separate kernels").
+#ifdef ECL_PROF
+#define PROF_ADD(dc, k, v) atomicAdd(&(dc)->prof[k], (unsigned long long)(v))
+#else
+#define PROF_ADD(dc, k, v) ((void)0)
+#endif
 constexpr int SLOTS = 4;                 // cached intra-tile neighbours per vertex and direction
 constexpr uint16_t NOSLOT = 0xFFFF;
-constexpr size_t TILE_DYN_SMEM = TILE * (4 + 4 + 8 + 8);   // values + slots: 48 KiB (+ 8 KiB static flags)
+template <int TT>
+constexpr size_t tile_dyn_smem() { return (size_t)TT * (4 + 4 + 8 + 8); }   // values + slots
 
 // slots are packed 4 x 16 bit in a 64-bit word (NOSLOT = empty).  A raised target w is
 // flagged in its owner's flag word (thread w/4 owns byte w%4).
@@ -422,20 +428,20 @@ __device__ __forceinline__ void add_slot(unsigned long long& pk, int& ns, unsign
     ns++;
 }
 
-template <bool SYNC>
-__global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t* __restrict__ cin,
+template <bool SYNC, int TT>
+__global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGraph g, int32_t* __restrict__ cin,
                                                                int32_t* __restrict__ cout, DevCounters* __restrict__ dc,
                                                                int pass, int first, uint8_t* __restrict__ dirty_cur,
                                                                uint8_t* __restrict__ dirty_next, int full) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    int* s_in = (int*)smem_raw;                              // [TILE]
-    int* s_out = s_in + TILE;                                // [TILE]
-    unsigned long long* s_nin = (unsigned long long*)(s_out + TILE);   // [TILE] intra in-neighbours
-    unsigned long long* s_nout = s_nin + TILE;                         // [TILE] intra out-neighbours
-    __shared__ unsigned s_fin[TILE_THREADS], s_fout[TILE_THREADS];   // raise flags, byte k = vertex 4t+k
+    int* s_in = (int*)smem_raw;                              // [TT]
+    int* s_out = s_in + TT;                                // [TT]
+    unsigned long long* s_nin = (unsigned long long*)(s_out + TT);   // [TT] intra in-neighbours
+    unsigned long long* s_nout = s_nin + TT;                         // [TT] intra out-neighbours
+    __shared__ unsigned s_fin[(TT / VPT)], s_fout[(TT / VPT)];   // raise flags, byte k = vertex 4t+k
     __shared__ int s_dirty;
     if (!pass_begin(dc, pass, first)) return;
-    const int ntiles = (g.na + TILE - 1) / TILE;
+    const int ntiles = (g.na + TT - 1) / TT;
     const int tile = (pass & 1) ? (ntiles - 1 - (int)blockIdx.x) : (int)blockIdx.x;
     const int tid = threadIdx.x;
     // dirty-tile skipping: a tile whose inputs did not change since its last visit is at
@@ -449,8 +455,8 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
         __syncthreads();
         if (!s_dirty) return;
     }
-    const int base = tile * TILE;
-    const int cnt = min(TILE, g.na - base);
+    const int base = tile * TT;
+    const int cnt = min(TT, g.na - base);
 
     int ob[VPT], oe[VPT], ib[VPT], ie[VPT], o_in[VPT], o_out[VPT];
     unsigned slow = 0;       // bit k: in-row of vertex k has > SLOTS intra neighbours; bit 4+k: out-row
@@ -492,13 +498,14 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
             if (full || x > o_in[k]) fin |= 1u << (8 * k);
             if (full || y > o_out[k]) fout |= 1u << (8 * k);
         }
-        if (v < TILE) {
+        if (v < TT) {
             s_in[v] = x;
             s_out[v] = y;
             s_nin[v] = ni;
             s_nout[v] = no;
         }
     }
+    if (tid == 0) PROF_ADD(dc, 0, 1);                         // tile visits
     // initial flags: this thread's four vertices in one word per direction
     s_fin[tid] = fin;
     s_fout[tid] = fout;
@@ -507,11 +514,14 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
     if (!SYNC) {
         for (;;) {
             int worked = 0;
+            if (tid == 0) PROF_ADD(dc, 1, 1);                 // block rounds
             for (;;) {                                       // drain this warp's flags
+                if ((tid & 31) == 0) PROF_ADD(dc, 2, 1);      // warp drain iterations
                 const unsigned wi = atomicExch(s_fin + tid, 0u), wo = atomicExch(s_fout + tid, 0u);
                 int any = 0;
                 if (wi | wo) {
                     worked = 1;
+                    PROF_ADD(dc, 3, __popc(wi) + __popc(wo));   // vertex pushes
 #pragma unroll
                     for (int k = 0; k < VPT; k++) {
                         const int v = tid * VPT + k;
@@ -560,7 +570,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
             if (dirty_next)
                 for (int e = ob[k]; e < oe[k]; e++) {
                     const int w = __ldg(g.oadj + e);
-                    if ((unsigned)(w - base) >= (unsigned)cnt) dirty_next[w / TILE] = 1;
+                    if ((unsigned)(w - base) >= (unsigned)cnt) dirty_next[w / TT] = 1;
                 }
         }
         if (y > o_out[k]) {
@@ -569,7 +579,7 @@ __global__ void __launch_bounds__(TILE_THREADS, 2) k_prop_tile(WGraph g, int32_t
             if (dirty_next)
                 for (int e = ib[k]; e < ie[k]; e++) {
                     const int u = __ldg(g.iadj + e);
-                    if ((unsigned)(u - base) >= (unsigned)cnt) dirty_next[u / TILE] = 1;
+                    if ((unsigned)(u - base) >= (unsigned)cnt) dirty_next[u / TT] = 1;
                 }
         }
     }

@@ -18,3 +18,4 @@ _, st = E.ecl_scc(rp, ci, lab, plan=plan, stats=True)
 torch.cuda.synchronize()
 torch.cuda.cudart().cudaProfilerStop()
 print({k: v for k, v in st.items() if k not in ("edges_kept",)})
+print('counters [visits, block_rounds, warp_drains, vertex_pushes]:', plan.counters()[:4])

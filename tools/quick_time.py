@@ -16,9 +16,10 @@ def run(name, g, flags=0, reps=5):
         a.record(); E.ecl_scc(rp, ci, lab, plan=plan); b.record(); torch.cuda.synchronize()
         ts.append(a.elapsed_time(b))
     t = float(np.median(ts))
-    print(f"{name:28s} flags={flags} n={g.n} m={g.nnz} t={t:.3f} ms  {g.nnz/t/1e3:.1f} Me/s  iters={st['iterations']} passes={st['passes']} per-iter={st['passes_iter'][:8]} ein={st['edges_in'][:6]}", flush=True)
+    cnt = plan.counters()[:4]
+    print(f"{name:28s} flags={flags} prof={cnt} n={g.n} m={g.nnz} t={t:.3f} ms  {g.nnz/t/1e3:.1f} Me/s  iters={st['iterations']} passes={st['passes']} per-iter={st['passes_iter'][:8]} ein={st['edges_in'][:6]}", flush=True)
 
-FLAGS = [0, E.IDENTITY_IDS, E.NO_DIRTY, E.IDENTITY_IDS | E.NO_DIRTY]
+FLAGS = [int(x) for x in os.environ.get('QT_FLAGS', '0,32,64,96').split(',')]
 
 if __name__ == "__main__":
     which = sys.argv[1:] or ["c2", "c4", "c3"]

@@ -387,10 +387,10 @@ __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ ch
 //      the intra-tile neighbours as 16-bit slots in shared memory;
 //   2. frontier propagation in shared memory: a vertex whose value rose pushes it to its
 //      intra-tile dependents (in along out-edges, out along in-edges) with shared-memory
-//      atomicMax, and a dependent that rose is flagged (bitmask words).  Each warp keeps
-//      draining the flags of its own 128 vertices (atomic fetch-and-clear, 32 vertices per
-//      SIMD step) so chains inside a warp's region need no block barrier; block rounds
-//      repeat until a round does no work.  Work is proportional to the number of raises;
+//      atomicMax, and a dependent that rose is flagged.  Each warp keeps draining the
+//      flags of its own 128 vertices (atomic fetch-and-clear) so chains inside a warp's
+//      region need no block barrier; block rounds repeat until a round does no work.
+//      Work is proportional to the number of raises, not to rounds x tile size;
 //   3. write raised signatures back and flag the out-of-tile dependents' tiles dirty.
 // Rows longer than HEAVY_T are skipped here (k_prop_heavy folds them in).  Tile order
 // alternates with the pass parity so values can ride the block schedule both ways.
@@ -408,17 +408,19 @@ constexpr uint16_t NOSLOT = 0xFFFF;
 template <int TT>
 constexpr size_t tile_dyn_smem() { return (size_t)TT * (4 + 4 + 8 + 8); }   // values + slots
 
-// Intra-tile neighbour slots: 4 x 16 bit in a 64-bit word, NOSLOT = empty.  A vertex with
-// more than SLOTS intra-tile neighbours in a direction carries SLOWBIT on slot 3 and
-// walks its global row instead.  Raise flags are bitmasks: word j covers tile vertices
-// 32j .. 32j+31; warp w owns words 4w .. 4w+3 (vertices 128w .. 128w+127).
-constexpr unsigned SLOWBIT = 0x8000u;
+// slots are packed 4 x 16 bit in a 64-bit word (NOSLOT = empty).  A raised target w is
+// flagged in its owner's flag word (thread w/4 owns byte w%4).
 __device__ __forceinline__ void flag_set(unsigned* __restrict__ fw, unsigned w) {
-    atomicOr(fw + (w >> 5), 1u << (w & 31));
+    atomicOr(fw + (w >> 2), 1u << (8 * (w & 3)));
 }
-__device__ __forceinline__ void raise_to(int* __restrict__ sig, unsigned* __restrict__ fw, unsigned w, int val,
-                                         int& any) {
-    if (sig[w] < val && atomicMax(sig + w, val) < val) { flag_set(fw, w); any = 1; }
+__device__ __forceinline__ void push_slots(unsigned long long nb, int val, int* __restrict__ sig,
+                                           unsigned* __restrict__ fw, int& any) {
+#pragma unroll
+    for (int q = 0; q < SLOTS; q++) {
+        const unsigned w = (unsigned)(nb >> (16 * q)) & 0xFFFFu;
+        if (w == NOSLOT) break;
+        if (sig[w] < val && atomicMax(sig + w, val) < val) { flag_set(fw, w); any = 1; }
+    }
 }
 __device__ __forceinline__ void add_slot(unsigned long long& pk, int& ns, unsigned idx) {
     pk &= ~(0xFFFFull << (16 * ns));
@@ -436,7 +438,7 @@ __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGrap
     int* s_out = s_in + TT;                                // [TT]
     unsigned long long* s_nin = (unsigned long long*)(s_out + TT);   // [TT] intra in-neighbours
     unsigned long long* s_nout = s_nin + TT;                         // [TT] intra out-neighbours
-    __shared__ unsigned s_fin[TT / 32], s_fout[TT / 32];   // raise flags (bitmasks, see above)
+    __shared__ unsigned s_fin[(TT / VPT)], s_fout[(TT / VPT)];   // raise flags, byte k = vertex 4t+k
     __shared__ int s_dirty;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + TT - 1) / TT;
@@ -457,7 +459,8 @@ __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGrap
     const int cnt = min(TT, g.na - base);
 
     int ob[VPT], oe[VPT], ib[VPT], ie[VPT], o_in[VPT], o_out[VPT];
-    unsigned fin = 0, fout = 0;             // bit k: vertex 4t+k starts flagged
+    unsigned slow = 0;       // bit k: in-row of vertex k has > SLOTS intra neighbours; bit 4+k: out-row
+    unsigned fin = 0, fout = 0;
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int v = tid * VPT + k;
@@ -482,7 +485,7 @@ __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGrap
                 if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) { x = max(x, ld_cg(cin + u)); continue; }
                 if (full) x = max(x, ld_cg(cin + u));   // see "full" above: heavy rows do not push
                 if (ns < SLOTS) add_slot(ni, ns, (unsigned)(u - base));
-                else ni |= (unsigned long long)SLOWBIT << 48;
+                else slow |= 1u << k;
             }
             ns = 0;
             for (int e = ob[k]; e < oe[k]; e++) {
@@ -490,10 +493,10 @@ __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGrap
                 if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) { y = max(y, ld_cg(cout + w)); continue; }
                 if (full) y = max(y, ld_cg(cout + w));
                 if (ns < SLOTS) add_slot(no, ns, (unsigned)(w - base));
-                else no |= (unsigned long long)SLOWBIT << 48;
+                else slow |= 1u << (4 + k);
             }
-            if (full || x > o_in[k]) fin |= 1u << k;
-            if (full || y > o_out[k]) fout |= 1u << k;
+            if (full || x > o_in[k]) fin |= 1u << (8 * k);
+            if (full || y > o_out[k]) fout |= 1u << (8 * k);
         }
         if (v < TT) {
             s_in[v] = x;
@@ -503,57 +506,52 @@ __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGrap
         }
     }
     if (tid == 0) PROF_ADD(dc, 0, 1);                         // tile visits
-    // initial flags (thread t's four vertices are bits 4(t%8) .. 4(t%8)+3 of word t/8)
-    if (tid < TT / 32) { s_fin[tid] = 0; s_fout[tid] = 0; }
+    // initial flags: this thread's four vertices in one word per direction
+    s_fin[tid] = fin;
+    s_fout[tid] = fout;
     __syncthreads();
-    if (fin) atomicOr(s_fin + (tid >> 3), fin << (4 * (tid & 7)));
-    if (fout) atomicOr(s_fout + (tid >> 3), fout << (4 * (tid & 7)));
-    __syncthreads();
-    // step 2: frontier propagation in shared memory.  A warp drains its own 8 flag words
-    // (4 per direction); each word is one SIMD step in which lane i pushes vertex 32j+i.
+    // step 2: frontier propagation in shared memory
     if (!SYNC) {
-        const int lane = tid & 31, warp = tid >> 5;
         for (;;) {
             int worked = 0;
-            for (;;) {
-                unsigned word = 0;
-                if (lane < 8) word = atomicExch((lane < 4 ? s_fin : s_fout) + warp * 4 + (lane & 3), 0u);
+            if (tid == 0) PROF_ADD(dc, 1, 1);                 // block rounds
+            for (;;) {                                       // drain this warp's flags
+                if ((tid & 31) == 0) PROF_ADD(dc, 2, 1);      // warp drain iterations
+                const unsigned wi = atomicExch(s_fin + tid, 0u), wo = atomicExch(s_fout + tid, 0u);
                 int any = 0;
-                if (__any_sync(FULL, word != 0)) {
+                if (wi | wo) {
                     worked = 1;
-#pragma unroll 1
-                    for (int j = 0; j < 8; j++) {
-                        const unsigned bits = __shfl_sync(FULL, word, j);
-                        if (!((bits >> lane) & 1u)) continue;
-                        const unsigned v = (unsigned)(warp * 128 + (j & 3) * 32 + lane);
-                        const bool dir_in = j < 4;           // v_in rose: push along out-edges
-                        int* sig = dir_in ? s_in : s_out;
-                        unsigned* fw = dir_in ? s_fin : s_fout;
-                        const int val = sig[v];
-                        const unsigned long long nb = dir_in ? s_nout[v] : s_nin[v];
+                    PROF_ADD(dc, 3, __popc(wi) + __popc(wo));   // vertex pushes
 #pragma unroll
-                        for (int q = 0; q < SLOTS; q++) {
-                            const unsigned w = (unsigned)(nb >> (16 * q)) & 0xFFFFu;
-                            if (w == NOSLOT) break;
-                            raise_to(sig, fw, w & ~SLOWBIT, val, any);
+                    for (int k = 0; k < VPT; k++) {
+                        const int v = tid * VPT + k;
+                        if ((wi >> (8 * k)) & 0xFF) {        // v_in rose: push along out-edges
+                            const int val = s_in[v];
+                            push_slots(s_nout[v], val, s_in, s_fin, any);
+                            if (slow & (1u << (4 + k)))
+                                for (int e = ob[k]; e < oe[k]; e++) {
+                                    const int w = __ldg(g.oadj + e) - base;
+                                    if ((unsigned)w < (unsigned)cnt && s_in[w] < val && atomicMax(s_in + w, val) < val) {
+                                        flag_set(s_fin, w); any = 1;
+                                    }
+                                }
                         }
-                        if ((unsigned)(nb >> 48) != NOSLOT && ((nb >> 48) & SLOWBIT)) {   // more than SLOTS
-                            const int gi = base + (int)v;
-                            const int32_t* adj = dir_in ? g.oadj : g.iadj;
-                            const int rb = dir_in ? __ldg(g.optr + gi) : __ldg(g.iptr + gi);
-                            const int re = dir_in ? __ldg(g.optr + gi + 1) : __ldg(g.iptr + gi + 1);
-                            int q = 0;
-                            for (int e = rb; e < re; e++) {
-                                const int w = __ldg(adj + e) - base;
-                                if ((unsigned)w >= (unsigned)cnt) continue;
-                                if (q++ < SLOTS) continue;           // already pushed via a slot
-                                raise_to(sig, fw, (unsigned)w, val, any);
-                            }
+                        if ((wo >> (8 * k)) & 0xFF) {        // v_out rose: push along in-edges
+                            const int val = s_out[v];
+                            push_slots(s_nin[v], val, s_out, s_fout, any);
+                            if (slow & (1u << k))
+                                for (int e = ib[k]; e < ie[k]; e++) {
+                                    const int u = __ldg(g.iadj + e) - base;
+                                    if ((unsigned)u < (unsigned)cnt && s_out[u] < val && atomicMax(s_out + u, val) < val) {
+                                        flag_set(s_fout, u); any = 1;
+                                    }
+                                }
                         }
                     }
                 }
                 __syncwarp();
-                if (!__any_sync(FULL, any)) break;           // raised nothing: region drained
+                // another pass while this warp raised something (possibly its own vertices)
+                if (!__any_sync(FULL, any)) break;
             }
             if (!__syncthreads_or(worked)) break;            // a round with no work: done
         }

@@ -82,8 +82,8 @@ typedef struct {
     int64_t vertices_in[ECL_SCC_TRACE_MAX];  /* vertices with a live edge in Phase 2     */
     int64_t edges_kept[ECL_SCC_TRACE_MAX];   /* edges kept by Phase 3 (before next trim) */
     int64_t passes_iter[ECL_SCC_TRACE_MAX];  /* global passes of Phase 2, per iteration  */
-    int64_t prop_bytes;                      /* algorithmic bytes of all Phase-2 passes
-                                                (SURVEY 8(d) accounting)      */
+    int64_t prop_bytes;                      /* algorithmic bytes of the Phase-2 work done
+                                                (SURVEY 8(d) terms over the visited tiles) */
     int64_t kernel_launches;                 /* kernels this call launched                */
     /* device time per stage (CUDA events on the call's stream), only with
        ECL_SCC_TIME_STAGES; 0 otherwise */

@@ -260,7 +260,7 @@ static double stage_ms(Plan* p, int k) {   // call after a stream sync
 int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, int32_t* labels,
               cudaStream_t s, ecl_scc_stats* st, int stop_iter, int32_t* dbg_in, int32_t* dbg_out) {
     if (st) memset(st, 0, sizeof(*st));
-    CK(cudaMemsetAsync(p->dc->prof, 0, sizeof(p->dc->prof), s));
+    CK(cudaMemsetAsync(p->dc->prof, 0, sizeof(p->dc->prof) + 3 * sizeof(unsigned long long), s));
     stage_mark(p, 0, s);
     if (!(p->flags & ECL_SCC_NO_VALIDATE) && n > 0) {
         CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
@@ -327,8 +327,6 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
                     st->passes_iter[iter - 1] = passes;
                 }
                 st->passes += passes;
-                // 4(n_p+1) offsets + 12 B/edge + 16 B/vertex
-                st->prop_bytes += (4 * ((int64_t)t.x + 1) + 12 * (int64_t)t.y + 16 * (int64_t)t.x) * passes;
             }
             if (stop_iter == iter) {
                 p->launches++; k_snapshot_left<<<grid_for(n, TPB), TPB, 0, s>>>(n, labels, dbg_in, dbg_out, P);
@@ -352,12 +350,17 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         CK(cudaMemcpyAsync(dbg_in, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
         CK(cudaMemcpyAsync(dbg_out, labels, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
     }
+    CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
     if (st) {
         st->iterations = iters;
         st->trace_len = std::min(iters, ECL_SCC_TRACE_MAX);
         st->kernel_launches = p->launches;
+        // SURVEY 8(d) accounting over the tiles actually visited: 4 B offset + 16 B own
+        // in/out read+write per vertex, 12 B per edge (index + both far-end signatures);
+        // heavy chunks: 8 B per edge (index + one far-end signature)
+        st->prop_bytes = (int64_t)(20 * p->hc->visit_v + 12 * p->hc->visit_e + 8 * p->hc->heavy_e);
     }
-    CK(cudaStreamSynchronize(s));
     return ECL_SCC_OK;
 }
 

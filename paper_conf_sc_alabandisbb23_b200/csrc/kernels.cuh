@@ -372,6 +372,7 @@ __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ ch
         int acc = 0;
         for (int e = k.beg + lane; e < k.end; e += WARP) acc = max(acc, ld_cg(sig + __ldg(adj + e)));
         acc = warp_max(acc);
+        if (lane == 0) atomicAdd(&dc->heavy_e, (unsigned long long)(k.end - k.beg));
         if (lane == 0 && acc > ld_cg(sig + k.i)) {
             if (atomicMax(sig + k.i, acc) < acc) ch = true;
         }
@@ -504,6 +505,17 @@ __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGrap
             s_nin[v] = ni;
             s_nout[v] = no;
         }
+    }
+    {
+        // honest roofline accounting: only visited tiles move bytes (SURVEY 8(d) per-vertex
+        // and per-edge terms applied to the tile's vertices and out-rows)
+        int me = 0;
+#pragma unroll
+        for (int k = 0; k < VPT; k++)
+            if (tid * VPT + k < cnt) me += __ldg(g.optr + base + tid * VPT + k + 1) - __ldg(g.optr + base + tid * VPT + k);
+        me = warp_sum(me);
+        if ((tid & 31) == 0 && me) atomicAdd(&dc->visit_e, (unsigned long long)me);
+        if (tid == 0) atomicAdd(&dc->visit_v, (unsigned long long)cnt);
     }
     if (tid == 0) PROF_ADD(dc, 0, 1);                         // tile visits
     // initial flags: this thread's four vertices in one word per direction

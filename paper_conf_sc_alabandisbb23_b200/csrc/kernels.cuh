@@ -34,7 +34,7 @@ struct Chunk {
 };
 
 // ------------------------------------------------------------------ init / validation
-__global__ void k_validate(int32_t n, int64_t nnz, const int32_t* __restrict__ rp,
+static __global__ void k_validate(int32_t n, int64_t nnz, const int32_t* __restrict__ rp,
                            const int32_t* __restrict__ ci, int* __restrict__ err) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -53,13 +53,13 @@ __global__ void k_validate(int32_t n, int64_t nnz, const int32_t* __restrict__ r
 }
 
 // ------------------------------------------------------------------ a1: CSR -> CSC
-__global__ void k_indeg(int64_t nnz, const int32_t* __restrict__ ci, int32_t* __restrict__ ideg) {
+static __global__ void k_indeg(int64_t nnz, const int32_t* __restrict__ ci, int32_t* __restrict__ ideg) {
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x)
         atomicAdd(&ideg[ci[e]], 1);
 }
 
 // one thread per source row; rows longer than HEAVY are spread over the warp
-__global__ void k_csc_scatter(int32_t n, const int32_t* __restrict__ rp, const int32_t* __restrict__ ci,
+static __global__ void k_csc_scatter(int32_t n, const int32_t* __restrict__ rp, const int32_t* __restrict__ ci,
                               const int32_t* __restrict__ iptr, int32_t* __restrict__ cursor,
                               int32_t* __restrict__ iadj) {
     const int lane = threadIdx.x & 31;
@@ -170,7 +170,7 @@ struct SurvivePred {
 
 // kept in/out degree per local vertex, plus the number of kept edges
 template <bool FIRST>
-__global__ void k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+static __global__ void k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                              int32_t* __restrict__ kin, int32_t* __restrict__ kout,
                              unsigned long long* __restrict__ kept) {
     const int lane = threadIdx.x & 31;
@@ -186,7 +186,7 @@ __global__ void k_keep_count(WGraph g, const int32_t* __restrict__ cin, const in
 
 // per-vertex surviving (kept, not trimmed) degrees and per-warp totals (alive, out, in)
 template <bool FIRST, bool TRIM>
-__global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                 const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
                                 int2* __restrict__ cnt, int4* __restrict__ wsum) {
     const int lane = threadIdx.x & 31;
@@ -213,7 +213,7 @@ __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const
 // with its signature s = max priority of its SCC; with raw IDs that is the label itself,
 // otherwise it is stored as -(s+1) and k_relabel_* turn it into the SCC's max vertex ID.
 template <bool FIRST>
-__global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                               const int2* __restrict__ cnt, const int4* __restrict__ wscan,
                               const int4* __restrict__ totals, int32_t* __restrict__ newidx,
                               int32_t* __restrict__ act2, int32_t* __restrict__ cin2, int32_t* __restrict__ cout2,
@@ -266,26 +266,26 @@ __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, const i
 // Final labels under priorities: an SCC is named by s = max priority; its label is the
 // largest vertex ID with signature s.  rep: the member with pi(v) == s seeds the slot;
 // max: the others fold in with atomicMax; apply: write the label.
-__global__ void k_relabel_rep(int32_t n, int32_t* __restrict__ labels, int32_t* __restrict__ slot, Prio P) {
+static __global__ void k_relabel_rep(int32_t n, int32_t* __restrict__ labels, int32_t* __restrict__ slot, Prio P) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         const int l = labels[v];
         if (l < 0 && (int)prio_of(P, (uint32_t)v) == -l - 1) slot[-l - 1] = (int)v;
     }
 }
-__global__ void k_relabel_max(int32_t n, const int32_t* __restrict__ labels, int32_t* __restrict__ slot, Prio P) {
+static __global__ void k_relabel_max(int32_t n, const int32_t* __restrict__ labels, int32_t* __restrict__ slot, Prio P) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         const int l = labels[v];
         if (l < 0 && (int)prio_of(P, (uint32_t)v) != -l - 1) atomicMax(slot - l - 1, (int)v);
     }
 }
-__global__ void k_relabel_apply(int32_t n, int32_t* __restrict__ labels, const int32_t* __restrict__ slot) {
+static __global__ void k_relabel_apply(int32_t n, int32_t* __restrict__ labels, const int32_t* __restrict__ slot) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         const int l = labels[v];
         if (l < 0) labels[v] = slot[-l - 1];
     }
 }
 // debug snapshot of the vertices that already left: their (in, out) in priority space
-__global__ void k_snapshot_left(int32_t n, const int32_t* __restrict__ labels, int32_t* __restrict__ din,
+static __global__ void k_snapshot_left(int32_t n, const int32_t* __restrict__ labels, int32_t* __restrict__ din,
                                 int32_t* __restrict__ dout, Prio P) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         const int l = labels[v];
@@ -326,7 +326,7 @@ __device__ __forceinline__ void emit_row(const int32_t* __restrict__ adj, int rb
 }
 
 template <bool FIRST, bool TRIM>
-__global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                   const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
                                   const int32_t* __restrict__ newidx, const int32_t* __restrict__ optr2,
                                   const int32_t* __restrict__ iptr2, int32_t* __restrict__ oadj2,
@@ -357,7 +357,7 @@ __device__ __forceinline__ bool pass_begin(DevCounters* dc, int pass, bool first
 
 // Heavy rows: one warp per chunk of a long row; the chunk max is folded in with
 // atomicMax (monotone, so concurrent chunks of one row commute).
-__global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ chunks, int nchunks, WGraph g,
+static __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ chunks, int nchunks, WGraph g,
                                                     int32_t* __restrict__ cin, int32_t* __restrict__ cout,
                                                     DevCounters* __restrict__ dc, int pass) {
     if (!pass_begin(dc, pass, true)) return;
@@ -430,7 +430,7 @@ __device__ __forceinline__ void add_slot(unsigned long long& pk, int& ns, unsign
 }
 
 template <bool SYNC, int TT>
-__global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGraph g, int32_t* __restrict__ cin,
+static __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGraph g, int32_t* __restrict__ cin,
                                                                int32_t* __restrict__ cout, DevCounters* __restrict__ dc,
                                                                int pass, int first, uint8_t* __restrict__ dirty_cur,
                                                                uint8_t* __restrict__ dirty_next, int full) {

@@ -11,7 +11,8 @@ for r in csv.DictReader(lines):
     key = (name, r["ID"])
     v = float(r["Metric Value"].replace(",", "") or 0)
     u = r.get("Metric Unit", "")
-    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-3, "usecond": 1, "msecond": 1e3}.get(u, 1)
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-3, "nsecond": 1e-3, "us": 1,
+             "usecond": 1, "ms": 1e3, "msecond": 1e3}.get(u, 1)
     per[key][r["Metric Name"]] += v * scale
 agg = collections.defaultdict(lambda: {"launches": 0, "dram_bytes": 0.0, "time_us": 0.0})
 for (name, _), m in per.items():

@@ -15,6 +15,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <string>
 #include <vector>
 
 #include "../../include/ecl_scc.h"
@@ -186,19 +187,49 @@ static int set_tile_attrs() {
 
 template <int TT>
 static int launch_tile(Plan* p, bool sync, const WGraph& g, int32_t* cin, int32_t* cout, int pass, int first,
-                       uint8_t* dcur, uint8_t* dnext, int full, cudaStream_t s) {
+                       uint8_t* dcur, uint8_t* dnext, int full, int theta, cudaStream_t s) {
     if (int r = set_tile_attrs<TT>()) return r;
     const unsigned ntiles = (unsigned)cdiv(g.na, TT);
     p->launches++;
-    if (sync) k_prop_tile<true, TT><<<ntiles, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, nullptr, nullptr, 1);
-    else k_prop_tile<false, TT><<<ntiles, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, dcur, dnext, full);
+    if (sync) k_prop_tile<true, TT><<<ntiles, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, nullptr, nullptr, 1, theta);
+    else k_prop_tile<false, TT><<<ntiles, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, dcur, dnext, full, theta);
     return ECL_SCC_OK;
 }
 
-static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int nchunks, cudaStream_t s,
+// Threshold stages: the top-K priorities of the working graph flood first (a vertex
+// reached by one of them already holds its final value: everything else is smaller), then
+// the next K, ..., then theta = 0.  K list: ECL_SCC_STAGES.
+static std::vector<int> stage_thresholds(int32_t n, int32_t na, bool identity) {
+    std::vector<int> th;
+    static std::vector<long long> Ks;
+    static bool init = false;
+    if (!init) {
+        const char* e = getenv("ECL_SCC_STAGES");
+        std::string spec = e ? e : "64,4096,262144";
+        size_t pos = 0;
+        while (pos < spec.size()) {
+            size_t q = spec.find(',', pos);
+            if (q == std::string::npos) q = spec.size();
+            const long long k = atoll(spec.substr(pos, q - pos).c_str());
+            if (k > 0) Ks.push_back(k);
+            pos = q + 1;
+        }
+        init = true;
+    }
+    (void)identity;
+    for (long long K : Ks)
+        if (K < na) {
+            const long long t = (long long)n - (long long)n * K / na;   // priorities are uniform on [0, n)
+            if (t > 0 && (th.empty() || t < th.back())) th.push_back((int)t);
+        }
+    th.push_back(0);
+    return th;
+}
+
+// a4-a6: Phase 2 to its fixed point.  Passes are enqueued in growing batches; a pass
+// whose predecessor changed nothing exits at once, so over-enqueueing costs only a launch.
+static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int nchunks, int32_t n, cudaStream_t s,
                      int64_t* passes_out) {
-    CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
-    CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
     const unsigned ntiles = (unsigned)cdiv(g.na, p->tile);
     const unsigned hgrid = (unsigned)std::min<int64_t>(cdiv(std::max(nchunks, 1), TPB / WARP), 148 * 8);
     const bool sync = (p->flags & ECL_SCC_SYNC_PASSES) != 0;
@@ -206,37 +237,45 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     // and a local fixed point per visit (not the SYNC ablation)
     const bool use_dirty = nchunks == 0 && !sync && !(p->flags & ECL_SCC_NO_DIRTY);
     uint8_t* D[2] = {p->dirty, p->dirty + p->dirty_cap};
-    if (use_dirty) {
-        CK(cudaMemsetAsync(D[0], 1, ntiles, s));
-        CK(cudaMemsetAsync(D[1], 0, ntiles, s));
-    }
-    int pass = 0;
-    int batch = 2;
-    for (;;) {
-        for (int k = 0; k < batch; k++, pass++) {
-            uint8_t* dc_ = use_dirty ? D[pass & 1] : nullptr;
-            uint8_t* dn_ = use_dirty ? D[(pass + 1) & 1] : nullptr;
-            if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>((const Chunk*)p->chunks, nchunks, g, cin, cout, p->dc, pass); }
-            const int full = (pass == 0 || nchunks > 0);
-            int r = ECL_SCC_OK;
-            switch (p->tile) {
-                case 512: r = launch_tile<512>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, s); break;
-                case 1024: r = launch_tile<1024>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, s); break;
-                case 4096: r = launch_tile<4096>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, s); break;
-                default: r = launch_tile<2048>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, s); break;
-            }
-            if (r) return r;
+    const std::vector<int> thetas = (p->flags & ECL_SCC_NO_STAGES) ? std::vector<int>{0}
+                                                                      : stage_thresholds(n, g.na, false);
+    int64_t total = 0;
+    for (const int theta : thetas) {
+        CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
+        CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
+        if (use_dirty) {
+            CK(cudaMemsetAsync(D[0], 1, ntiles, s));
+            CK(cudaMemsetAsync(D[1], 0, ntiles, s));
         }
-        CK(cudaGetLastError());
-        CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));
-        if (p->hc->changed[(pass - 1) & (RING - 1)] == 0) break;
-        // a monotone max over int32 IDs cannot take more passes than this
-        if ((int64_t)pass > 4 * (int64_t)g.na + 1024)
-            return fail(ECL_SCC_ECUDA, "internal: Phase 2 did not converge after %d passes", pass);
-        batch = std::min(batch * 2, RING / 2);
+        int pass = 0;
+        int batch = 2;
+        for (;;) {
+            for (int k = 0; k < batch; k++, pass++) {
+                uint8_t* dc_ = use_dirty ? D[pass & 1] : nullptr;
+                uint8_t* dn_ = use_dirty ? D[(pass + 1) & 1] : nullptr;
+                if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>((const Chunk*)p->chunks, nchunks, g, cin, cout, p->dc, pass, theta); }
+                const int full = (pass == 0 || nchunks > 0);
+                int r = ECL_SCC_OK;
+                switch (p->tile) {
+                    case 512: r = launch_tile<512>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, theta, s); break;
+                    case 1024: r = launch_tile<1024>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, theta, s); break;
+                    case 4096: r = launch_tile<4096>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, theta, s); break;
+                    default: r = launch_tile<2048>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, theta, s); break;
+                }
+                if (r) return r;
+            }
+            CK(cudaGetLastError());
+            CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));
+            if (p->hc->changed[(pass - 1) & (RING - 1)] == 0) break;
+            // a monotone max over int32 IDs cannot take more passes than this
+            if ((int64_t)pass > 4 * (int64_t)g.na + 1024)
+                return fail(ECL_SCC_ECUDA, "internal: Phase 2 did not converge after %d passes", pass);
+            batch = std::min(batch * 2, RING / 2);
+        }
+        total += (int64_t)p->hc->passes;
     }
-    *passes_out = (int64_t)p->hc->passes;
+    *passes_out = total;
     return ECL_SCC_OK;
 }
 
@@ -312,7 +351,7 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             if (t.y == 0) break;                                   // no live edge: done
             int64_t passes = 0;
             stage_mark(p, 4, s);
-            r = propagate(p, g, p->cin[ob], p->cout[ob], nchunks, s, &passes);
+            r = propagate(p, g, p->cin[ob], p->cout[ob], nchunks, n, s, &passes);
             if (r) return r;
             stage_mark(p, 5, s);
             if (st && (p->flags & ECL_SCC_TIME_STAGES)) {

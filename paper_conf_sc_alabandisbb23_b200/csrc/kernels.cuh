@@ -355,11 +355,16 @@ __device__ __forceinline__ bool pass_begin(DevCounters* dc, int pass, bool first
     return true;
 }
 
+// Threshold stages: within a stage only signature values
+// >= theta take part in propagation; smaller values wait for a later stage.  The last
+// stage has theta = 0, so the final state is the ordinary fixed point.
+__device__ __forceinline__ int eff(int x, int theta) { return x >= theta ? x : -1; }
+
 // Heavy rows: one warp per chunk of a long row; the chunk max is folded in with
 // atomicMax (monotone, so concurrent chunks of one row commute).
 static __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ chunks, int nchunks, WGraph g,
                                                     int32_t* __restrict__ cin, int32_t* __restrict__ cout,
-                                                    DevCounters* __restrict__ dc, int pass) {
+                                                    DevCounters* __restrict__ dc, int pass, int theta) {
     if (!pass_begin(dc, pass, true)) return;
     const int lane = threadIdx.x & 31;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -370,7 +375,7 @@ static __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restri
         const int32_t* adj = k.dir ? g.iadj : g.oadj;
         int32_t* sig = k.dir ? cin : cout;
         int acc = 0;
-        for (int e = k.beg + lane; e < k.end; e += WARP) acc = max(acc, ld_cg(sig + __ldg(adj + e)));
+        for (int e = k.beg + lane; e < k.end; e += WARP) acc = max(acc, eff(ld_cg(sig + __ldg(adj + e)), theta));
         acc = warp_max(acc);
         if (lane == 0) atomicAdd(&dc->heavy_e, (unsigned long long)(k.end - k.beg));
         if (lane == 0 && acc > ld_cg(sig + k.i)) {
@@ -395,7 +400,8 @@ static __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restri
 //   3. write raised signatures back and flag the out-of-tile dependents' tiles dirty.
 // Rows longer than HEAVY_T are skipped here (k_prop_heavy folds them in).  Tile order
 // alternates with the pass parity so values can ride the block schedule both ways.
-// full: every vertex starts flagged and step 1 also pulls the intra-tile neighbours'
+// theta: threshold stage (only values >= theta propagate).
+// full: every vertex (with a value >= theta) starts flagged and step 1 also pulls the intra-tile neighbours'
 // values (first visit of a phase, and every visit when heavy rows exist: an intra-tile
 // edge whose source row is heavy is not in any push list, so it is covered by the pull).
 // SYNC = ablation: no step 2 (one relaxation per pass, "separate kernels").
@@ -433,7 +439,7 @@ template <bool SYNC, int TT>
 static __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGraph g, int32_t* __restrict__ cin,
                                                                int32_t* __restrict__ cout, DevCounters* __restrict__ dc,
                                                                int pass, int first, uint8_t* __restrict__ dirty_cur,
-                                                               uint8_t* __restrict__ dirty_next, int full) {
+                                                               uint8_t* __restrict__ dirty_next, int full, int theta) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     int* s_in = (int*)smem_raw;                              // [TT]
     int* s_out = s_in + TT;                                // [TT]
@@ -483,21 +489,21 @@ static __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_til
             int ns = 0;
             for (int e = ib[k]; e < ie[k]; e++) {
                 const int u = __ldg(g.iadj + e);
-                if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) { x = max(x, ld_cg(cin + u)); continue; }
-                if (full) x = max(x, ld_cg(cin + u));   // see "full" above: heavy rows do not push
+                if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) { x = max(x, eff(ld_cg(cin + u), theta)); continue; }
+                if (full) x = max(x, eff(ld_cg(cin + u), theta));   // see "full" above: heavy rows do not push
                 if (ns < SLOTS) add_slot(ni, ns, (unsigned)(u - base));
                 else slow |= 1u << k;
             }
             ns = 0;
             for (int e = ob[k]; e < oe[k]; e++) {
                 const int w = __ldg(g.oadj + e);
-                if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) { y = max(y, ld_cg(cout + w)); continue; }
-                if (full) y = max(y, ld_cg(cout + w));
+                if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) { y = max(y, eff(ld_cg(cout + w), theta)); continue; }
+                if (full) y = max(y, eff(ld_cg(cout + w), theta));
                 if (ns < SLOTS) add_slot(no, ns, (unsigned)(w - base));
                 else slow |= 1u << (4 + k);
             }
-            if (full || x > o_in[k]) fin |= 1u << (8 * k);
-            if (full || y > o_out[k]) fout |= 1u << (8 * k);
+            if ((full && x >= theta) || x > o_in[k]) fin |= 1u << (8 * k);
+            if ((full && y >= theta) || y > o_out[k]) fout |= 1u << (8 * k);
         }
         if (v < TT) {
             s_in[v] = x;

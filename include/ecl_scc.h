@@ -70,8 +70,8 @@ typedef enum {
                                       priorities pi(v) (reading 16); labels are
                                       identical either way */
 #define ECL_SCC_NO_DIRTY 0x40u    /* ablation: visit every tile in every Phase-2 pass */
-#define ECL_SCC_NO_STAGES 0x80u   /* ablation: release every priority at once in Phase 2
-                                     (no threshold stages) */
+#define ECL_SCC_STAGED 0x80u      /* Phase 2 in threshold stages: the top-K priorities
+                                     propagate first (ECL_SCC_STAGES env, default off) */
 
 #define ECL_SCC_TRACE_MAX 64
 

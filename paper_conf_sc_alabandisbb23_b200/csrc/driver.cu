@@ -237,8 +237,8 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     // and a local fixed point per visit (not the SYNC ablation)
     const bool use_dirty = nchunks == 0 && !sync && !(p->flags & ECL_SCC_NO_DIRTY);
     uint8_t* D[2] = {p->dirty, p->dirty + p->dirty_cap};
-    const std::vector<int> thetas = (p->flags & ECL_SCC_NO_STAGES) ? std::vector<int>{0}
-                                                                      : stage_thresholds(n, g.na, false);
+    const std::vector<int> thetas = (p->flags & ECL_SCC_STAGED) ? stage_thresholds(n, g.na, false)
+                                                                   : std::vector<int>{0};
     int64_t total = 0;
     for (const int theta : thetas) {
         CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
@@ -274,6 +274,9 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             batch = std::min(batch * 2, RING / 2);
         }
         total += (int64_t)p->hc->passes;
+        if (getenv("ECL_SCC_DEBUG"))
+            fprintf(stderr, "[ecl_scc] na=%d m=%d theta=%d passes=%llu visited_vertices=%llu\n", g.na,
+                    (int)0, theta, (unsigned long long)p->hc->passes, (unsigned long long)p->hc->visit_v);
     }
     *passes_out = total;
     return ECL_SCC_OK;

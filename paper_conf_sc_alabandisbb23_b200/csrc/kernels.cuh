@@ -424,8 +424,9 @@ __device__ __forceinline__ void push_slots(unsigned long long nb, int val, int* 
                                            unsigned* __restrict__ fw, int& any) {
 #pragma unroll
     for (int q = 0; q < SLOTS; q++) {
-        const unsigned w = (unsigned)(nb >> (16 * q)) & 0xFFFFu;
+        unsigned w = (unsigned)(nb >> (16 * q)) & 0xFFFFu;
         if (w == NOSLOT) break;
+        w &= 0x7FFFu;                                  // slot 3 may carry the SLOW mark
         if (sig[w] < val && atomicMax(sig + w, val) < val) { flag_set(fw, w); any = 1; }
     }
 }
@@ -435,17 +436,20 @@ __device__ __forceinline__ void add_slot(unsigned long long& pk, int& ns, unsign
     ns++;
 }
 
+// slots: SLOWBIT on slot 3 marks a vertex with more than SLOTS intra-tile neighbours in
+// that direction (it walks its global row for the rest)
+constexpr unsigned long long SLOW_MARK = 0x8000ull << 48;
+
 template <bool SYNC, int TT>
-static __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_tile(WGraph g, int32_t* __restrict__ cin,
-                                                               int32_t* __restrict__ cout, DevCounters* __restrict__ dc,
-                                                               int pass, int first, uint8_t* __restrict__ dirty_cur,
-                                                               uint8_t* __restrict__ dirty_next, int full, int theta) {
+static __global__ void __launch_bounds__(TT / VPT, (1536 / (TT / VPT)) > 0 ? 1536 / (TT / VPT) : 1)
+k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, DevCounters* __restrict__ dc, int pass,
+            int first, uint8_t* __restrict__ dirty_cur, uint8_t* __restrict__ dirty_next, int full, int theta) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    int* s_in = (int*)smem_raw;                              // [TT]
-    int* s_out = s_in + TT;                                // [TT]
-    unsigned long long* s_nin = (unsigned long long*)(s_out + TT);   // [TT] intra in-neighbours
-    unsigned long long* s_nout = s_nin + TT;                         // [TT] intra out-neighbours
-    __shared__ unsigned s_fin[(TT / VPT)], s_fout[(TT / VPT)];   // raise flags, byte k = vertex 4t+k
+    int* s_in = (int*)smem_raw;                                        // [TT]
+    int* s_out = s_in + TT;                                            // [TT]
+    unsigned long long* s_nin = (unsigned long long*)(s_out + TT);     // [TT] intra in-neighbours
+    unsigned long long* s_nout = s_nin + TT;                           // [TT] intra out-neighbours
+    __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];             // raise flags, byte k = vertex 4t+k
     __shared__ int s_dirty;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + TT - 1) / TT;
@@ -465,45 +469,44 @@ static __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_til
     const int base = tile * TT;
     const int cnt = min(TT, g.na - base);
 
-    int ob[VPT], oe[VPT], ib[VPT], ie[VPT], o_in[VPT], o_out[VPT];
-    unsigned slow = 0;       // bit k: in-row of vertex k has > SLOTS intra neighbours; bit 4+k: out-row
+    // ---- step 1: rows, out-of-tile pulls (global, L2-coherent), intra-tile slots
     unsigned fin = 0, fout = 0;
+    int me = 0;                                   // out-edges of the visited rows (accounting)
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int v = tid * VPT + k;
-        ob[k] = oe[k] = ib[k] = ie[k] = 0;
-        o_in[k] = o_out[k] = 0;
         int x = 0, y = 0;
         unsigned long long ni = ~0ull, no = ~0ull;
         if (v < cnt) {
             const int gi = base + v;
-            ob[k] = __ldg(g.optr + gi); oe[k] = __ldg(g.optr + gi + 1);
-            ib[k] = __ldg(g.iptr + gi); ie[k] = __ldg(g.iptr + gi + 1);
-            if (oe[k] - ob[k] > HEAVY_T) ob[k] = oe[k];       // heavy: reduced elsewhere
-            if (ie[k] - ib[k] > HEAVY_T) ib[k] = ie[k];
-            o_in[k] = ld_cg(cin + gi);
-            o_out[k] = ld_cg(cout + gi);
-            x = o_in[k];
-            y = o_out[k];
-            // step 1: out-of-tile neighbours from global memory, intra-tile ones cached
+            int ob = __ldg(g.optr + gi);
+            const int oe = __ldg(g.optr + gi + 1);
+            int ib = __ldg(g.iptr + gi);
+            const int ie = __ldg(g.iptr + gi + 1);
+            me += oe - ob;
+            if (oe - ob > HEAVY_T) ob = oe;       // heavy: reduced by k_prop_heavy
+            if (ie - ib > HEAVY_T) ib = ie;
+            const int x0 = ld_cg(cin + gi), y0 = ld_cg(cout + gi);
+            x = x0;
+            y = y0;
             int ns = 0;
-            for (int e = ib[k]; e < ie[k]; e++) {
+            for (int e = ib; e < ie; e++) {
                 const int u = __ldg(g.iadj + e);
                 if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) { x = max(x, eff(ld_cg(cin + u), theta)); continue; }
                 if (full) x = max(x, eff(ld_cg(cin + u), theta));   // see "full" above: heavy rows do not push
                 if (ns < SLOTS) add_slot(ni, ns, (unsigned)(u - base));
-                else slow |= 1u << k;
+                else ni |= SLOW_MARK;
             }
             ns = 0;
-            for (int e = ob[k]; e < oe[k]; e++) {
+            for (int e = ob; e < oe; e++) {
                 const int w = __ldg(g.oadj + e);
                 if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) { y = max(y, eff(ld_cg(cout + w), theta)); continue; }
                 if (full) y = max(y, eff(ld_cg(cout + w), theta));
                 if (ns < SLOTS) add_slot(no, ns, (unsigned)(w - base));
-                else slow |= 1u << (4 + k);
+                else no |= SLOW_MARK;
             }
-            if ((full && x >= theta) || x > o_in[k]) fin |= 1u << (8 * k);
-            if ((full && y >= theta) || y > o_out[k]) fout |= 1u << (8 * k);
+            if ((full && x >= theta) || x > x0) fin |= 1u << (8 * k);
+            if ((full && y >= theta) || y > y0) fout |= 1u << (8 * k);
         }
         if (v < TT) {
             s_in[v] = x;
@@ -513,22 +516,16 @@ static __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_til
         }
     }
     {
-        // honest roofline accounting: only visited tiles move bytes (SURVEY 8(d) per-vertex
-        // and per-edge terms applied to the tile's vertices and out-rows)
-        int me = 0;
-#pragma unroll
-        for (int k = 0; k < VPT; k++)
-            if (tid * VPT + k < cnt) me += __ldg(g.optr + base + tid * VPT + k + 1) - __ldg(g.optr + base + tid * VPT + k);
+        // honest roofline accounting: only visited tiles move bytes (SURVEY 8(d) terms)
         me = warp_sum(me);
         if ((tid & 31) == 0 && me) atomicAdd(&dc->visit_e, (unsigned long long)me);
         if (tid == 0) atomicAdd(&dc->visit_v, (unsigned long long)cnt);
     }
     if (tid == 0) PROF_ADD(dc, 0, 1);                         // tile visits
-    // initial flags: this thread's four vertices in one word per direction
     s_fin[tid] = fin;
     s_fout[tid] = fout;
     __syncthreads();
-    // step 2: frontier propagation in shared memory
+    // ---- step 2: frontier propagation in shared memory
     if (!SYNC) {
         for (;;) {
             int worked = 0;
@@ -545,9 +542,10 @@ static __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_til
                         const int v = tid * VPT + k;
                         if ((wi >> (8 * k)) & 0xFF) {        // v_in rose: push along out-edges
                             const int val = s_in[v];
-                            push_slots(s_nout[v], val, s_in, s_fin, any);
-                            if (slow & (1u << (4 + k)))
-                                for (int e = ob[k]; e < oe[k]; e++) {
+                            const unsigned long long nb = s_nout[v];
+                            push_slots(nb, val, s_in, s_fin, any);
+                            if ((nb & SLOW_MARK) && (nb >> 48) != 0xFFFFull)
+                                for (int e = __ldg(g.optr + base + v), ee = __ldg(g.optr + base + v + 1); e < ee; e++) {
                                     const int w = __ldg(g.oadj + e) - base;
                                     if ((unsigned)w < (unsigned)cnt && s_in[w] < val && atomicMax(s_in + w, val) < val) {
                                         flag_set(s_fin, w); any = 1;
@@ -556,9 +554,10 @@ static __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_til
                         }
                         if ((wo >> (8 * k)) & 0xFF) {        // v_out rose: push along in-edges
                             const int val = s_out[v];
-                            push_slots(s_nin[v], val, s_out, s_fout, any);
-                            if (slow & (1u << k))
-                                for (int e = ib[k]; e < ie[k]; e++) {
+                            const unsigned long long nb = s_nin[v];
+                            push_slots(nb, val, s_out, s_fout, any);
+                            if ((nb & SLOW_MARK) && (nb >> 48) != 0xFFFFull)
+                                for (int e = __ldg(g.iptr + base + v), ee = __ldg(g.iptr + base + v + 1); e < ee; e++) {
                                     const int u = __ldg(g.iadj + e) - base;
                                     if ((unsigned)u < (unsigned)cnt && s_out[u] < val && atomicMax(s_out + u, val) < val) {
                                         flag_set(s_fout, u); any = 1;
@@ -574,28 +573,30 @@ static __global__ void __launch_bounds__(TT / VPT, 1024 / (TT / VPT)) k_prop_til
             if (!__syncthreads_or(worked)) break;            // a round with no work: done
         }
     }
-    // step 3: write back; a raised v_in must reach the out-neighbours' tiles, a raised
-    // v_out the in-neighbours' tiles (next pass)
+    // ---- step 3: write back; a raised v_in must reach the out-neighbours' tiles, a
+    // raised v_out the in-neighbours' tiles (next pass).  Only this tile writes its
+    // vertices, so global memory still holds the values read in step 1.
     int ch = 0;
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int v = tid * VPT + k;
         if (v >= cnt) continue;
+        const int gi = base + v;
         const int x = s_in[v], y = s_out[v];
-        if (x > o_in[k]) {
-            cin[base + v] = x;
+        if (x > ld_cg(cin + gi)) {
+            cin[gi] = x;
             ch = 1;
             if (dirty_next)
-                for (int e = ob[k]; e < oe[k]; e++) {
+                for (int e = __ldg(g.optr + gi), ee = __ldg(g.optr + gi + 1); e < ee; e++) {
                     const int w = __ldg(g.oadj + e);
                     if ((unsigned)(w - base) >= (unsigned)cnt) dirty_next[w / TT] = 1;
                 }
         }
-        if (y > o_out[k]) {
-            cout[base + v] = y;
+        if (y > ld_cg(cout + gi)) {
+            cout[gi] = y;
             ch = 1;
             if (dirty_next)
-                for (int e = ib[k]; e < ie[k]; e++) {
+                for (int e = __ldg(g.iptr + gi), ee = __ldg(g.iptr + gi + 1); e < ee; e++) {
                     const int u = __ldg(g.iadj + e);
                     if ((unsigned)(u - base) >= (unsigned)cnt) dirty_next[u / TT] = 1;
                 }

@@ -532,7 +532,10 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
             if (tid == 0) PROF_ADD(dc, 1, 1);                 // block rounds
             for (;;) {                                       // drain this warp's flags
                 if ((tid & 31) == 0) PROF_ADD(dc, 2, 1);      // warp drain iterations
-                const unsigned wi = atomicExch(s_fin + tid, 0u), wo = atomicExch(s_fout + tid, 0u);
+                // plain load first: a shared atomic costs a full pipe pass per lane
+                unsigned wi = ((volatile unsigned*)s_fin)[tid], wo = ((volatile unsigned*)s_fout)[tid];
+                if (wi) wi = atomicExch(s_fin + tid, 0u);
+                if (wo) wo = atomicExch(s_fout + tid, 0u);
                 int any = 0;
                 if (wi | wo) {
                     worked = 1;

@@ -450,6 +450,7 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
     unsigned long long* s_nin = (unsigned long long*)(s_out + TT);     // [TT] intra in-neighbours
     unsigned long long* s_nout = s_nin + TT;                           // [TT] intra out-neighbours
     __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];             // raise flags, byte k = vertex 4t+k
+    __shared__ unsigned short s_queue[2 * TT];                         // per-warp item queues
     __shared__ int s_dirty;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + TT - 1) / TT;
@@ -525,47 +526,58 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
     s_fin[tid] = fin;
     s_fout[tid] = fout;
     __syncthreads();
-    // ---- step 2: frontier propagation in shared memory
+    // ---- step 2: frontier propagation in shared memory.  Each warp drains the flags of
+    // its own 128 vertices: flagged (vertex, direction) items are compacted into a
+    // per-warp queue (ballot-free: popc + warp prefix sum) so all lanes run the same push
+    // path; block rounds repeat until a round does no work.
     if (!SYNC) {
+        const int lane = tid & 31, wq0 = (tid >> 5) * (2 * 32 * VPT);
         for (;;) {
             int worked = 0;
             if (tid == 0) PROF_ADD(dc, 1, 1);                 // block rounds
             for (;;) {                                       // drain this warp's flags
-                if ((tid & 31) == 0) PROF_ADD(dc, 2, 1);      // warp drain iterations
+                if (lane == 0) PROF_ADD(dc, 2, 1);            // warp drain iterations
                 // plain load first: a shared atomic costs a full pipe pass per lane
                 unsigned wi = ((volatile unsigned*)s_fin)[tid], wo = ((volatile unsigned*)s_fout)[tid];
                 if (wi) wi = atomicExch(s_fin + tid, 0u);
                 if (wo) wo = atomicExch(s_fout + tid, 0u);
+                // one bit per item: bits 0-3 in-direction of vertex 4t+k, bits 4-7 out-direction
+                const unsigned items = ((wi & 0x01u) | ((wi >> 7) & 0x02u) | ((wi >> 14) & 0x04u) | ((wi >> 21) & 0x08u)) |
+                                       (((wo & 0x01u) | ((wo >> 7) & 0x02u) | ((wo >> 14) & 0x04u) | ((wo >> 21) & 0x08u)) << 4);
+                const int c = __popc(items);
+                const int incl = warp_incl_scan(c, lane);
+                const int total = __shfl_sync(FULL, incl, 31);
+                if (total == 0) break;                       // region drained
+                worked = 1;
+                PROF_ADD(dc, 3, c);                          // vertex pushes
+                {
+                    int pos = wq0 + incl - c;
+                    unsigned it = items;
+                    while (it) {
+                        const int bit = __ffs(it) - 1;
+                        it &= it - 1;
+                        s_queue[pos++] = (unsigned short)(((tid * VPT + (bit & 3)) << 1) | (bit >> 2));
+                    }
+                }
+                __syncwarp();
                 int any = 0;
-                if (wi | wo) {
-                    worked = 1;
-                    PROF_ADD(dc, 3, __popc(wi) + __popc(wo));   // vertex pushes
-#pragma unroll
-                    for (int k = 0; k < VPT; k++) {
-                        const int v = tid * VPT + k;
-                        if ((wi >> (8 * k)) & 0xFF) {        // v_in rose: push along out-edges
-                            const int val = s_in[v];
-                            const unsigned long long nb = s_nout[v];
-                            push_slots(nb, val, s_in, s_fin, any);
-                            if ((nb & SLOW_MARK) && (nb >> 48) != 0xFFFFull)
-                                for (int e = __ldg(g.optr + base + v), ee = __ldg(g.optr + base + v + 1); e < ee; e++) {
-                                    const int w = __ldg(g.oadj + e) - base;
-                                    if ((unsigned)w < (unsigned)cnt && s_in[w] < val && atomicMax(s_in + w, val) < val) {
-                                        flag_set(s_fin, w); any = 1;
-                                    }
-                                }
-                        }
-                        if ((wo >> (8 * k)) & 0xFF) {        // v_out rose: push along in-edges
-                            const int val = s_out[v];
-                            const unsigned long long nb = s_nin[v];
-                            push_slots(nb, val, s_out, s_fout, any);
-                            if ((nb & SLOW_MARK) && (nb >> 48) != 0xFFFFull)
-                                for (int e = __ldg(g.iptr + base + v), ee = __ldg(g.iptr + base + v + 1); e < ee; e++) {
-                                    const int u = __ldg(g.iadj + e) - base;
-                                    if ((unsigned)u < (unsigned)cnt && s_out[u] < val && atomicMax(s_out + u, val) < val) {
-                                        flag_set(s_fout, u); any = 1;
-                                    }
-                                }
+                for (int q = lane; q < total; q += 32) {
+                    const unsigned item = s_queue[wq0 + q];
+                    const int v = (int)(item >> 1);
+                    const bool dir_out = item & 1u;           // v_out rose: push along in-edges
+                    int* sig = dir_out ? s_out : s_in;
+                    unsigned* fw = dir_out ? s_fout : s_fin;
+                    const int val = sig[v];
+                    const unsigned long long nb = dir_out ? s_nin[v] : s_nout[v];
+                    push_slots(nb, val, sig, fw, any);
+                    if ((nb & SLOW_MARK) && (nb >> 48) != 0xFFFFull) {
+                        const int32_t* ptr = dir_out ? g.iptr : g.optr;
+                        const int32_t* adj = dir_out ? g.iadj : g.oadj;
+                        for (int e = __ldg(ptr + base + v), ee = __ldg(ptr + base + v + 1); e < ee; e++) {
+                            const int w = __ldg(adj + e) - base;
+                            if ((unsigned)w < (unsigned)cnt && sig[w] < val && atomicMax(sig + w, val) < val) {
+                                flag_set(fw, w); any = 1;
+                            }
                         }
                     }
                 }

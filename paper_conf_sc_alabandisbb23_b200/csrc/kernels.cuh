@@ -469,6 +469,9 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
     }
     const int base = tile * TT;
     const int cnt = min(TT, g.na - base);
+#ifdef ECL_PROF
+    const long long t_start = clock64();
+#endif
 
     // ---- step 1: rows, out-of-tile pulls (global, L2-coherent), intra-tile slots
     unsigned fin = 0, fout = 0;
@@ -526,6 +529,9 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
     s_fin[tid] = fin;
     s_fout[tid] = fout;
     __syncthreads();
+#ifdef ECL_PROF
+    const long long t_step1 = clock64();
+#endif
     // ---- step 2: frontier propagation in shared memory.  Each warp drains the flags of
     // its own 128 vertices: flagged (vertex, direction) items are compacted into a
     // per-warp queue (ballot-free: popc + warp prefix sum) so all lanes run the same push
@@ -588,6 +594,10 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
             if (!__syncthreads_or(worked)) break;            // a round with no work: done
         }
     }
+#ifdef ECL_PROF
+    __syncthreads();
+    const long long t_step2 = clock64();
+#endif
     // ---- step 3: write back; a raised v_in must reach the out-neighbours' tiles, a
     // raised v_out the in-neighbours' tiles (next pass).  Only this tile writes its
     // vertices, so global memory still holds the values read in step 1.
@@ -618,6 +628,14 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
         }
     }
     if (__syncthreads_or(ch) && tid == 0) dc->changed[pass & (RING - 1)] = 1;
+#ifdef ECL_PROF
+    if (tid == 0) {
+        const long long t_end = clock64();
+        PROF_ADD(dc, 4, t_step1 - t_start);
+        PROF_ADD(dc, 5, t_step2 - t_step1);
+        PROF_ADD(dc, 6, t_end - t_step2);
+    }
+#endif
 }
 
 }  // namespace eclscc

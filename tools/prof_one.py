@@ -18,4 +18,6 @@ _, st = E.ecl_scc(rp, ci, lab, plan=plan, stats=True)
 torch.cuda.synchronize()
 torch.cuda.cudart().cudaProfilerStop()
 print({k: v for k, v in st.items() if k not in ("edges_kept",)})
-print('counters [visits, block_rounds, warp_drains, vertex_pushes]:', plan.counters()[:4])
+c = plan.counters()
+print('counters [visits, block_rounds, warp_drains, vertex_pushes]:', c[:4])
+if c[0]: print('cycles per visit: step1 %.0f step2 %.0f step3 %.0f' % (c[4]/c[0], c[5]/c[0], c[6]/c[0]))

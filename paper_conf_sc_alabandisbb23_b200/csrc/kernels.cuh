@@ -536,13 +536,20 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
     // its own 128 vertices: flagged (vertex, direction) items are compacted into a
     // per-warp queue (ballot-free: popc + warp prefix sum) so all lanes run the same push
     // path; block rounds repeat until a round does no work.
+#ifdef ECL_PROF
+    unsigned prof_rounds = 0, prof_drains = 0, prof_pushes = 0;
+#endif
     if (!SYNC) {
         const int lane = tid & 31, wq0 = (tid >> 5) * (2 * 32 * VPT);
         for (;;) {
             int worked = 0;
-            if (tid == 0) PROF_ADD(dc, 1, 1);                 // block rounds
+#ifdef ECL_PROF
+            if (tid == 0) prof_rounds++;
+#endif
             for (;;) {                                       // drain this warp's flags
-                if (lane == 0) PROF_ADD(dc, 2, 1);            // warp drain iterations
+#ifdef ECL_PROF
+                if (lane == 0) prof_drains++;
+#endif
                 // plain load first: a shared atomic costs a full pipe pass per lane
                 unsigned wi = ((volatile unsigned*)s_fin)[tid], wo = ((volatile unsigned*)s_fout)[tid];
                 if (wi) wi = atomicExch(s_fin + tid, 0u);
@@ -555,7 +562,9 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
                 const int total = __shfl_sync(FULL, incl, 31);
                 if (total == 0) break;                       // region drained
                 worked = 1;
-                PROF_ADD(dc, 3, c);                          // vertex pushes
+#ifdef ECL_PROF
+                prof_pushes += c;
+#endif
                 {
                     int pos = wq0 + incl - c;
                     unsigned it = items;
@@ -597,6 +606,9 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
 #ifdef ECL_PROF
     __syncthreads();
     const long long t_step2 = clock64();
+    prof_pushes = warp_sum(prof_pushes);
+    if ((tid & 31) == 0) { PROF_ADD(dc, 2, prof_drains); PROF_ADD(dc, 3, prof_pushes); }
+    if (tid == 0) PROF_ADD(dc, 1, prof_rounds);
 #endif
     // ---- step 3: write back; a raised v_in must reach the out-neighbours' tiles, a
     // raised v_out the in-neighbours' tiles (next pass).  Only this tile writes its

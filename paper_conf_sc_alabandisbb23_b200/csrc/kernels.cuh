@@ -413,7 +413,7 @@ static __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restri
 constexpr int SLOTS = 4;                 // cached intra-tile neighbours per vertex and direction
 constexpr uint16_t NOSLOT = 0xFFFF;
 template <int TT>
-constexpr size_t tile_dyn_smem() { return (size_t)TT * (4 + 4 + 8 + 8 + 2); }   // values, slots, degree bytes
+constexpr size_t tile_dyn_smem() { return (size_t)TT * (4 + 4 + 8 + 8); }   // values + slots
 
 // slots are packed 4 x 16 bit in a 64-bit word (NOSLOT = empty).  A raised target w is
 // flagged in its owner's flag word (thread w/4 owns byte w%4).
@@ -436,42 +436,26 @@ __device__ __forceinline__ void add_slot(unsigned long long& pk, int& ns, unsign
     ns++;
 }
 
-// per-warp scratch for step 1/3 (row offsets of the warp's 128 vertices) and step 2 (item queue)
-constexpr int WSCRATCH = 132;   // ints per warp
-
-// first j in [0, n) with off[j + 1] > e (the row that owns edge e); off is ascending
-__device__ __forceinline__ int owner_of(const int* __restrict__ off, int n, int e) {
-    int lo = 0, hi = n - 1;
-    while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (off[mid] <= e) lo = mid; else hi = mid - 1;
-    }
-    return lo;
-}
-// byte counters packed 4 per word (vertex v -> word v/4, byte v%4); returns the old byte
-__device__ __forceinline__ unsigned bump_byte(unsigned* __restrict__ w, int v) {
-    return (atomicAdd(w + (v >> 2), 1u << (8 * (v & 3))) >> (8 * (v & 3))) & 0xFFu;
-}
+// slots: SLOWBIT on slot 3 marks a vertex with more than SLOTS intra-tile neighbours in
+// that direction (it walks its global row for the rest)
+constexpr unsigned long long SLOW_MARK = 0x8000ull << 48;
 
 template <bool SYNC, int TT>
 static __global__ void __launch_bounds__(TT / VPT, (1536 / (TT / VPT)) > 0 ? 1536 / (TT / VPT) : 1)
 k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, DevCounters* __restrict__ dc, int pass,
             int first, uint8_t* __restrict__ dirty_cur, uint8_t* __restrict__ dirty_next, int full, int theta) {
-    constexpr int NW = TT / VPT / 32;                                  // warps; each owns 128 vertices
     extern __shared__ __align__(16) unsigned char smem_raw[];
     int* s_in = (int*)smem_raw;                                        // [TT]
     int* s_out = s_in + TT;                                            // [TT]
     unsigned long long* s_nin = (unsigned long long*)(s_out + TT);     // [TT] intra in-neighbours
     unsigned long long* s_nout = s_nin + TT;                           // [TT] intra out-neighbours
-    unsigned* s_cin = (unsigned*)(s_nout + TT);                        // [TT/4] intra in-degree bytes
-    unsigned* s_cout = s_cin + TT / 4;                                 // [TT/4] intra out-degree bytes
     __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];             // raise flags, byte k = vertex 4t+k
-    __shared__ int s_scratch[NW * WSCRATCH];                           // per-warp offsets / item queue
+    __shared__ unsigned short s_queue[2 * TT];                         // per-warp item queues
     __shared__ int s_dirty;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + TT - 1) / TT;
     const int tile = (pass & 1) ? (ntiles - 1 - (int)blockIdx.x) : (int)blockIdx.x;
-    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    const int tid = threadIdx.x;
     // dirty-tile skipping: a tile whose inputs did not change since its last visit is at
     // its local fixed point already.  The read flag is cleared here, so after pass p the
     // buffer read in pass p is all zero and pass p+1 can fill it for pass p+2.
@@ -485,83 +469,78 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
     }
     const int base = tile * TT;
     const int cnt = min(TT, g.na - base);
-    int* off = s_scratch + wid * WSCRATCH;
-    const int wb = wid * 128, nv = max(0, min(128, cnt - wb));
 #ifdef ECL_PROF
     const long long t_start = clock64();
 #endif
 
-    // ---- step 1a: the tile's signatures (coalesced), empty slots, zero counters and flags
-    for (int v = tid; v < TT; v += TT / VPT) {
-        s_in[v] = v < cnt ? ld_cg(cin + base + v) : 0;
-        s_out[v] = v < cnt ? ld_cg(cout + base + v) : 0;
-        s_nin[v] = ~0ull;
-        s_nout[v] = ~0ull;
-    }
-    for (int w = tid; w < TT / 4; w += TT / VPT) { s_cin[w] = 0; s_cout[w] = 0; }
-    s_fin[tid] = 0;
-    s_fout[tid] = 0;
-    __syncthreads();
-    // ---- step 1b: warp-cooperative, edge-parallel over the warp's rows (coalesced
-    // adjacency loads, many in flight): out-of-tile neighbours are pulled from global
-    // memory (Alg. 1 l.10-11) with shared atomicMax; intra-tile neighbours go to the slots
-    int me = 0;
-    for (int dir = 0; dir < 2; dir++) {
-        const int32_t* ptr = dir ? g.optr : g.iptr;            // dir 0: in-rows, 1: out-rows
-        const int32_t* adj = dir ? g.oadj : g.iadj;
-        const int32_t* gsig = dir ? cout : cin;
-        int* ssig = dir ? s_out : s_in;
-        unsigned long long* slots = dir ? s_nout : s_nin;
-        unsigned* ccount = dir ? s_cout : s_cin;
-        unsigned* fw = dir ? s_fout : s_fin;
-        if (nv > 0) {
-            for (int j = lane; j <= nv; j += 32) off[j] = __ldg(ptr + base + wb + j);
-            __syncwarp();
-            const int e0 = off[0], e1 = off[nv];
-            if (dir) me = e1 - e0;
-            for (int e = e0 + lane; e < e1; e += 32) {
-                const int j = owner_of(off, nv, e);
-                if (off[j + 1] - off[j] > HEAVY_T) continue;   // heavy row: k_prop_heavy
-                const int v = wb + j;
-                const int x = __ldg(adj + e);
-                if (SYNC || (unsigned)(x - base) >= (unsigned)cnt) {
-                    const int val = eff(ld_cg(gsig + x), theta);
-                    if (val > ssig[v] && atomicMax(ssig + v, val) < val) flag_set(fw, v);
-                } else {
-                    const unsigned q = bump_byte(ccount, v);
-                    if (q < SLOTS) ((unsigned short*)(slots + v))[q] = (unsigned short)(x - base);
-                    if (full) {                              // heavy rows do not push: pull once
-                        const int val = eff(ssig[x - base], theta);
-                        if (val > ssig[v] && atomicMax(ssig + v, val) < val) flag_set(fw, v);
-                    }
-                }
+    // ---- step 1: rows, out-of-tile pulls (global, L2-coherent), intra-tile slots
+    unsigned fin = 0, fout = 0;
+    int me = 0;                                   // out-edges of the visited rows (accounting)
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int v = tid * VPT + k;
+        int x = 0, y = 0;
+        unsigned long long ni = ~0ull, no = ~0ull;
+        if (v < cnt) {
+            const int gi = base + v;
+            int ob = __ldg(g.optr + gi);
+            const int oe = __ldg(g.optr + gi + 1);
+            int ib = __ldg(g.iptr + gi);
+            const int ie = __ldg(g.iptr + gi + 1);
+            me += oe - ob;
+            if (oe - ob > HEAVY_T) ob = oe;       // heavy: reduced by k_prop_heavy
+            if (ie - ib > HEAVY_T) ib = ie;
+            const int x0 = ld_cg(cin + gi), y0 = ld_cg(cout + gi);
+            x = x0;
+            y = y0;
+            int ns = 0;
+            for (int e = ib; e < ie; e++) {
+                const int u = __ldg(g.iadj + e);
+                if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) { x = max(x, eff(ld_cg(cin + u), theta)); continue; }
+                if (full) x = max(x, eff(ld_cg(cin + u), theta));   // see "full" above: heavy rows do not push
+                if (ns < SLOTS) add_slot(ni, ns, (unsigned)(u - base));
+                else ni |= SLOW_MARK;
             }
-            __syncwarp();
+            ns = 0;
+            for (int e = ob; e < oe; e++) {
+                const int w = __ldg(g.oadj + e);
+                if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) { y = max(y, eff(ld_cg(cout + w), theta)); continue; }
+                if (full) y = max(y, eff(ld_cg(cout + w), theta));
+                if (ns < SLOTS) add_slot(no, ns, (unsigned)(w - base));
+                else no |= SLOW_MARK;
+            }
+            if ((full && x >= theta) || x > x0) fin |= 1u << (8 * k);
+            if ((full && y >= theta) || y > y0) fout |= 1u << (8 * k);
+        }
+        if (v < TT) {
+            s_in[v] = x;
+            s_out[v] = y;
+            s_nin[v] = ni;
+            s_nout[v] = no;
         }
     }
-    me = warp_sum(me);
-    if (lane == 0 && me) atomicAdd(&dc->visit_e, (unsigned long long)me);
-    if (tid == 0) {
-        atomicAdd(&dc->visit_v, (unsigned long long)cnt);
-        PROF_ADD(dc, 0, 1);                                    // tile visits
+    {
+        // honest roofline accounting: only visited tiles move bytes (SURVEY 8(d) terms)
+        me = warp_sum(me);
+        if ((tid & 31) == 0 && me) atomicAdd(&dc->visit_e, (unsigned long long)me);
+        if (tid == 0) atomicAdd(&dc->visit_v, (unsigned long long)cnt);
     }
-    __syncthreads();
-    if (full)                                                  // first visit: every live value pushes
-        for (int v = tid; v < cnt; v += TT / VPT) {
-            if (s_in[v] >= theta) flag_set(s_fin, v);
-            if (s_out[v] >= theta) flag_set(s_fout, v);
-        }
+    if (tid == 0) PROF_ADD(dc, 0, 1);                         // tile visits
+    s_fin[tid] = fin;
+    s_fout[tid] = fout;
     __syncthreads();
 #ifdef ECL_PROF
     const long long t_step1 = clock64();
-    unsigned prof_rounds = 0, prof_drains = 0, prof_pushes = 0;
 #endif
     // ---- step 2: frontier propagation in shared memory.  Each warp drains the flags of
     // its own 128 vertices: flagged (vertex, direction) items are compacted into a
-    // per-warp queue so all lanes run the same push path; block rounds repeat until a
-    // round does no work.
+    // per-warp queue (ballot-free: popc + warp prefix sum) so all lanes run the same push
+    // path; block rounds repeat until a round does no work.
+#ifdef ECL_PROF
+    unsigned prof_rounds = 0, prof_drains = 0, prof_pushes = 0;
+#endif
     if (!SYNC) {
-        unsigned short* queue = (unsigned short*)off;          // 2 x 128 items
+        const int lane = tid & 31, wq0 = (tid >> 5) * (2 * 32 * VPT);
         for (;;) {
             int worked = 0;
 #ifdef ECL_PROF
@@ -587,27 +566,26 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
                 prof_pushes += c;
 #endif
                 {
-                    int pos = incl - c;
+                    int pos = wq0 + incl - c;
                     unsigned it = items;
                     while (it) {
                         const int bit = __ffs(it) - 1;
                         it &= it - 1;
-                        queue[pos++] = (unsigned short)(((tid * VPT + (bit & 3)) << 1) | (bit >> 2));
+                        s_queue[pos++] = (unsigned short)(((tid * VPT + (bit & 3)) << 1) | (bit >> 2));
                     }
                 }
                 __syncwarp();
                 int any = 0;
                 for (int q = lane; q < total; q += 32) {
-                    const unsigned item = queue[q];
+                    const unsigned item = s_queue[wq0 + q];
                     const int v = (int)(item >> 1);
                     const bool dir_out = item & 1u;           // v_out rose: push along in-edges
                     int* sig = dir_out ? s_out : s_in;
                     unsigned* fw = dir_out ? s_fout : s_fin;
                     const int val = sig[v];
-                    push_slots(dir_out ? s_nin[v] : s_nout[v], val, sig, fw, any);
-                    // more than SLOTS intra-tile dependents: walk the global row
-                    const unsigned deg = ((dir_out ? s_cin : s_cout)[v >> 2] >> (8 * (v & 3))) & 0xFFu;
-                    if (deg > SLOTS) {
+                    const unsigned long long nb = dir_out ? s_nin[v] : s_nout[v];
+                    push_slots(nb, val, sig, fw, any);
+                    if ((nb & SLOW_MARK) && (nb >> 48) != 0xFFFFull) {
                         const int32_t* ptr = dir_out ? g.iptr : g.optr;
                         const int32_t* adj = dir_out ? g.iadj : g.oadj;
                         for (int e = __ldg(ptr + base + v), ee = __ldg(ptr + base + v + 1); e < ee; e++) {
@@ -629,42 +607,39 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
     __syncthreads();
     const long long t_step2 = clock64();
     prof_pushes = warp_sum(prof_pushes);
-    if (lane == 0) { PROF_ADD(dc, 2, prof_drains); PROF_ADD(dc, 3, prof_pushes); }
+    if ((tid & 31) == 0) { PROF_ADD(dc, 2, prof_drains); PROF_ADD(dc, 3, prof_pushes); }
     if (tid == 0) PROF_ADD(dc, 1, prof_rounds);
 #endif
-    // ---- step 3a: write back raised signatures (coalesced); only this tile writes its
-    // vertices, so global memory still holds the values read in step 1a.  The flag words
-    // (all zero after step 2) now mark what was raised.
+    // ---- step 3: write back; a raised v_in must reach the out-neighbours' tiles, a
+    // raised v_out the in-neighbours' tiles (next pass).  Only this tile writes its
+    // vertices, so global memory still holds the values read in step 1.
     int ch = 0;
-    for (int v = tid; v < cnt; v += TT / VPT) {
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int v = tid * VPT + k;
+        if (v >= cnt) continue;
+        const int gi = base + v;
         const int x = s_in[v], y = s_out[v];
-        if (x > ld_cg(cin + base + v)) { cin[base + v] = x; flag_set(s_fin, v); ch = 1; }
-        if (y > ld_cg(cout + base + v)) { cout[base + v] = y; flag_set(s_fout, v); ch = 1; }
-    }
-    const int any_ch = __syncthreads_or(ch);
-    // ---- step 3b: a raised v_in must reach the out-neighbours' tiles, a raised v_out the
-    // in-neighbours' tiles: mark them dirty for the next pass (edge-parallel per warp)
-    if (dirty_next && any_ch && nv > 0) {
-        for (int dir = 0; dir < 2; dir++) {
-            const unsigned* fw = dir ? s_fout : s_fin;         // raised in-values use out-rows
-            const unsigned mine = fw[wb / 4 + lane];           // the warp's 128 vertices = 32 words
-            if (!__any_sync(FULL, mine != 0)) continue;
-            const int32_t* ptr = dir ? g.iptr : g.optr;
-            const int32_t* adj = dir ? g.iadj : g.oadj;
-            for (int j = lane; j <= nv; j += 32) off[j] = __ldg(ptr + base + wb + j);
-            __syncwarp();
-            const int e0 = off[0], e1 = off[nv];
-            for (int e = e0 + lane; e < e1; e += 32) {
-                const int j = owner_of(off, nv, e);
-                const int v = wb + j;
-                if (!((fw[v >> 2] >> (8 * (v & 3))) & 0xFFu)) continue;
-                const int x = __ldg(adj + e);
-                if ((unsigned)(x - base) >= (unsigned)cnt) dirty_next[x / TT] = 1;
-            }
-            __syncwarp();
+        if (x > ld_cg(cin + gi)) {
+            cin[gi] = x;
+            ch = 1;
+            if (dirty_next)
+                for (int e = __ldg(g.optr + gi), ee = __ldg(g.optr + gi + 1); e < ee; e++) {
+                    const int w = __ldg(g.oadj + e);
+                    if ((unsigned)(w - base) >= (unsigned)cnt) dirty_next[w / TT] = 1;
+                }
+        }
+        if (y > ld_cg(cout + gi)) {
+            cout[gi] = y;
+            ch = 1;
+            if (dirty_next)
+                for (int e = __ldg(g.iptr + gi), ee = __ldg(g.iptr + gi + 1); e < ee; e++) {
+                    const int u = __ldg(g.iadj + e);
+                    if ((unsigned)(u - base) >= (unsigned)cnt) dirty_next[u / TT] = 1;
+                }
         }
     }
-    if (any_ch && tid == 0) dc->changed[pass & (RING - 1)] = 1;
+    if (__syncthreads_or(ch) && tid == 0) dc->changed[pass & (RING - 1)] = 1;
 #ifdef ECL_PROF
     if (tid == 0) {
         const long long t_end = clock64();

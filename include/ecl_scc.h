@@ -70,6 +70,8 @@ typedef enum {
                                       priorities pi(v) (reading 16); labels are
                                       identical either way */
 #define ECL_SCC_NO_DIRTY 0x40u    /* ablation: visit every tile in every Phase-2 pass */
+#define ECL_SCC_NO_SWEEP 0x100u   /* Phase 2 in synchronous passes over dirty tiles instead of
+                                     dependency-ordered sweeps */
 #define ECL_SCC_STAGED 0x80u      /* Phase 2 in threshold stages: the top-K priorities
                                      propagate first (ECL_SCC_STAGES env, default off) */
 

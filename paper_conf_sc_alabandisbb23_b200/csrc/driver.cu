@@ -89,6 +89,14 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     e = e ? e : A((void**)&p->bsum, (size_t)p->bsum_cap * sizeof(int4));
     e = e ? e : A((void**)&p->chunks, (size_t)p->chunk_cap * sizeof(Chunk));
     e = e ? e : A((void**)&p->dirty, 2 * (size_t)p->dirty_cap);
+    e = e ? e : A((void**)&p->nb_cnt, (size_t)p->dirty_cap * 4);
+    e = e ? e : A((void**)&p->nb_list, (size_t)p->dirty_cap * NBCAP * 4);
+    e = e ? e : A((void**)&p->done, (size_t)p->dirty_cap * 4);
+    e = e ? e : A((void**)&p->mark, (size_t)p->dirty_cap * 4);
+    e = e ? e : A((void**)&p->sweep_ctr, 16);
+    if (e == cudaSuccess) e = cudaMemset(p->done, 0, (size_t)p->dirty_cap * 4);
+    if (e == cudaSuccess) e = cudaMemset(p->mark, 0, (size_t)p->dirty_cap * 4);
+    p->epoch = 0;
     e = e ? e : A((void**)&p->dc, sizeof(DevCounters));
     if (e == cudaSuccess) e = cudaMallocHost((void**)&p->hc, sizeof(DevCounters));
     if (e != cudaSuccess) {
@@ -107,6 +115,7 @@ void plan_free(Plan* p) {
     cudaFree(p->kin); cudaFree(p->kout); cudaFree(p->newidx); cudaFree(p->cnt);
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
     cudaFree(p->dirty);
+    cudaFree(p->nb_cnt); cudaFree(p->nb_list); cudaFree(p->done); cudaFree(p->mark); cudaFree(p->sweep_ctr);
     cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
     if (p->hc) cudaFreeHost(p->hc);
     if (p->ev_ok)
@@ -196,6 +205,55 @@ static int launch_tile(Plan* p, bool sync, const WGraph& g, int32_t* cin, int32_
     return ECL_SCC_OK;
 }
 
+// Sweep mode: dependency-ordered sweeps over the tiles,
+// alternating forward / backward, until a sweep raises nothing.  Returns 1 in *used if it
+// ran (0: the tile graph was too dense -- the caller falls back to pass mode).
+template <int TT>
+static int sweep_phase(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, cudaStream_t s, int64_t* sweeps,
+                       int* used) {
+    *used = 0;
+    const int ntiles = (int)cdiv(g.na, TT);
+    static int resident = 0;
+    if (!resident) {
+        if (int r = set_tile_attrs<TT>()) return r;
+        CK(cudaFuncSetAttribute(k_sweep_tile<TT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tile_dyn_smem<TT>()));
+        int per_sm = 0, dev = 0, sms = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sweep_tile<TT>, TT / VPT, tile_dyn_smem<TT>()));
+        CK(cudaGetDevice(&dev));
+        CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+        resident = std::max(1, per_sm) * sms;
+    }
+    CK(cudaMemsetAsync(p->sweep_ctr, 0, 16, s));
+    CK(cudaMemsetAsync(&p->dc->err, 0, 4, s));
+    p->launches++;
+    k_tile_nbrs<TT><<<ntiles, 256, 0, s>>>(g, p->nb_cnt, p->nb_list, p->sweep_ctr + 2);
+    CK(cudaGetLastError());
+    int h[3];
+    CK(cudaMemcpyAsync(h, p->sweep_ctr, 12, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (h[2]) return ECL_SCC_OK;                                   // overflow: use passes
+    *used = 1;
+    const unsigned grid = (unsigned)std::min(ntiles, resident);
+    int64_t k = 0;
+    for (;; k++) {
+        if (k > 4 * (int64_t)g.na + 1024) return fail(ECL_SCC_ECUDA, "internal: sweeps did not converge");
+        const int epoch = ++p->epoch;
+        CK(cudaMemsetAsync(p->sweep_ctr, 0, 8, s));
+        p->launches++;
+        k_sweep_tile<TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, p->nb_cnt, p->nb_list, p->done,
+                                                                    p->mark, p->sweep_ctr, epoch, k == 0, (int)(k & 1),
+                                                                    p->sweep_ctr + 1);
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(h, p->sweep_ctr, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(&h[2], &p->dc->err, 4, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (h[2] == 2) return fail(ECL_SCC_ECUDA, "internal: sweep dependency wait timed out");
+        if (!h[1]) break;                                          // nothing raised: fixed point
+    }
+    *sweeps = k + 1;
+    return ECL_SCC_OK;
+}
+
 // Threshold stages: the top-K priorities of the working graph flood first (a vertex
 // reached by one of them already holds its final value: everything else is smaller), then
 // the next K, ..., then theta = 0.  K list: ECL_SCC_STAGES.
@@ -240,6 +298,22 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     const std::vector<int> thetas = (p->flags & ECL_SCC_STAGED) ? stage_thresholds(n, g.na, false)
                                                                    : std::vector<int>{0};
     int64_t total = 0;
+    if (!sync && nchunks == 0 && !(p->flags & (ECL_SCC_NO_SWEEP | ECL_SCC_STAGED))) {
+        int used = 0, r = ECL_SCC_OK;
+        switch (p->tile) {
+            case 512: r = sweep_phase<512>(p, g, cin, cout, s, &total, &used); break;
+            case 1024: r = sweep_phase<1024>(p, g, cin, cout, s, &total, &used); break;
+            case 4096: r = sweep_phase<4096>(p, g, cin, cout, s, &total, &used); break;
+            default: r = sweep_phase<2048>(p, g, cin, cout, s, &total, &used); break;
+        }
+        if (r) return r;
+        if (used) {
+            if (getenv("ECL_SCC_DEBUG"))
+                fprintf(stderr, "[ecl_scc] sweep mode na=%d sweeps=%lld\n", g.na, (long long)total);
+            *passes_out = total;
+            return ECL_SCC_OK;
+        }
+    }
     for (const int theta : thetas) {
         CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
         CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));

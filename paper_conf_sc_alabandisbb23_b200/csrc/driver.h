@@ -34,6 +34,10 @@ struct Plan {
     uint8_t* dirty;                      // 2 x dirty_cap tile flags (Phase-2 skipping)
     int64_t dirty_cap;
     int tile;                            // Phase-2 tile size (vertices per CTA)
+    int *nb_cnt, *nb_list;               // sweep mode: neighbour tiles of each tile
+    int *done, *mark;                    // sweep mode: per-tile done / dirty epochs
+    int* sweep_ctr;                      // [0] tile counter, [1] changed, [2] overflow
+    int epoch;                           // sweep epoch (monotone over the plan's life)
     int64_t launches;                    // kernels launched by the current call
     cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
     bool ev_ok;

@@ -440,33 +440,48 @@ __device__ __forceinline__ void add_slot(unsigned long long& pk, int& ns, unsign
 // that direction (it walks its global row for the rest)
 constexpr unsigned long long SLOW_MARK = 0x8000ull << 48;
 
-template <bool SYNC, int TT>
-static __global__ void __launch_bounds__(TT / VPT, (1536 / (TT / VPT)) > 0 ? 1536 / (TT / VPT) : 1)
-k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, DevCounters* __restrict__ dc, int pass,
-            int first, uint8_t* __restrict__ dirty_cur, uint8_t* __restrict__ dirty_next, int full, int theta) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    int* s_in = (int*)smem_raw;                                        // [TT]
-    int* s_out = s_in + TT;                                            // [TT]
-    unsigned long long* s_nin = (unsigned long long*)(s_out + TT);     // [TT] intra in-neighbours
-    unsigned long long* s_nout = s_nin + TT;                           // [TT] intra out-neighbours
-    __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];             // raise flags, byte k = vertex 4t+k
-    __shared__ unsigned short s_queue[2 * TT];                         // per-warp item queues
-    __shared__ int s_dirty;
-    if (!pass_begin(dc, pass, first)) return;
-    const int ntiles = (g.na + TT - 1) / TT;
-    const int tile = (pass & 1) ? (ntiles - 1 - (int)blockIdx.x) : (int)blockIdx.x;
-    const int tid = threadIdx.x;
-    // dirty-tile skipping: a tile whose inputs did not change since its last visit is at
-    // its local fixed point already.  The read flag is cleared here, so after pass p the
-    // buffer read in pass p is all zero and pass p+1 can fill it for pass p+2.
-    if (dirty_cur) {
-        if (tid == 0) {
-            s_dirty = dirty_cur[tile];
-            dirty_cur[tile] = 0;
-        }
-        __syncthreads();
-        if (!s_dirty) return;
+// Shared-memory working set of one tile visit (dynamic shared memory + static arrays).
+template <int TT>
+struct TileSmem {
+    int* s_in;
+    int* s_out;
+    unsigned long long* s_nin;
+    unsigned long long* s_nout;
+    unsigned* s_fin;
+    unsigned* s_fout;
+    unsigned short* s_queue;
+};
+
+// dirty marking of the tiles that depend on a raised value (pass mode: byte flags for
+// the next pass; sweep mode: the current sweep epoch)
+struct MarkNext {
+    uint8_t* next;
+    __device__ __forceinline__ bool on() const { return next != nullptr; }
+    __device__ __forceinline__ void operator()(int t) const { next[t] = 1; }
+};
+struct MarkEpoch {
+    int* mark;
+    int epoch;
+    __device__ __forceinline__ bool on() const { return true; }
+    __device__ __forceinline__ void operator()(int t) const {
+        if (((volatile int*)mark)[t] != epoch) mark[t] = epoch;
     }
+};
+
+// One block-local fixed point of tile `tile` (steps 1-3 above).  Returns non-zero in
+// every thread if a signature was raised.
+template <bool SYNC, int TT, typename Mark>
+__device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__ cin, int32_t* __restrict__ cout,
+                                          DevCounters* __restrict__ dc, int tile, int full, int theta, Mark mark,
+                                          const TileSmem<TT>& S) {
+    int* s_in = S.s_in;
+    int* s_out = S.s_out;
+    unsigned long long* s_nin = S.s_nin;
+    unsigned long long* s_nout = S.s_nout;
+    unsigned* s_fin = S.s_fin;
+    unsigned* s_fout = S.s_fout;
+    unsigned short* s_queue = S.s_queue;
+    const int tid = threadIdx.x;
     const int base = tile * TT;
     const int cnt = min(TT, g.na - base);
 #ifdef ECL_PROF
@@ -623,23 +638,23 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
         if (x > ld_cg(cin + gi)) {
             cin[gi] = x;
             ch = 1;
-            if (dirty_next)
+            if (mark.on())
                 for (int e = __ldg(g.optr + gi), ee = __ldg(g.optr + gi + 1); e < ee; e++) {
                     const int w = __ldg(g.oadj + e);
-                    if ((unsigned)(w - base) >= (unsigned)cnt) dirty_next[w / TT] = 1;
+                    if ((unsigned)(w - base) >= (unsigned)cnt) mark(w / TT);
                 }
         }
         if (y > ld_cg(cout + gi)) {
             cout[gi] = y;
             ch = 1;
-            if (dirty_next)
+            if (mark.on())
                 for (int e = __ldg(g.iptr + gi), ee = __ldg(g.iptr + gi + 1); e < ee; e++) {
                     const int u = __ldg(g.iadj + e);
-                    if ((unsigned)(u - base) >= (unsigned)cnt) dirty_next[u / TT] = 1;
+                    if ((unsigned)(u - base) >= (unsigned)cnt) mark(u / TT);
                 }
         }
     }
-    if (__syncthreads_or(ch) && tid == 0) dc->changed[pass & (RING - 1)] = 1;
+    const int any_ch = __syncthreads_or(ch);
 #ifdef ECL_PROF
     if (tid == 0) {
         const long long t_end = clock64();
@@ -648,6 +663,161 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
         PROF_ADD(dc, 6, t_end - t_step2);
     }
 #endif
+    return any_ch;
+}
+
+template <bool SYNC, int TT>
+static __global__ void __launch_bounds__(TT / VPT, (1536 / (TT / VPT)) > 0 ? 1536 / (TT / VPT) : 1)
+k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, DevCounters* __restrict__ dc, int pass,
+            int first, uint8_t* __restrict__ dirty_cur, uint8_t* __restrict__ dirty_next, int full, int theta) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];             // raise flags, byte k = vertex 4t+k
+    __shared__ unsigned short s_queue[2 * TT];                         // per-warp item queues
+    __shared__ int s_dirty;
+    TileSmem<TT> S;
+    S.s_in = (int*)smem_raw;
+    S.s_out = S.s_in + TT;
+    S.s_nin = (unsigned long long*)(S.s_out + TT);
+    S.s_nout = S.s_nin + TT;
+    S.s_fin = s_fin;
+    S.s_fout = s_fout;
+    S.s_queue = s_queue;
+    if (!pass_begin(dc, pass, first)) return;
+    const int ntiles = (g.na + TT - 1) / TT;
+    const int tile = (pass & 1) ? (ntiles - 1 - (int)blockIdx.x) : (int)blockIdx.x;
+    const int tid = threadIdx.x;
+    // dirty-tile skipping: a tile whose inputs did not change since its last visit is at
+    // its local fixed point already.  The read flag is cleared here, so after pass p the
+    // buffer read in pass p is all zero and pass p+1 can fill it for pass p+2.
+    if (dirty_cur) {
+        if (tid == 0) {
+            s_dirty = dirty_cur[tile];
+            dirty_cur[tile] = 0;
+        }
+        __syncthreads();
+        if (!s_dirty) return;
+    }
+    const int ch = tile_visit<SYNC, TT>(g, cin, cout, dc, tile, full, theta, MarkNext{dirty_next}, S);
+    if (ch && tid == 0) dc->changed[pass & (RING - 1)] = 1;
+}
+
+// ---------------------------------------------------------------------- sweep mode
+// Neighbour tiles of every tile (distinct tiles holding an endpoint of one of its edges),
+// for the dependency-ordered sweeps.  One CTA per tile, set in shared memory; more than
+// NBCAP neighbours sets *overflow (the driver then uses pass mode).
+constexpr int NBCAP = 64;
+template <int TT>
+static __global__ void __launch_bounds__(256) k_tile_nbrs(WGraph g, int* __restrict__ nb_cnt, int* __restrict__ nb_list,
+                                                          int* __restrict__ overflow) {
+    __shared__ int set[2 * NBCAP];
+    __shared__ int n_set, ovf;
+    const int tile = blockIdx.x, base = tile * TT, cnt = min(TT, g.na - base);
+    for (int i = threadIdx.x; i < 2 * NBCAP; i += blockDim.x) set[i] = -1;
+    if (threadIdx.x == 0) { n_set = 0; ovf = 0; }
+    __syncthreads();
+    for (int v = threadIdx.x; v < cnt; v += blockDim.x) {
+        for (int dir = 0; dir < 2; dir++) {
+            const int32_t* ptr = dir ? g.iptr : g.optr;
+            const int32_t* adj = dir ? g.iadj : g.oadj;
+            for (int e = ptr[base + v], ee = ptr[base + v + 1]; e < ee; e++) {
+                const int t = adj[e] / TT;
+                if (t == tile) continue;
+                unsigned h = ((unsigned)t * 2654435761u) & (2 * NBCAP - 1);
+                for (int probe = 0; probe < 2 * NBCAP; probe++) {
+                    const int cur = set[h];
+                    if (cur == t) break;
+                    if (cur == -1) {
+                        const int old = atomicCAS(set + h, -1, t);
+                        if (old == -1) {
+                            if (atomicAdd(&n_set, 1) >= NBCAP) ovf = 1;
+                            break;
+                        }
+                        if (old == t) break;
+                    }
+                    h = (h + 1) & (2 * NBCAP - 1);
+                    if (probe == 2 * NBCAP - 1) ovf = 1;
+                }
+            }
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int k = 0;
+        if (!ovf)
+            for (int i = 0; i < 2 * NBCAP; i++)
+                if (set[i] >= 0) nb_list[tile * NBCAP + k++] = set[i];
+        nb_cnt[tile] = k;
+        if (ovf) *overflow = 1;
+    }
+}
+
+__device__ __forceinline__ int ld_acquire(const int* p) {
+    int v;
+    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(int* p, int v) {
+    asm volatile("st.release.gpu.global.b32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+
+// One dependency-ordered sweep (persistent CTAs).  Tiles are taken in index order
+// (backward when dir = 1) from a counter; a tile first waits until every neighbour tile
+// that precedes it in this order has finished (done[] >= epoch), so values flowing along
+// the order cross any number of tiles in one sweep.  It is visited if it is the first
+// sweep of the phase or a neighbour raised one of its inputs since the previous sweep
+// (mark >= epoch - 1); then it publishes done = epoch.  Dependencies against the order
+// are left to the next sweep; a sweep without any raise certifies the fixed point.
+template <int TT>
+static __global__ void __launch_bounds__(TT / VPT, (1536 / (TT / VPT)) > 0 ? 1536 / (TT / VPT) : 1)
+k_sweep_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, DevCounters* __restrict__ dc,
+             const int* __restrict__ nb_cnt, const int* __restrict__ nb_list, int* __restrict__ done,
+             int* __restrict__ mark, int* __restrict__ counter, int epoch, int first_sweep, int dir,
+             int* __restrict__ changed) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];
+    __shared__ unsigned short s_queue[2 * TT];
+    __shared__ int s_idx, s_go;
+    TileSmem<TT> S;
+    S.s_in = (int*)smem_raw;
+    S.s_out = S.s_in + TT;
+    S.s_nin = (unsigned long long*)(S.s_out + TT);
+    S.s_nout = S.s_nin + TT;
+    S.s_fin = s_fin;
+    S.s_fout = s_fout;
+    S.s_queue = s_queue;
+    const int ntiles = (g.na + TT - 1) / TT;
+    const int tid = threadIdx.x;
+    int ch_any = 0;
+    for (;;) {
+        if (tid == 0) s_idx = atomicAdd(counter, 1);
+        __syncthreads();
+        const int idx = s_idx;
+        if (idx >= ntiles) break;
+        const int tile = dir ? ntiles - 1 - idx : idx;
+        // wait for the preceding neighbours (all of them were taken earlier: no deadlock)
+        const int nn = nb_cnt[tile];
+        for (int j = tid; j < nn; j += blockDim.x) {
+            const int nb = nb_list[tile * NBCAP + j];
+            if (dir ? nb > tile : nb < tile) {
+                // bounded wait (a bug must not hang the GPU): give up after ~1 s
+                for (unsigned spin = 0; ld_acquire(done + nb) < epoch; spin++) {
+                    if (spin > (1u << 24)) { dc->err = 2; break; }
+                    __nanosleep(64);
+                }
+            }
+        }
+        __syncthreads();
+        if (tid == 0) s_go = first_sweep || ld_acquire(mark + tile) >= epoch - 1;
+        __syncthreads();
+        if (s_go) {
+            const int ch = tile_visit<false, TT>(g, cin, cout, dc, tile, first_sweep, 0, MarkEpoch{mark, epoch}, S);
+            ch_any |= ch;
+            __threadfence();
+        }
+        __syncthreads();
+        if (tid == 0) st_release(done + tile, epoch);
+    }
+    if (ch_any && tid == 0) *changed = 1;
 }
 
 }  // namespace eclscc

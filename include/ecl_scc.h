@@ -70,8 +70,9 @@ typedef enum {
                                       priorities pi(v) (reading 16); labels are
                                       identical either way */
 #define ECL_SCC_NO_DIRTY 0x40u    /* ablation: visit every tile in every Phase-2 pass */
-#define ECL_SCC_NO_SWEEP 0x100u   /* Phase 2 in synchronous passes over dirty tiles instead of
-                                     dependency-ordered sweeps */
+#define ECL_SCC_SWEEP 0x100u      /* Phase 2 as dependency-ordered forward/backward tile
+                                     sweeps instead of passes (experimental; pays off only
+                                     when the tile graph is close to a DAG in ID order) */
 #define ECL_SCC_STAGED 0x80u      /* Phase 2 in threshold stages: the top-K priorities
                                      propagate first (ECL_SCC_STAGES env, default off) */
 

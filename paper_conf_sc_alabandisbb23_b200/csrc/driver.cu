@@ -298,7 +298,7 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     const std::vector<int> thetas = (p->flags & ECL_SCC_STAGED) ? stage_thresholds(n, g.na, false)
                                                                    : std::vector<int>{0};
     int64_t total = 0;
-    if (!sync && nchunks == 0 && !(p->flags & (ECL_SCC_NO_SWEEP | ECL_SCC_STAGED))) {
+    if (!sync && nchunks == 0 && (p->flags & ECL_SCC_SWEEP) && !(p->flags & ECL_SCC_STAGED)) {
         int used = 0, r = ECL_SCC_OK;
         switch (p->tile) {
             case 512: r = sweep_phase<512>(p, g, cin, cout, s, &total, &used); break;

@@ -468,6 +468,23 @@ struct MarkEpoch {
     }
 };
 
+// flag the intra-tile vertices in slot word nb (and, for a slow row, the rest of the
+// global row) for a re-pull: plain byte stores
+__device__ __forceinline__ void notify(unsigned long long nb, const int32_t* __restrict__ ptr,
+                                       const int32_t* __restrict__ adj, int base, int cnt, int v, uint8_t* f) {
+#pragma unroll
+    for (int k = 0; k < SLOTS; k++) {
+        const unsigned w = (unsigned)(nb >> (16 * k)) & 0xFFFFu;
+        if (w == NOSLOT) break;
+        ((volatile uint8_t*)f)[w & 0x7FFFu] = 1;
+    }
+    if ((nb & SLOW_MARK) && (nb >> 48) != 0xFFFFull)
+        for (int e = __ldg(ptr + base + v), ee = __ldg(ptr + base + v + 1); e < ee; e++) {
+            const int w = __ldg(adj + e) - base;
+            if ((unsigned)w < (unsigned)cnt) ((volatile uint8_t*)f)[w] = 1;
+        }
+}
+
 // One block-local fixed point of tile `tile` (steps 1-3 above).  Returns non-zero in
 // every thread if a signature was raised.
 template <bool SYNC, int TT, typename Mark>
@@ -541,19 +558,34 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
         if (tid == 0) atomicAdd(&dc->visit_v, (unsigned long long)cnt);
     }
     if (tid == 0) PROF_ADD(dc, 0, 1);                         // tile visits
-    s_fin[tid] = fin;
-    s_fout[tid] = fout;
+    // ---- step 1b: recompute flags (pull model).  Byte k of s_fin[t] / s_fout[t] asks
+    // vertex 4t+k to re-pull v_in / v_out from its intra-tile neighbours.  First visit:
+    // everybody; otherwise the intra-tile dependents of what step 1 raised.
+    s_fin[tid] = full ? 0x01010101u : 0u;
+    s_fout[tid] = full ? 0x01010101u : 0u;
+    __syncthreads();
+    if (!full && (fin | fout)) {
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            const int v = tid * VPT + k;
+            if ((fin >> (8 * k)) & 0xFF) notify(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
+            if ((fout >> (8 * k)) & 0xFF) notify(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
+        }
+    }
     __syncthreads();
 #ifdef ECL_PROF
     const long long t_step1 = clock64();
-#endif
-    // ---- step 2: frontier propagation in shared memory.  Each warp drains the flags of
-    // its own 128 vertices: flagged (vertex, direction) items are compacted into a
-    // per-warp queue (ballot-free: popc + warp prefix sum) so all lanes run the same push
-    // path; block rounds repeat until a round does no work.
-#ifdef ECL_PROF
     unsigned prof_rounds = 0, prof_drains = 0, prof_pushes = 0;
 #endif
+    // ---- step 2: local fixed point in shared memory, owner-computes pull (Alg. 1
+    // l.10-11 on intra-tile edges).  A flagged vertex re-pulls the max over its intra
+    // neighbours (slots, or its global row when it has more than SLOTS of them); if it
+    // rises it stores the value (single writer) and flags its dependents with plain byte
+    // stores after a block fence.  A thread takes its flag words with an exchange (only
+    // when non-zero), which orders it after every setter it consumed.  Flagged items of a
+    // warp are compacted into a per-warp queue so all lanes run the same path; each warp
+    // drains its own 128 vertices, block rounds repeat until a round does no work.  No
+    // shared-memory atomic touches the signatures.
     if (!SYNC) {
         const int lane = tid & 31, wq0 = (tid >> 5) * (2 * 32 * VPT);
         for (;;) {
@@ -565,11 +597,9 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
 #ifdef ECL_PROF
                 if (lane == 0) prof_drains++;
 #endif
-                // plain load first: a shared atomic costs a full pipe pass per lane
                 unsigned wi = ((volatile unsigned*)s_fin)[tid], wo = ((volatile unsigned*)s_fout)[tid];
                 if (wi) wi = atomicExch(s_fin + tid, 0u);
                 if (wo) wo = atomicExch(s_fout + tid, 0u);
-                // one bit per item: bits 0-3 in-direction of vertex 4t+k, bits 4-7 out-direction
                 const unsigned items = ((wi & 0x01u) | ((wi >> 7) & 0x02u) | ((wi >> 14) & 0x04u) | ((wi >> 21) & 0x08u)) |
                                        (((wo & 0x01u) | ((wo >> 7) & 0x02u) | ((wo >> 14) & 0x04u) | ((wo >> 21) & 0x08u)) << 4);
                 const int c = __popc(items);
@@ -590,30 +620,41 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
                     }
                 }
                 __syncwarp();
+                __threadfence_block();
                 int any = 0;
                 for (int q = lane; q < total; q += 32) {
                     const unsigned item = s_queue[wq0 + q];
                     const int v = (int)(item >> 1);
-                    const bool dir_out = item & 1u;           // v_out rose: push along in-edges
+                    const bool dir_out = item & 1u;
                     int* sig = dir_out ? s_out : s_in;
-                    unsigned* fw = dir_out ? s_fout : s_fin;
-                    const int val = sig[v];
-                    const unsigned long long nb = dir_out ? s_nin[v] : s_nout[v];
-                    push_slots(nb, val, sig, fw, any);
-                    if ((nb & SLOW_MARK) && (nb >> 48) != 0xFFFFull) {
-                        const int32_t* ptr = dir_out ? g.iptr : g.optr;
-                        const int32_t* adj = dir_out ? g.iadj : g.oadj;
-                        for (int e = __ldg(ptr + base + v), ee = __ldg(ptr + base + v + 1); e < ee; e++) {
-                            const int w = __ldg(adj + e) - base;
-                            if ((unsigned)w < (unsigned)cnt && sig[w] < val && atomicMax(sig + w, val) < val) {
-                                flag_set(fw, w); any = 1;
-                            }
+                    // pull: v_in from in-neighbours, v_out from out-neighbours
+                    const unsigned long long src = dir_out ? s_nout[v] : s_nin[v];
+                    const int32_t* sptr = dir_out ? g.optr : g.iptr;
+                    const int32_t* sadj = dir_out ? g.oadj : g.iadj;
+                    const int old = ((volatile int*)sig)[v];
+                    int val = old;
+#pragma unroll
+                    for (int k = 0; k < SLOTS; k++) {
+                        unsigned w = (unsigned)(src >> (16 * k)) & 0xFFFFu;
+                        if (w == NOSLOT) break;
+                        val = max(val, ((volatile int*)sig)[w & 0x7FFFu]);
+                    }
+                    if ((src & SLOW_MARK) && (src >> 48) != 0xFFFFull)
+                        for (int e = __ldg(sptr + base + v), ee = __ldg(sptr + base + v + 1); e < ee; e++) {
+                            const int w = __ldg(sadj + e) - base;
+                            if ((unsigned)w < (unsigned)cnt) val = max(val, ((volatile int*)sig)[w]);
                         }
+                    if (val > old) {
+                        ((volatile int*)sig)[v] = val;
+                        __threadfence_block();
+                        // dependents: out-neighbours re-pull v_in, in-neighbours re-pull v_out
+                        if (dir_out) notify(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
+                        else notify(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
+                        any = 1;
                     }
                 }
                 __syncwarp();
-                // another pass while this warp raised something (possibly its own vertices)
-                if (!__any_sync(FULL, any)) break;
+                if (!__any_sync(FULL, any)) break;           // raised nothing: region drained
             }
             if (!__syncthreads_or(worked)) break;            // a round with no work: done
         }

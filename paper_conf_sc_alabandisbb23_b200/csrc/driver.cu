@@ -87,7 +87,9 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     e = e ? e : A((void**)&p->wsum, (size_t)p->nw_cap * sizeof(int4));
     e = e ? e : A((void**)&p->wscan, (size_t)p->nw_cap * sizeof(int4));
     e = e ? e : A((void**)&p->bsum, (size_t)p->bsum_cap * sizeof(int4));
-    e = e ? e : A((void**)&p->chunks, (size_t)p->chunk_cap * sizeof(Chunk));
+    e = e ? e : A((void**)&p->chunks, 2 * (size_t)p->chunk_cap * sizeof(Chunk));
+    e = e ? e : A((void**)&p->chunk_cnt, (size_t)p->chunk_cap * sizeof(int));
+    e = e ? e : A((void**)&p->hcnt, n1 * sizeof(int2));
     e = e ? e : A((void**)&p->dirty, 2 * (size_t)p->dirty_cap);
     e = e ? e : A((void**)&p->nb_cnt, (size_t)p->dirty_cap * 4);
     e = e ? e : A((void**)&p->nb_list, (size_t)p->dirty_cap * NBCAP * 4);
@@ -114,6 +116,7 @@ void plan_free(Plan* p) {
     }
     cudaFree(p->kin); cudaFree(p->kout); cudaFree(p->newidx); cudaFree(p->cnt);
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
+    cudaFree(p->chunk_cnt); cudaFree(p->hcnt);
     cudaFree(p->dirty);
     cudaFree(p->nb_cnt); cudaFree(p->nb_list); cudaFree(p->done); cudaFree(p->mark); cudaFree(p->sweep_ctr);
     cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
@@ -149,13 +152,35 @@ __global__ void k_scatter_sigs(int32_t na, const int32_t* __restrict__ act, cons
 
 // --------------------------------------------------------------------------- steps
 // a1: CSC of the input graph into buffer 0 (in-degree histogram, scan, scatter)
+static Chunk* chunk_buf(Plan* p, int b) { return (Chunk*)p->chunks + (size_t)b * p->chunk_cap; }
+
+static int read_nchunks(Plan* p, cudaStream_t s, int* out) {
+    CK(cudaMemcpyAsync(&p->hc->nchunks, &p->dc->nchunks, sizeof(int), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (p->hc->nchunks > p->chunk_cap) return fail(ECL_SCC_ECUDA, "internal: long-row chunk list overflow");
+    *out = p->hc->nchunks;
+    return ECL_SCC_OK;
+}
+static unsigned chunk_grid(int nchunks) { return (unsigned)std::max<int64_t>(1, cdiv(nchunks, TPB / WARP)); }
+
+// a1: CSC of the input graph into buffer 0 (in-degree histogram, scan, scatter; long
+// rows by chunks) and the chunk list of the input graph (buffer p->cb)
 static int build_csc(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, cudaStream_t s) {
+    p->cb = 0;
+    Chunk* ch = chunk_buf(p, p->cb);
+    CK(cudaMemsetAsync(&p->dc->nchunks, 0, sizeof(int), s));
+    p->launches++; k_ingest_chunks<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, 0, ch, &p->dc->nchunks, (int)p->chunk_cap);
     CK(cudaMemsetAsync(p->kin, 0, sizeof(int32_t) * (size_t)(n + 1), s));
     p->launches++; k_indeg<<<grid_for(nnz, TPB), TPB, 0, s>>>(nnz, ci, p->kin);
     int r = scan_excl<I1>(p, (const I1*)p->kin, n, (I1*)p->iptr[0], (I1*)&p->dc->grand1, p->bsum, 1, s);
     if (r) return r;
     CK(cudaMemsetAsync(p->kout, 0, sizeof(int32_t) * (size_t)n, s));
     p->launches++; k_csc_scatter<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, ci, p->iptr[0], p->kout, p->iadj[0]);
+    int nout = 0;
+    if ((r = read_nchunks(p, s, &nout))) return r;
+    if (nout) { p->launches++; k_csc_scatter_chunks<<<chunk_grid(nout), TPB, 0, s>>>(ch, nout, ci, p->iptr[0], p->kout, p->iadj[0]); }
+    p->launches++; k_ingest_chunks<<<grid_for(n, TPB), TPB, 0, s>>>(n, p->iptr[0], 1, ch, &p->dc->nchunks, (int)p->chunk_cap);
+    if ((r = read_nchunks(p, s, &p->nchunks_cur))) return r;
     CK(cudaGetLastError());
     return ECL_SCC_OK;
 }
@@ -167,17 +192,30 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
                               int32_t* labels, const Prio& P, cudaStream_t s) {
     const unsigned grid = grid_for(g.na, TPB);
     const int64_t nw = (int64_t)grid * (TPB / WARP);
+    const int nc = p->nchunks_cur, chunked = nc > 0;
+    const Chunk* cur = chunk_buf(p, p->cb);
     CK(cudaMemsetAsync(&p->dc->kept, 0, sizeof(unsigned long long), s));
     CK(cudaMemsetAsync(&p->dc->nchunks, 0, sizeof(int), s));
-    p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, &p->dc->kept);
-    p->launches++; k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->cnt, p->wsum);
+    p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, &p->dc->kept, chunked, p->hcnt);
+    if (chunked) {
+        p->launches += 2;
+        k_keep_chunks<FIRST><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kin, p->kout, &p->dc->kept);
+        k_count_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kin, p->kout, p->chunk_cnt, p->hcnt);
+    }
+    p->launches++; k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->cnt, p->wsum, chunked, p->hcnt);
     int r = scan_excl<I3>(p, (const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
     if (r) return r;
     p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
-                                              (Chunk*)p->chunks, &p->dc->nchunks, (int)p->chunk_cap, P);
+                                              chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P);
     p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->newidx, p->optr[ob],
-                                                          p->iptr[ob], p->oadj[ob], p->iadj[ob]);
+                                                          p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked);
+    if (chunked) {
+        p->launches++;
+        k_scatter_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kin, p->kout, p->chunk_cnt,
+                                                                     p->newidx, p->optr[ob], p->iptr[ob], p->oadj[ob], p->iadj[ob]);
+    }
+    p->cb ^= 1;                                   // the next graph's chunk list is now current
     CK(cudaGetLastError());
     return ECL_SCC_OK;
 }
@@ -327,7 +365,7 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             for (int k = 0; k < batch; k++, pass++) {
                 uint8_t* dc_ = use_dirty ? D[pass & 1] : nullptr;
                 uint8_t* dn_ = use_dirty ? D[(pass + 1) & 1] : nullptr;
-                if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>((const Chunk*)p->chunks, nchunks, g, cin, cout, p->dc, pass, theta); }
+                if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>(chunk_buf(p, p->cb), nchunks, g, cin, cout, p->dc, pass, theta); }
                 const int full = (pass == 0 || nchunks > 0);
                 int r = ECL_SCC_OK;
                 switch (p->tile) {
@@ -419,6 +457,7 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             }
             const int4 t = p->hc->totals;
             const int nchunks = p->hc->nchunks;
+            p->nchunks_cur = nchunks;
             if (st && iter >= 2 && iter - 2 < ECL_SCC_TRACE_MAX) st->edges_kept[iter - 2] = (int64_t)p->hc->kept;
             if (t.y != t.z) return fail(ECL_SCC_ECUDA, "internal: CSR/CSC survivor mismatch %d vs %d", t.y, t.z);
             if (nchunks > p->chunk_cap) return fail(ECL_SCC_ECUDA, "internal: heavy chunk list overflow");

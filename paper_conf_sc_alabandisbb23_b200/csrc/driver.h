@@ -23,7 +23,11 @@ struct Plan {
     int2* cnt;                           // per-vertex surviving (out, in) degree
     int4 *wsum, *wscan;                  // per-warp compaction counts and their prefix
     void* bsum;                          // scan block totals
-    void* chunks;                        // heavy-row chunks (Chunk[chunk_cap])
+    void* chunks;                        // long-row chunks, 2 x Chunk[chunk_cap] (current / next graph)
+    int* chunk_cnt;                      // survivors per chunk of the current graph
+    int2* hcnt;                          // survivors of a vertex's long rows
+    int cb;                              // which chunk buffer belongs to the current graph
+    int nchunks_cur;                     // chunks of the current graph
     int32_t *dbg_tmp;                    // unused placeholder
     DevCounters* dc;                     // device counters
     DevCounters* hc;                     // pinned host mirror

@@ -31,6 +31,7 @@ struct Chunk {
     int32_t i;      // local vertex
     int32_t dir;    // 0: out-row (pull cout), 1: in-row (pull cin)
     int32_t beg, end;
+    int32_t first;  // index of the first chunk of the same row (rows are contiguous runs)
 };
 
 // ------------------------------------------------------------------ init / validation
@@ -67,6 +68,7 @@ static __global__ void k_csc_scatter(int32_t n, const int32_t* __restrict__ rp, 
     const bool valid = u < n;
     int b = 0, e = 0;
     if (valid) { b = rp[u]; e = rp[u + 1]; }
+    if (e - b > HEAVY_T) e = b;                          // long row: k_csc_scatter_chunks
     if (valid && e - b <= HEAVY)
         for (int k = b; k < e; k++) {
             const int w = ci[k];
@@ -123,8 +125,10 @@ __device__ __forceinline__ RowCtx load_row(const WGraph& g, int64_t i, const int
 
 // count edges of one row (light: by the lane, heavy: by the whole warp) that satisfy P
 template <typename P>
-__device__ __forceinline__ int count_row(const int32_t* __restrict__ adj, int rb, int re, bool go, int lane, P pred) {
+__device__ __forceinline__ int count_row(const int32_t* __restrict__ adj, int rb, int re, bool go, int lane, P pred,
+                                         bool chunked = false) {
     int c = 0;
+    if (chunked && re - rb > HEAVY_T) go = false;      // long row: the chunk kernels count it
     if (go && re - rb <= HEAVY)
         for (int e = rb; e < re; e++) c += pred(__ldg(adj + e));
     unsigned hm = __ballot_sync(FULL, go && re - rb > HEAVY);
@@ -172,14 +176,14 @@ struct SurvivePred {
 template <bool FIRST>
 static __global__ void k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                              int32_t* __restrict__ kin, int32_t* __restrict__ kout,
-                             unsigned long long* __restrict__ kept) {
+                             unsigned long long* __restrict__ kept, int chunked, int2* __restrict__ hcnt) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
     KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout};
-    const int co = count_row(g.oadj, r.ob, r.oe, r.live, lane, pred);
-    const int ci = count_row(g.iadj, r.ib, r.ie, r.live, lane, pred);
-    if (r.valid) { kin[i] = ci; kout[i] = co; }
+    const int co = count_row(g.oadj, r.ob, r.oe, r.live, lane, pred, chunked);
+    const int ci = count_row(g.iadj, r.ib, r.ie, r.live, lane, pred, chunked);
+    if (r.valid) { kin[i] = ci; kout[i] = co; hcnt[i] = make_int2(0, 0); }
     const int s = warp_sum(co);
     if (lane == 0 && s) atomicAdd(kept, (unsigned long long)s);
 }
@@ -188,7 +192,8 @@ static __global__ void k_keep_count(WGraph g, const int32_t* __restrict__ cin, c
 template <bool FIRST, bool TRIM>
 static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                 const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
-                                int2* __restrict__ cnt, int4* __restrict__ wsum) {
+                                int2* __restrict__ cnt, int4* __restrict__ wsum, int chunked,
+                                const int2* __restrict__ hcnt) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
@@ -198,8 +203,13 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
     } else {
         const bool go = r.live && !trimmed(kin, kout, (int)i);
         SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
-        nout = count_row(g.oadj, r.ob, r.oe, go, lane, pred);
-        nin = count_row(g.iadj, r.ib, r.ie, go, lane, pred);
+        nout = count_row(g.oadj, r.ob, r.oe, go, lane, pred, chunked);
+        nin = count_row(g.iadj, r.ib, r.ie, go, lane, pred, chunked);
+        if (chunked && r.valid) {                       // long rows: counted by k_count_chunks
+            const int2 h = hcnt[i];
+            nout += h.x;
+            nin += h.y;
+        }
     }
     if (r.valid) cnt[i] = make_int2(nout, nin);
     const int alive = (nout + nin) > 0;
@@ -249,7 +259,7 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
                 const int nc = (deg + CHUNK - 1) / CHUNK;
                 const int at = atomicAdd(nchunks, nc);
                 for (int k = 0; k < nc && at + k < chunk_cap; k++)
-                    chunks[at + k] = Chunk{j, dir, beg + k * CHUNK, min(beg + (k + 1) * CHUNK, beg + deg)};
+                    chunks[at + k] = Chunk{j, dir, beg + k * CHUNK, min(beg + (k + 1) * CHUNK, beg + deg), at};
             }
         }
     } else {
@@ -299,7 +309,8 @@ static __global__ void k_snapshot_left(int32_t n, const int32_t* __restrict__ la
 template <typename P>
 __device__ __forceinline__ void emit_row(const int32_t* __restrict__ adj, int rb, int re, bool go, int pos,
                                          const int32_t* __restrict__ newidx, int32_t* __restrict__ dst, int lane,
-                                         P pred) {
+                                         P pred, bool chunked = false) {
+    if (chunked && re - rb > HEAVY_T) go = false;      // long row: k_scatter_chunks writes it
     if (go && re - rb <= HEAVY) {
         for (int e = rb; e < re; e++) {
             const int x = __ldg(adj + e);
@@ -330,7 +341,7 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
                                   const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
                                   const int32_t* __restrict__ newidx, const int32_t* __restrict__ optr2,
                                   const int32_t* __restrict__ iptr2, int32_t* __restrict__ oadj2,
-                                  int32_t* __restrict__ iadj2) {
+                                  int32_t* __restrict__ iadj2, int chunked) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
@@ -339,8 +350,115 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
     int po = 0, pi = 0;
     if (go) { po = optr2[j]; pi = iptr2[j]; }
     SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
-    emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred);
-    emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred);
+    emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred, chunked);
+    emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred, chunked);
+}
+
+// ------------------------------------------------------------------ long rows in chunks
+// Rows longer than HEAVY_T are split into CHUNK-edge pieces (one warp each) in every
+// compaction kernel, so a 100k-edge hub costs 200 warps, not one.  Counts are folded in
+// with atomics; the scatter places a chunk after the survivors of the earlier chunks of
+// its row (chunk_cnt prefix), so rows stay stable.
+template <bool FIRST>
+static __global__ void __launch_bounds__(256) k_keep_chunks(WGraph g, const Chunk* __restrict__ chunks, int nchunks,
+                                                            const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+                                                            int32_t* __restrict__ kin, int32_t* __restrict__ kout,
+                                                            unsigned long long* __restrict__ kept) {
+    const int lane = threadIdx.x & 31;
+    const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (c >= nchunks) return;
+    const Chunk k = chunks[c];
+    const int a = FIRST ? 0 : cin[k.i], b = FIRST ? 0 : cout[k.i];
+    if (!FIRST && a == b) return;                        // finished owner keeps nothing
+    const int32_t* adj = k.dir ? g.iadj : g.oadj;
+    int cc = 0;
+    for (int e = k.beg + lane; e < k.end; e += WARP) cc += keep_edge<FIRST>(k.i, a, b, __ldg(adj + e), cin, cout);
+    cc = warp_sum(cc);
+    if (lane == 0 && cc) {
+        atomicAdd(k.dir ? kin + k.i : kout + k.i, cc);
+        if (!k.dir) atomicAdd(kept, (unsigned long long)cc);
+    }
+}
+template <bool FIRST, bool TRIM>
+static __global__ void __launch_bounds__(256) k_count_chunks(WGraph g, const Chunk* __restrict__ chunks, int nchunks,
+                                                             const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+                                                             const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
+                                                             int* __restrict__ chunk_cnt, int2* __restrict__ hcnt) {
+    const int lane = threadIdx.x & 31;
+    const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (c >= nchunks) return;
+    const Chunk k = chunks[c];
+    const int a = FIRST ? 0 : cin[k.i], b = FIRST ? 0 : cout[k.i];
+    int cc = 0;
+    if ((FIRST || a != b) && !(TRIM && trimmed(kin, kout, k.i))) {
+        const int32_t* adj = k.dir ? g.iadj : g.oadj;
+        SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kin, kout};
+        for (int e = k.beg + lane; e < k.end; e += WARP) cc += pred(__ldg(adj + e));
+        cc = warp_sum(cc);
+    }
+    if (lane == 0) {
+        chunk_cnt[c] = cc;
+        if (cc) atomicAdd(k.dir ? &hcnt[k.i].y : &hcnt[k.i].x, cc);
+    }
+}
+template <bool FIRST, bool TRIM>
+static __global__ void __launch_bounds__(256) k_scatter_chunks(WGraph g, const Chunk* __restrict__ chunks, int nchunks,
+                                                               const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+                                                               const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
+                                                               const int* __restrict__ chunk_cnt,
+                                                               const int32_t* __restrict__ newidx,
+                                                               const int32_t* __restrict__ optr2, const int32_t* __restrict__ iptr2,
+                                                               int32_t* __restrict__ oadj2, int32_t* __restrict__ iadj2) {
+    const int lane = threadIdx.x & 31;
+    const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (c >= nchunks) return;
+    const Chunk k = chunks[c];
+    if (chunk_cnt[c] == 0) return;
+    const int j = newidx[k.i];
+    // survivors of the earlier chunks of this row
+    int before = 0;
+    for (int q = k.first + lane; q < (int)c; q += WARP) before += chunk_cnt[q];
+    before = warp_sum(before);
+    int pos = (k.dir ? iptr2[j] : optr2[j]) + before;
+    const int a = FIRST ? 0 : cin[k.i], b = FIRST ? 0 : cout[k.i];
+    const int32_t* adj = k.dir ? g.iadj : g.oadj;
+    int32_t* dst = k.dir ? iadj2 : oadj2;
+    SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kin, kout};
+    for (int base = k.beg; base < k.end; base += WARP) {
+        const int e = base + lane;
+        int x = 0;
+        if (e < k.end) x = __ldg(adj + e);
+        const bool keep = (e < k.end) && pred(x);
+        const unsigned bm = __ballot_sync(FULL, keep);
+        if (keep) dst[pos + __popc(bm & ((1u << lane) - 1))] = __ldg(newidx + x);
+        pos += __popc(bm);
+    }
+}
+// chunk list of the input graph (CSR rows from row_ptr, CSC rows from iptr)
+static __global__ void k_ingest_chunks(int32_t n, const int32_t* __restrict__ ptr, int dir, Chunk* __restrict__ chunks,
+                                       int* __restrict__ nchunks, int chunk_cap) {
+    const int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (v >= n) return;
+    const int beg = ptr[v], deg = ptr[v + 1] - beg;
+    if (deg <= HEAVY_T) return;
+    const int nc = (deg + CHUNK - 1) / CHUNK;
+    const int at = atomicAdd(nchunks, nc);
+    for (int k = 0; k < nc && at + k < chunk_cap; k++)
+        chunks[at + k] = Chunk{(int32_t)v, dir, beg + k * CHUNK, min(beg + (k + 1) * CHUNK, beg + deg), at};
+}
+// CSC scatter of long CSR rows (input graph)
+static __global__ void __launch_bounds__(256) k_csc_scatter_chunks(const Chunk* __restrict__ chunks, int nchunks,
+                                                                   const int32_t* __restrict__ ci, const int32_t* __restrict__ iptr,
+                                                                   int32_t* __restrict__ cursor, int32_t* __restrict__ iadj) {
+    const int lane = threadIdx.x & 31;
+    const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (c >= nchunks) return;
+    const Chunk k = chunks[c];
+    if (k.dir) return;
+    for (int e = k.beg + lane; e < k.end; e += WARP) {
+        const int w = ci[e];
+        iadj[iptr[w] + atomicAdd(&cursor[w], 1)] = k.i;
+    }
 }
 
 // ------------------------------------------------------------------ Phase 2

@@ -283,9 +283,21 @@ static __global__ void k_relabel_rep(int32_t n, int32_t* __restrict__ labels, in
     }
 }
 static __global__ void k_relabel_max(int32_t n, const int32_t* __restrict__ labels, int32_t* __restrict__ slot, Prio P) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-        const int l = labels[v];
-        if (l < 0 && (int)prio_of(P, (uint32_t)v) != -l - 1) atomicMax(slot - l - 1, (int)v);
+    // lanes that target the same slot (a giant SCC: most of them) combine first, so the
+    // slot sees one atomic per group instead of one per vertex
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t start = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    for (int64_t v0 = start - (threadIdx.x & 31); v0 < n; v0 += stride) {
+        const int64_t v = v0 + (threadIdx.x & 31);
+        int key = -1, val = -1;
+        if (v < n) {
+            const int l = labels[v];
+            if (l < 0 && (int)prio_of(P, (uint32_t)v) != -l - 1) { key = -l - 1; val = (int)v; }
+        }
+        const unsigned grp = __match_any_sync(FULL, key);
+        int m = val;
+        for (unsigned g = grp; g; g &= g - 1) m = max(m, __shfl_sync(grp, val, __ffs(g) - 1));
+        if (key >= 0 && (threadIdx.x & 31) == __ffs(grp) - 1) atomicMax(slot + key, m);
     }
 }
 static __global__ void k_relabel_apply(int32_t n, int32_t* __restrict__ labels, const int32_t* __restrict__ slot) {
@@ -828,7 +840,8 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
 template <bool SYNC, int TT>
 static __global__ void __launch_bounds__(TT / VPT, (1536 / (TT / VPT)) > 0 ? 1536 / (TT / VPT) : 1)
 k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, DevCounters* __restrict__ dc, int pass,
-            int first, uint8_t* __restrict__ dirty_cur, uint8_t* __restrict__ dirty_next, int full, int theta) {
+            int first, uint8_t* __restrict__ dirty_cur, uint8_t* __restrict__ dirty_next, int full, int theta,
+            int run) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];             // raise flags, byte k = vertex 4t+k
     __shared__ unsigned short s_queue[2 * TT];                         // per-warp item queues
@@ -843,21 +856,30 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
     S.s_queue = s_queue;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + TT - 1) / TT;
-    const int tile = (pass & 1) ? (ntiles - 1 - (int)blockIdx.x) : (int)blockIdx.x;
     const int tid = threadIdx.x;
-    // dirty-tile skipping: a tile whose inputs did not change since its last visit is at
-    // its local fixed point already.  The read flag is cleared here, so after pass p the
-    // buffer read in pass p is all zero and pass p+1 can fill it for pass p+2.
-    if (dirty_cur) {
-        if (tid == 0) {
-            s_dirty = dirty_cur[tile];
-            dirty_cur[tile] = 0;
+    int ch_any = 0;
+    // Each CTA walks a run of `run` consecutive tiles in order (reversed on odd passes):
+    // a tile then sees the tile before it in the run already finished (Gauss-Seidel along
+    // the run), while different runs proceed in parallel.
+    for (int j = 0; j < run; j++) {
+        const int idx = (int)blockIdx.x * run + ((pass & 1) ? run - 1 - j : j);
+        if (idx >= ntiles) continue;
+        const int tile = (pass & 1) ? ntiles - 1 - idx : idx;
+        // dirty-tile skipping: a tile whose inputs did not change since its last visit is
+        // at its local fixed point already.  The read flag is cleared here, so after pass p
+        // the buffer read in pass p is all zero and pass p+1 can fill it for pass p+2.
+        if (dirty_cur) {
+            if (tid == 0) {
+                s_dirty = dirty_cur[tile];
+                dirty_cur[tile] = 0;
+            }
+            __syncthreads();
+            if (!s_dirty) continue;
         }
-        __syncthreads();
-        if (!s_dirty) return;
+        ch_any |= tile_visit<SYNC, TT>(g, cin, cout, dc, tile, full, theta, MarkNext{dirty_next}, S);
+        __syncthreads();                                     // shared memory is reused by the next tile
     }
-    const int ch = tile_visit<SYNC, TT>(g, cin, cout, dc, tile, full, theta, MarkNext{dirty_next}, S);
-    if (ch && tid == 0) dc->changed[pass & (RING - 1)] = 1;
+    if (ch_any && tid == 0) dc->changed[pass & (RING - 1)] = 1;
 }
 
 // ---------------------------------------------------------------------- sweep mode

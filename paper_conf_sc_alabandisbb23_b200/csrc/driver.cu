@@ -236,20 +236,12 @@ template <int TT>
 static int launch_tile(Plan* p, bool sync, const WGraph& g, int32_t* cin, int32_t* cout, int pass, int first,
                        uint8_t* dcur, uint8_t* dnext, int full, int theta, cudaStream_t s) {
     if (int r = set_tile_attrs<TT>()) return r;
-    static int resident = 0;
-    if (!resident) {
-        int per_sm = 0, dev = 0, sms = 0;
-        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_tile<false, TT>, TT / VPT, tile_dyn_smem<TT>()));
-        CK(cudaGetDevice(&dev));
-        CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-        resident = std::max(1, per_sm) * sms;
-    }
     const int64_t ntiles = cdiv(g.na, TT);
-    // runs of consecutive tiles per CTA (Gauss-Seidel along a run); ECL_SCC_RUN=1 gives
-    // one tile per CTA
+    // runs of consecutive tiles per CTA (Gauss-Seidel along a run).  Measured on C4: run
+    // 4 beats 1 (-14%), longer runs starve the SMs (fewer CTAs than resident slots).
     static int run_env = -1;
-    if (run_env < 0) run_env = getenv("ECL_SCC_RUN") ? std::max(1, atoi(getenv("ECL_SCC_RUN"))) : 0;
-    const int run = run_env ? run_env : (int)std::max<int64_t>(1, cdiv(ntiles, resident));
+    if (run_env < 0) run_env = getenv("ECL_SCC_RUN") ? std::max(1, atoi(getenv("ECL_SCC_RUN"))) : 4;
+    const int run = (int)std::min<int64_t>(run_env, std::max<int64_t>(1, ntiles / (2 * 148)));
     const unsigned grid = (unsigned)cdiv(ntiles, run);
     p->launches++;
     if (sync) k_prop_tile<true, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, nullptr, nullptr, 1, theta, run);

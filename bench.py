@@ -148,7 +148,7 @@ def reference_arm(args):
     v = g.nnz / t / 1e6
     line = {"impl": "reference", "metric": "SCC detection Medges/s", "value": round(v, 3), "unit": "Medges/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 3),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int32",
             "data": "synthetic", "config": workload(args, g),
             "cpu_baseline": {"value": round(v, 3), "unit": "Medges/s", "cores": 1, "kind": "oracle",
                              "sample": f"full graph ({g.n} vertices, {g.nnz} edges), O1 Tarjan+max-relabel, "

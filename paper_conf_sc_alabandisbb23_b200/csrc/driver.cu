@@ -243,9 +243,12 @@ static int launch_tile(Plan* p, bool sync, const WGraph& g, int32_t* cin, int32_
     if (run_env < 0) run_env = getenv("ECL_SCC_RUN") ? std::max(1, atoi(getenv("ECL_SCC_RUN"))) : 4;
     const int run = (int)std::min<int64_t>(run_env, std::max<int64_t>(1, ntiles / (2 * 148)));
     const unsigned grid = (unsigned)cdiv(ntiles, run);
+    static int kcap = -1;    // >0: bounded SIMD rounds in shared memory instead of drains
+    if (kcap < 0) kcap = getenv("ECL_SCC_KCAP") ? std::max(0, atoi(getenv("ECL_SCC_KCAP"))) : 0;
+    const int kc = dnext ? kcap : 0;   // the cap needs dirty marking to resume
     p->launches++;
-    if (sync) k_prop_tile<true, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, nullptr, nullptr, 1, theta, run);
-    else k_prop_tile<false, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, dcur, dnext, full, theta, run);
+    if (sync) k_prop_tile<true, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, nullptr, nullptr, 1, theta, run, 0);
+    else k_prop_tile<false, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, dcur, dnext, full, theta, run, kc);
     return ECL_SCC_OK;
 }
 

@@ -620,7 +620,7 @@ __device__ __forceinline__ void notify(unsigned long long nb, const int32_t* __r
 template <bool SYNC, int TT, typename Mark>
 __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__ cin, int32_t* __restrict__ cout,
                                           DevCounters* __restrict__ dc, int tile, int full, int theta, Mark mark,
-                                          const TileSmem<TT>& S) {
+                                          const TileSmem<TT>& S, int kcap = 0, int* capped = nullptr) {
     int* s_in = S.s_in;
     int* s_out = S.s_out;
     unsigned long long* s_nin = S.s_nin;
@@ -716,7 +716,42 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
     // warp are compacted into a per-warp queue so all lanes run the same path; each warp
     // drains its own 128 vertices, block rounds repeat until a round does no work.  No
     // shared-memory atomic touches the signatures.
-    if (!SYNC) {
+    if (!SYNC && kcap > 0) {
+        // bounded variant: at most kcap SIMD Jacobi rounds over the slots (each thread
+        // re-pulls its four vertices every round); a tile still changing after kcap rounds
+        // reports `capped` and is revisited in the next pass
+        for (int r = 0; r < kcap; r++) {
+            int any = 0;
+#pragma unroll
+            for (int k = 0; k < VPT; k++) {
+                const int v = tid * VPT + k;
+                if (v >= cnt) continue;
+                for (int dir = 0; dir < 2; dir++) {
+                    int* sig = dir ? s_out : s_in;
+                    const unsigned long long src = dir ? s_nout[v] : s_nin[v];
+                    const int old = ((volatile int*)sig)[v];
+                    int val = old;
+#pragma unroll
+                    for (int q = 0; q < SLOTS; q++) {
+                        const unsigned w = (unsigned)(src >> (16 * q)) & 0xFFFFu;
+                        if (w == NOSLOT) break;
+                        val = max(val, ((volatile int*)sig)[w & 0x7FFFu]);
+                    }
+                    if ((src & SLOW_MARK) && (src >> 48) != 0xFFFFull) {
+                        const int32_t* sptr = dir ? g.optr : g.iptr;
+                        const int32_t* sadj = dir ? g.oadj : g.iadj;
+                        for (int e = __ldg(sptr + base + v), ee = __ldg(sptr + base + v + 1); e < ee; e++) {
+                            const int w = __ldg(sadj + e) - base;
+                            if ((unsigned)w < (unsigned)cnt) val = max(val, ((volatile int*)sig)[w]);
+                        }
+                    }
+                    if (val > old) { ((volatile int*)sig)[v] = val; any = 1; }
+                }
+            }
+            if (!__syncthreads_or(any)) break;
+            if (r == kcap - 1 && capped) *capped = 1;
+        }
+    } else if (!SYNC) {
         const int lane = tid & 31, wq0 = (tid >> 5) * (2 * 32 * VPT);
         for (;;) {
             int worked = 0;
@@ -841,7 +876,7 @@ template <bool SYNC, int TT>
 static __global__ void __launch_bounds__(TT / VPT, (1536 / (TT / VPT)) > 0 ? 1536 / (TT / VPT) : 1)
 k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, DevCounters* __restrict__ dc, int pass,
             int first, uint8_t* __restrict__ dirty_cur, uint8_t* __restrict__ dirty_next, int full, int theta,
-            int run) {
+            int run, int kcap) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];             // raise flags, byte k = vertex 4t+k
     __shared__ unsigned short s_queue[2 * TT];                         // per-warp item queues
@@ -876,7 +911,9 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
             __syncthreads();
             if (!s_dirty) continue;
         }
-        ch_any |= tile_visit<SYNC, TT>(g, cin, cout, dc, tile, full, theta, MarkNext{dirty_next}, S);
+        int capped = 0;
+        ch_any |= tile_visit<SYNC, TT>(g, cin, cout, dc, tile, full, theta, MarkNext{dirty_next}, S, kcap, &capped);
+        if (capped && dirty_next && tid == 0) dirty_next[tile] = 1;   // not converged: come back
         __syncthreads();                                     // shared memory is reused by the next tile
     }
     if (ch_any && tid == 0) dc->changed[pass & (RING - 1)] = 1;

@@ -13,7 +13,8 @@
 extern "C" int64_t tilesim(int32_t n, const int32_t* rp, const int32_t* ci, const int32_t* tile_of, int32_t ntiles,
                            const int32_t* prio, int64_t* out /* passes, visits, visited_vertices, raises */, int heap,
                            int gs /* 1: Gauss-Seidel across tiles, alternating order */,
-                           const int32_t* order /* tile dispatch order (nullptr: index) */, int32_t window) {
+                           const int32_t* order /* tile dispatch order (nullptr: index) */, int32_t window,
+                           int32_t kround /* >0: exactly kround Jacobi rounds inside a tile instead of its fixed point */) {
     // CSC
     std::vector<int32_t> cp(n + 1, 0), cr(rp[n]);
     for (int64_t e = 0; e < rp[n]; e++) cp[ci[e] + 1]++;
@@ -67,7 +68,22 @@ extern "C" int64_t tilesim(int32_t n, const int32_t* rp, const int32_t* ci, cons
                 qi.push_back(v); qo.push_back(v); inq_in[v] = inq_out[v] = 1;
             }
             // step 2: local fixed point by pushes (FIFO, or max-value-first with heap=1)
-            if (heap) {
+            if (kround > 0) {
+                qi.clear(); qo.clear();
+                for (int v : members[t]) inq_in[v] = inq_out[v] = 0;
+                std::vector<int32_t> ti, to;
+                for (int r = 0; r < kround; r++) {
+                    ti.clear(); to.clear();
+                    for (int v : members[t]) {
+                        int x = vin[v], y = vout[v];
+                        for (int e = cp[v]; e < cp[v + 1]; e++) { int u = cr[e]; if (tile_of[u] == t) x = std::max(x, vin[u]); }
+                        for (int e = rp[v]; e < rp[v + 1]; e++) { int w = ci[e]; if (tile_of[w] == t) y = std::max(y, vout[w]); }
+                        ti.push_back(x); to.push_back(y);
+                    }
+                    size_t k = 0;
+                    for (int v : members[t]) { if (ti[k] > vin[v]) { vin[v] = ti[k]; raises++; } if (to[k] > vout[v]) { vout[v] = to[k]; raises++; } k++; }
+                }
+            } else if (heap) {
                 std::priority_queue<std::pair<int,int>> hi, ho;
                 for (int v : members[t]) { hi.push({vin[v], v}); ho.push({vout[v], v}); }
                 qi.clear(); qo.clear();

@@ -91,6 +91,7 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     e = e ? e : A((void**)&p->chunk_cnt, (size_t)p->chunk_cap * sizeof(int));
     e = e ? e : A((void**)&p->hcnt, n1 * sizeof(int2));
     e = e ? e : A((void**)&p->dirty, 2 * (size_t)p->dirty_cap);
+    e = e ? e : A((void**)&p->lvl, n1);
     e = e ? e : A((void**)&p->nb_cnt, (size_t)p->dirty_cap * 4);
     e = e ? e : A((void**)&p->nb_list, (size_t)p->dirty_cap * NBCAP * 4);
     e = e ? e : A((void**)&p->done, (size_t)p->dirty_cap * 4);
@@ -117,7 +118,7 @@ void plan_free(Plan* p) {
     cudaFree(p->kin); cudaFree(p->kout); cudaFree(p->newidx); cudaFree(p->cnt);
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
     cudaFree(p->chunk_cnt); cudaFree(p->hcnt);
-    cudaFree(p->dirty);
+    cudaFree(p->dirty); cudaFree(p->lvl);
     cudaFree(p->nb_cnt); cudaFree(p->nb_list); cudaFree(p->done); cudaFree(p->mark); cudaFree(p->sweep_ctr);
     cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
     if (p->hc) cudaFreeHost(p->hc);
@@ -246,9 +247,12 @@ static int launch_tile(Plan* p, bool sync, const WGraph& g, int32_t* cin, int32_
     static int kcap = -1;    // >0: bounded SIMD rounds in shared memory instead of drains
     if (kcap < 0) kcap = getenv("ECL_SCC_KCAP") ? std::max(0, atoi(getenv("ECL_SCC_KCAP"))) : 0;
     const int kc = dnext ? kcap : 0;   // the cap needs dirty marking to resume
+    static int levels = -1;  // level sweeps inside a tile (needs dirty mode: levels built on the first pass)
+    if (levels < 0) levels = getenv("ECL_SCC_LEVELS") ? atoi(getenv("ECL_SCC_LEVELS")) : 0;
+    uint8_t* lv = (levels && dnext && TT >= 1024) ? p->lvl : nullptr;
     p->launches++;
-    if (sync) k_prop_tile<true, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, nullptr, nullptr, 1, theta, run, 0);
-    else k_prop_tile<false, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, dcur, dnext, full, theta, run, kc);
+    if (sync) k_prop_tile<true, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, nullptr, nullptr, 1, theta, run, 0, nullptr);
+    else k_prop_tile<false, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, dcur, dnext, full, theta, run, kc, lv);
     return ECL_SCC_OK;
 }
 

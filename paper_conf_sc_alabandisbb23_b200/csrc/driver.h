@@ -38,6 +38,7 @@ struct Plan {
     uint8_t* dirty;                      // 2 x dirty_cap tile flags (Phase-2 skipping)
     int64_t dirty_cap;
     int tile;                            // Phase-2 tile size (vertices per CTA)
+    uint8_t* lvl;                        // level-sweep mode: intra-tile level per vertex
     int *nb_cnt, *nb_list;               // sweep mode: neighbour tiles of each tile
     int *done, *mark;                    // sweep mode: per-tile done / dirty epochs
     int* sweep_ctr;                      // [0] tile counter, [1] changed, [2] overflow

@@ -579,8 +579,26 @@ struct TileSmem {
     unsigned long long* s_nout;
     unsigned* s_fin;
     unsigned* s_fout;
-    unsigned short* s_queue;
+    unsigned short* s_queue;      // drain item queues; level-sweep order + level starts
+    uint8_t* s_lv;                // level-sweep: intra-tile level of each vertex
 };
+
+// pull of one vertex over its slots (and its global row when it is a slow row)
+__device__ __forceinline__ int pull_slots(const int* sig, unsigned long long src, const int32_t* __restrict__ sptr,
+                                          const int32_t* __restrict__ sadj, int base, int cnt, int v, int val) {
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+        const unsigned w = (unsigned)(src >> (16 * q)) & 0xFFFFu;
+        if (w == 0xFFFFu) break;
+        val = max(val, ((volatile const int*)sig)[w & 0x7FFFu]);
+    }
+    if ((src & (0x8000ull << 48)) && (src >> 48) != 0xFFFFull)
+        for (int e = __ldg(sptr + base + v), ee = __ldg(sptr + base + v + 1); e < ee; e++) {
+            const int w = __ldg(sadj + e) - base;
+            if ((unsigned)w < (unsigned)cnt) val = max(val, ((volatile const int*)sig)[w]);
+        }
+    return val;
+}
 
 // dirty marking of the tiles that depend on a raised value (pass mode: byte flags for
 // the next pass; sweep mode: the current sweep epoch)
@@ -620,7 +638,8 @@ __device__ __forceinline__ void notify(unsigned long long nb, const int32_t* __r
 template <bool SYNC, int TT, typename Mark>
 __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__ cin, int32_t* __restrict__ cout,
                                           DevCounters* __restrict__ dc, int tile, int full, int theta, Mark mark,
-                                          const TileSmem<TT>& S, int kcap = 0, int* capped = nullptr) {
+                                          const TileSmem<TT>& S, int kcap = 0, int* capped = nullptr,
+                                          uint8_t* __restrict__ lvl = nullptr) {
     int* s_in = S.s_in;
     int* s_out = S.s_out;
     unsigned long long* s_nin = S.s_nin;
@@ -716,6 +735,120 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
     // warp are compacted into a per-warp queue so all lanes run the same path; each warp
     // drains its own 128 vertices, block rounds repeat until a round does no work.  No
     // shared-memory atomic touches the signatures.
+    // ---- step 2 (level-sweep variant): intra-tile levels (longest path from the tile's
+    // sources over intra edges, by relaxation, capped) are computed on the first visit of
+    // a phase and kept in `lvl`; every visit then pulls v_in in ascending and v_out in
+    // descending level order -- one pull per vertex per sweep for the acyclic part -- and
+    // checks with one Jacobi round; cycles left over fall through to the drain loop.
+    bool need_drain = true;
+    if (!SYNC && lvl && kcap == 0) {
+        int* s_L = (int*)S.s_queue;                          // [TT] ints during the level build
+        uint8_t* s_lv = S.s_lv;
+        if (full) {
+            for (int v = tid; v < TT; v += TT / VPT) s_L[v] = 0;
+            __syncthreads();
+            for (int r = 0; r < 64; r++) {
+                int any = 0;
+#pragma unroll
+                for (int k = 0; k < VPT; k++) {
+                    const int v = tid * VPT + k;
+                    if (v >= cnt) continue;
+                    const unsigned long long src = s_nin[v];
+                    int l = ((volatile int*)s_L)[v];
+                    const int l0 = l;
+#pragma unroll
+                    for (int q = 0; q < 4; q++) {
+                        const unsigned w = (unsigned)(src >> (16 * q)) & 0xFFFFu;
+                        if (w == 0xFFFFu) break;
+                        l = max(l, ((volatile int*)s_L)[w & 0x7FFFu] + 1);
+                    }
+                    l = min(l, 250);
+                    if (l > l0) { ((volatile int*)s_L)[v] = l; any = 1; }
+                }
+                if (!__syncthreads_or(any)) break;
+            }
+            for (int v = tid; v < cnt; v += TT / VPT) {
+                s_lv[v] = (uint8_t)s_L[v];
+                lvl[base + v] = (uint8_t)s_L[v];
+            }
+        } else {
+            for (int v = tid; v < cnt; v += TT / VPT) s_lv[v] = __ldg(lvl + base + v);
+        }
+        __syncthreads();
+        // counting sort by level: order[] (u16) and level starts in the queue area
+        unsigned short* order = S.s_queue;
+        int* lstart = (int*)(S.s_queue + TT);                  // [257]
+        for (int i = tid; i < 257; i += TT / VPT) lstart[i] = 0;
+        __syncthreads();
+        for (int v = tid; v < cnt; v += TT / VPT) atomicAdd(lstart + s_lv[v] + 1, 1);
+        __syncthreads();
+        if (tid < 32) {                                        // exclusive scan of 256 bins by one warp
+            int carry = 0;
+            for (int b0 = 0; b0 < 256; b0 += 32) {
+                const int x = lstart[b0 + 1 + tid];
+                const int inc = warp_incl_scan(x, tid);
+                lstart[b0 + 1 + tid] = carry + inc;
+                carry += __shfl_sync(FULL, inc, 31);
+            }
+        }
+        __syncthreads();
+        int maxl = 0;
+        for (int v = tid; v < cnt; v += TT / VPT) maxl = max(maxl, (int)s_lv[v]);
+        // scatter (positions via a per-level cursor reusing the s_fin area)
+        int* cursor = (int*)S.s_fin;                           // >= 256 ints (TT/VPT >= 256)
+        for (int i = tid; i < 256; i += TT / VPT) cursor[i] = 0;
+        __syncthreads();
+        for (int v = tid; v < cnt; v += TT / VPT) {
+            const int l = s_lv[v];
+            order[lstart[l] + atomicAdd(cursor + l, 1)] = (unsigned short)v;
+        }
+        // every thread needs the maximum level
+        maxl = __reduce_max_sync(FULL, maxl);
+        __shared__ int s_maxl;
+        if (tid == 0) s_maxl = 0;
+        __syncthreads();
+        if ((tid & 31) == 0) atomicMax(&s_maxl, maxl);
+        __syncthreads();
+        maxl = s_maxl;
+        for (int rep = 0; rep < 3 && need_drain; rep++) {
+            // sweeps: v_in at level l (ascending), v_out at level maxl-l (descending)
+            for (int l = 0; l <= maxl; l++) {
+                for (int i = lstart[l] + tid; i < lstart[l + 1]; i += TT / VPT) {
+                    const int v = order[i];
+                    const int old = ((volatile int*)s_in)[v];
+                    const int val = pull_slots(s_in, s_nin[v], g.iptr, g.iadj, base, cnt, v, old);
+                    if (val > old) ((volatile int*)s_in)[v] = val;
+                }
+                const int lo = maxl - l;
+                for (int i = lstart[lo] + tid; i < lstart[lo + 1]; i += TT / VPT) {
+                    const int v = order[i];
+                    const int old = ((volatile int*)s_out)[v];
+                    const int val = pull_slots(s_out, s_nout[v], g.optr, g.oadj, base, cnt, v, old);
+                    if (val > old) ((volatile int*)s_out)[v] = val;
+                }
+                __syncthreads();
+            }
+            // check: one Jacobi round; no change means the local fixed point
+            int any = 0;
+#pragma unroll
+            for (int k = 0; k < VPT; k++) {
+                const int v = tid * VPT + k;
+                if (v >= cnt) continue;
+                int old = ((volatile int*)s_in)[v];
+                int val = pull_slots(s_in, s_nin[v], g.iptr, g.iadj, base, cnt, v, old);
+                if (val > old) { ((volatile int*)s_in)[v] = val; any = 1; }
+                old = ((volatile int*)s_out)[v];
+                val = pull_slots(s_out, s_nout[v], g.optr, g.oadj, base, cnt, v, old);
+                if (val > old) { ((volatile int*)s_out)[v] = val; any = 1; }
+            }
+            need_drain = __syncthreads_or(any) != 0;
+        }
+        if (need_drain) {                                      // cycles: finish with the drains
+            s_fin[tid] = 0x01010101u;
+            s_fout[tid] = 0x01010101u;
+        }
+        __syncthreads();
+    }
     if (!SYNC && kcap > 0) {
         // bounded variant: at most kcap SIMD Jacobi rounds over the slots (each thread
         // re-pulls its four vertices every round); a tile still changing after kcap rounds
@@ -751,7 +884,7 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
             if (!__syncthreads_or(any)) break;
             if (r == kcap - 1 && capped) *capped = 1;
         }
-    } else if (!SYNC) {
+    } else if (!SYNC && need_drain) {
         const int lane = tid & 31, wq0 = (tid >> 5) * (2 * 32 * VPT);
         for (;;) {
             int worked = 0;
@@ -876,10 +1009,11 @@ template <bool SYNC, int TT>
 static __global__ void __launch_bounds__(TT / VPT, (1536 / (TT / VPT)) > 0 ? 1536 / (TT / VPT) : 1)
 k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, DevCounters* __restrict__ dc, int pass,
             int first, uint8_t* __restrict__ dirty_cur, uint8_t* __restrict__ dirty_next, int full, int theta,
-            int run, int kcap) {
+            int run, int kcap, uint8_t* __restrict__ lvl) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];             // raise flags, byte k = vertex 4t+k
-    __shared__ unsigned short s_queue[2 * TT];                         // per-warp item queues
+    __shared__ unsigned short s_queue[2 * TT + 2 * 260];               // per-warp item queues / level order
+    __shared__ uint8_t s_lv[TT];
     __shared__ int s_dirty;
     TileSmem<TT> S;
     S.s_in = (int*)smem_raw;
@@ -889,6 +1023,7 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
     S.s_fin = s_fin;
     S.s_fout = s_fout;
     S.s_queue = s_queue;
+    S.s_lv = s_lv;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + TT - 1) / TT;
     const int tid = threadIdx.x;
@@ -912,7 +1047,7 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
             if (!s_dirty) continue;
         }
         int capped = 0;
-        ch_any |= tile_visit<SYNC, TT>(g, cin, cout, dc, tile, full, theta, MarkNext{dirty_next}, S, kcap, &capped);
+        ch_any |= tile_visit<SYNC, TT>(g, cin, cout, dc, tile, full, theta, MarkNext{dirty_next}, S, kcap, &capped, lvl);
         if (capped && dirty_next && tid == 0) dirty_next[tile] = 1;   // not converged: come back
         __syncthreads();                                     // shared memory is reused by the next tile
     }

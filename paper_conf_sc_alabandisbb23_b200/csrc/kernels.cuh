@@ -942,34 +942,13 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
                             const int w = __ldg(sadj + e) - base;
                             if ((unsigned)w < (unsigned)cnt) val = max(val, ((volatile int*)sig)[w]);
                         }
-                    if (val > old && atomicMax(sig + v, val) < val) {
+                    if (val > old) {
+                        ((volatile int*)sig)[v] = val;
                         __threadfence_block();
                         // dependents: out-neighbours re-pull v_in, in-neighbours re-pull v_out
                         if (dir_out) notify(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
                         else notify(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
                         any = 1;
-                        // chase: re-pull a dependent inside this warp's region right away
-                        // (its flag stays set, so a later drain re-checks it)
-                        int cur = v;
-                        for (int hop = 0; hop < 8; hop++) {
-                            const unsigned long long dep = dir_out ? s_nin[cur] : s_nout[cur];
-                            int w = -1;
-#pragma unroll
-                            for (int q = 0; q < SLOTS; q++) {
-                                const unsigned x = (unsigned)(dep >> (16 * q)) & 0xFFFFu;
-                                if (x == NOSLOT) break;
-                                const int xx = (int)(x & 0x7FFFu);
-                                if (w < 0 && (xx >> 7) == (tid >> 5)) w = xx;
-                            }
-                            if (w < 0) break;
-                            const int ow = ((volatile int*)sig)[w];
-                            const int vw = pull_slots(sig, dir_out ? s_nout[w] : s_nin[w], sptr, sadj, base, cnt, w, ow);
-                            if (!(vw > ow && atomicMax(sig + w, vw) < vw)) break;
-                            __threadfence_block();
-                            if (dir_out) notify(s_nin[w], g.iptr, g.iadj, base, cnt, w, (uint8_t*)s_fout);
-                            else notify(s_nout[w], g.optr, g.oadj, base, cnt, w, (uint8_t*)s_fin);
-                            cur = w;
-                        }
                     }
                 }
                 __syncwarp();

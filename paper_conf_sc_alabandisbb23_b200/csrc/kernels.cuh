@@ -1044,7 +1044,9 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
                 dirty_cur[tile] = 0;
             }
             __syncthreads();
-            if (!s_dirty) continue;
+            const int d = s_dirty;
+            __syncthreads();             // everyone has read s_dirty before thread 0 rewrites it
+            if (!d) continue;
         }
         int capped = 0;
         ch_any |= tile_visit<SYNC, TT>(g, cin, cout, dc, tile, full, theta, MarkNext{dirty_next}, S, kcap, &capped, lvl);

@@ -225,3 +225,17 @@ def test_c5_batched_meshes():
     torch.cuda.synchronize()
     for g, lab in zip(graphs, labs):
         np.testing.assert_array_equal(lab.cpu().numpy(), oracle.tarjan_labels(g.row_ptr, g.col_idx))
+
+
+def test_repeated_runs_with_plan_reuse_are_stable():
+    """Races show up under repetition: the same plan, several graphs and orders, many runs."""
+    graphs = [gen.mesh(60, gen.ordinate(d), seed=4 + d, order=o, **gen.C4_MESH)
+              for d, o in ((0, "lex"), (9, "blocked8"), (40, "lex"))]
+    plan = E.Plan(max(g.n for g in graphs), max(g.nnz for g in graphs))
+    for g in graphs:
+        truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+        rp, ci = dev(g)
+        for _ in range(4):
+            lab = E.ecl_scc(rp, ci, plan=plan)
+            torch.cuda.synchronize()
+            np.testing.assert_array_equal(lab.cpu().numpy(), truth)

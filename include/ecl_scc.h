@@ -73,6 +73,9 @@ typedef enum {
 #define ECL_SCC_SWEEP 0x100u      /* Phase 2 as dependency-ordered forward/backward tile
                                      sweeps instead of passes (experimental; pays off only
                                      when the tile graph is close to a DAG in ID order) */
+#define ECL_SCC_NO_REORDER 0x200u /* keep the caller's vertex numbering as the storage order
+                                     (by default graphs without rows longer than 64 edges and
+                                     n >= 16384 are renumbered into BFS-Voronoi cells) */
 #define ECL_SCC_STAGED 0x80u      /* Phase 2 in threshold stages: the top-K priorities
                                      propagate first (ECL_SCC_STAGES env, default off) */
 

@@ -22,6 +22,7 @@
 #include "common.cuh"
 #include "kernels.cuh"
 #include "scan.cuh"
+#include "reorder.cuh"
 #include "driver.h"
 
 namespace eclscc {
@@ -92,6 +93,15 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     e = e ? e : A((void**)&p->hcnt, n1 * sizeof(int2));
     e = e ? e : A((void**)&p->dirty, 2 * (size_t)p->dirty_cap);
     e = e ? e : A((void**)&p->lvl, n1);
+    e = e ? e : A((void**)&p->rp2, n1 * 4);
+    e = e ? e : A((void**)&p->ci2, m * 4);
+    e = e ? e : A((void**)&p->orig, n1 * 4);
+    e = e ? e : A((void**)&p->pos, n1 * 4);
+    e = e ? e : A((void**)&p->cellv, n1 * 4);
+    e = e ? e : A((void**)&p->fa, n1 * 4);
+    e = e ? e : A((void**)&p->fb, n1 * 4);
+    e = e ? e : A((void**)&p->cellbuf, 3 * (((size_t)p->n_cap >> reo::CELL_SHIFT) + 2) * 4);
+    e = e ? e : A((void**)&p->rcnt, 16);
     e = e ? e : A((void**)&p->nb_cnt, (size_t)p->dirty_cap * 4);
     e = e ? e : A((void**)&p->nb_list, (size_t)p->dirty_cap * NBCAP * 4);
     e = e ? e : A((void**)&p->done, (size_t)p->dirty_cap * 4);
@@ -119,6 +129,8 @@ void plan_free(Plan* p) {
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
     cudaFree(p->chunk_cnt); cudaFree(p->hcnt);
     cudaFree(p->dirty); cudaFree(p->lvl);
+    cudaFree(p->rp2); cudaFree(p->ci2); cudaFree(p->orig); cudaFree(p->pos); cudaFree(p->cellv);
+    cudaFree(p->fa); cudaFree(p->fb); cudaFree(p->cellbuf); cudaFree(p->rcnt);
     cudaFree(p->nb_cnt); cudaFree(p->nb_list); cudaFree(p->done); cudaFree(p->mark); cudaFree(p->sweep_ctr);
     cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
     if (p->hc) cudaFreeHost(p->hc);
@@ -144,11 +156,13 @@ __global__ void k_iota(int32_t n, int32_t* __restrict__ out) {
 }
 // debug snapshot: signatures of the active vertices over the labels of the others
 __global__ void k_scatter_sigs(int32_t na, const int32_t* __restrict__ act, const int32_t* __restrict__ cin,
-                               const int32_t* __restrict__ cout, int32_t* __restrict__ din, int32_t* __restrict__ dout) {
+                               const int32_t* __restrict__ cout, int32_t* __restrict__ din, int32_t* __restrict__ dout,
+                               const int32_t* __restrict__ orig) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= na) return;
-    din[act[i]] = cin[i];
-    dout[act[i]] = cout[i];
+    const int v = orig ? orig[act[i]] : act[i];
+    din[v] = cin[i];
+    dout[v] = cout[i];
 }
 
 // --------------------------------------------------------------------------- steps
@@ -186,6 +200,44 @@ static int build_csc(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const i
     return ECL_SCC_OK;
 }
 
+// Storage reordering (reorder.cuh): BFS-Voronoi cells become runs of consecutive storage
+// IDs; fills p->rp2 / p->ci2 (permuted CSR) and p->orig (storage -> caller ID).  Needs the
+// CSC of the input (buffer 0).
+static int reorder_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t* ci, cudaStream_t s) {
+    const unsigned gs = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
+    CK(cudaMemsetAsync(p->rcnt, 0, 16, s));
+    p->launches++; reo::k_seed2<<<gs, TPB, 0, s>>>(n, p->cellv, p->fa, p->rcnt);
+    int h[3] = {0, 0, 0};
+    for (int r = 0;; ) {
+        for (int k = 0; k < 16; k++, r++) {
+            p->launches++;
+            reo::k_bfs_level<<<148 * 8, TPB, 0, s>>>(p->fa, p->fb, p->rcnt, r, rp, ci, p->iptr[0], p->iadj[0], p->cellv);
+        }
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(h, p->rcnt, 12, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (h[r % 3] == 0) break;                      // the frontier of level r is empty
+        if (r > n + 32) return fail(ECL_SCC_ECUDA, "internal: reorder BFS did not finish");
+    }
+    const int64_t nkeys = ((int64_t)n >> reo::CELL_SHIFT) + 1;
+    int32_t* hist = p->cellbuf;
+    int32_t* start = p->cellbuf + (nkeys + 1);
+    int32_t* cursor = p->kout;                         // free until the first compaction
+    CK(cudaMemsetAsync(hist, 0, sizeof(int32_t) * (size_t)(nkeys + 1), s));
+    p->launches++; reo::k_cell_hist<<<gs, TPB, 0, s>>>(n, p->cellv, hist);
+    int r = scan_excl<I1>(p, (const I1*)hist, nkeys, (I1*)start, (I1*)&p->dc->grand1, p->bsum, 1, s);
+    if (r) return r;
+    CK(cudaMemsetAsync(cursor, 0, sizeof(int32_t) * (size_t)(nkeys + 1), s));
+    p->launches++; reo::k_cell_place<<<gs, TPB, 0, s>>>(n, p->cellv, start, cursor, p->pos, p->orig);
+    p->launches++; reo::k_perm_deg<<<gs, TPB, 0, s>>>(n, rp, p->pos, p->kin);
+    r = scan_excl<I1>(p, (const I1*)p->kin, n, (I1*)p->rp2, (I1*)&p->dc->grand1, p->bsum, 1, s);
+    if (r) return r;
+    p->launches++; reo::k_perm_fill<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, ci, p->pos, p->rp2, p->ci2);
+    CK(cudaGetLastError());
+    (void)nnz;
+    return ECL_SCC_OK;
+}
+
 // a7 + a2 + a3 + a8: Phase 3 edge removal, Trim-1, compaction into buffer `ob` with the
 // Phase-1 reset of the survivors and the final labels of the vertices that leave
 template <bool FIRST, bool TRIM>
@@ -208,7 +260,7 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     if (r) return r;
     p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
-                                              chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P);
+                                              chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur);
     p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked);
     if (chunked) {
@@ -449,6 +501,15 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         if (stop_iter > 0) CK(cudaMemsetAsync(labels, 0, sizeof(int32_t) * (size_t)n, s));
         int r = build_csc(p, n, nnz, rp, ci, s);
         if (r) return r;
+        p->orig_cur = nullptr;
+        // storage reordering for graphs without long rows (meshes); results do not depend on it
+        if (!(p->flags & ECL_SCC_NO_REORDER) && p->nchunks_cur == 0 && n >= 8 * TILE) {
+            if ((r = reorder_graph(p, n, nnz, rp, ci, s))) return r;
+            rp = p->rp2;
+            ci = p->ci2;
+            if ((r = build_csc(p, n, nnz, rp, ci, s))) return r;
+            p->orig_cur = p->orig;
+        }
         stage_mark(p, 1, s);
         WGraph g{nullptr, rp, ci, p->iptr[0], p->iadj[0], n};
         const int32_t *cin = nullptr, *cout = nullptr;          // identity (l.3-6) in the input
@@ -498,7 +559,7 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             }
             if (stop_iter == iter) {
                 p->launches++; k_snapshot_left<<<grid_for(n, TPB), TPB, 0, s>>>(n, labels, dbg_in, dbg_out, P);
-                p->launches++; k_scatter_sigs<<<grid_for(t.x, TPB), TPB, 0, s>>>(t.x, g.act, cin, cout, dbg_in, dbg_out);
+                p->launches++; k_scatter_sigs<<<grid_for(t.x, TPB), TPB, 0, s>>>(t.x, g.act, cin, cout, dbg_in, dbg_out, p->orig_cur);
                 CK(cudaGetLastError());
                 stopped = true;
                 break;

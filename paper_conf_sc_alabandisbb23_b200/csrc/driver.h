@@ -39,6 +39,9 @@ struct Plan {
     int64_t dirty_cap;
     int tile;                            // Phase-2 tile size (vertices per CTA)
     uint8_t* lvl;                        // level-sweep mode: intra-tile level per vertex
+    // storage reordering (reorder.cuh): permuted input CSR and the storage -> caller ID map
+    int32_t *rp2, *ci2, *orig, *pos, *cellv, *fa, *fb, *cellbuf, *rcnt;
+    const int32_t* orig_cur;             // orig when the current run is reordered, else null
     int *nb_cnt, *nb_list;               // sweep mode: neighbour tiles of each tile
     int *done, *mark;                    // sweep mode: per-tile done / dirty epochs
     int* sweep_ctr;                      // [0] tile counter, [1] changed, [2] overflow

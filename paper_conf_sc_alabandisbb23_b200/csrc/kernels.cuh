@@ -228,7 +228,8 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
                               const int4* __restrict__ totals, int32_t* __restrict__ newidx,
                               int32_t* __restrict__ act2, int32_t* __restrict__ cin2, int32_t* __restrict__ cout2,
                               int32_t* __restrict__ optr2, int32_t* __restrict__ iptr2, int32_t* __restrict__ labels,
-                              Chunk* __restrict__ chunks, int* __restrict__ nchunks, int chunk_cap, Prio P) {
+                              Chunk* __restrict__ chunks, int* __restrict__ nchunks, int chunk_cap, Prio P,
+                              const int32_t* __restrict__ orig) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i == 0) {
@@ -244,11 +245,12 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
     const int po = warp_incl_scan(c.x, lane) - c.x + base.y;
     const int pi = warp_incl_scan(c.y, lane) - c.y + base.z;
     if (!valid) return;
-    const int v = g.act ? g.act[i] : (int)i;
+    const int v = g.act ? g.act[i] : (int)i;          // storage ID
+    const int ov = orig ? orig[v] : v;                 // caller's ID (reorder.cuh)
     if (alive) {
         newidx[i] = j;
         act2[j] = v;
-        const int pv = (int)prio_of(P, (uint32_t)v);
+        const int pv = (int)prio_of(P, (uint32_t)ov);
         cin2[j] = pv;       // Phase 1: v_in <- v_id, v_out <- v_id for the unfinished
         cout2[j] = pv;
         optr2[j] = po;
@@ -264,12 +266,12 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
         }
     } else {
         newidx[i] = -1;
-        int lab = v;    // unfinished (or trimmed) and edgeless: a singleton SCC
+        int lab = ov;   // unfinished (or trimmed) and edgeless: a singleton SCC
         if (!FIRST) {
             const int a = cin[i], b = cout[i];
             if (a == b) lab = P.ids ? a : -(a + 1);
         }
-        labels[v] = lab;
+        labels[ov] = lab;
     }
 }
 

@@ -239,3 +239,18 @@ def test_repeated_runs_with_plan_reuse_are_stable():
             lab = E.ecl_scc(rp, ci, plan=plan)
             torch.cuda.synchronize()
             np.testing.assert_array_equal(lab.cpu().numpy(), truth)
+
+
+def test_storage_reordering_keeps_labels_and_traces():
+    """Graphs without long rows and n >= 16384 are renumbered into BFS-Voronoi cells
+    internally (reorder.cuh); labels, per-iteration edge counts and signatures must be
+    those of the caller's numbering."""
+    g = gen.mesh(16, gen.ordinate(5), seed=7, order="lex", **gen.C4_MESH)    # n = 24576
+    truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+    la, sa = gpu_labels(g)
+    lb, sb = gpu_labels(g, E.NO_REORDER)
+    np.testing.assert_array_equal(la, truth)
+    np.testing.assert_array_equal(lb, truth)
+    assert sa["edges_in"] == sb["edges_in"] and sa["iterations"] == sb["iterations"]
+    check_trace(g, trim=True, max_iters=3)
+    check_trace(g, trim=True, flags=E.IDENTITY_IDS, max_iters=3)

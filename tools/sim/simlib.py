@@ -12,7 +12,8 @@ def run(g, tile_of, pr, heap=0, gs=0, order=None, window=1):
     out = np.zeros(4, dtype=np.int64)
     nt = int(tile_of.max()) + 1
     L.tilesim(ctypes.c_int32(g.n), P(g.row_ptr), P(g.col_idx), P(tile_of), ctypes.c_int32(nt), P(pr), P(out),
-              ctypes.c_int(heap), ctypes.c_int(gs), P(order) if order is not None else None, ctypes.c_int32(window))
+              ctypes.c_int(heap), ctypes.c_int(gs), P(order) if order is not None else None, ctypes.c_int32(window),
+              ctypes.c_int32(0))
     return out
 
 def mesh_coords(N, n):

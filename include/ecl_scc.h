@@ -74,8 +74,11 @@ typedef enum {
                                      sweeps instead of passes (experimental; pays off only
                                      when the tile graph is close to a DAG in ID order) */
 #define ECL_SCC_NO_REORDER 0x200u /* keep the caller's vertex numbering as the storage order
-                                     (by default graphs without rows longer than 64 edges and
-                                     n >= 16384 are renumbered into BFS-Voronoi cells) */
+                                     (by default graphs without rows longer than 64 edges,
+                                     n >= 16384 and fewer than 85% of the edges inside
+                                     2048-ID ranges are renumbered into BFS-Voronoi cells) */
+#define ECL_SCC_FORCE_REORDER 0x400u /* renumber into BFS-Voronoi cells whenever the graph has
+                                        no row longer than 64 edges (tests, ablation) */
 #define ECL_SCC_STAGED 0x80u      /* Phase 2 in threshold stages: the top-K priorities
                                      propagate first (ECL_SCC_STAGES env, default off) */
 

@@ -62,18 +62,22 @@ static __global__ void k_indeg(int64_t nnz, const int32_t* __restrict__ ci, int3
 // one thread per source row; rows longer than HEAVY are spread over the warp
 static __global__ void k_csc_scatter(int32_t n, const int32_t* __restrict__ rp, const int32_t* __restrict__ ci,
                               const int32_t* __restrict__ iptr, int32_t* __restrict__ cursor,
-                              int32_t* __restrict__ iadj) {
+                              int32_t* __restrict__ iadj, unsigned long long* __restrict__ local_e) {
     const int lane = threadIdx.x & 31;
     const int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const bool valid = u < n;
     int b = 0, e = 0;
     if (valid) { b = rp[u]; e = rp[u + 1]; }
     if (e - b > HEAVY_T) e = b;                          // long row: k_csc_scatter_chunks
+    unsigned nloc = 0;                                   // storage locality of the numbering
     if (valid && e - b <= HEAVY)
         for (int k = b; k < e; k++) {
             const int w = ci[k];
+            nloc += ((w ^ (int)u) >> 11) == 0;
             iadj[iptr[w] + atomicAdd(&cursor[w], 1)] = (int32_t)u;
         }
+    nloc = __reduce_add_sync(FULL, nloc);
+    if (lane == 0 && nloc) atomicAdd(local_e, (unsigned long long)nloc);
     unsigned hm = __ballot_sync(FULL, valid && e - b > HEAVY);
     while (hm) {
         const int src = __ffs(hm) - 1;

@@ -72,6 +72,41 @@ static __global__ void k_cell_place(int32_t n, const int32_t* __restrict__ key, 
         orig[j] = (int)v;
     }
 }
+// one CTA per cell: sort the cell's storage slots by caller ID (bitonic sort in shared
+// memory), so that a tile holding part of a cell holds a compact piece of it (the
+// atomic placement above leaves the members in arbitrary order).  Cells larger than
+// SORT_MAX keep the arbitrary order (only the pass count depends on it).
+constexpr int SORT_MAX = 8192;
+constexpr int SORT_THREADS = 1024;
+static __global__ void __launch_bounds__(SORT_THREADS) k_cell_sort(int64_t nkeys, const int32_t* __restrict__ start,
+                                                                  int32_t* __restrict__ orig, int32_t* __restrict__ pos) {
+    __shared__ int32_t sk[SORT_MAX];
+    for (int64_t c = blockIdx.x; c < nkeys; c += gridDim.x) {
+        const int b = start[c], sz = start[c + 1] - b;
+        if (sz <= 1 || sz > SORT_MAX) continue;
+        int m = 1;
+        while (m < sz) m <<= 1;
+        for (int k = threadIdx.x; k < m; k += SORT_THREADS) sk[k] = k < sz ? orig[b + k] : 0x7FFFFFFF;
+        __syncthreads();
+        for (int k = 2; k <= m; k <<= 1)
+            for (int j = k >> 1; j > 0; j >>= 1) {
+                for (int t = threadIdx.x; t < m; t += SORT_THREADS) {
+                    const int o = t ^ j;
+                    if (o > t) {
+                        const int x = sk[t], y = sk[o];
+                        if (((t & k) == 0) == (x > y)) { sk[t] = y; sk[o] = x; }
+                    }
+                }
+                __syncthreads();
+            }
+        for (int k = threadIdx.x; k < sz; k += SORT_THREADS) {
+            const int v = sk[k];
+            orig[b + k] = v;
+            pos[v] = b + k;
+        }
+        __syncthreads();
+    }
+}
 static __global__ void k_perm_deg(int32_t n, const int32_t* __restrict__ rp, const int32_t* __restrict__ pos,
                                   int32_t* __restrict__ deg) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)

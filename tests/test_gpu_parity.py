@@ -94,19 +94,20 @@ def test_random_small_graphs_labels_and_traces():
         edges = [(rng.randrange(n), rng.randrange(n)) for _ in range(m)]
         g = gen.from_edges(n, edges)
         truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-        for flags in (0, E.NO_TRIM, E.IDENTITY_IDS, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP):
+        for flags in (0, E.NO_TRIM, E.IDENTITY_IDS, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER):
             lab, _ = gpu_labels(g, flags)
             np.testing.assert_array_equal(lab, truth, err_msg=f"trial {trial} flags {flags}")
         if trial % 10 == 0:
             check_trace(g, trim=True)
             check_trace(g, trim=False)
             check_trace(g, trim=True, flags=E.IDENTITY_IDS)
+            check_trace(g, trim=True, flags=E.FORCE_REORDER)
 
 
 def test_c1_gnm_2000_8000():
     g = gen.config("c1")
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-    for flags in (0, E.IDENTITY_IDS, E.NO_TRIM, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP):
+    for flags in (0, E.IDENTITY_IDS, E.NO_TRIM, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER):
         lab, _ = gpu_labels(g, flags)
         np.testing.assert_array_equal(lab, truth)
     check_trace(g, trim=True)
@@ -247,10 +248,10 @@ def test_storage_reordering_keeps_labels_and_traces():
     those of the caller's numbering."""
     g = gen.mesh(16, gen.ordinate(5), seed=7, order="lex", **gen.C4_MESH)    # n = 24576
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-    la, sa = gpu_labels(g)
+    la, sa = gpu_labels(g, E.FORCE_REORDER)
     lb, sb = gpu_labels(g, E.NO_REORDER)
     np.testing.assert_array_equal(la, truth)
     np.testing.assert_array_equal(lb, truth)
     assert sa["edges_in"] == sb["edges_in"] and sa["iterations"] == sb["iterations"]
-    check_trace(g, trim=True, max_iters=3)
-    check_trace(g, trim=True, flags=E.IDENTITY_IDS, max_iters=3)
+    check_trace(g, trim=True, flags=E.FORCE_REORDER, max_iters=3)
+    check_trace(g, trim=True, flags=E.IDENTITY_IDS | E.FORCE_REORDER, max_iters=3)

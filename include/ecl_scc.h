@@ -79,6 +79,8 @@ typedef enum {
                                      2048-ID ranges are renumbered into BFS-Voronoi cells) */
 #define ECL_SCC_FORCE_REORDER 0x400u /* renumber into BFS-Voronoi cells whenever the graph has
                                         no row longer than 64 edges (tests, ablation) */
+#define ECL_SCC_NO_PACK 0x800u    /* ablation: Phase 2 re-walks the CSR/CSC rows on every tile
+                                     visit instead of reading per-iteration tile packs */
 #define ECL_SCC_STAGED 0x80u      /* Phase 2 in threshold stages: the top-K priorities
                                      propagate first (ECL_SCC_STAGES env, default off) */
 

@@ -23,6 +23,7 @@
 #include "kernels.cuh"
 #include "scan.cuh"
 #include "reorder.cuh"
+#include "pack.cuh"
 #include "driver.h"
 
 namespace eclscc {
@@ -134,6 +135,7 @@ void plan_free(Plan* p) {
     cudaFree(p->fa); cudaFree(p->fb); cudaFree(p->cellbuf); cudaFree(p->rcnt);
     cudaFree(p->nb_cnt); cudaFree(p->nb_list); cudaFree(p->done); cudaFree(p->mark); cudaFree(p->sweep_ctr);
     cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
+    cudaFree(p->pnin); cudaFree(p->pnout); cudaFree(p->ext); cudaFree(p->ext_cnt);
     if (p->hc) cudaFreeHost(p->hc);
     if (p->ev_ok)
         for (int k = 0; k < 6; k++) cudaEventDestroy(p->ev[k]);
@@ -404,6 +406,28 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     const std::vector<int> thetas = (p->flags & ECL_SCC_STAGED) ? stage_thresholds(n, g.na, false)
                                                                    : std::vector<int>{0};
     int64_t total = 0;
+    // tile packs (pack.cuh): the default for graphs without long rows
+    static int env_variant = -1;   // the KCAP / LEVELS experiments run on the tile kernel
+    if (env_variant < 0) env_variant = (getenv("ECL_SCC_KCAP") || getenv("ECL_SCC_LEVELS")) ? 1 : 0;
+    const bool use_pack = use_dirty && p->tile == PACK_TT && thetas.size() == 1 && !env_variant &&
+                          !(p->flags & (ECL_SCC_NO_PACK | ECL_SCC_SWEEP)) && g.na > 0;
+    if (use_pack) {
+        if (!p->pnin) {                                  // first use: sized for the plan
+            const size_t np = (size_t)cdiv((int64_t)p->n_cap + 1, PACK_TT) * PACK_TT + PACK_TT;
+            cudaError_t e = cudaMalloc((void**)&p->pnin, np * 8);
+            if (e == cudaSuccess) e = cudaMalloc((void**)&p->pnout, np * 8);
+            if (e == cudaSuccess) e = cudaMalloc((void**)&p->ext, 2 * (size_t)p->m_cap * sizeof(int2) + 16);
+            if (e == cudaSuccess) e = cudaMalloc((void**)&p->ext_cnt, (size_t)p->dirty_cap * 4);
+            if (e != cudaSuccess) {
+                cudaGetLastError();
+                return fail(ECL_SCC_ENOMEM, "tile pack allocation: %s", cudaGetErrorString(e));
+            }
+            CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tile_dyn_smem<PACK_TT>()));
+        }
+        p->launches++;
+        k_tile_pack<<<ntiles, PACK_TH, 0, s>>>(g, p->pnin, p->pnout, p->ext, p->ext_cnt);
+        CK(cudaGetLastError());
+    }
     if (!sync && nchunks == 0 && (p->flags & ECL_SCC_SWEEP) && !(p->flags & ECL_SCC_STAGED)) {
         int used = 0, r = ECL_SCC_OK;
         switch (p->tile) {
@@ -436,6 +460,15 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                 if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>(chunk_buf(p, p->cb), nchunks, g, cin, cout, p->dc, pass, theta); }
                 const int full = (pass == 0 || nchunks > 0);
                 int r = ECL_SCC_OK;
+                if (use_pack) {
+                    static int run_env = -1;
+                    if (run_env < 0) run_env = getenv("ECL_SCC_RUN") ? std::max(1, atoi(getenv("ECL_SCC_RUN"))) : 4;
+                    const int run = (int)std::min<int64_t>(run_env, std::max<int64_t>(1, ntiles / (2 * 148)));
+                    p->launches++;
+                    k_prop_pack<<<(unsigned)cdiv(ntiles, run), PACK_TH, tile_dyn_smem<PACK_TT>(), s>>>(
+                        g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, pass, nchunks == 0, dc_, dn_, full, run);
+                    continue;
+                }
                 switch (p->tile) {
                     case 512: r = launch_tile<512>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, theta, s); break;
                     case 1024: r = launch_tile<1024>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, theta, s); break;

@@ -46,6 +46,9 @@ struct Plan {
     int *done, *mark;                    // sweep mode: per-tile done / dirty epochs
     int* sweep_ctr;                      // [0] tile counter, [1] changed, [2] overflow
     int epoch;                           // sweep epoch (monotone over the plan's life)
+    unsigned long long *pnin, *pnout;    // tile packs (pack.cuh): slot words per local vertex
+    int2* ext;                           // tile packs: cut edges per tile
+    int* ext_cnt;                        // tile packs: cut edges of each tile
     int64_t launches;                    // kernels launched by the current call
     cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
     bool ev_ok;

@@ -639,6 +639,88 @@ __device__ __forceinline__ void notify(unsigned long long nb, const int32_t* __r
         }
 }
 
+// Step 2 drain loop (see tile_visit): owner-computes pulls over the intra-tile slots until
+// no flag is left.  Shared by the tile and the tile-pack kernels.
+__device__ __forceinline__ void drain_local(const WGraph& g, int* __restrict__ s_in, int* __restrict__ s_out,
+                                            const unsigned long long* __restrict__ s_nin,
+                                            const unsigned long long* __restrict__ s_nout,
+                                            unsigned* __restrict__ s_fin, unsigned* __restrict__ s_fout,
+                                            unsigned short* __restrict__ s_queue, int base, int cnt,
+                                            unsigned& prof_rounds, unsigned& prof_drains, unsigned& prof_pushes) {
+    const int tid = threadIdx.x;
+    const int lane = tid & 31, wq0 = (tid >> 5) * (2 * 32 * VPT);
+    for (;;) {
+        int worked = 0;
+#ifdef ECL_PROF
+        if (tid == 0) prof_rounds++;
+#endif
+        for (;;) {                                       // drain this warp's flags
+#ifdef ECL_PROF
+            if (lane == 0) prof_drains++;
+#endif
+            unsigned wi = ((volatile unsigned*)s_fin)[tid], wo = ((volatile unsigned*)s_fout)[tid];
+            if (wi) wi = atomicExch(s_fin + tid, 0u);
+            if (wo) wo = atomicExch(s_fout + tid, 0u);
+            const unsigned items = ((wi & 0x01u) | ((wi >> 7) & 0x02u) | ((wi >> 14) & 0x04u) | ((wi >> 21) & 0x08u)) |
+                                   (((wo & 0x01u) | ((wo >> 7) & 0x02u) | ((wo >> 14) & 0x04u) | ((wo >> 21) & 0x08u)) << 4);
+            const int c = __popc(items);
+            const int incl = warp_incl_scan(c, lane);
+            const int total = __shfl_sync(FULL, incl, 31);
+            if (total == 0) break;                       // region drained
+            worked = 1;
+#ifdef ECL_PROF
+            prof_pushes += c;
+#endif
+            {
+                int pos = wq0 + incl - c;
+                unsigned it = items;
+                while (it) {
+                    const int bit = __ffs(it) - 1;
+                    it &= it - 1;
+                    s_queue[pos++] = (unsigned short)(((tid * VPT + (bit & 3)) << 1) | (bit >> 2));
+                }
+            }
+            __syncwarp();
+            __threadfence_block();
+            int any = 0;
+            for (int q = lane; q < total; q += 32) {
+                const unsigned item = s_queue[wq0 + q];
+                const int v = (int)(item >> 1);
+                const bool dir_out = item & 1u;
+                int* sig = dir_out ? s_out : s_in;
+                // pull: v_in from in-neighbours, v_out from out-neighbours
+                const unsigned long long src = dir_out ? s_nout[v] : s_nin[v];
+                const int32_t* sptr = dir_out ? g.optr : g.iptr;
+                const int32_t* sadj = dir_out ? g.oadj : g.iadj;
+                const int old = ((volatile int*)sig)[v];
+                int val = old;
+#pragma unroll
+                for (int k = 0; k < SLOTS; k++) {
+                    unsigned w = (unsigned)(src >> (16 * k)) & 0xFFFFu;
+                    if (w == NOSLOT) break;
+                    val = max(val, ((volatile int*)sig)[w & 0x7FFFu]);
+                }
+                if ((src & SLOW_MARK) && (src >> 48) != 0xFFFFull)
+                    for (int e = __ldg(sptr + base + v), ee = __ldg(sptr + base + v + 1); e < ee; e++) {
+                        const int w = __ldg(sadj + e) - base;
+                        if ((unsigned)w < (unsigned)cnt) val = max(val, ((volatile int*)sig)[w]);
+                    }
+                if (val > old) {
+                    ((volatile int*)sig)[v] = val;
+                    __threadfence_block();
+                    // dependents: out-neighbours re-pull v_in, in-neighbours re-pull v_out
+                    if (dir_out) notify(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
+                    else notify(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
+                    any = 1;
+                }
+            }
+            __syncwarp();
+            if (!__any_sync(FULL, any)) break;           // raised nothing: region drained
+        }
+        if (!__syncthreads_or(worked)) break;            // a round with no work: done
+    }
+}
+
 // One block-local fixed point of tile `tile` (steps 1-3 above).  Returns non-zero in
 // every thread if a signature was raised.
 template <bool SYNC, int TT, typename Mark>
@@ -891,77 +973,11 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
             if (r == kcap - 1 && capped) *capped = 1;
         }
     } else if (!SYNC && need_drain) {
-        const int lane = tid & 31, wq0 = (tid >> 5) * (2 * 32 * VPT);
-        for (;;) {
-            int worked = 0;
-#ifdef ECL_PROF
-            if (tid == 0) prof_rounds++;
+#ifndef ECL_PROF
+        unsigned prof_rounds = 0, prof_drains = 0, prof_pushes = 0;
 #endif
-            for (;;) {                                       // drain this warp's flags
-#ifdef ECL_PROF
-                if (lane == 0) prof_drains++;
-#endif
-                unsigned wi = ((volatile unsigned*)s_fin)[tid], wo = ((volatile unsigned*)s_fout)[tid];
-                if (wi) wi = atomicExch(s_fin + tid, 0u);
-                if (wo) wo = atomicExch(s_fout + tid, 0u);
-                const unsigned items = ((wi & 0x01u) | ((wi >> 7) & 0x02u) | ((wi >> 14) & 0x04u) | ((wi >> 21) & 0x08u)) |
-                                       (((wo & 0x01u) | ((wo >> 7) & 0x02u) | ((wo >> 14) & 0x04u) | ((wo >> 21) & 0x08u)) << 4);
-                const int c = __popc(items);
-                const int incl = warp_incl_scan(c, lane);
-                const int total = __shfl_sync(FULL, incl, 31);
-                if (total == 0) break;                       // region drained
-                worked = 1;
-#ifdef ECL_PROF
-                prof_pushes += c;
-#endif
-                {
-                    int pos = wq0 + incl - c;
-                    unsigned it = items;
-                    while (it) {
-                        const int bit = __ffs(it) - 1;
-                        it &= it - 1;
-                        s_queue[pos++] = (unsigned short)(((tid * VPT + (bit & 3)) << 1) | (bit >> 2));
-                    }
-                }
-                __syncwarp();
-                __threadfence_block();
-                int any = 0;
-                for (int q = lane; q < total; q += 32) {
-                    const unsigned item = s_queue[wq0 + q];
-                    const int v = (int)(item >> 1);
-                    const bool dir_out = item & 1u;
-                    int* sig = dir_out ? s_out : s_in;
-                    // pull: v_in from in-neighbours, v_out from out-neighbours
-                    const unsigned long long src = dir_out ? s_nout[v] : s_nin[v];
-                    const int32_t* sptr = dir_out ? g.optr : g.iptr;
-                    const int32_t* sadj = dir_out ? g.oadj : g.iadj;
-                    const int old = ((volatile int*)sig)[v];
-                    int val = old;
-#pragma unroll
-                    for (int k = 0; k < SLOTS; k++) {
-                        unsigned w = (unsigned)(src >> (16 * k)) & 0xFFFFu;
-                        if (w == NOSLOT) break;
-                        val = max(val, ((volatile int*)sig)[w & 0x7FFFu]);
-                    }
-                    if ((src & SLOW_MARK) && (src >> 48) != 0xFFFFull)
-                        for (int e = __ldg(sptr + base + v), ee = __ldg(sptr + base + v + 1); e < ee; e++) {
-                            const int w = __ldg(sadj + e) - base;
-                            if ((unsigned)w < (unsigned)cnt) val = max(val, ((volatile int*)sig)[w]);
-                        }
-                    if (val > old) {
-                        ((volatile int*)sig)[v] = val;
-                        __threadfence_block();
-                        // dependents: out-neighbours re-pull v_in, in-neighbours re-pull v_out
-                        if (dir_out) notify(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
-                        else notify(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
-                        any = 1;
-                    }
-                }
-                __syncwarp();
-                if (!__any_sync(FULL, any)) break;           // raised nothing: region drained
-            }
-            if (!__syncthreads_or(worked)) break;            // a round with no work: done
-        }
+        drain_local(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, s_queue, base, cnt, prof_rounds, prof_drains,
+                    prof_pushes);
     }
 #ifdef ECL_PROF
     __syncthreads();

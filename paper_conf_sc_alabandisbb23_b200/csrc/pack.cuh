@@ -1,0 +1,244 @@
+// pack.cuh -- Phase 2 over per-iteration tile packs (k_prop_pack).
+//
+// The tile kernel (kernels.cuh, k_prop_tile) re-walks the CSR and CSC rows of its 2048
+// vertices on every visit to find the intra-tile neighbours (16-bit slots) and the
+// out-of-tile ones (global pulls); on meshes a tile is visited ~10 times per outer
+// iteration and that walk -- three dependent global loads per row -- was half of the
+// visit.  The working graph does not change during Phase 2, so once per outer iteration
+// k_tile_pack writes each tile's shared-memory image:
+//   pnin[i], pnout[i]  the slot words of local vertex i (the s_nin / s_nout encoding,
+//                      SLOW_MARK for more than SLOTS intra-tile neighbours)
+//   ext[off(t) ..]     the tile's cut edges as {far-end local index, v | dir << 15}:
+//                      dir 0 = in-edge u -> v (v_in pulls in[u]; a raised v_out marks
+//                      tile(u)), dir 1 = out-edge v -> w (v_out pulls out[w]; a raised
+//                      v_in marks tile(w)); off(t) = optr[t*TT] + iptr[t*TT] (a tile
+//                      never has more cut edges than edges), ext_cnt[t] entries.
+// and every visit of k_prop_pack then reads its tile with coalesced vector loads and its
+// cut edges as a flat list (one gather each), runs the same local fixed point
+// (drain_local), and writes back / marks dirty tiles from the same list.  Alg. 1 l.10-11
+// are unchanged: every live edge is either a slot pull or a cut-edge pull.
+#pragma once
+#include "kernels.cuh"
+
+namespace eclscc {
+
+constexpr int PACK_TT = TILE;                 // 2048 vertices per tile
+constexpr int PACK_TH = TILE_THREADS;         // 512 threads, 4 vertices each
+constexpr unsigned EXT_DIR = 0x8000u;
+
+// one CTA per tile: slot words and cut-edge list (graphs without rows longer than HEAVY_T)
+static __global__ void __launch_bounds__(PACK_TH) k_tile_pack(WGraph g, unsigned long long* __restrict__ pnin,
+                                                              unsigned long long* __restrict__ pnout,
+                                                              int2* __restrict__ ext, int* __restrict__ ext_cnt) {
+    __shared__ int s_n;
+    const int tid = threadIdx.x, tile = blockIdx.x;
+    const int base = tile * PACK_TT, cnt = min(PACK_TT, g.na - base);
+    const int64_t off = (int64_t)__ldg(g.optr + base) + __ldg(g.iptr + base);
+    if (tid == 0) s_n = 0;
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        const int v = tid * VPT + k;
+        unsigned long long ni = ~0ull, no = ~0ull;
+        if (v < cnt) {
+            const int gi = base + v;
+            int ns = 0;
+            for (int e = __ldg(g.iptr + gi), ee = __ldg(g.iptr + gi + 1); e < ee; e++) {
+                const int u = __ldg(g.iadj + e);
+                if ((unsigned)(u - base) >= (unsigned)cnt) {
+                    ext[off + atomicAdd(&s_n, 1)] = make_int2(u, v);
+                    continue;
+                }
+                if (ns < SLOTS) add_slot(ni, ns, (unsigned)(u - base));
+                else ni |= SLOW_MARK;
+            }
+            ns = 0;
+            for (int e = __ldg(g.optr + gi), ee = __ldg(g.optr + gi + 1); e < ee; e++) {
+                const int w = __ldg(g.oadj + e);
+                if ((unsigned)(w - base) >= (unsigned)cnt) {
+                    ext[off + atomicAdd(&s_n, 1)] = make_int2(w, v | (int)EXT_DIR);
+                    continue;
+                }
+                if (ns < SLOTS) add_slot(no, ns, (unsigned)(w - base));
+                else no |= SLOW_MARK;
+            }
+        }
+        pnin[(int64_t)base + v] = ni;       // the pack arrays are padded to whole tiles
+        pnout[(int64_t)base + v] = no;
+    }
+    __syncthreads();
+    if (tid == 0) ext_cnt[tile] = s_n;
+}
+
+// One visit of tile `tile` from its pack.  Returns non-zero in every thread if a
+// signature was raised.
+__device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__ cin, int32_t* __restrict__ cout,
+                                          const unsigned long long* __restrict__ pnin,
+                                          const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext,
+                                          const int* __restrict__ ext_cnt, DevCounters* __restrict__ dc, int tile,
+                                          int full, uint8_t* __restrict__ dnext, const TileSmem<PACK_TT>& S) {
+    int* s_in = S.s_in;
+    int* s_out = S.s_out;
+    unsigned long long* s_nin = S.s_nin;
+    unsigned long long* s_nout = S.s_nout;
+    unsigned* s_fin = S.s_fin;
+    unsigned* s_fout = S.s_fout;
+    const int tid = threadIdx.x;
+    const int base = tile * PACK_TT;
+    const int cnt = min(PACK_TT, g.na - base);
+    const int v0 = tid * VPT;
+    const int ne = __ldg(ext_cnt + tile);
+    const int2* E = ext + (int64_t)__ldg(g.optr + base) + __ldg(g.iptr + base);
+
+    // ---- step 1: own values and slot words (coalesced 16-byte loads), then the cut-edge
+    // pulls (Alg. 1 l.10-11 across the tile boundary), folded in with shared atomicMax
+    {
+        const ulonglong2* a = (const ulonglong2*)(pnin + base + v0);
+        const ulonglong2* b = (const ulonglong2*)(pnout + base + v0);
+        ulonglong2* sa = (ulonglong2*)(s_nin + v0);
+        ulonglong2* sb = (ulonglong2*)(s_nout + v0);
+        sa[0] = __ldg(a);
+        sa[1] = __ldg(a + 1);
+        sb[0] = __ldg(b);
+        sb[1] = __ldg(b + 1);
+    }
+    int x0[VPT], y0[VPT];
+    {
+        if (v0 + VPT <= cnt) {
+            const int4 x = __ldcg((const int4*)(cin + base + v0));
+            const int4 y = __ldcg((const int4*)(cout + base + v0));
+            x0[0] = x.x; x0[1] = x.y; x0[2] = x.z; x0[3] = x.w;
+            y0[0] = y.x; y0[1] = y.y; y0[2] = y.z; y0[3] = y.w;
+        } else {
+#pragma unroll
+            for (int k = 0; k < VPT; k++) {
+                x0[k] = v0 + k < cnt ? ld_cg(cin + base + v0 + k) : 0;
+                y0[k] = v0 + k < cnt ? ld_cg(cout + base + v0 + k) : 0;
+            }
+        }
+        *(int4*)(s_in + v0) = make_int4(x0[0], x0[1], x0[2], x0[3]);
+        *(int4*)(s_out + v0) = make_int4(y0[0], y0[1], y0[2], y0[3]);
+    }
+    if (tid == 0) {                                   // roofline accounting (SURVEY 8(d) terms)
+        atomicAdd(&dc->visit_v, (unsigned long long)cnt);
+        atomicAdd(&dc->visit_e, (unsigned long long)(__ldg(g.optr + base + cnt) - __ldg(g.optr + base)));
+    }
+    __syncthreads();
+    for (int i = tid; i < ne; i += PACK_TH) {
+        const int2 e = __ldg(E + i);
+        const int v = e.y & 0x7FFF;
+        int* sig = (e.y & EXT_DIR) ? s_out : s_in;
+        const int val = ld_cg(((e.y & EXT_DIR) ? cout : cin) + e.x);
+        if (val > ((volatile int*)sig)[v]) atomicMax(sig + v, val);
+    }
+    __syncthreads();
+    // ---- step 1b: flags.  First visit of a phase: every vertex; otherwise the intra-tile
+    // dependents of what the cut-edge pulls raised.
+    unsigned fin = 0, fout = 0;
+#pragma unroll
+    for (int k = 0; k < VPT; k++) {
+        if (v0 + k >= cnt) continue;
+        if (full || s_in[v0 + k] > x0[k]) fin |= 1u << (8 * k);
+        if (full || s_out[v0 + k] > y0[k]) fout |= 1u << (8 * k);
+    }
+    s_fin[tid] = full ? fin : 0u;
+    s_fout[tid] = full ? fout : 0u;
+    __syncthreads();
+    if (!full && (fin | fout)) {
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            const int v = v0 + k;
+            if ((fin >> (8 * k)) & 0xFF) notify(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
+            if ((fout >> (8 * k)) & 0xFF) notify(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
+        }
+    }
+    __syncthreads();
+    // ---- step 2: local fixed point in shared memory (same drain loop as k_prop_tile)
+    {
+        unsigned r0 = 0, r1 = 0, r2 = 0;
+        drain_local(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, S.s_queue, base, cnt, r0, r1, r2);
+    }
+    // ---- step 3: write back (whole 16-byte groups; only this CTA writes these vertices
+    // during the pass, so global memory still holds the originals: re-read rather than
+    // kept in registers across step 2) and record which directions rose, for the marks
+    unsigned rin = 0, rout = 0;
+    if (v0 + VPT <= cnt) {
+        const int4 xs = *(const int4*)(s_in + v0);
+        const int4 a = __ldcg((const int4*)(cin + base + v0));
+        rin = (xs.x > a.x ? 1u : 0u) | (xs.y > a.y ? 0x100u : 0u) | (xs.z > a.z ? 0x10000u : 0u) |
+              (xs.w > a.w ? 0x1000000u : 0u);
+        if (rin) __stcg((int4*)(cin + base + v0), xs);
+        const int4 ys = *(const int4*)(s_out + v0);
+        const int4 b = __ldcg((const int4*)(cout + base + v0));
+        rout = (ys.x > b.x ? 1u : 0u) | (ys.y > b.y ? 0x100u : 0u) | (ys.z > b.z ? 0x10000u : 0u) |
+               (ys.w > b.w ? 0x1000000u : 0u);
+        if (rout) __stcg((int4*)(cout + base + v0), ys);
+    } else {
+        for (int k = 0; k < VPT && v0 + k < cnt; k++) {
+            const int gi = base + v0 + k;
+            const int xv = s_in[v0 + k], yv = s_out[v0 + k];
+            if (xv > ld_cg(cin + gi)) { cin[gi] = xv; rin |= 1u << (8 * k); }
+            if (yv > ld_cg(cout + gi)) { cout[gi] = yv; rout |= 1u << (8 * k); }
+        }
+    }
+    const int any = __syncthreads_or((int)(rin | rout));   // also: every drain flag is consumed
+    if (any && dnext) {
+        s_fin[tid] = rin;
+        s_fout[tid] = rout;
+        __syncthreads();
+        const uint8_t* bi = (const uint8_t*)s_fin;
+        const uint8_t* bo = (const uint8_t*)s_fout;
+        for (int i = tid; i < ne; i += PACK_TH) {
+            const int2 e = __ldg(E + i);
+            const int v = e.y & 0x7FFF;
+            // in-edge u -> v: a raised v_out reaches u; out-edge v -> w: a raised v_in reaches w
+            if (((e.y & EXT_DIR) ? bi[v] : bo[v]) != 0) dnext[e.x / PACK_TT] = 1;
+        }
+    }
+    return any;
+}
+
+// Phase-2 pass over the packs (pass protocol, dirty skipping and runs as k_prop_tile)
+static __global__ void __launch_bounds__(PACK_TH, 1536 / PACK_TH)
+k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, const unsigned long long* __restrict__ pnin,
+            const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext, const int* __restrict__ ext_cnt,
+            DevCounters* __restrict__ dc, int pass, int first, uint8_t* __restrict__ dirty_cur,
+            uint8_t* __restrict__ dirty_next, int full, int run) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ unsigned s_fin[PACK_TH], s_fout[PACK_TH];
+    __shared__ unsigned short s_queue[2 * PACK_TT];
+    __shared__ int s_dirty;
+    TileSmem<PACK_TT> S;
+    S.s_in = (int*)smem_raw;
+    S.s_out = S.s_in + PACK_TT;
+    S.s_nin = (unsigned long long*)(S.s_out + PACK_TT);
+    S.s_nout = S.s_nin + PACK_TT;
+    S.s_fin = s_fin;
+    S.s_fout = s_fout;
+    S.s_queue = s_queue;
+    S.s_lv = nullptr;
+    if (!pass_begin(dc, pass, first)) return;
+    const int ntiles = (g.na + PACK_TT - 1) / PACK_TT;
+    const int tid = threadIdx.x;
+    int ch_any = 0;
+    for (int j = 0; j < run; j++) {
+        const int idx = (int)blockIdx.x * run + ((pass & 1) ? run - 1 - j : j);
+        if (idx >= ntiles) continue;
+        const int tile = (pass & 1) ? ntiles - 1 - idx : idx;
+        if (dirty_cur) {
+            if (tid == 0) {
+                s_dirty = dirty_cur[tile];
+                dirty_cur[tile] = 0;
+            }
+            __syncthreads();
+            const int d = s_dirty;
+            __syncthreads();
+            if (!d) continue;
+        }
+        ch_any |= pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, dirty_next, S);
+        __syncthreads();
+    }
+    if (ch_any && tid == 0) dc->changed[pass & (RING - 1)] = 1;
+}
+
+}  // namespace eclscc

@@ -422,7 +422,7 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                 cudaGetLastError();
                 return fail(ECL_SCC_ENOMEM, "tile pack allocation: %s", cudaGetErrorString(e));
             }
-            CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tile_dyn_smem<PACK_TT>()));
+            CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
         }
         p->launches++;
         k_tile_pack<<<ntiles, PACK_TH, 0, s>>>(g, p->pnin, p->pnout, p->ext, p->ext_cnt);
@@ -465,7 +465,7 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                     if (run_env < 0) run_env = getenv("ECL_SCC_RUN") ? std::max(1, atoi(getenv("ECL_SCC_RUN"))) : 4;
                     const int run = (int)std::min<int64_t>(run_env, std::max<int64_t>(1, ntiles / (2 * 148)));
                     p->launches++;
-                    k_prop_pack<<<(unsigned)cdiv(ntiles, run), PACK_TH, tile_dyn_smem<PACK_TT>(), s>>>(
+                    k_prop_pack<<<(unsigned)cdiv(ntiles, run), PACK_TH, pack_dyn_smem(), s>>>(
                         g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, pass, nchunks == 0, dc_, dn_, full, run);
                     continue;
                 }

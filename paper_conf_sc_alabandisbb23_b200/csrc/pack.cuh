@@ -25,6 +25,131 @@ namespace eclscc {
 constexpr int PACK_TT = TILE;                 // 2048 vertices per tile
 constexpr int PACK_TH = TILE_THREADS;         // 512 threads, 4 vertices each
 constexpr unsigned EXT_DIR = 0x8000u;
+// Pack slot encoding: four 16-bit local indices per word; an empty slot holds PACK_TT, the
+// index of a sentinel entry (value 0 <= every priority, scratch flag byte), so pulls and
+// notifications run without branches; bit 63 (slot 3, only set when all four slots are
+// used) marks a row with more than SLOTS intra-tile neighbours (SLOW_MARK).
+constexpr unsigned long long PSLOTS_EMPTY = 0x0800080008000800ull;
+static_assert(PACK_TT == 0x800, "PSLOTS_EMPTY encodes PACK_TT");
+
+__device__ __forceinline__ int ppull(const int* sig, unsigned long long src, int val) {
+    const unsigned lo = (unsigned)src, hi = (unsigned)(src >> 32);
+    const volatile int* s = (const volatile int*)sig;
+    const int a = s[lo & 0xFFFFu], b = s[lo >> 16], c = s[hi & 0xFFFFu], d = s[(hi >> 16) & 0x7FFFu];
+    return max(max(val, a), max(b, max(c, d)));
+}
+__device__ __forceinline__ void pnotify(unsigned long long nb, uint8_t* f) {
+    const unsigned lo = (unsigned)nb, hi = (unsigned)(nb >> 32);
+    volatile uint8_t* x = (volatile uint8_t*)f;
+    x[lo & 0xFFFFu] = 1;
+    x[lo >> 16] = 1;
+    x[hi & 0xFFFFu] = 1;
+    x[(hi >> 16) & 0x7FFFu] = 1;
+}
+// the rest of a slow row (more than SLOTS intra-tile neighbours): walk the global row
+__device__ __noinline__ int pull_slow(const int* sig, const int32_t* __restrict__ ptr, const int32_t* __restrict__ adj,
+                                      int base, int cnt, int v, int val) {
+    for (int e = __ldg(ptr + base + v), ee = __ldg(ptr + base + v + 1); e < ee; e++) {
+        const int w = __ldg(adj + e) - base;
+        if ((unsigned)w < (unsigned)cnt) val = max(val, ((volatile const int*)sig)[w]);
+    }
+    return val;
+}
+__device__ __noinline__ void notify_slow(const int32_t* __restrict__ ptr, const int32_t* __restrict__ adj, int base,
+                                         int cnt, int v, uint8_t* f) {
+    for (int e = __ldg(ptr + base + v), ee = __ldg(ptr + base + v + 1); e < ee; e++) {
+        const int w = __ldg(adj + e) - base;
+        if ((unsigned)w < (unsigned)cnt) ((volatile uint8_t*)f)[w] = 1;
+    }
+}
+__device__ __forceinline__ void pnotify_full(unsigned long long nb, const int32_t* __restrict__ ptr,
+                                             const int32_t* __restrict__ adj, int base, int cnt, int v, uint8_t* f) {
+    pnotify(nb, f);
+    if (nb & SLOW_MARK) notify_slow(ptr, adj, base, cnt, v, f);
+}
+
+// Step 2 for the pack kernel: the drain loop of drain_local (kernels.cuh) with the
+// sentinel slot encoding (branch-free pulls and notifications) and a multiply-based
+// gather of the four flag bytes of a thread.
+__device__ __forceinline__ unsigned gather4(unsigned w) {      // byte k (0/1) -> bit k
+    return (((w & 0x01010101u) * 0x01020408u) >> 24) & 0xFu;
+}
+__device__ __forceinline__ void drain_pack(const WGraph& g, int* __restrict__ s_in, int* __restrict__ s_out,
+                                           const unsigned long long* __restrict__ s_nin,
+                                           const unsigned long long* __restrict__ s_nout,
+                                           unsigned* __restrict__ s_fin, unsigned* __restrict__ s_fout,
+                                           unsigned short* __restrict__ s_queue, int base, int cnt,
+                                           unsigned& prof_rounds, unsigned& prof_drains, unsigned& prof_pushes) {
+    const int tid = threadIdx.x;
+    const int lane = tid & 31, wq0 = (tid >> 5) * (2 * 32 * VPT);
+    for (;;) {
+        int worked = 0;
+#ifdef ECL_PROF
+        if (tid == 0) prof_rounds++;
+#endif
+        for (;;) {
+#ifdef ECL_PROF
+            if (lane == 0) prof_drains++;
+#endif
+            unsigned wi = ((volatile unsigned*)s_fin)[tid], wo = ((volatile unsigned*)s_fout)[tid];
+            if (wi) wi = atomicExch(s_fin + tid, 0u);
+            if (wo) wo = atomicExch(s_fout + tid, 0u);
+            const unsigned items = gather4(wi) | (gather4(wo) << 4);
+            const int c = __popc(items);
+            const int incl = warp_incl_scan(c, lane);
+            const int total = __shfl_sync(FULL, incl, 31);
+            if (total == 0) break;
+            worked = 1;
+#ifdef ECL_PROF
+            prof_pushes += c;
+#endif
+            {
+                int pos = wq0 + incl - c;
+                unsigned it = items;
+                while (it) {
+                    const int bit = __ffs(it) - 1;
+                    it &= it - 1;
+                    s_queue[pos++] = (unsigned short)(((tid * VPT + (bit & 3)) << 1) | (bit >> 2));
+                }
+            }
+            __syncwarp();
+            __threadfence_block();
+            int any = 0;
+            for (int q = lane; q < total; q += 32) {
+                const unsigned item = s_queue[wq0 + q];
+                const int v = (int)(item >> 1);
+                if (item & 1u) {                                 // v_out from the out-neighbours
+                    const unsigned long long src = s_nout[v];
+                    const int old = ((volatile int*)s_out)[v];
+                    int val = ppull(s_out, src, old);
+                    if (src & SLOW_MARK) val = pull_slow(s_out, g.optr, g.oadj, base, cnt, v, val);
+                    if (val > old) {
+                        ((volatile int*)s_out)[v] = val;
+                        __threadfence_block();
+                        pnotify_full(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
+                        any = 1;
+                    }
+                } else {                                         // v_in from the in-neighbours
+                    const unsigned long long src = s_nin[v];
+                    const int old = ((volatile int*)s_in)[v];
+                    int val = ppull(s_in, src, old);
+                    if (src & SLOW_MARK) val = pull_slow(s_in, g.iptr, g.iadj, base, cnt, v, val);
+                    if (val > old) {
+                        ((volatile int*)s_in)[v] = val;
+                        __threadfence_block();
+                        pnotify_full(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
+                        any = 1;
+                    }
+                }
+            }
+            __syncwarp();
+            if (!__any_sync(FULL, any)) break;
+        }
+        if (!__syncthreads_or(worked)) break;
+    }
+}
+
+constexpr size_t pack_dyn_smem() { return (size_t)(PACK_TT + 4) * 4 * 2 + (size_t)PACK_TT * 8 * 2; }
 
 // one CTA per tile: slot words and cut-edge list (graphs without rows longer than HEAVY_T)
 static __global__ void __launch_bounds__(PACK_TH) k_tile_pack(WGraph g, unsigned long long* __restrict__ pnin,
@@ -39,7 +164,7 @@ static __global__ void __launch_bounds__(PACK_TH) k_tile_pack(WGraph g, unsigned
 #pragma unroll
     for (int k = 0; k < VPT; k++) {
         const int v = tid * VPT + k;
-        unsigned long long ni = ~0ull, no = ~0ull;
+        unsigned long long ni = PSLOTS_EMPTY, no = PSLOTS_EMPTY;
         if (v < cnt) {
             const int gi = base + v;
             int ns = 0;
@@ -89,6 +214,10 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
     const int v0 = tid * VPT;
     const int ne = __ldg(ext_cnt + tile);
     const int2* E = ext + (int64_t)__ldg(g.optr + base) + __ldg(g.iptr + base);
+#ifdef ECL_PROF
+    const long long t_start = clock64();
+    if (tid == 0) PROF_ADD(dc, 0, 1);
+#endif
 
     // ---- step 1: own values and slot words (coalesced 16-byte loads), then the cut-edge
     // pulls (Alg. 1 l.10-11 across the tile boundary), folded in with shared atomicMax
@@ -148,16 +277,28 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
 #pragma unroll
         for (int k = 0; k < VPT; k++) {
             const int v = v0 + k;
-            if ((fin >> (8 * k)) & 0xFF) notify(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
-            if ((fout >> (8 * k)) & 0xFF) notify(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
+            if ((fin >> (8 * k)) & 0xFF) pnotify_full(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
+            if ((fout >> (8 * k)) & 0xFF) pnotify_full(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
         }
     }
     __syncthreads();
     // ---- step 2: local fixed point in shared memory (same drain loop as k_prop_tile)
+#ifdef ECL_PROF
+    const long long t_step1 = clock64();
+#endif
     {
         unsigned r0 = 0, r1 = 0, r2 = 0;
-        drain_local(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, S.s_queue, base, cnt, r0, r1, r2);
+        drain_pack(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, S.s_queue, base, cnt, r0, r1, r2);
+#ifdef ECL_PROF
+        r2 = warp_sum(r2);
+        if ((tid & 31) == 0) { PROF_ADD(dc, 2, r1); PROF_ADD(dc, 3, r2); }
+        if (tid == 0) PROF_ADD(dc, 1, r0);
+#endif
     }
+#ifdef ECL_PROF
+    __syncthreads();
+    const long long t_step2 = clock64();
+#endif
     // ---- step 3: write back (whole 16-byte groups; only this CTA writes these vertices
     // during the pass, so global memory still holds the originals: re-read rather than
     // kept in registers across step 2) and record which directions rose, for the marks
@@ -195,6 +336,15 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
             if (((e.y & EXT_DIR) ? bi[v] : bo[v]) != 0) dnext[e.x / PACK_TT] = 1;
         }
     }
+#ifdef ECL_PROF
+    __syncthreads();
+    if (tid == 0) {
+        const long long t_end = clock64();
+        PROF_ADD(dc, 4, t_step1 - t_start);
+        PROF_ADD(dc, 5, t_step2 - t_step1);
+        PROF_ADD(dc, 6, t_end - t_step2);
+    }
+#endif
     return any;
 }
 
@@ -205,14 +355,15 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
             DevCounters* __restrict__ dc, int pass, int first, uint8_t* __restrict__ dirty_cur,
             uint8_t* __restrict__ dirty_next, int full, int run) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ unsigned s_fin[PACK_TH], s_fout[PACK_TH];
+    __shared__ unsigned s_fin[PACK_TH + 1], s_fout[PACK_TH + 1];      // + the sentinel's scratch byte
     __shared__ unsigned short s_queue[2 * PACK_TT];
     __shared__ int s_dirty;
     TileSmem<PACK_TT> S;
-    S.s_in = (int*)smem_raw;
-    S.s_out = S.s_in + PACK_TT;
-    S.s_nin = (unsigned long long*)(S.s_out + PACK_TT);
+    S.s_in = (int*)smem_raw;                                          // [PACK_TT] + sentinel
+    S.s_out = S.s_in + PACK_TT + 4;
+    S.s_nin = (unsigned long long*)(S.s_out + PACK_TT + 4);
     S.s_nout = S.s_nin + PACK_TT;
+    if (threadIdx.x == 0) { S.s_in[PACK_TT] = 0; S.s_out[PACK_TT] = 0; }   // <= every priority
     S.s_fin = s_fin;
     S.s_fout = s_fout;
     S.s_queue = s_queue;

@@ -81,6 +81,8 @@ typedef enum {
                                         no row longer than 64 edges (tests, ablation) */
 #define ECL_SCC_NO_PACK 0x800u    /* ablation: Phase 2 re-walks the CSR/CSC rows on every tile
                                      visit instead of reading per-iteration tile packs */
+#define ECL_SCC_NO_ASYNC 0x1000u  /* ablation: Phase 2 as global passes (one launch each)
+                                     instead of one persistent launch with a tile queue */
 #define ECL_SCC_STAGED 0x80u      /* Phase 2 in threshold stages: the top-K priorities
                                      propagate first (ECL_SCC_STAGES env, default off) */
 
@@ -90,7 +92,10 @@ typedef enum {
 typedef struct {
     int32_t iterations;                      /* outer iterations that ran Phase 2        */
     int32_t trace_len;                       /* min(iterations, ECL_SCC_TRACE_MAX)       */
-    int64_t passes;                          /* global Phase-2 passes, all iterations    */
+    int64_t passes;                          /* global Phase-2 passes, all iterations; in
+                                                the asynchronous mode (default for graphs
+                                                without long rows): tile visits / tiles,
+                                                rounded up, per iteration               */
     int64_t edges_in[ECL_SCC_TRACE_MAX];     /* live edges entering Phase 2 (after trim) */
     int64_t vertices_in[ECL_SCC_TRACE_MAX];  /* vertices with a live edge in Phase 2     */
     int64_t edges_kept[ECL_SCC_TRACE_MAX];   /* edges kept by Phase 3 (before next trim) */

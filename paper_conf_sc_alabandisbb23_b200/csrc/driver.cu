@@ -136,6 +136,7 @@ void plan_free(Plan* p) {
     cudaFree(p->nb_cnt); cudaFree(p->nb_list); cudaFree(p->done); cudaFree(p->mark); cudaFree(p->sweep_ctr);
     cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
     cudaFree(p->pnin); cudaFree(p->pnout); cudaFree(p->ext); cudaFree(p->ext_cnt);
+    cudaFree(p->aq_state); cudaFree(p->aq_seen); cudaFree(p->aq_ctr);
     if (p->hc) cudaFreeHost(p->hc);
     if (p->ev_ok)
         for (int k = 0; k < 6; k++) cudaEventDestroy(p->ev[k]);
@@ -427,6 +428,37 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
         p->launches++;
         k_tile_pack<<<ntiles, PACK_TH, 0, s>>>(g, p->pnin, p->pnout, p->ext, p->ext_cnt);
         CK(cudaGetLastError());
+        if (!(p->flags & ECL_SCC_NO_ASYNC)) {          // one persistent launch (pack.cuh)
+            if (!p->aq_state) {
+                const size_t nt = (size_t)p->dirty_cap;
+                cudaError_t e = cudaMalloc((void**)&p->aq_state, nt * 4);
+                if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_seen, nt);
+                if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_ctr, 32);
+                if (e != cudaSuccess) {
+                    cudaGetLastError();
+                    return fail(ECL_SCC_ENOMEM, "async queue allocation: %s", cudaGetErrorString(e));
+                }
+                CK(cudaFuncSetAttribute(k_prop_async, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
+                int per_sm = 0, dev = 0, sms = 0;
+                CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_async, PACK_TH, pack_dyn_smem()));
+                CK(cudaGetDevice(&dev));
+                CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+                p->aq_resident = std::max(1, per_sm) * sms;
+            }
+            AsyncQ Q{p->aq_state, p->aq_seen, p->aq_ctr};
+            CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
+            CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
+            p->launches += 2;
+            k_async_init<<<grid_for((int64_t)ntiles, TPB), TPB, 0, s>>>(Q, (int)ntiles);
+            k_prop_async<<<(unsigned)std::min<int64_t>(ntiles, p->aq_resident), PACK_TH, pack_dyn_smem(), s>>>(
+                g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, Q);
+            CK(cudaGetLastError());
+            CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));
+            if (p->hc->err == 3) return fail(ECL_SCC_ECUDA, "internal: asynchronous Phase 2 stalled (watchdog)");
+            *passes_out = (int64_t)cdiv((int64_t)p->hc->passes, ntiles);   // sweep equivalents
+            return ECL_SCC_OK;
+        }
     }
     if (!sync && nchunks == 0 && (p->flags & ECL_SCC_SWEEP) && !(p->flags & ECL_SCC_STAGED)) {
         int used = 0, r = ECL_SCC_OK;

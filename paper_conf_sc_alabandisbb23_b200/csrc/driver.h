@@ -49,6 +49,10 @@ struct Plan {
     unsigned long long *pnin, *pnout;    // tile packs (pack.cuh): slot words per local vertex
     int2* ext;                           // tile packs: cut edges per tile
     int* ext_cnt;                        // tile packs: cut edges of each tile
+    int* aq_state;                       // asynchronous Phase 2 (pack.cuh AsyncQ)
+    uint8_t* aq_seen;
+    unsigned long long* aq_ctr;
+    int64_t aq_resident;                 // resident CTAs of k_prop_async
     int64_t launches;                    // kernels launched by the current call
     cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
     bool ev_ok;

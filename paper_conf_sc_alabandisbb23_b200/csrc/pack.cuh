@@ -197,11 +197,12 @@ static __global__ void __launch_bounds__(PACK_TH) k_tile_pack(WGraph g, unsigned
 
 // One visit of tile `tile` from its pack.  Returns non-zero in every thread if a
 // signature was raised.
+template <typename Mark>
 __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__ cin, int32_t* __restrict__ cout,
                                           const unsigned long long* __restrict__ pnin,
                                           const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext,
                                           const int* __restrict__ ext_cnt, DevCounters* __restrict__ dc, int tile,
-                                          int full, uint8_t* __restrict__ dnext, const TileSmem<PACK_TT>& S) {
+                                          int full, Mark mark, const TileSmem<PACK_TT>& S) {
     int* s_in = S.s_in;
     int* s_out = S.s_out;
     unsigned long long* s_nin = S.s_nin;
@@ -323,7 +324,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
         }
     }
     const int any = __syncthreads_or((int)(rin | rout));   // also: every drain flag is consumed
-    if (any && dnext) {
+    if (any && mark.on()) {
         s_fin[tid] = rin;
         s_fout[tid] = rout;
         __syncthreads();
@@ -333,7 +334,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
             const int2 e = __ldg(E + i);
             const int v = e.y & 0x7FFF;
             // in-edge u -> v: a raised v_out reaches u; out-edge v -> w: a raised v_in reaches w
-            if (((e.y & EXT_DIR) ? bi[v] : bo[v]) != 0) dnext[e.x / PACK_TT] = 1;
+            if (((e.y & EXT_DIR) ? bi[v] : bo[v]) != 0) mark(e.x / PACK_TT);
         }
     }
 #ifdef ECL_PROF
@@ -386,10 +387,142 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
             __syncthreads();
             if (!d) continue;
         }
-        ch_any |= pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, dirty_next, S);
+        ch_any |= pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkNext{dirty_next}, S);
         __syncthreads();
     }
     if (ch_any && tid == 0) dc->changed[pass & (RING - 1)] = 1;
+}
+
+// ------------------------------------------------------------------ asynchronous mode
+// Phase 2 as ONE persistent launch per outer iteration ("asynchronous", P:204
+// "persistent threads") at tile granularity, without pass barriers.  A global sweep cursor
+// runs over the tiles, ascending and descending in turn (the alternating pass order of
+// k_prop_pack); resident CTAs claim the next dirty tile under the cursor, so a tile
+// dirtied ahead of the cursor is visited in the same sweep (Gauss-Seidel between tiles)
+// and no CTA waits for the slowest visit of a pass.
+// Tile state machine (tstate): 0 clean, 1 dirty, 2 running, 3 running + dirtied again.
+//   mark(t):   0 -> 1 (pending++); 2 -> 3; 1, 3 unchanged
+//   claim(t):  1 -> 2 (the first visit of a tile in the phase is a full one)
+//   finish(t): 2 -> 0 (pending--); 3 -> 1
+// pending counts tiles in states 1-3.  A visit's marks (pending++) precede its own
+// finish (pending--), so pending == 0 means no visit is running and every tile's last
+// visit saw its final inputs: the Phase-2 fixed point (Alg. 1 l.7-14).  Values are
+// written (st.cg) and fenced before the marks; a claimer fences after its claim and reads
+// through L2, so it sees every value written before the state change it observed.
+struct AsyncQ {
+    int* tstate;                  // [ntiles]
+    uint8_t* tseen;               // [ntiles] visited in this phase
+    unsigned long long* ctr;      // [0] cursor, [1] pending, [2] stop
+};
+__device__ __forceinline__ void aq_mark(const AsyncQ& Q, int t) {
+    int st = *(volatile int*)(Q.tstate + t);
+    for (;;) {
+        if (st == 1 || st == 3) return;
+        const int old = atomicCAS(Q.tstate + t, st, st == 0 ? 1 : 3);
+        if (old == st) break;
+        st = old;
+    }
+    if (st == 0) atomicAdd(Q.ctr + 1, 1ull);
+}
+static __global__ void k_async_init(AsyncQ Q, int ntiles) {
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < ntiles; t += gridDim.x * blockDim.x) {
+        Q.tstate[t] = 1;
+        Q.tseen[t] = 0;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) { Q.ctr[0] = 0; Q.ctr[1] = (unsigned long long)ntiles; Q.ctr[2] = 0; }
+}
+
+// marks of one visit, deduplicated per neighbour tile in a shared-memory hash set
+constexpr int MSET = 256;
+struct MarkSet {
+    int* set;
+    AsyncQ Q;
+    __device__ __forceinline__ bool on() const { return true; }
+    __device__ __forceinline__ void operator()(int t) const {
+        unsigned h = ((unsigned)t * 0x9E3779B1u) >> 24;          // MSET = 256 slots
+        for (int k = 0; k < 16; k++, h = (h + 1) & (MSET - 1)) {
+            const int cur = ((volatile int*)set)[h];
+            if (cur == t) return;
+            if (cur == -1) {
+                const int old = atomicCAS(set + h, -1, t);
+                if (old == -1 || old == t) return;
+            }
+        }
+        __threadfence();                                          // crowded set: mark directly
+        aq_mark(Q, t);
+    }
+};
+
+static __global__ void __launch_bounds__(PACK_TH, 1536 / PACK_TH)
+k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, const unsigned long long* __restrict__ pnin,
+             const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext, const int* __restrict__ ext_cnt,
+             DevCounters* __restrict__ dc, AsyncQ Q) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ unsigned s_fin[PACK_TH + 1], s_fout[PACK_TH + 1];
+    __shared__ unsigned short s_queue[2 * PACK_TT];
+    __shared__ int s_set[MSET];
+    __shared__ int s_tile, s_full;
+    TileSmem<PACK_TT> S;
+    S.s_in = (int*)smem_raw;
+    S.s_out = S.s_in + PACK_TT + 4;
+    S.s_nin = (unsigned long long*)(S.s_out + PACK_TT + 4);
+    S.s_nout = S.s_nin + PACK_TT;
+    S.s_fin = s_fin;
+    S.s_fout = s_fout;
+    S.s_queue = s_queue;
+    S.s_lv = nullptr;
+    const int tid = threadIdx.x;
+    const int ntiles = (g.na + PACK_TT - 1) / PACK_TT;
+    if (tid == 0) { S.s_in[PACK_TT] = 0; S.s_out[PACK_TT] = 0; }
+    volatile unsigned long long* ctr = Q.ctr;
+    long long t0 = clock64();
+    for (;;) {
+        if (tid == 0) {
+            int t = -1;
+            for (unsigned miss = 0;; miss++) {
+                if (ctr[1] == 0 || ctr[2]) break;                 // fixed point (or watchdog stop)
+                const unsigned long long pos = atomicAdd(Q.ctr, 1ull);
+                const unsigned long long k = pos / (unsigned)ntiles;
+                const int off = (int)(pos - k * (unsigned)ntiles);
+                const int c = (k & 1) ? ntiles - 1 - off : off;
+                if (((volatile int*)Q.tstate)[c] == 1 && atomicCAS(Q.tstate + c, 1, 2) == 1) {
+                    t = c;
+                    break;
+                }
+                if (miss >= (unsigned)ntiles) {                   // a whole sweep without work
+                    __nanosleep(256);
+                    if (clock64() - t0 > (1ll << 36)) {           // ~30 s idle: protocol bug
+                        atomicExch(&dc->err, 3);
+                        atomicExch(Q.ctr + 2, 1ull);
+                        break;
+                    }
+                }
+            }
+            if (t >= 0) {
+                t0 = clock64();
+                atomicAdd(&dc->passes, 1ull);                     // tile visits of the phase
+                __threadfence();                                  // claim before the value reads
+                s_full = Q.tseen[t] == 0;
+                Q.tseen[t] = 1;
+            }
+            s_tile = t;
+        }
+        for (int i = tid; i < MSET; i += PACK_TH) s_set[i] = -1;
+        __syncthreads();
+        const int tile = s_tile, full = s_full;
+        if (tile < 0) break;
+        pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S);
+        __threadfence();                                          // values before marks
+        __syncthreads();
+        for (int i = tid; i < MSET; i += PACK_TH)
+            if (s_set[i] >= 0) aq_mark(Q, s_set[i]);
+        __threadfence();
+        __syncthreads();                                          // marks (pending++) before finish
+        if (tid == 0) {
+            if (atomicCAS(Q.tstate + tile, 2, 0) == 2) atomicAdd(Q.ctr + 1, ~0ull);
+            else atomicExch(Q.tstate + tile, 1);
+        }
+    }
 }
 
 }  // namespace eclscc

@@ -94,7 +94,7 @@ def test_random_small_graphs_labels_and_traces():
         edges = [(rng.randrange(n), rng.randrange(n)) for _ in range(m)]
         g = gen.from_edges(n, edges)
         truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-        for flags in (0, E.NO_TRIM, E.IDENTITY_IDS, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER, E.NO_PACK):
+        for flags in (0, E.NO_TRIM, E.IDENTITY_IDS, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER, E.NO_PACK, E.NO_ASYNC):
             lab, _ = gpu_labels(g, flags)
             np.testing.assert_array_equal(lab, truth, err_msg=f"trial {trial} flags {flags}")
         if trial % 10 == 0:
@@ -107,7 +107,7 @@ def test_random_small_graphs_labels_and_traces():
 def test_c1_gnm_2000_8000():
     g = gen.config("c1")
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-    for flags in (0, E.IDENTITY_IDS, E.NO_TRIM, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER, E.NO_PACK):
+    for flags in (0, E.IDENTITY_IDS, E.NO_TRIM, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER, E.NO_PACK, E.NO_ASYNC):
         lab, _ = gpu_labels(g, flags)
         np.testing.assert_array_equal(lab, truth)
     check_trace(g, trim=True)

@@ -446,12 +446,18 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                 p->aq_resident = std::max(1, per_sm) * sms;
             }
             AsyncQ Q{p->aq_state, p->aq_seen, p->aq_ctr};
+            // tiles per claim: runs pay when there are many tiles per resident CTA (measured:
+            // C4 iteration 1, 18 tiles per CTA, best at 8; C2, ~1 tile per CTA, best at 1)
+            static int claim_env = -1;                      // tuning knob ECL_SCC_CLAIM
+            if (claim_env < 0) claim_env = getenv("ECL_SCC_CLAIM") ? std::min(32, std::max(1, atoi(getenv("ECL_SCC_CLAIM")))) : 0;
+            const int claim = claim_env ? claim_env
+                                        : (int)std::min<int64_t>(8, std::max<int64_t>(1, ntiles / (2 * p->aq_resident)));
             CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
             CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
             p->launches += 2;
             k_async_init<<<grid_for((int64_t)ntiles, TPB), TPB, 0, s>>>(Q, (int)ntiles);
             k_prop_async<<<(unsigned)std::min<int64_t>(ntiles, p->aq_resident), PACK_TH, pack_dyn_smem(), s>>>(
-                g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, Q);
+                g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, Q, claim);
             CK(cudaGetLastError());
             CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
             CK(cudaStreamSynchronize(s));

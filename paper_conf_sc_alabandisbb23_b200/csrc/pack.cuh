@@ -324,6 +324,12 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
         }
     }
     const int any = __syncthreads_or((int)(rin | rout));   // also: every drain flag is consumed
+#ifdef ECL_PROF
+    {
+        const int nr = warp_sum(__popc(rin) + __popc(rout));   // raised vertex-directions
+        if ((tid & 31) == 0 && nr) PROF_ADD(dc, 7, nr);
+    }
+#endif
     if (any && mark.on()) {
         s_fin[tid] = rin;
         s_fout[tid] = rout;
@@ -432,6 +438,8 @@ static __global__ void k_async_init(AsyncQ Q, int ntiles) {
     if (blockIdx.x == 0 && threadIdx.x == 0) { Q.ctr[0] = 0; Q.ctr[1] = (unsigned long long)ntiles; Q.ctr[2] = 0; }
 }
 
+constexpr int CLAIM_MAX = 32;     // sweep positions per claim (a CTA's run of tiles), <= a warp
+
 // marks of one visit, deduplicated per neighbour tile in a shared-memory hash set
 constexpr int MSET = 256;
 struct MarkSet {
@@ -456,12 +464,13 @@ struct MarkSet {
 static __global__ void __launch_bounds__(PACK_TH, 1536 / PACK_TH)
 k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, const unsigned long long* __restrict__ pnin,
              const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext, const int* __restrict__ ext_cnt,
-             DevCounters* __restrict__ dc, AsyncQ Q) {
+             DevCounters* __restrict__ dc, AsyncQ Q, int claim) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ unsigned s_fin[PACK_TH + 1], s_fout[PACK_TH + 1];
     __shared__ unsigned short s_queue[2 * PACK_TT];
     __shared__ int s_set[MSET];
-    __shared__ int s_tile, s_full;
+    __shared__ int s_claim[CLAIM_MAX], s_nclaim;
+    __shared__ uint8_t s_seen[CLAIM_MAX];
     TileSmem<PACK_TT> S;
     S.s_in = (int*)smem_raw;
     S.s_out = S.s_in + PACK_TT + 4;
@@ -477,51 +486,68 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
     volatile unsigned long long* ctr = Q.ctr;
     long long t0 = clock64();
     for (;;) {
-        if (tid == 0) {
-            int t = -1;
-            for (unsigned miss = 0;; miss++) {
-                if (ctr[1] == 0 || ctr[2]) break;                 // fixed point (or watchdog stop)
-                const unsigned long long pos = atomicAdd(Q.ctr, 1ull);
-                const unsigned long long k = pos / (unsigned)ntiles;
-                const int off = (int)(pos - k * (unsigned)ntiles);
-                const int c = (k & 1) ? ntiles - 1 - off : off;
-                if (((volatile int*)Q.tstate)[c] == 1 && atomicCAS(Q.tstate + c, 1, 2) == 1) {
-                    t = c;
-                    break;
+        // warp 0 claims: one cursor step covers CLAIM consecutive sweep positions, every
+        // dirty tile among them is claimed and the CTA visits them in sweep order (a run)
+        if (tid < 32) {
+            const int lane = tid;
+            int got = 0, stop = 0;
+            for (unsigned miss = 0;; miss += claim) {
+                if (lane == 0) stop = (ctr[1] == 0 || ctr[2]) ? 1 : 0;   // fixed point / watchdog
+                if (__shfl_sync(FULL, stop, 0)) break;
+                unsigned long long pos = 0;
+                if (lane == 0) pos = atomicAdd(Q.ctr, (unsigned long long)claim);
+                pos = __shfl_sync(FULL, pos, 0) + (unsigned)lane;
+                bool mine = false;
+                int c = 0;
+                if (lane < claim) {
+                    const unsigned long long k = pos / (unsigned)ntiles;
+                    const int off = (int)(pos - k * (unsigned)ntiles);
+                    c = (k & 1) ? ntiles - 1 - off : off;
+                    mine = ((volatile int*)Q.tstate)[c] == 1 && atomicCAS(Q.tstate + c, 1, 2) == 1;
                 }
-                if (miss >= (unsigned)ntiles) {                   // a whole sweep without work
+                const unsigned m = __ballot_sync(FULL, mine);
+                if (mine) {
+                    const int slot = __popc(m & ((1u << lane) - 1));
+                    s_claim[slot] = c;
+                    atomicAdd(&dc->passes, 1ull);                  // tile visits of the phase
+                    s_seen[slot] = Q.tseen[c];
+                    Q.tseen[c] = 1;
+                }
+                if (m) { got = __popc(m); break; }
+                if (miss >= (unsigned)ntiles) {                    // a whole sweep without work
                     __nanosleep(256);
-                    if (clock64() - t0 > (1ll << 36)) {           // ~30 s idle: protocol bug
+                    if (lane == 0 && clock64() - t0 > (1ll << 36)) {   // ~30 s idle: protocol bug
                         atomicExch(&dc->err, 3);
                         atomicExch(Q.ctr + 2, 1ull);
-                        break;
                     }
                 }
             }
-            if (t >= 0) {
-                t0 = clock64();
-                atomicAdd(&dc->passes, 1ull);                     // tile visits of the phase
-                __threadfence();                                  // claim before the value reads
-                s_full = Q.tseen[t] == 0;
-                Q.tseen[t] = 1;
+            if (lane == 0) {
+                s_nclaim = got;
+                if (got) t0 = clock64();
             }
-            s_tile = t;
+            __threadfence();                                      // claims before the value reads
         }
-        for (int i = tid; i < MSET; i += PACK_TH) s_set[i] = -1;
         __syncthreads();
-        const int tile = s_tile, full = s_full;
-        if (tile < 0) break;
-        pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S);
-        __threadfence();                                          // values before marks
-        __syncthreads();
-        for (int i = tid; i < MSET; i += PACK_TH)
-            if (s_set[i] >= 0) aq_mark(Q, s_set[i]);
-        __threadfence();
-        __syncthreads();                                          // marks (pending++) before finish
-        if (tid == 0) {
-            if (atomicCAS(Q.tstate + tile, 2, 0) == 2) atomicAdd(Q.ctr + 1, ~0ull);
-            else atomicExch(Q.tstate + tile, 1);
+        const int nclaim = s_nclaim;
+        if (nclaim == 0) break;
+        for (int j = 0; j < nclaim; j++) {
+            const int tile = s_claim[j], full = s_seen[j] == 0;
+            for (int i = tid; i < MSET; i += PACK_TH) s_set[i] = -1;
+            __syncthreads();
+            pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S);
+            __threadfence();                                      // values before marks
+            __syncthreads();
+            for (int i = tid; i < MSET; i += PACK_TH)
+                if (s_set[i] >= 0) aq_mark(Q, s_set[i]);
+            __threadfence();
+            __syncthreads();                                      // marks (pending++) before finish
+            if (tid == 0) {
+                if (atomicCAS(Q.tstate + tile, 2, 0) == 2) atomicAdd(Q.ctr + 1, ~0ull);
+                else atomicExch(Q.tstate + tile, 1);
+            }
         }
+        __syncthreads();                                          // s_claim is rewritten next
     }
 }
 

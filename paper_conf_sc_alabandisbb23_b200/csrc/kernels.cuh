@@ -101,11 +101,12 @@ template <bool FIRST>
 __device__ __forceinline__ bool keep_edge(int owner, int a, int b, int other, const int32_t* __restrict__ cin,
                                           const int32_t* __restrict__ cout) {
     if (FIRST) return other != owner;
-    return __ldg(cin + other) == a && __ldg(cout + other) == b;
+    // both loads are issued unconditionally (no short circuit): callers batch these gathers
+    return (__ldg(cin + other) == a) & (__ldg(cout + other) == b);
 }
 // Trim-1 on the kept graph: no kept in-edge or no kept out-edge
 __device__ __forceinline__ bool trimmed(const int32_t* __restrict__ kin, const int32_t* __restrict__ kout, int x) {
-    return __ldg(kin + x) == 0 || __ldg(kout + x) == 0;
+    return (__ldg(kin + x) == 0) | (__ldg(kout + x) == 0);
 }
 
 struct RowCtx {
@@ -130,10 +131,10 @@ __device__ __forceinline__ RowCtx load_row(const WGraph& g, int64_t i, const int
 // count edges of one row (light: by the lane, heavy: by the whole warp) that satisfy P
 template <typename P>
 __device__ __forceinline__ int count_row(const int32_t* __restrict__ adj, int rb, int re, bool go, int lane, P pred,
-                                         bool chunked = false) {
+                                         bool chunked = false, bool light = true) {
     int c = 0;
     if (chunked && re - rb > HEAVY_T) go = false;      // long row: the chunk kernels count it
-    if (go && re - rb <= HEAVY)
+    if (light && go && re - rb <= HEAVY)
         for (int e = rb; e < re; e++) c += pred(__ldg(adj + e));
     unsigned hm = __ballot_sync(FULL, go && re - rb > HEAVY);
     while (hm) {
@@ -167,7 +168,7 @@ struct SurvivePred {
     int i, a, b;
     const int32_t *cin, *cout, *kin, *kout;
     __device__ __forceinline__ bool operator()(int k) const {
-        return keep_edge<FIRST>(i, a, b, k, cin, cout) && !(TRIM && trimmed(kin, kout, k));
+        return keep_edge<FIRST>(i, a, b, k, cin, cout) & !(TRIM && trimmed(kin, kout, k));
     }
     __device__ __forceinline__ SurvivePred bcast(int src) const {
         SurvivePred p = *this;
@@ -175,6 +176,56 @@ struct SurvivePred {
         return p;
     }
 };
+
+// Light rows (<= HEAVY edges) of both directions of one vertex, in batches of 4 edges per
+// direction: the adjacency loads of a batch, then all the predicate gathers, are issued
+// before any result is used (memory-level parallelism; a thread used to walk its rows one
+// dependent load after another).  Invalid slots evaluate the predicate on `self`.
+template <typename P>
+__device__ __forceinline__ void count_light2(const int32_t* __restrict__ oadj, int ob, int no,
+                                             const int32_t* __restrict__ iadj, int ib, int ni, int self, P pred,
+                                             int& co, int& ci) {
+    for (int k = 0; k < no || k < ni; k += 4) {
+        int xo[4], xi[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            xo[q] = k + q < no ? __ldg(oadj + ob + k + q) : self;
+            xi[q] = k + q < ni ? __ldg(iadj + ib + k + q) : self;
+        }
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            co += (int)pred(xo[q]) & (int)(k + q < no);
+            ci += (int)pred(xi[q]) & (int)(k + q < ni);
+        }
+    }
+}
+template <typename P>
+__device__ __forceinline__ void emit_light2(const int32_t* __restrict__ oadj, int ob, int no, int po,
+                                            int32_t* __restrict__ odst, const int32_t* __restrict__ iadj, int ib,
+                                            int ni, int pi, int32_t* __restrict__ idst, int self,
+                                            const int32_t* __restrict__ newidx, P pred) {
+    for (int k = 0; k < no || k < ni; k += 4) {
+        int xo[4], xi[4], yo[4], yi[4];
+        bool so[4], si[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            xo[q] = k + q < no ? __ldg(oadj + ob + k + q) : self;
+            xi[q] = k + q < ni ? __ldg(iadj + ib + k + q) : self;
+        }
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            so[q] = pred(xo[q]) & (k + q < no);
+            si[q] = pred(xi[q]) & (k + q < ni);
+            yo[q] = __ldg(newidx + xo[q]);
+            yi[q] = __ldg(newidx + xi[q]);
+        }
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            if (so[q]) odst[po++] = yo[q];
+            if (si[q]) idst[pi++] = yi[q];
+        }
+    }
+}
 
 // kept in/out degree per local vertex, plus the number of kept edges
 template <bool FIRST>
@@ -185,9 +236,16 @@ static __global__ void k_keep_count(WGraph g, const int32_t* __restrict__ cin, c
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
     KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout};
-    const int co = count_row(g.oadj, r.ob, r.oe, r.live, lane, pred, chunked);
-    const int ci = count_row(g.iadj, r.ib, r.ie, r.live, lane, pred, chunked);
-    if (r.valid) { kin[i] = ci; kout[i] = co; hcnt[i] = make_int2(0, 0); }
+    int co = 0, ci = 0;
+    count_light2(g.oadj, r.ob, r.live && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, g.iadj, r.ib,
+                 r.live && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, (int)(r.valid ? i : 0), pred, co, ci);
+    co += count_row(g.oadj, r.ob, r.oe, r.live, lane, pred, chunked, false);
+    ci += count_row(g.iadj, r.ib, r.ie, r.live, lane, pred, chunked, false);
+    if (r.valid) {
+        kin[i] = ci;
+        kout[i] = co;
+        if (chunked) hcnt[i] = make_int2(0, 0);
+    }
     const int s = warp_sum(co);
     if (lane == 0 && s) atomicAdd(kept, (unsigned long long)s);
 }
@@ -207,8 +265,10 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
     } else {
         const bool go = r.live && !trimmed(kin, kout, (int)i);
         SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
-        nout = count_row(g.oadj, r.ob, r.oe, go, lane, pred, chunked);
-        nin = count_row(g.iadj, r.ib, r.ie, go, lane, pred, chunked);
+        count_light2(g.oadj, r.ob, go && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, g.iadj, r.ib,
+                     go && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, (int)(r.valid ? i : 0), pred, nout, nin);
+        nout += count_row(g.oadj, r.ob, r.oe, go, lane, pred, chunked, false);
+        nin += count_row(g.iadj, r.ib, r.ie, go, lane, pred, chunked, false);
         if (chunked && r.valid) {                       // long rows: counted by k_count_chunks
             const int2 h = hcnt[i];
             nout += h.x;
@@ -327,9 +387,9 @@ static __global__ void k_snapshot_left(int32_t n, const int32_t* __restrict__ la
 template <typename P>
 __device__ __forceinline__ void emit_row(const int32_t* __restrict__ adj, int rb, int re, bool go, int pos,
                                          const int32_t* __restrict__ newidx, int32_t* __restrict__ dst, int lane,
-                                         P pred, bool chunked = false) {
+                                         P pred, bool chunked = false, bool light = true) {
     if (chunked && re - rb > HEAVY_T) go = false;      // long row: k_scatter_chunks writes it
-    if (go && re - rb <= HEAVY) {
+    if (light && go && re - rb <= HEAVY) {
         for (int e = rb; e < re; e++) {
             const int x = __ldg(adj + e);
             if (pred(x)) dst[pos++] = __ldg(newidx + x);
@@ -368,8 +428,10 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
     int po = 0, pi = 0;
     if (go) { po = optr2[j]; pi = iptr2[j]; }
     SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
-    emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred, chunked);
-    emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred, chunked);
+    emit_light2(g.oadj, r.ob, go && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, po, oadj2, g.iadj, r.ib,
+                go && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, pi, iadj2, (int)(r.valid ? i : 0), newidx, pred);
+    emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred, chunked, false);
+    emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred, chunked, false);
 }
 
 // ------------------------------------------------------------------ long rows in chunks

@@ -55,6 +55,7 @@ static inline unsigned grid_for(int64_t work, int threads) {
 }
 
 constexpr int TPB = 256;
+static_assert(TPB == TPB_COMPACT, "k_keep_count reduces over TPB_COMPACT threads");
 constexpr double REORDER_LOCALITY = 0.85;   // measured: C4 lex 0.77, blocked8 0.91
 
 // --------------------------------------------------------------------------- plan

@@ -228,8 +228,9 @@ __device__ __forceinline__ void emit_light2(const int32_t* __restrict__ oadj, in
 }
 
 // kept in/out degree per local vertex, plus the number of kept edges
+constexpr int TPB_COMPACT = 256;     // block size of the compaction kernels (driver TPB)
 template <bool FIRST>
-static __global__ void k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                              int32_t* __restrict__ kin, int32_t* __restrict__ kout,
                              unsigned long long* __restrict__ kept, int chunked, int2* __restrict__ hcnt) {
     const int lane = threadIdx.x & 31;
@@ -246,8 +247,16 @@ static __global__ void k_keep_count(WGraph g, const int32_t* __restrict__ cin, c
         kout[i] = co;
         if (chunked) hcnt[i] = make_int2(0, 0);
     }
+    // one atomic per block (one per warp on a single address serialised ~0.5M atomics in L2)
+    __shared__ int s_kept[TPB_COMPACT / WARP];
     const int s = warp_sum(co);
-    if (lane == 0 && s) atomicAdd(kept, (unsigned long long)s);
+    if (lane == 0) s_kept[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int t = 0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); w++) t += s_kept[w];
+        if (t) atomicAdd(kept, (unsigned long long)t);
+    }
 }
 
 // per-vertex surviving (kept, not trimmed) degrees and per-warp totals (alive, out, in)
@@ -568,6 +577,7 @@ static __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restri
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     bool ch = false;
+    long long ne = 0;                              // edges reduced by this warp (accounting)
     for (int64_t c = wid; c < nchunks; c += nw) {
         const Chunk k = chunks[c];
         const int32_t* adj = k.dir ? g.iadj : g.oadj;
@@ -575,11 +585,12 @@ static __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restri
         int acc = 0;
         for (int e = k.beg + lane; e < k.end; e += WARP) acc = max(acc, eff(ld_cg(sig + __ldg(adj + e)), theta));
         acc = warp_max(acc);
-        if (lane == 0) atomicAdd(&dc->heavy_e, (unsigned long long)(k.end - k.beg));
+        ne += k.end - k.beg;
         if (lane == 0 && acc > ld_cg(sig + k.i)) {
             if (atomicMax(sig + k.i, acc) < acc) ch = true;
         }
     }
+    if (lane == 0 && ne) atomicAdd(&dc->heavy_e, (unsigned long long)ne);
     if (__any_sync(FULL, ch) && lane == 0) dc->changed[pass & (RING - 1)] = 1;
 }
 
@@ -852,9 +863,11 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
     }
     {
         // honest roofline accounting: only visited tiles move bytes (SURVEY 8(d) terms)
-        me = warp_sum(me);
-        if ((tid & 31) == 0 && me) atomicAdd(&dc->visit_e, (unsigned long long)me);
-        if (tid == 0) atomicAdd(&dc->visit_v, (unsigned long long)cnt);
+        (void)me;                                 // = optr[base + cnt] - optr[base], one atomic per visit
+        if (tid == 0) {
+            atomicAdd(&dc->visit_e, (unsigned long long)(__ldg(g.optr + base + cnt) - __ldg(g.optr + base)));
+            atomicAdd(&dc->visit_v, (unsigned long long)cnt);
+        }
     }
     if (tid == 0) PROF_ADD(dc, 0, 1);                         // tile visits
     // ---- step 1b: recompute flags (pull model).  Byte k of s_fin[t] / s_fout[t] asks

@@ -340,8 +340,16 @@ def ours(args):
         pms = sum(s["ms_prop"] for s in rstats) / len(rstats)
         launches = sum(s["passes"] for s in rstats) / len(rstats)
         achieved = pb / (pms * 1e-3) / 1e9 if pms > 0 else None
-        traffic = roofline_traffic("k_prop_tile")
-        roof = {"bound": "hbm", "kernel": "Phase 2 (k_prop_tile + k_prop_heavy)",
+        # the dominant kernel: k_prop_async (one persistent launch per outer iteration) on
+        # graphs without long rows, the pass kernels k_prop_tile + k_prop_heavy otherwise
+        async_path = args.config != "c3"
+        kname = "k_prop_async" if async_path else "k_prop_tile"
+        traffic = roofline_traffic(kname)
+        iters = sum(s["iterations"] for s in rstats) / len(rstats)
+        roof = {"bound": "hbm",
+                "kernel": ("Phase 2 (k_tile_pack + k_prop_async)" if async_path
+                           else "Phase 2 (k_prop_tile + k_prop_heavy)"),
+                "algorithmic_bytes_per_launch": int(pb / iters) if async_path and iters else None,
                 "achieved": round(achieved, 1) if achieved else None, "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4) if achieved else None,
                 "traffic": traffic, "peak_source": peak_src,

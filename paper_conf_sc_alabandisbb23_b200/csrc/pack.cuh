@@ -202,7 +202,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
                                           const unsigned long long* __restrict__ pnin,
                                           const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext,
                                           const int* __restrict__ ext_cnt, DevCounters* __restrict__ dc, int tile,
-                                          int full, Mark mark, const TileSmem<PACK_TT>& S) {
+                                          int full, Mark mark, const TileSmem<PACK_TT>& S, int next = -1) {
     int* s_in = S.s_in;
     int* s_out = S.s_out;
     unsigned long long* s_nin = S.s_nin;
@@ -283,6 +283,18 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
         }
     }
     __syncthreads();
+    // the next tile of this CTA's run: pull its pack rows and values into L2 while this one
+    // drains (384 lines of 128 B, one per thread; L2 is coherent, so racing writers are fine)
+    if (next >= 0 && tid < 384) {
+        const int nb = next * PACK_TT;
+        const char* line;
+        if (tid < 128) line = (const char*)(pnin + nb) + 128 * tid;
+        else if (tid < 256) line = (const char*)(pnout + nb) + 128 * (tid - 128);
+        else if (tid < 320) line = (const char*)(cin + nb) + 128 * (tid - 256);
+        else line = (const char*)(cout + nb) + 128 * (tid - 320);
+        if (tid < 256 || nb + 32 * ((tid - 256) & 63) < g.na)
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(line));
+    }
     // ---- step 2: local fixed point in shared memory (same drain loop as k_prop_tile)
 #ifdef ECL_PROF
     const long long t_step1 = clock64();
@@ -535,7 +547,8 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             const int tile = s_claim[j], full = s_seen[j] == 0;
             for (int i = tid; i < MSET; i += PACK_TH) s_set[i] = -1;
             __syncthreads();
-            pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S);
+            pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S,
+                       j + 1 < nclaim ? s_claim[j + 1] : -1);
             __threadfence();                                      // values before marks
             __syncthreads();
             for (int i = tid; i < MSET; i += PACK_TH)

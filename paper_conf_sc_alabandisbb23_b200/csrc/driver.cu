@@ -230,7 +230,7 @@ static int reorder_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, con
     int32_t* start = p->cellbuf + (nkeys + 1);
     int32_t* cursor = p->kout;                         // free until the first compaction
     CK(cudaMemsetAsync(hist, 0, sizeof(int32_t) * (size_t)(nkeys + 1), s));
-    p->launches++; reo::k_cell_hist<<<gs, TPB, 0, s>>>(n, p->cellv, hist);
+    p->launches++; reo::k_cell_hist_agg<<<gs, TPB, 0, s>>>(n, p->cellv, hist);
     int r = scan_excl<I1>(p, (const I1*)hist, nkeys, (I1*)start, (I1*)&p->dc->grand1, p->bsum, 1, s);
     if (r) return r;
     CK(cudaMemsetAsync(cursor, 0, sizeof(int32_t) * (size_t)(nkeys + 1), s));

@@ -32,15 +32,35 @@ static __global__ void k_bfs_level(int32_t* __restrict__ fa, int32_t* __restrict
     int32_t* next = (r & 1) ? fa : fb;
     const int nf = ld_vol(cnt + r % 3);
     if (blockIdx.x == 0 && threadIdx.x == 0) cnt[(r + 2) % 3] = 0;
-    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nf; k += (int64_t)gridDim.x * blockDim.x) {
-        const int u = front[k], c = ld_cg(cell + u);
-        for (int dir = 0; dir < 2; dir++) {
-            const int32_t* p = dir ? cp : rp;
-            const int32_t* a = dir ? cr : ci;
-            for (int e = p[u]; e < p[u + 1]; e++) {
-                const int w = a[e];
-                if (ld_cg(cell + w) != NOLAB) continue;
-                if (atomicCAS(cell + w, NOLAB, c) == NOLAB) next[atomicAdd(cnt + (r + 1) % 3, 1)] = w;
+    const int lane = threadIdx.x & 31;
+    // whole warps iterate (ballots below); appends are warp-aggregated: one atomic per warp
+    // and round instead of one per claimed vertex on a single counter
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t k0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x - lane; k0 < nf; k0 += stride) {
+        const int64_t k = k0 + lane;
+        const bool act = k < nf;
+        int u = 0, c = 0, b0 = 0, e0 = 0, b1 = 0, e1 = 0;
+        if (act) {
+            u = front[k];
+            c = ld_cg(cell + u);
+            b0 = rp[u]; e0 = rp[u + 1]; b1 = cp[u]; e1 = cp[u + 1];
+        }
+        int n0 = e0 - b0, n1 = e1 - b1;
+        for (int j = 0;; j++) {                        // j-th neighbour of every lane's vertex
+            const bool has = j < n0 + n1;
+            if (!__any_sync(FULL, has)) break;
+            bool got = false;
+            int w = 0;
+            if (has) {
+                w = j < n0 ? ci[b0 + j] : cr[b1 + j - n0];
+                got = ld_cg(cell + w) == NOLAB && atomicCAS(cell + w, NOLAB, c) == NOLAB;
+            }
+            const unsigned m = __ballot_sync(FULL, got);
+            if (m) {
+                int at = 0;
+                if (lane == __ffs(m) - 1) at = atomicAdd(cnt + (r + 1) % 3, __popc(m));
+                at = __shfl_sync(FULL, at, __ffs(m) - 1);
+                if (got) next[at + __popc(m & ((1u << lane) - 1))] = w;
             }
         }
     }
@@ -54,22 +74,38 @@ static __global__ void k_seed2(int32_t n, int32_t* __restrict__ cell, int32_t* _
 }
 // cell key (seed ID >> CELL_SHIFT: nearly unique per cell, ordered like the seeds);
 // vertices no seed reached form cells of their own ID range
-static __global__ void k_cell_hist(int32_t n, int32_t* __restrict__ lab, int32_t* __restrict__ hist) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-        int c = lab[v];
-        if (c == NOLAB) c = (int)v;
-        c >>= CELL_SHIFT;
-        lab[v] = c;
-        atomicAdd(hist + c, 1);
+// lanes with equal keys (consecutive vertices mostly share a cell) add once per group
+static __global__ void k_cell_hist_agg(int32_t n, int32_t* __restrict__ lab, int32_t* __restrict__ hist) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t v0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x - lane; v0 < n; v0 += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t v = v0 + lane;
+        int c = -1;
+        if (v < n) {
+            c = lab[v];
+            if (c == NOLAB) c = (int)v;
+            c >>= CELL_SHIFT;
+            lab[v] = c;
+        }
+        const unsigned grp = __match_any_sync(FULL, c);
+        if (c >= 0 && lane == __ffs(grp) - 1) atomicAdd(hist + c, __popc(grp));
     }
 }
 static __global__ void k_cell_place(int32_t n, const int32_t* __restrict__ key, const int32_t* __restrict__ start,
                                     int32_t* __restrict__ cursor, int32_t* __restrict__ pos, int32_t* __restrict__ orig) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-        const int c = key[v];
-        const int j = start[c] + atomicAdd(cursor + c, 1);
-        pos[v] = j;
-        orig[j] = (int)v;
+    const int lane = threadIdx.x & 31;
+    for (int64_t v0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x - lane; v0 < n; v0 += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t v = v0 + lane;
+        const int c = v < n ? key[v] : -1;
+        const unsigned grp = __match_any_sync(FULL, c);       // one atomic per key group
+        const int leader = __ffs(grp) - 1;
+        int at = 0;
+        if (c >= 0 && lane == leader) at = atomicAdd(cursor + c, __popc(grp));
+        at = __shfl_sync(FULL, at, leader);
+        if (c >= 0) {
+            const int j = start[c] + at + __popc(grp & ((1u << lane) - 1));
+            pos[v] = j;
+            orig[j] = (int)v;
+        }
     }
 }
 // one CTA per cell: sort the cell's storage slots by caller ID (bitonic sort in shared

@@ -83,6 +83,10 @@ typedef enum {
                                      visit instead of reading per-iteration tile packs */
 #define ECL_SCC_NO_ASYNC 0x1000u  /* ablation: Phase 2 as global passes (one launch each)
                                      instead of one persistent launch with a tile queue */
+#define ECL_SCC_TAIL 0x2000u      /* opt-in: once the working graph has at most 32768 vertices,
+                                     run the remaining outer iterations in one cooperative
+                                     launch (tail.cuh) instead of compacting each time
+                                     (measured: no gain on C2/C4) */
 #define ECL_SCC_STAGED 0x80u      /* Phase 2 in threshold stages: the top-K priorities
                                      propagate first (ECL_SCC_STAGES env, default off) */
 
@@ -108,6 +112,8 @@ typedef struct {
     double ms_ingest;                        /* validation + CSC build                    */
     double ms_compact;                       /* Phase 3 + trim + compaction + Phase 1     */
     double ms_prop;                          /* Phase 2 (all passes)                      */
+    double ms_prop_iter[ECL_SCC_TRACE_MAX];  /* Phase 2 of outer iteration k+1            */
+    double ms_compact_iter[ECL_SCC_TRACE_MAX]; /* Phase 3 + compaction before iteration k+1 */
 } ecl_scc_stats;
 
 typedef struct ecl_scc_plan_s* ecl_scc_plan_t;

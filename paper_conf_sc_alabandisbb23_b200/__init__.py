@@ -20,7 +20,7 @@ _LIB_PATH = os.path.join(_HERE, "libeclscc.so")
 OK, EINVAL, ERANGE, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED = range(7)
 NO_TRIM, NO_VALIDATE, SYNC_PASSES, TIME_STAGES = 0x1, 0x4, 0x8, 0x10
 IDENTITY_IDS, NO_DIRTY, STAGED, SWEEP, NO_REORDER = 0x20, 0x40, 0x80, 0x100, 0x200
-FORCE_REORDER, NO_PACK, NO_ASYNC = 0x400, 0x800, 0x1000
+FORCE_REORDER, NO_PACK, NO_ASYNC, TAIL = 0x400, 0x800, 0x1000, 0x2000
 TRACE_MAX = 64
 
 _lib = None
@@ -38,7 +38,8 @@ class Stats(ctypes.Structure):
                 ("edges_in", ctypes.c_int64 * TRACE_MAX), ("vertices_in", ctypes.c_int64 * TRACE_MAX),
                 ("edges_kept", ctypes.c_int64 * TRACE_MAX), ("passes_iter", ctypes.c_int64 * TRACE_MAX),
                 ("prop_bytes", ctypes.c_int64), ("kernel_launches", ctypes.c_int64),
-                ("ms_ingest", ctypes.c_double), ("ms_compact", ctypes.c_double), ("ms_prop", ctypes.c_double)]
+                ("ms_ingest", ctypes.c_double), ("ms_compact", ctypes.c_double), ("ms_prop", ctypes.c_double),
+                ("ms_prop_iter", ctypes.c_double * TRACE_MAX), ("ms_compact_iter", ctypes.c_double * TRACE_MAX)]
 
     def as_dict(self) -> dict:
         k = self.trace_len
@@ -47,7 +48,9 @@ class Stats(ctypes.Structure):
                     ms_compact=self.ms_compact, ms_prop=self.ms_prop,
                     edges_in=list(self.edges_in[:k]), vertices_in=list(self.vertices_in[:k]),
                     edges_kept=list(self.edges_kept[:max(k - 1, 0)]),
-                    passes_iter=list(self.passes_iter[:k]))
+                    passes_iter=list(self.passes_iter[:k]),
+                    ms_prop_iter=[round(x, 4) for x in self.ms_prop_iter[:k]],
+                    ms_compact_iter=[round(x, 4) for x in self.ms_compact_iter[:k + 1]])
 
 
 def lib() -> ctypes.CDLL:

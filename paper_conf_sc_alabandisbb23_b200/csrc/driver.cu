@@ -24,6 +24,7 @@
 #include "scan.cuh"
 #include "reorder.cuh"
 #include "pack.cuh"
+#include "tail.cuh"
 #include "driver.h"
 
 namespace eclscc {
@@ -138,6 +139,8 @@ void plan_free(Plan* p) {
     cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
     cudaFree(p->pnin); cudaFree(p->pnout); cudaFree(p->ext); cudaFree(p->ext_cnt);
     cudaFree(p->aq_state); cudaFree(p->aq_seen); cudaFree(p->aq_ctr);
+    cudaFree(p->tail_dev);
+    if (p->tail_host) cudaFreeHost(p->tail_host);
     if (p->hc) cudaFreeHost(p->hc);
     if (p->ev_ok)
         for (int k = 0; k < 6; k++) cudaEventDestroy(p->ev[k]);
@@ -191,15 +194,16 @@ static int build_csc(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const i
     CK(cudaMemsetAsync(&p->dc->nchunks, 0, sizeof(int), s));
     p->launches++; k_ingest_chunks<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, 0, ch, &p->dc->nchunks, (int)p->chunk_cap);
     CK(cudaMemsetAsync(p->kin, 0, sizeof(int32_t) * (size_t)(n + 1), s));
-    p->launches++; k_indeg<<<grid_for(nnz, TPB), TPB, 0, s>>>(nnz, ci, p->kin);
+    // per-edge ranks in the second working buffer (free until the first compaction)
+    int32_t* rank = p->oadj[1];
+    p->launches++; k_indeg_rank<<<(unsigned)std::min<int64_t>(grid_for(nnz, TPB), 148 * 8), TPB, 0, s>>>(nnz, ci, p->kin, rank);
     int r = scan_excl<I1>(p, (const I1*)p->kin, n, (I1*)p->iptr[0], (I1*)&p->dc->grand1, p->bsum, 1, s);
     if (r) return r;
-    CK(cudaMemsetAsync(p->kout, 0, sizeof(int32_t) * (size_t)n, s));
     CK(cudaMemsetAsync(&p->dc->local_e, 0, sizeof(unsigned long long), s));
-    p->launches++; k_csc_scatter<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, ci, p->iptr[0], p->kout, p->iadj[0], &p->dc->local_e);
+    p->launches++; k_csc_scatter<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, ci, p->iptr[0], rank, p->iadj[0], &p->dc->local_e);
     int nout = 0;
     if ((r = read_nchunks(p, s, &nout))) return r;
-    if (nout) { p->launches++; k_csc_scatter_chunks<<<chunk_grid(nout), TPB, 0, s>>>(ch, nout, ci, p->iptr[0], p->kout, p->iadj[0]); }
+    if (nout) { p->launches++; k_csc_scatter_chunks<<<chunk_grid(nout), TPB, 0, s>>>(ch, nout, ci, p->iptr[0], rank, p->iadj[0]); }
     p->launches++; k_ingest_chunks<<<grid_for(n, TPB), TPB, 0, s>>>(n, p->iptr[0], 1, ch, &p->dc->nchunks, (int)p->chunk_cap);
     if ((r = read_nchunks(p, s, &p->nchunks_cur))) return r;
     CK(cudaGetLastError());
@@ -534,6 +538,58 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     return ECL_SCC_OK;
 }
 
+// Device-resident tail (tail.cuh): every remaining outer iteration of a small working graph
+// in one cooperative launch.  Threshold: live vertices (env ECL_SCC_TAIL_V).
+static int tail_threshold() {
+    static int v = -1;
+    if (v < 0) v = getenv("ECL_SCC_TAIL_V") ? std::max(0, atoi(getenv("ECL_SCC_TAIL_V"))) : 32768;
+    return v;
+}
+static int run_tail(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int32_t* labels, const Prio& P, int iter,
+                    bool trim, cudaStream_t s, TailTrace** out) {
+    if (!p->tail_dev) {
+        cudaError_t e = cudaMalloc(&p->tail_dev, sizeof(TailTrace));
+        if (e == cudaSuccess) e = cudaMallocHost(&p->tail_host, sizeof(TailTrace));
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(ECL_SCC_ENOMEM, "tail trace allocation: %s", cudaGetErrorString(e));
+        }
+        int per_sm = 0, dev = 0, sms = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_tail<false>, TAIL_TH, 0));
+        CK(cudaGetDevice(&dev));
+        CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+        p->tail_resident = std::max(1, std::min(per_sm, 1) * sms);    // one CTA per SM
+    }
+    TailTrace* T = (TailTrace*)p->tail_dev;
+    CK(cudaMemsetAsync(T, 0, sizeof(TailTrace), s));
+    // one CTA up to 2048 vertices (block barriers, L1-served re-reads), else ~2 vertices per
+    // thread (measured: one CTA on 7.5k vertices took 43 us per pass, 27 CTAs ~9 us)
+    int G = g.na <= 2048 ? 1 : (int)std::min<int64_t>(p->tail_resident, cdiv(g.na, 2 * TAIL_TH));
+    G = std::max(G, 1);
+    int32_t na = g.na;
+    const int32_t* act = g.act;
+    const int32_t* optr = g.optr;
+    int32_t* oadj = (int32_t*)g.oadj;
+    const int32_t* iptr = g.iptr;
+    int32_t* iadj = (int32_t*)g.iadj;
+    int32_t* kin = p->kin;
+    int32_t* kout = p->kout;
+    int32_t* alive = p->newidx;
+    const int32_t* orig = p->orig_cur;
+    int first = iter, tr = trim ? 1 : 0;
+    DevCounters* dc = p->dc;
+    void* args[] = {&na, &act, &optr, &oadj, &iptr, &iadj, &cin, &cout, &kin, &kout, &alive, &labels,
+                    (void*)&P, &orig, &first, &tr, &T, &dc};
+    p->launches++;
+    if (G == 1) CK(cudaLaunchCooperativeKernel((const void*)k_tail<true>, dim3(1), dim3(TAIL_TH), args, 0, s));
+    else CK(cudaLaunchCooperativeKernel((const void*)k_tail<false>, dim3(G), dim3(TAIL_TH), args, 0, s));
+    CK(cudaMemcpyAsync(p->tail_host, T, sizeof(TailTrace), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    *out = (TailTrace*)p->tail_host;
+    if ((*out)->err) return fail(ECL_SCC_ECUDA, "internal: tail did not terminate");
+    return ECL_SCC_OK;
+}
+
 // stage timing: events 2k/2k+1 bracket stage k (0 ingest, 1 compaction, 2 Phase 2)
 static void stage_mark(Plan* p, int ev, cudaStream_t s) {
     if (!(p->flags & ECL_SCC_TIME_STAGES)) return;
@@ -612,7 +668,9 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             CK(cudaStreamSynchronize(s));
             if (st) {
                 if (iter == 1) st->ms_ingest += stage_ms(p, 0);
-                st->ms_compact += stage_ms(p, 1);
+                const double mc = stage_ms(p, 1);
+                st->ms_compact += mc;
+                if (iter - 1 < ECL_SCC_TRACE_MAX) st->ms_compact_iter[iter - 1] = mc;
             }
             const int4 t = p->hc->totals;
             const int nchunks = p->hc->nchunks;
@@ -624,6 +682,36 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             cin = p->cin[ob];
             cout = p->cout[ob];
             if (t.y == 0) break;                                   // no live edge: done
+            // (the Phase-2 ablation flags keep their own Phase 2 to the end)
+            const uint32_t no_tail = ECL_SCC_SYNC_PASSES | ECL_SCC_NO_DIRTY | ECL_SCC_STAGED | ECL_SCC_SWEEP |
+                                     ECL_SCC_NO_PACK | ECL_SCC_NO_ASYNC;
+            if ((p->flags & ECL_SCC_TAIL) && !(p->flags & no_tail) && nchunks == 0 && stop_iter == 0 &&
+                t.x <= tail_threshold()) {
+                // the rest of the outer loop on the device (tail.cuh)
+                stage_mark(p, 4, s);
+                TailTrace* T = nullptr;
+                r = run_tail(p, g, p->cin[ob], p->cout[ob], labels, P, iter, trim, s, &T);
+                if (r) return r;
+                stage_mark(p, 5, s);
+                if (st && (p->flags & ECL_SCC_TIME_STAGES)) {
+                    CK(cudaEventSynchronize(p->ev[5]));
+                    const double mp = stage_ms(p, 2);
+                    st->ms_prop += mp;
+                    if (iter - 1 < ECL_SCC_TRACE_MAX) st->ms_prop_iter[iter - 1] = mp;
+                }
+                iters = T->last_iter;
+                if (st) {
+                    for (int k = iter; k <= T->last_iter; k++) {
+                        if (k - 1 >= ECL_SCC_TRACE_MAX) break;
+                        st->edges_in[k - 1] = k == iter ? t.y : T->edges_in[k - 1];
+                        st->vertices_in[k - 1] = k == iter ? t.x : T->vertices_in[k - 1];
+                        st->passes_iter[k - 1] = T->passes[k - 1];
+                        st->passes += T->passes[k - 1];
+                        if (k >= 2 && k > iter) st->edges_kept[k - 2] = T->edges_kept[k - 2];
+                    }
+                }
+                break;
+            }
             int64_t passes = 0;
             stage_mark(p, 4, s);
             r = propagate(p, g, p->cin[ob], p->cout[ob], nchunks, n, s, &passes);
@@ -631,7 +719,9 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             stage_mark(p, 5, s);
             if (st && (p->flags & ECL_SCC_TIME_STAGES)) {
                 CK(cudaEventSynchronize(p->ev[5]));
-                st->ms_prop += stage_ms(p, 2);
+                const double mp = stage_ms(p, 2);
+                st->ms_prop += mp;
+                if (iter - 1 < ECL_SCC_TRACE_MAX) st->ms_prop_iter[iter - 1] = mp;
             }
             iters = iter;
             if (st) {

@@ -53,6 +53,9 @@ struct Plan {
     uint8_t* aq_seen;
     unsigned long long* aq_ctr;
     int64_t aq_resident;                 // resident CTAs of k_prop_async
+    void* tail_dev;                      // tail.cuh TailTrace (device) and its pinned mirror
+    void* tail_host;
+    int tail_resident;                   // co-resident CTAs of k_tail
     int64_t launches;                    // kernels launched by the current call
     cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
     bool ev_ok;

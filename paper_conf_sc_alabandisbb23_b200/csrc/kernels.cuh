@@ -54,27 +54,51 @@ static __global__ void k_validate(int32_t n, int64_t nnz, const int32_t* __restr
 }
 
 // ------------------------------------------------------------------ a1: CSR -> CSC
-static __global__ void k_indeg(int64_t nnz, const int32_t* __restrict__ ci, int32_t* __restrict__ ideg) {
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x)
-        atomicAdd(&ideg[ci[e]], 1);
+// in-degree histogram and, per edge, its rank among the in-edges of its destination:
+// edge-parallel returning atomics (no per-row serial chain), four independent per thread
+static __global__ void __launch_bounds__(256) k_indeg_rank(int64_t nnz, const int32_t* __restrict__ ci,
+                                                           int32_t* __restrict__ ideg, int32_t* __restrict__ rank) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t e0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e0 < nnz; e0 += 4 * stride) {
+        int w[4], r[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) w[q] = e0 + q * stride < nnz ? __ldg(ci + e0 + q * stride) : -1;
+#pragma unroll
+        for (int q = 0; q < 4; q++) r[q] = w[q] >= 0 ? atomicAdd(&ideg[w[q]], 1) : 0;
+#pragma unroll
+        for (int q = 0; q < 4; q++)
+            if (w[q] >= 0) rank[e0 + q * stride] = r[q];
+    }
 }
 
-// one thread per source row; rows longer than HEAVY are spread over the warp
-static __global__ void k_csc_scatter(int32_t n, const int32_t* __restrict__ rp, const int32_t* __restrict__ ci,
-                              const int32_t* __restrict__ iptr, int32_t* __restrict__ cursor,
+// one thread per source row: edge k = u -> w lands at iadj[iptr[w] + rank[k]]; rows longer
+// than HEAVY are spread over the warp, rows longer than HEAVY_T go to k_csc_scatter_chunks
+static __global__ void __launch_bounds__(256) k_csc_scatter(int32_t n, const int32_t* __restrict__ rp, const int32_t* __restrict__ ci,
+                              const int32_t* __restrict__ iptr, const int32_t* __restrict__ rank,
                               int32_t* __restrict__ iadj, unsigned long long* __restrict__ local_e) {
     const int lane = threadIdx.x & 31;
     const int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const bool valid = u < n;
     int b = 0, e = 0;
-    if (valid) { b = rp[u]; e = rp[u + 1]; }
+    if (valid) { b = __ldg(rp + u); e = __ldg(rp + u + 1); }
     if (e - b > HEAVY_T) e = b;                          // long row: k_csc_scatter_chunks
     unsigned nloc = 0;                                   // storage locality of the numbering
     if (valid && e - b <= HEAVY)
-        for (int k = b; k < e; k++) {
-            const int w = ci[k];
-            nloc += ((w ^ (int)u) >> 11) == 0;
-            iadj[iptr[w] + atomicAdd(&cursor[w], 1)] = (int32_t)u;
+        for (int k = b; k < e; k += 4) {                 // loads of a batch issued before use
+            int w[4], r[4], o[4];
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                w[q] = k + q < e ? __ldg(ci + k + q) : 0;
+                r[q] = k + q < e ? __ldg(rank + k + q) : 0;
+            }
+#pragma unroll
+            for (int q = 0; q < 4; q++) o[q] = __ldg(iptr + w[q]);
+#pragma unroll
+            for (int q = 0; q < 4; q++)
+                if (k + q < e) {
+                    nloc += ((w[q] ^ (int)u) >> 11) == 0;
+                    iadj[o[q] + r[q]] = (int32_t)u;
+                }
         }
     nloc = __reduce_add_sync(FULL, nloc);
     if (lane == 0 && nloc) atomicAdd(local_e, (unsigned long long)nloc);
@@ -84,10 +108,7 @@ static __global__ void k_csc_scatter(int32_t n, const int32_t* __restrict__ rp, 
         hm &= hm - 1;
         const int sb = __shfl_sync(FULL, b, src), se = __shfl_sync(FULL, e, src);
         const int su = __shfl_sync(FULL, (int)u, src);
-        for (int k = sb + lane; k < se; k += WARP) {
-            const int w = ci[k];
-            iadj[iptr[w] + atomicAdd(&cursor[w], 1)] = su;
-        }
+        for (int k = sb + lane; k < se; k += WARP) iadj[__ldg(iptr + __ldg(ci + k)) + __ldg(rank + k)] = su;
     }
 }
 
@@ -538,16 +559,13 @@ static __global__ void k_ingest_chunks(int32_t n, const int32_t* __restrict__ pt
 // CSC scatter of long CSR rows (input graph)
 static __global__ void __launch_bounds__(256) k_csc_scatter_chunks(const Chunk* __restrict__ chunks, int nchunks,
                                                                    const int32_t* __restrict__ ci, const int32_t* __restrict__ iptr,
-                                                                   int32_t* __restrict__ cursor, int32_t* __restrict__ iadj) {
+                                                                   const int32_t* __restrict__ rank, int32_t* __restrict__ iadj) {
     const int lane = threadIdx.x & 31;
     const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (c >= nchunks) return;
     const Chunk k = chunks[c];
     if (k.dir) return;
-    for (int e = k.beg + lane; e < k.end; e += WARP) {
-        const int w = ci[e];
-        iadj[iptr[w] + atomicAdd(&cursor[w], 1)] = k.i;
-    }
+    for (int e = k.beg + lane; e < k.end; e += WARP) iadj[__ldg(iptr + __ldg(ci + e)) + __ldg(rank + e)] = k.i;
 }
 
 // ------------------------------------------------------------------ Phase 2

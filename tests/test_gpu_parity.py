@@ -94,11 +94,13 @@ def test_random_small_graphs_labels_and_traces():
         edges = [(rng.randrange(n), rng.randrange(n)) for _ in range(m)]
         g = gen.from_edges(n, edges)
         truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-        for flags in (0, E.NO_TRIM, E.IDENTITY_IDS, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER, E.NO_PACK, E.NO_ASYNC):
+        for flags in (0, E.TAIL, E.NO_TRIM, E.NO_TRIM | E.TAIL, E.IDENTITY_IDS, E.IDENTITY_IDS | E.TAIL,
+                      E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER, E.NO_PACK, E.NO_ASYNC):
             lab, _ = gpu_labels(g, flags)
             np.testing.assert_array_equal(lab, truth, err_msg=f"trial {trial} flags {flags}")
         if trial % 10 == 0:
             check_trace(g, trim=True)
+            check_trace(g, trim=True, flags=E.TAIL)
             check_trace(g, trim=False)
             check_trace(g, trim=True, flags=E.IDENTITY_IDS)
             check_trace(g, trim=True, flags=E.FORCE_REORDER)
@@ -107,10 +109,13 @@ def test_random_small_graphs_labels_and_traces():
 def test_c1_gnm_2000_8000():
     g = gen.config("c1")
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-    for flags in (0, E.IDENTITY_IDS, E.NO_TRIM, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER, E.NO_PACK, E.NO_ASYNC):
+    for flags in (0, E.TAIL, E.IDENTITY_IDS, E.NO_TRIM, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER,
+                  E.NO_PACK, E.NO_ASYNC):
         lab, _ = gpu_labels(g, flags)
         np.testing.assert_array_equal(lab, truth)
     check_trace(g, trim=True)
+    check_trace(g, trim=True, flags=E.TAIL)
+    check_trace(g, trim=False, flags=E.TAIL)
     check_trace(g, trim=False)
     check_trace(g, trim=True, flags=E.IDENTITY_IDS)
 
@@ -136,6 +141,13 @@ def test_edge_cases():
     # long path (deep DAG): identity
     g = gen.from_edges(n, np.stack([perm[:-1], perm[1:]], 1))
     np.testing.assert_array_equal(gpu_labels(g)[0], np.arange(n))
+    # the same two inside the device-resident tail (tail.cuh): one CTA and a multi-CTA grid
+    for nn in (1500, 30000):
+        pp = np.random.default_rng(nn).permutation(nn)
+        g = gen.from_edges(nn, np.stack([pp, np.roll(pp, -1)], 1))
+        assert (gpu_labels(g, E.TAIL)[0] == nn - 1).all()
+        g = gen.from_edges(nn, np.stack([pp[:-1], pp[1:]], 1))
+        np.testing.assert_array_equal(gpu_labels(g, E.TAIL)[0], np.arange(nn))
     # disjoint k-cycles on consecutive IDs
     k = 5
     e = [(b * k + i, b * k + (i + 1) % k) for b in range(1000) for i in range(k)]
@@ -193,11 +205,13 @@ def test_plan_reuse_and_stream():
 def test_c2_mesh_1m(order):
     g = gen.config("c2", order=order)
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-    lab, st = gpu_labels(g)
-    np.testing.assert_array_equal(lab, truth)
     pi = prio(g.n)
     tr = oracle.ecl_scc(*(lambda h: (h.row_ptr, h.col_idx))(relabel(g, pi)), trim=True)
-    assert st["edges_in"] == tr.edges_in[:64] and st["iterations"] == tr.iterations
+    for fl in (0, E.TAIL):
+        lab, st = gpu_labels(g, fl)
+        np.testing.assert_array_equal(lab, truth)
+        assert st["edges_in"] == tr.edges_in[:64] and st["iterations"] == tr.iterations
+        assert st["edges_kept"] == tr.edges_kept[:st["iterations"] - 1]
     lab, st = gpu_labels(g, E.IDENTITY_IDS)
     np.testing.assert_array_equal(lab, truth)
     tr = oracle.ecl_scc(g.row_ptr, g.col_idx, trim=True)

@@ -54,8 +54,11 @@ static __global__ void k_validate(int32_t n, int64_t nnz, const int32_t* __restr
 }
 
 // ------------------------------------------------------------------ a1: CSR -> CSC
-// in-degree histogram and, per edge, its rank among the in-edges of its destination:
-// edge-parallel returning atomics (no per-row serial chain), four independent per thread
+// in-degree histogram and (RANK) per edge its rank among the in-edges of its destination:
+// edge-parallel returning atomics (no per-row serial chain), four independent per thread.
+// Without RANK (power-law inputs: returning atomics on hub destinations serialise) the
+// histogram uses fire-and-forget reductions and the scatter takes cursor atomics.
+template <bool RANK>
 static __global__ void __launch_bounds__(256) k_indeg_rank(int64_t nnz, const int32_t* __restrict__ ci,
                                                            int32_t* __restrict__ ideg, int32_t* __restrict__ rank) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -64,17 +67,27 @@ static __global__ void __launch_bounds__(256) k_indeg_rank(int64_t nnz, const in
 #pragma unroll
         for (int q = 0; q < 4; q++) w[q] = e0 + q * stride < nnz ? __ldg(ci + e0 + q * stride) : -1;
 #pragma unroll
-        for (int q = 0; q < 4; q++) r[q] = w[q] >= 0 ? atomicAdd(&ideg[w[q]], 1) : 0;
+        for (int q = 0; q < 4; q++) {
+            if (!RANK && w[q] >= 0) atomicAdd(&ideg[w[q]], 1);
+            r[q] = RANK && w[q] >= 0 ? atomicAdd(&ideg[w[q]], 1) : 0;
+        }
+        if (RANK)
 #pragma unroll
-        for (int q = 0; q < 4; q++)
-            if (w[q] >= 0) rank[e0 + q * stride] = r[q];
+            for (int q = 0; q < 4; q++)
+                if (w[q] >= 0) rank[e0 + q * stride] = r[q];
     }
 }
 
-// one thread per source row: edge k = u -> w lands at iadj[iptr[w] + rank[k]]; rows longer
-// than HEAVY are spread over the warp, rows longer than HEAVY_T go to k_csc_scatter_chunks
+// one thread per source row: edge k = u -> w lands at iadj[iptr[w] + rank[k]] (RANK) or at
+// a cursor slot; rows longer than HEAVY are spread over the warp, rows longer than HEAVY_T
+// go to k_csc_scatter_chunks
+template <bool RANK>
+__device__ __forceinline__ int csc_slot(const int32_t* __restrict__ rank, int32_t* cursor, int k, int w) {
+    return RANK ? __ldg(rank + k) : atomicAdd(cursor + w, 1);
+}
+template <bool RANK>
 static __global__ void __launch_bounds__(256) k_csc_scatter(int32_t n, const int32_t* __restrict__ rp, const int32_t* __restrict__ ci,
-                              const int32_t* __restrict__ iptr, const int32_t* __restrict__ rank,
+                              const int32_t* __restrict__ iptr, const int32_t* __restrict__ rank, int32_t* cursor,
                               int32_t* __restrict__ iadj, unsigned long long* __restrict__ local_e) {
     const int lane = threadIdx.x & 31;
     const int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -89,7 +102,7 @@ static __global__ void __launch_bounds__(256) k_csc_scatter(int32_t n, const int
 #pragma unroll
             for (int q = 0; q < 4; q++) {
                 w[q] = k + q < e ? __ldg(ci + k + q) : 0;
-                r[q] = k + q < e ? __ldg(rank + k + q) : 0;
+                r[q] = RANK && k + q < e ? __ldg(rank + k + q) : 0;
             }
 #pragma unroll
             for (int q = 0; q < 4; q++) o[q] = __ldg(iptr + w[q]);
@@ -97,7 +110,7 @@ static __global__ void __launch_bounds__(256) k_csc_scatter(int32_t n, const int
             for (int q = 0; q < 4; q++)
                 if (k + q < e) {
                     nloc += ((w[q] ^ (int)u) >> 11) == 0;
-                    iadj[o[q] + r[q]] = (int32_t)u;
+                    iadj[o[q] + (RANK ? r[q] : atomicAdd(cursor + w[q], 1))] = (int32_t)u;
                 }
         }
     nloc = __reduce_add_sync(FULL, nloc);
@@ -108,7 +121,10 @@ static __global__ void __launch_bounds__(256) k_csc_scatter(int32_t n, const int
         hm &= hm - 1;
         const int sb = __shfl_sync(FULL, b, src), se = __shfl_sync(FULL, e, src);
         const int su = __shfl_sync(FULL, (int)u, src);
-        for (int k = sb + lane; k < se; k += WARP) iadj[__ldg(iptr + __ldg(ci + k)) + __ldg(rank + k)] = su;
+        for (int k = sb + lane; k < se; k += WARP) {
+            const int w = __ldg(ci + k);
+            iadj[__ldg(iptr + w) + csc_slot<RANK>(rank, cursor, k, w)] = su;
+        }
     }
 }
 
@@ -198,14 +214,14 @@ struct SurvivePred {
     }
 };
 
-// Light rows (<= HEAVY edges) of both directions of one vertex, in batches of 4 edges per
-// direction: the adjacency loads of a batch, then all the predicate gathers, are issued
-// before any result is used (memory-level parallelism; a thread used to walk its rows one
-// dependent load after another).  Invalid slots evaluate the predicate on `self`.
+// Light rows as bit masks (bit k = entry k of the row satisfies the predicate).  Phase 3
+// evaluates keep() once, in k_keep_count; k_compact_count then gathers only the trim
+// degrees of the kept entries and k_compact_scatter only the new indices of the
+// survivors (the predicates used to be re-evaluated, with their gathers, in all three).
 template <typename P>
-__device__ __forceinline__ void count_light2(const int32_t* __restrict__ oadj, int ob, int no,
-                                             const int32_t* __restrict__ iadj, int ib, int ni, int self, P pred,
-                                             int& co, int& ci) {
+__device__ __forceinline__ void mask_light2(const int32_t* __restrict__ oadj, int ob, int no,
+                                            const int32_t* __restrict__ iadj, int ib, int ni, int self, P pred,
+                                            unsigned& mo, unsigned& mi) {
     for (int k = 0; k < no || k < ni; k += 4) {
         int xo[4], xi[4];
 #pragma unroll
@@ -215,36 +231,45 @@ __device__ __forceinline__ void count_light2(const int32_t* __restrict__ oadj, i
         }
 #pragma unroll
         for (int q = 0; q < 4; q++) {
-            co += (int)pred(xo[q]) & (int)(k + q < no);
-            ci += (int)pred(xi[q]) & (int)(k + q < ni);
+            mo |= (unsigned)((int)pred(xo[q]) & (int)(k + q < no)) << (k + q);
+            mi |= (unsigned)((int)pred(xi[q]) & (int)(k + q < ni)) << (k + q);
         }
     }
 }
-template <typename P>
-__device__ __forceinline__ void emit_light2(const int32_t* __restrict__ oadj, int ob, int no, int po,
-                                            int32_t* __restrict__ odst, const int32_t* __restrict__ iadj, int ib,
-                                            int ni, int pi, int32_t* __restrict__ idst, int self,
-                                            const int32_t* __restrict__ newidx, P pred) {
-    for (int k = 0; k < no || k < ni; k += 4) {
-        int xo[4], xi[4], yo[4], yi[4];
-        bool so[4], si[4];
+// keep the set bits of m whose entry's far end is not trimmed (batches of 4 entries)
+__device__ __forceinline__ unsigned trim_mask(const int32_t* __restrict__ adj, int b, unsigned m, int self,
+                                              const int32_t* __restrict__ kin, const int32_t* __restrict__ kout) {
+    unsigned out = 0;
+    while (m) {
+        int k[4], x[4];
 #pragma unroll
         for (int q = 0; q < 4; q++) {
-            xo[q] = k + q < no ? __ldg(oadj + ob + k + q) : self;
-            xi[q] = k + q < ni ? __ldg(iadj + ib + k + q) : self;
+            k[q] = m ? __ffs(m) - 1 : -1;
+            m &= m - 1;
         }
 #pragma unroll
-        for (int q = 0; q < 4; q++) {
-            so[q] = pred(xo[q]) & (k + q < no);
-            si[q] = pred(xi[q]) & (k + q < ni);
-            yo[q] = __ldg(newidx + xo[q]);
-            yi[q] = __ldg(newidx + xi[q]);
-        }
+        for (int q = 0; q < 4; q++) x[q] = k[q] >= 0 ? __ldg(adj + b + k[q]) : self;
+#pragma unroll
+        for (int q = 0; q < 4; q++)
+            if (k[q] >= 0 && !trimmed(kin, kout, x[q])) out |= 1u << k[q];
+    }
+    return out;
+}
+// write the entries of m (in row order) as new local indices from dst[pos]
+__device__ __forceinline__ void emit_mask(const int32_t* __restrict__ adj, int b, unsigned m, int self,
+                                          const int32_t* __restrict__ newidx, int32_t* __restrict__ dst, int pos) {
+    while (m) {
+        int k[4], y[4];
 #pragma unroll
         for (int q = 0; q < 4; q++) {
-            if (so[q]) odst[po++] = yo[q];
-            if (si[q]) idst[pi++] = yi[q];
+            k[q] = m ? __ffs(m) - 1 : -1;
+            m &= m - 1;
         }
+#pragma unroll
+        for (int q = 0; q < 4; q++) y[q] = __ldg(newidx + (k[q] >= 0 ? __ldg(adj + b + k[q]) : self));
+#pragma unroll
+        for (int q = 0; q < 4; q++)
+            if (k[q] >= 0) dst[pos++] = y[q];
     }
 }
 
@@ -253,19 +278,22 @@ constexpr int TPB_COMPACT = 256;     // block size of the compaction kernels (dr
 template <bool FIRST>
 static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                              int32_t* __restrict__ kin, int32_t* __restrict__ kout,
-                             unsigned long long* __restrict__ kept, int chunked, int2* __restrict__ hcnt) {
+                             unsigned long long* __restrict__ kept, int chunked, int2* __restrict__ hcnt,
+                             uint2* __restrict__ emask) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
     KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout};
-    int co = 0, ci = 0;
-    count_light2(g.oadj, r.ob, r.live && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, g.iadj, r.ib,
-                 r.live && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, (int)(r.valid ? i : 0), pred, co, ci);
+    unsigned mo = 0, mi = 0;
+    mask_light2(g.oadj, r.ob, r.live && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, g.iadj, r.ib,
+                r.live && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, (int)(r.valid ? i : 0), pred, mo, mi);
+    int co = __popc(mo), ci = __popc(mi);
     co += count_row(g.oadj, r.ob, r.oe, r.live, lane, pred, chunked, false);
     ci += count_row(g.iadj, r.ib, r.ie, r.live, lane, pred, chunked, false);
     if (r.valid) {
         kin[i] = ci;
         kout[i] = co;
+        emask[i] = make_uint2(mo, mi);
         if (chunked) hcnt[i] = make_int2(0, 0);
     }
     // one atomic per block (one per warp on a single address serialised ~0.5M atomics in L2)
@@ -285,18 +313,24 @@ template <bool FIRST, bool TRIM>
 static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                 const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
                                 int2* __restrict__ cnt, int4* __restrict__ wsum, int chunked,
-                                const int2* __restrict__ hcnt) {
+                                const int2* __restrict__ hcnt, uint2* __restrict__ emask) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
     int nout = 0, nin = 0;
     if (!TRIM) {
-        if (r.live) { nout = kout[i]; nin = kin[i]; }
+        if (r.live) { nout = kout[i]; nin = kin[i]; }   // survivors = kept: the masks stand
     } else {
         const bool go = r.live && !trimmed(kin, kout, (int)i);
         SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
-        count_light2(g.oadj, r.ob, go && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, g.iadj, r.ib,
-                     go && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, (int)(r.valid ? i : 0), pred, nout, nin);
+        if (r.valid) {                                   // light rows: the kept entries' far ends
+            const uint2 km = emask[i];
+            const unsigned so = go && r.oe - r.ob <= HEAVY ? trim_mask(g.oadj, r.ob, km.x, (int)i, kin, kout) : 0u;
+            const unsigned si = go && r.ie - r.ib <= HEAVY ? trim_mask(g.iadj, r.ib, km.y, (int)i, kin, kout) : 0u;
+            emask[i] = make_uint2(so, si);
+            nout = __popc(so);
+            nin = __popc(si);
+        }
         nout += count_row(g.oadj, r.ob, r.oe, go, lane, pred, chunked, false);
         nin += count_row(g.iadj, r.ib, r.ie, go, lane, pred, chunked, false);
         if (chunked && r.valid) {                       // long rows: counted by k_count_chunks
@@ -449,17 +483,21 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
                                   const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
                                   const int32_t* __restrict__ newidx, const int32_t* __restrict__ optr2,
                                   const int32_t* __restrict__ iptr2, int32_t* __restrict__ oadj2,
-                                  int32_t* __restrict__ iadj2, int chunked) {
+                                  int32_t* __restrict__ iadj2, int chunked, const uint2* __restrict__ emask) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
     const int j = r.valid ? newidx[i] : -1;
     const bool go = j >= 0;
     int po = 0, pi = 0;
-    if (go) { po = optr2[j]; pi = iptr2[j]; }
+    if (go) {
+        po = optr2[j];
+        pi = iptr2[j];
+        const uint2 sm = emask[i];                     // light rows: the survivors' bits
+        if (r.oe - r.ob <= HEAVY) emit_mask(g.oadj, r.ob, sm.x, (int)i, newidx, oadj2, po);
+        if (r.ie - r.ib <= HEAVY) emit_mask(g.iadj, r.ib, sm.y, (int)i, newidx, iadj2, pi);
+    }
     SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
-    emit_light2(g.oadj, r.ob, go && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, po, oadj2, g.iadj, r.ib,
-                go && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, pi, iadj2, (int)(r.valid ? i : 0), newidx, pred);
     emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred, chunked, false);
     emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred, chunked, false);
 }
@@ -557,15 +595,20 @@ static __global__ void k_ingest_chunks(int32_t n, const int32_t* __restrict__ pt
         chunks[at + k] = Chunk{(int32_t)v, dir, beg + k * CHUNK, min(beg + (k + 1) * CHUNK, beg + deg), at};
 }
 // CSC scatter of long CSR rows (input graph)
+template <bool RANK>
 static __global__ void __launch_bounds__(256) k_csc_scatter_chunks(const Chunk* __restrict__ chunks, int nchunks,
                                                                    const int32_t* __restrict__ ci, const int32_t* __restrict__ iptr,
-                                                                   const int32_t* __restrict__ rank, int32_t* __restrict__ iadj) {
+                                                                   const int32_t* __restrict__ rank, int32_t* cursor,
+                                                                   int32_t* __restrict__ iadj) {
     const int lane = threadIdx.x & 31;
     const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (c >= nchunks) return;
     const Chunk k = chunks[c];
     if (k.dir) return;
-    for (int e = k.beg + lane; e < k.end; e += WARP) iadj[__ldg(iptr + __ldg(ci + e)) + __ldg(rank + e)] = k.i;
+    for (int e = k.beg + lane; e < k.end; e += WARP) {
+        const int w = __ldg(ci + e);
+        iadj[__ldg(iptr + w) + csc_slot<RANK>(rank, cursor, e, w)] = k.i;
+    }
 }
 
 // ------------------------------------------------------------------ Phase 2

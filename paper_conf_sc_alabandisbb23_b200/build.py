@@ -32,7 +32,7 @@ def deps() -> list[str]:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
-    if os.environ.get("ECL_PROF") == "1":
+    if os.environ.get("ECL_PROF") == "1" or os.environ.get("ECL_NVCC_EXTRA"):
         force = True
     if not force and os.path.exists(LIB):
         t = os.path.getmtime(LIB)
@@ -41,6 +41,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     inc, lib = nccl_dirs()
     tmp = LIB + f".tmp{os.getpid()}"
     extra = ["-DECL_PROF"] if os.environ.get("ECL_PROF") == "1" else []
+    extra += os.environ.get("ECL_NVCC_EXTRA", "").split()       # development: variant -D flags
     cmd = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", *extra, "-Xcompiler", "-fPIC", "-shared",
            "-I", os.path.join(ROOT, "include"), "-I", inc, "-o", tmp, *sources(),
            "-L", lib, "-l:libnccl.so.2", f"-Xlinker", f"-rpath={lib}"]

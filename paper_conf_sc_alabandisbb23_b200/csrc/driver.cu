@@ -441,6 +441,8 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                 return fail(ECL_SCC_ENOMEM, "tile pack allocation: %s", cudaGetErrorString(e));
             }
             CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
+            CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                    (int)cudaSharedmemCarveoutMaxShared));
         }
         p->launches++;
         k_tile_pack<<<ntiles, PACK_TH, 0, s>>>(g, p->pnin, p->pnout, p->ext, p->ext_cnt);
@@ -456,11 +458,14 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                     return fail(ECL_SCC_ENOMEM, "async queue allocation: %s", cudaGetErrorString(e));
                 }
                 CK(cudaFuncSetAttribute(k_prop_async, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
+                CK(cudaFuncSetAttribute(k_prop_async, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                        (int)cudaSharedmemCarveoutMaxShared));
                 int per_sm = 0, dev = 0, sms = 0;
                 CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_async, PACK_TH, pack_dyn_smem()));
                 CK(cudaGetDevice(&dev));
                 CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
                 p->aq_resident = std::max(1, per_sm) * sms;
+                if (getenv("ECL_SCC_DEBUG")) fprintf(stderr, "[ecl_scc] k_prop_async: %d CTAs per SM\n", per_sm);
             }
             AsyncQ Q{p->aq_state, p->aq_seen, p->aq_ctr};
             // tiles per claim: runs pay when there are many tiles per resident CTA (measured:

@@ -24,6 +24,9 @@ namespace eclscc {
 
 constexpr int PACK_TT = TILE;                 // 2048 vertices per tile
 constexpr int PACK_TH = TILE_THREADS;         // 512 threads, 4 vertices each
+#ifndef PACK_MINB
+#define PACK_MINB 3                           // resident CTAs per SM the kernels are built for
+#endif
 constexpr unsigned EXT_DIR = 0x8000u;
 // Pack slot encoding: four 16-bit local indices per word; an empty slot holds PACK_TT, the
 // index of a sentinel entry (value 0 <= every priority, scratch flag byte), so pulls and
@@ -119,6 +122,72 @@ __device__ __forceinline__ void drain_pack(const WGraph& g, int* __restrict__ s_
                 const unsigned item = s_queue[wq0 + q];
                 const int v = (int)(item >> 1);
                 if (item & 1u) {                                 // v_out from the out-neighbours
+                    const unsigned long long src = s_nout[v];
+                    const int old = ((volatile int*)s_out)[v];
+                    int val = ppull(s_out, src, old);
+                    if (src & SLOW_MARK) val = pull_slow(s_out, g.optr, g.oadj, base, cnt, v, val);
+                    if (val > old) {
+                        ((volatile int*)s_out)[v] = val;
+                        __threadfence_block();
+                        pnotify_full(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
+                        any = 1;
+                    }
+                } else {                                         // v_in from the in-neighbours
+                    const unsigned long long src = s_nin[v];
+                    const int old = ((volatile int*)s_in)[v];
+                    int val = ppull(s_in, src, old);
+                    if (src & SLOW_MARK) val = pull_slow(s_in, g.iptr, g.iadj, base, cnt, v, val);
+                    if (val > old) {
+                        ((volatile int*)s_in)[v] = val;
+                        __threadfence_block();
+                        pnotify_full(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
+                        any = 1;
+                    }
+                }
+            }
+            __syncwarp();
+            if (!__any_sync(FULL, any)) break;
+        }
+        if (!__syncthreads_or(worked)) break;
+    }
+}
+
+// Step 2 without the per-warp queue: every lane pulls its own flagged items directly (at
+// most VPT vertices x 2 directions).  With owner-computes pulls a drain round rarely holds
+// more than one item per lane, so the queue's warp scan and shared-memory round trip cost
+// more than the divergence they avoid.
+__device__ __forceinline__ void drain_direct(const WGraph& g, int* __restrict__ s_in, int* __restrict__ s_out,
+                                             const unsigned long long* __restrict__ s_nin,
+                                             const unsigned long long* __restrict__ s_nout,
+                                             unsigned* __restrict__ s_fin, unsigned* __restrict__ s_fout, int base,
+                                             int cnt, unsigned& prof_rounds, unsigned& prof_drains,
+                                             unsigned& prof_pushes) {
+    const int tid = threadIdx.x;
+    const int v0 = tid * VPT;
+    for (;;) {
+        int worked = 0;
+#ifdef ECL_PROF
+        if (tid == 0) prof_rounds++;
+#endif
+        for (;;) {
+#ifdef ECL_PROF
+            if ((tid & 31) == 0) prof_drains++;
+#endif
+            unsigned wi = ((volatile unsigned*)s_fin)[tid], wo = ((volatile unsigned*)s_fout)[tid];
+            if (wi) wi = atomicExch(s_fin + tid, 0u);
+            if (wo) wo = atomicExch(s_fout + tid, 0u);
+            unsigned items = gather4(wi) | (gather4(wo) << 4);
+            if (!__any_sync(FULL, items != 0)) break;
+            worked = 1;
+#ifdef ECL_PROF
+            prof_pushes += __popc(items);
+#endif
+            int any = 0;
+            while (items) {
+                const int bit = __ffs(items) - 1;
+                items &= items - 1;
+                const int v = v0 + (bit & 3);
+                if (bit & 4) {                                   // v_out from the out-neighbours
                     const unsigned long long src = s_nout[v];
                     const int old = ((volatile int*)s_out)[v];
                     int val = ppull(s_out, src, old);
@@ -301,7 +370,11 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
 #endif
     {
         unsigned r0 = 0, r1 = 0, r2 = 0;
+#ifdef ECL_DRAIN_QUEUE
         drain_pack(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, S.s_queue, base, cnt, r0, r1, r2);
+#else
+        drain_direct(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, base, cnt, r0, r1, r2);
+#endif
 #ifdef ECL_PROF
         r2 = warp_sum(r2);
         if ((tid & 31) == 0) { PROF_ADD(dc, 2, r1); PROF_ADD(dc, 3, r2); }
@@ -368,14 +441,18 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
 }
 
 // Phase-2 pass over the packs (pass protocol, dirty skipping and runs as k_prop_tile)
-static __global__ void __launch_bounds__(PACK_TH, 1536 / PACK_TH)
+static __global__ void __launch_bounds__(PACK_TH, PACK_MINB)
 k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, const unsigned long long* __restrict__ pnin,
             const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext, const int* __restrict__ ext_cnt,
             DevCounters* __restrict__ dc, int pass, int first, uint8_t* __restrict__ dirty_cur,
             uint8_t* __restrict__ dirty_next, int full, int run) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ unsigned s_fin[PACK_TH + 1], s_fout[PACK_TH + 1];      // + the sentinel's scratch byte
+#ifdef ECL_DRAIN_QUEUE
     __shared__ unsigned short s_queue[2 * PACK_TT];
+#else
+    unsigned short* s_queue = nullptr;
+#endif
     __shared__ int s_dirty;
     TileSmem<PACK_TT> S;
     S.s_in = (int*)smem_raw;                                          // [PACK_TT] + sentinel
@@ -473,13 +550,17 @@ struct MarkSet {
     }
 };
 
-static __global__ void __launch_bounds__(PACK_TH, 1536 / PACK_TH)
+static __global__ void __launch_bounds__(PACK_TH, PACK_MINB)
 k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, const unsigned long long* __restrict__ pnin,
              const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext, const int* __restrict__ ext_cnt,
              DevCounters* __restrict__ dc, AsyncQ Q, int claim) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ unsigned s_fin[PACK_TH + 1], s_fout[PACK_TH + 1];
+#ifdef ECL_DRAIN_QUEUE
     __shared__ unsigned short s_queue[2 * PACK_TT];
+#else
+    unsigned short* s_queue = nullptr;
+#endif
     __shared__ int s_set[MSET];
     __shared__ int s_claim[CLAIM_MAX], s_nclaim;
     __shared__ uint8_t s_seen[CLAIM_MAX];

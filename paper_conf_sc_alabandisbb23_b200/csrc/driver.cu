@@ -481,10 +481,9 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             k_prop_async<<<(unsigned)std::min<int64_t>(ntiles, p->aq_resident), PACK_TH, pack_dyn_smem(), s>>>(
                 g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, Q, claim);
             CK(cudaGetLastError());
-            CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
-            CK(cudaStreamSynchronize(s));
-            if (p->hc->err == 3) return fail(ECL_SCC_ECUDA, "internal: asynchronous Phase 2 stalled (watchdog)");
-            *passes_out = (int64_t)cdiv((int64_t)p->hc->passes, ntiles);   // sweep equivalents
+            // no stream synchronisation here: the watchdog word and the visit count are read
+            // with the counters of the next compaction (resolve_prop in run_graph)
+            *passes_out = -(int64_t)ntiles;
             return ECL_SCC_OK;
         }
     }
@@ -607,6 +606,16 @@ static int run_tail(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int32
     return ECL_SCC_OK;
 }
 
+// the deferred check of an asynchronous Phase 2 (propagate() returned -ntiles as its pass
+// count): after a stream synchronisation p->hc holds its watchdog word and visit count
+static int resolve_prop(Plan* p, int64_t* passes) {
+    if (*passes >= 0) return ECL_SCC_OK;
+    const int64_t ntiles = -*passes;
+    if (p->hc->err == 3) return fail(ECL_SCC_ECUDA, "internal: asynchronous Phase 2 stalled (watchdog)");
+    *passes = cdiv((int64_t)p->hc->passes, ntiles);              // sweep equivalents
+    return ECL_SCC_OK;
+}
+
 // stage timing: events 2k/2k+1 bracket stage k (0 ingest, 1 compaction, 2 Phase 2)
 static void stage_mark(Plan* p, int ev, cudaStream_t s) {
     if (!(p->flags & ECL_SCC_TIME_STAGES)) return;
@@ -672,6 +681,18 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         WGraph g{nullptr, rp, ci, p->iptr[0], p->iadj[0], n};
         const int32_t *cin = nullptr, *cout = nullptr;          // identity (l.3-6) in the input
         int ob = 1;
+        int64_t pend_passes = 0;                                 // deferred Phase-2 check
+        int pend_iter = 0;
+        auto resolve = [&]() -> int {
+            if (!pend_iter) return ECL_SCC_OK;
+            if (int e = resolve_prop(p, &pend_passes)) return e;
+            if (st) {
+                if (pend_iter - 1 < ECL_SCC_TRACE_MAX) st->passes_iter[pend_iter - 1] = pend_passes;
+                st->passes += pend_passes;
+            }
+            pend_iter = 0;
+            return ECL_SCC_OK;
+        };
         for (int iter = 1;; iter++) {
             if (iter > n + 2) return fail(ECL_SCC_ECUDA, "internal: outer loop exceeded n+2 iterations");
             stage_mark(p, 2, s);
@@ -683,6 +704,7 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             stage_mark(p, 3, s);
             CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
             CK(cudaStreamSynchronize(s));
+            if ((r = resolve())) return r;
             if (st) {
                 if (iter == 1) st->ms_ingest += stage_ms(p, 0);
                 const double mc = stage_ms(p, 1);
@@ -741,15 +763,23 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
                 if (iter - 1 < ECL_SCC_TRACE_MAX) st->ms_prop_iter[iter - 1] = mp;
             }
             iters = iter;
-            if (st) {
-                if (iter - 1 < ECL_SCC_TRACE_MAX) {
-                    st->edges_in[iter - 1] = t.y;
-                    st->vertices_in[iter - 1] = t.x;
-                    st->passes_iter[iter - 1] = passes;
+            if (st && iter - 1 < ECL_SCC_TRACE_MAX) {
+                st->edges_in[iter - 1] = t.y;
+                st->vertices_in[iter - 1] = t.x;
+            }
+            pend_passes = passes;
+            pend_iter = iter;
+            if (passes >= 0 || (p->flags & ECL_SCC_TIME_STAGES)) {   // already synchronised
+                if ((p->flags & ECL_SCC_TIME_STAGES) && passes < 0) {
+                    CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+                    CK(cudaStreamSynchronize(s));
                 }
-                st->passes += passes;
+                if ((r = resolve())) return r;
             }
             if (stop_iter == iter) {
+                CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+                CK(cudaStreamSynchronize(s));
+                if ((r = resolve())) return r;
                 p->launches++; k_snapshot_left<<<grid_for(n, TPB), TPB, 0, s>>>(n, labels, dbg_in, dbg_out, P);
                 p->launches++; k_scatter_sigs<<<grid_for(t.x, TPB), TPB, 0, s>>>(t.x, g.act, cin, cout, dbg_in, dbg_out, p->orig_cur);
                 CK(cudaGetLastError());

@@ -424,6 +424,7 @@ static __global__ void k_relabel_max(int32_t n, const int32_t* __restrict__ labe
             const int l = labels[v];
             if (l < 0 && (int)prio_of(P, (uint32_t)v) != -l - 1) { key = -l - 1; val = (int)v; }
         }
+        if (!__any_sync(FULL, key >= 0)) continue;           // singletons only (most warps)
         const unsigned grp = __match_any_sync(FULL, key);
         int m = val;
         for (unsigned g = grp; g; g &= g - 1) m = max(m, __shfl_sync(grp, val, __ffs(g) - 1));

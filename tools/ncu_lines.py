@@ -14,6 +14,7 @@ for b in blocks[1:]:
     i_inst = hdr.index("Instructions Executed")
     for r in rd:
         if len(r) <= i_inst: continue
+        if not r[i_line].strip(): continue     # SASS rows of the cuda,sass listing (already in their line)
         try: samp = float(r[i_samp] or 0); inst = float(r[i_inst] or 0)
         except ValueError: continue
         a = agg[(path, r[i_line])]

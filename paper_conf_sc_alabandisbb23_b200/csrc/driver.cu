@@ -58,6 +58,12 @@ static inline unsigned grid_for(int64_t work, int threads) {
 constexpr int TPB = 256;
 static_assert(TPB == TPB_COMPACT, "k_keep_count reduces over TPB_COMPACT threads");
 constexpr double REORDER_LOCALITY = 0.85;   // measured: C4 lex 0.77, blocked8 0.91
+// the reordering's cost is mostly per BFS level (launches, host checks): below this size it
+// does not pay back (measured: C2 lex, 1M vertices, 2.98 ms without vs 3.95 ms with)
+constexpr int32_t REORDER_MIN_N = 1 << 22;
+// a block-local fixed point pays only if tiles hold a real share of the edges (measured:
+// C3, random IDs, ~0 local edges: 8.2 ms with plain Jacobi passes vs 9.3 ms)
+constexpr double LOCAL_FP_LOCALITY = 0.25;
 
 // --------------------------------------------------------------------------- plan
 int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
@@ -416,7 +422,8 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                      int64_t* passes_out) {
     const unsigned ntiles = (unsigned)cdiv(g.na, p->tile);
     const unsigned hgrid = (unsigned)std::min<int64_t>(cdiv(std::max(nchunks, 1), TPB / WARP), 148 * 8);
-    const bool sync = (p->flags & ECL_SCC_SYNC_PASSES) != 0;
+    // plain Jacobi passes: the ablation flag, or graphs whose tiles hold almost no edges
+    const bool sync = (p->flags & ECL_SCC_SYNC_PASSES) != 0 || (p->low_locality && nchunks > 0);
     // dirty-tile skipping needs every raise to be seen by the tile kernel (no heavy rows)
     // and a local fixed point per visit (not the SYNC ablation)
     const bool use_dirty = nchunks == 0 && !sync && !(p->flags & ECL_SCC_NO_DIRTY);
@@ -663,13 +670,14 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         // fewer than REORDER_LOCALITY of the edges inside 2048-ID ranges; results do not
         // depend on it, only the number of Phase-2 passes does
         bool reorder = false;
+        unsigned long long loc = 0;                     // edges inside 2048-ID ranges
+        CK(cudaMemcpyAsync(&loc, &p->dc->local_e, sizeof(loc), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        p->low_locality = (double)loc < LOCAL_FP_LOCALITY * (double)nnz;
         if ((p->flags & ECL_SCC_FORCE_REORDER) && p->nchunks_cur == 0) reorder = true;
-        else if (!(p->flags & ECL_SCC_NO_REORDER) && p->nchunks_cur == 0 && n >= 8 * TILE) {
-            unsigned long long loc = 0;
-            CK(cudaMemcpyAsync(&loc, &p->dc->local_e, sizeof(loc), cudaMemcpyDeviceToHost, s));
-            CK(cudaStreamSynchronize(s));
+        else if (!(p->flags & ECL_SCC_NO_REORDER) && p->nchunks_cur == 0 && n >= REORDER_MIN_N)
             reorder = (double)loc < REORDER_LOCALITY * (double)nnz;
-        }
+        if (reorder) p->low_locality = false;
         if (reorder) {
             if ((r = reorder_graph(p, n, nnz, rp, ci, s))) return r;
             rp = p->rp2;

@@ -60,6 +60,7 @@ struct Plan {
     int64_t launches;                    // kernels launched by the current call
     cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
     bool ev_ok;
+    bool low_locality;                   // fewer than 25% of the input edges inside 2048-ID ranges
 };
 
 int fail(int status, const char* fmt, ...);

@@ -168,6 +168,16 @@ def test_heavy_vertices():
     for flags in (0, E.NO_TRIM, E.IDENTITY_IDS):
         np.testing.assert_array_equal(gpu_labels(g, flags)[0], truth)
     check_trace(g, trim=True, max_iters=3)
+    # hubs in a graph whose edges all lie inside one 2048-ID range: the pass kernels keep
+    # their block-local fixed point (high locality), the long rows go through k_prop_heavy
+    n = 2000
+    src = np.concatenate([np.full(900, 7), rng.integers(0, n, 900), rng.integers(0, n, 3000)])
+    dst = np.concatenate([rng.integers(0, n, 900), np.full(900, 1999), rng.integers(0, n, 3000)])
+    g = gen.from_edges(n, np.stack([src, dst], 1))
+    truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+    for flags in (0, E.NO_TRIM, E.IDENTITY_IDS):
+        np.testing.assert_array_equal(gpu_labels(g, flags)[0], truth)
+    check_trace(g, trim=True)
 
 
 def test_invalid_input_reports_erange():

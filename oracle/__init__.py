@@ -12,6 +12,9 @@ Functions (each cites the passage it follows; P:n = /root/reference/PAPER.md lin
 * ``ecl_scc(row_ptr, col_idx, reset_all=False, compress=False, trim=False, snap_iter=0)``
   -- O2: Alg. 1 in the paper's order with Jacobi Phase-2 rounds and the
   per-iteration trace.  Flags follow the readings in DESIGN.md.
+* ``scc_levels(row_ptr, col_idx, labels)`` -- O4: the sweep levels of the SCC condensation
+  (Table 2's "DAG depth"): Kahn's algorithm on the condensation, level = longest path
+  from a source SCC.  Returns (levels per vertex, depth).
 
 Both live in ``oracle.c`` and run single-threaded.  Pins: tests/test_oracle.py.
 """
@@ -56,6 +59,8 @@ def _load():
         lib.oracle_ecl_scc.argtypes = [ctypes.c_int32, i64p, i32p, ctypes.c_uint32, i32p,
                                        ctypes.c_int32, i64p, i64p, i64p,
                                        ctypes.c_int32, i32p, i32p]
+        lib.oracle_scc_levels.restype = ctypes.c_int32
+        lib.oracle_scc_levels.argtypes = [ctypes.c_int32, i64p, i32p, i32p, i32p]
         _lib = lib
     return _lib
 
@@ -86,6 +91,22 @@ def tarjan_labels(row_ptr, col_idx) -> np.ndarray:
     if r < 0:
         raise MemoryError("oracle_tarjan_labels")
     return labels
+
+
+def scc_levels(row_ptr, col_idx, labels) -> tuple[np.ndarray, int]:
+    """O4: (level of each vertex's SCC in the condensation DAG, depth = max level + 1)."""
+    n, rp, ci = _csr(row_ptr, col_idx)
+    lab = np.ascontiguousarray(labels, dtype=np.int32)
+    levels = np.empty(n, dtype=np.int32)
+    if n == 0:
+        return levels, 0
+    d = _load().oracle_scc_levels(n, _p(rp, ctypes.c_int64), _p(ci, ctypes.c_int32),
+                                  _p(lab, ctypes.c_int32), _p(levels, ctypes.c_int32))
+    if d == -1:
+        raise MemoryError("oracle_scc_levels")
+    if d == -2:
+        raise ValueError("labels do not induce an acyclic condensation")
+    return levels, int(d)
 
 
 @dataclass

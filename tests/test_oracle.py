@@ -345,3 +345,88 @@ def test_p169_claim_counterexample():
     s = oracle.ecl_scc(rp, ci, snap_iter=1)
     assert s.snap_in[5] == 5 and s.snap_out[5] == 5
     np.testing.assert_array_equal(s.labels, np.arange(10))
+
+
+# ---------------------------------------------------------------- O4: sweep levels
+def brute_levels(n, edges, labels):
+    """level of each vertex's SCC = longest condensation path ending there, by enumerating
+    every path from every SCC with a depth-first search (exponential: tiny graphs only)."""
+    comps = sorted({int(l) for l in labels})
+    succ = {c: set() for c in comps}
+    for u, v in edges:
+        a, b = int(labels[u]), int(labels[v])
+        if a != b:
+            succ[a].add(b)
+    best = {c: 0 for c in comps}
+
+    def walk(c, length):
+        best[c] = max(best[c], length)
+        for d in succ[c]:
+            walk(d, length + 1)
+
+    for c in comps:
+        walk(c, 0)
+    return np.array([best[int(labels[v])] for v in range(n)], dtype=np.int32)
+
+
+def test_levels_vs_bruteforce_paths():
+    rng = random.Random(11)
+    for trial in range(300):
+        n = rng.randrange(1, 11)
+        edges = random_edges(rng, n, rng.randrange(0, 2 * n + 1))
+        rp, ci = csr_from_edges(n, edges)
+        lab = brute_labels(n, edges)
+        lv, depth = oracle.scc_levels(rp, ci, lab)
+        exp = brute_levels(n, edges, lab)
+        np.testing.assert_array_equal(lv, exp, err_msg=f"trial {trial}")
+        assert depth == exp.max() + 1
+
+
+def test_levels_closed_forms_and_invariants():
+    rng = np.random.default_rng(3)
+    # a path in random ID order: level = position on the path
+    n = 5000
+    perm = rng.permutation(n)
+    rp, ci = csr_from_edges(n, np.stack([perm[:-1], perm[1:]], 1))
+    lv, depth = oracle.scc_levels(rp, ci, np.arange(n))
+    pos = np.empty(n, dtype=np.int32)
+    pos[perm] = np.arange(n)
+    np.testing.assert_array_equal(lv, pos)
+    assert depth == n
+    # disjoint cycles: every SCC is a source
+    k = 7
+    e = [(b * k + i, b * k + (i + 1) % k) for b in range(50) for i in range(k)]
+    rp, ci = csr_from_edges(350, e)
+    lv, depth = oracle.scc_levels(rp, ci, oracle.tarjan_labels(rp, ci))
+    assert (lv == 0).all() and depth == 1
+    # a chain of 3-cycles: cycle j has level j
+    e = [(3 * j + i, 3 * j + (i + 1) % 3) for j in range(40) for i in range(3)] + \
+        [(3 * j + 2, 3 * (j + 1)) for j in range(39)]
+    rp, ci = csr_from_edges(120, e)
+    lv, depth = oracle.scc_levels(rp, ci, oracle.tarjan_labels(rp, ci))
+    np.testing.assert_array_equal(lv, np.arange(120) // 3)
+    assert depth == 40
+    # invariants on random graphs: every inter-SCC edge climbs >= 1 level; every SCC above
+    # level 0 has a predecessor exactly one level below (the longest path is tight)
+    r = random.Random(5)
+    for _ in range(20):
+        n = r.randrange(50, 400)
+        edges = random_edges(r, n, r.randrange(0, 3 * n))
+        rp, ci = csr_from_edges(n, edges)
+        lab = oracle.tarjan_labels(rp, ci)
+        lv, depth = oracle.scc_levels(rp, ci, lab)
+        tight = np.zeros(n, bool)
+        for u, v in edges:
+            if lab[u] != lab[v]:
+                assert lv[v] >= lv[u] + 1
+                if lv[v] == lv[u] + 1:
+                    tight[lab[v]] = True
+        reps = np.unique(lab)
+        assert all(tight[c] for c in reps if lv[c] > 0)
+        assert depth == lv.max() + 1 == condensation_depth(n, edges, lab)
+
+
+def test_levels_reject_cyclic_labels():
+    rp, ci = csr_from_edges(3, [(0, 1), (1, 0)])
+    with pytest.raises(ValueError):
+        oracle.scc_levels(rp, ci, np.array([0, 1, 2]))       # 0 and 1 labelled apart: a cycle

@@ -153,6 +153,21 @@ int ecl_scc_batched(int32_t G, const int32_t* n, const int64_t* nnz,
                     int32_t* const* labels_out, ecl_scc_stream_t stream, ecl_scc_plan_t plan,
                     ecl_scc_stats* stats);
 
+/* ---- after SCC detection: the sweep schedule ------------------------------------ */
+/* Levels of the SCC condensation (the step after SCC detection in the RTE application:
+ * a transport sweep starts "from nodes with no incoming edges"; the paper tabulates
+ * the condensation's "DAG depth" per mesh, Table 2).  levels_out[v] = length of the longest
+ * path of the condensation DAG that ends in v's SCC (source SCCs: 0); SCCs of one level can
+ * be swept concurrently.  *depth_out (host, nullable) = max level + 1 (0 for n == 0).
+ * row_ptr/col_idx: the same device CSR given to ecl_scc(); labels: its device labels_out
+ * (any labelling that gives every SCC, and only it, one value in [0, n)).  levels_out:
+ * n int32, device, written.  Uses the plan's buffers as workspace (NULL: a temporary
+ * plan).  Synchronous on `stream`.  Errors: EINVAL (arguments), ERANGE (a label outside
+ * [0, n), or labels that induce a cyclic condensation, i.e. not the SCC partition). */
+int ecl_scc_levels(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx,
+                   const int32_t* labels, int32_t* levels_out, int32_t* depth_out,
+                   ecl_scc_stream_t stream, ecl_scc_plan_t plan);
+
 /* ---- multi-GPU: one large graph, edge-partitioned by source rows (SPMD) ---------- */
 typedef struct ecl_scc_comm_s* ecl_scc_comm_t;
 

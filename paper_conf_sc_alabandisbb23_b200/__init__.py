@@ -80,6 +80,7 @@ def lib() -> ctypes.CDLL:
         "ecl_scc_last_error": [],
         "ecl_scc_version": [],
         "ecl_scc_plan_counters": [vp, vp],
+        "ecl_scc_levels": [i32, i64, vp, vp, vp, vp, vp, vp, vp],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -96,7 +97,7 @@ ABI_SYMBOLS = ("ecl_scc", "ecl_scc_async", "ecl_scc_debug_run", "ecl_scc_plan_cr
                "ecl_scc_plan_destroy", "ecl_scc_batched", "ecl_scc_get_unique_id",
                "ecl_scc_comm_create", "ecl_scc_comm_destroy", "ecl_scc_partitioned",
                "ecl_scc_partitioned_emulated", "ecl_scc_partition_rows", "ecl_scc_status_string",
-               "ecl_scc_last_error", "ecl_scc_version", "ecl_scc_plan_counters")
+               "ecl_scc_last_error", "ecl_scc_version", "ecl_scc_plan_counters", "ecl_scc_levels")
 
 
 def status_string(s: int) -> str:
@@ -163,6 +164,23 @@ def ecl_scc(row_ptr: torch.Tensor, col_idx: torch.Tensor, labels_out: torch.Tens
                                _dev_i32(labels_out, "labels_out"), _stream(stream),
                                plan.handle if plan else None, ctypes.byref(st) if st else None), "ecl_scc")
     return (labels_out, st.as_dict()) if stats else labels_out
+
+
+def ecl_scc_levels(row_ptr: torch.Tensor, col_idx: torch.Tensor, labels: torch.Tensor,
+                   levels_out: torch.Tensor | None = None, stream=None, plan: Plan | None = None):
+    """Sweep levels of the SCC condensation (Table 2 "DAG depth"): returns (levels per
+    vertex = longest condensation path ending in its SCC, depth = max level + 1).  `labels`
+    are ecl_scc()'s output for the same graph."""
+    n = row_ptr.numel() - 1
+    nnz = col_idx.numel()
+    if levels_out is None:
+        levels_out = torch.empty(max(n, 0), dtype=torch.int32, device=row_ptr.device)
+    depth = ctypes.c_int32(0)
+    _check(lib().ecl_scc_levels(n, nnz, _dev_i32(row_ptr, "row_ptr"), _dev_i32(col_idx, "col_idx") if nnz else None,
+                                _dev_i32(labels, "labels"), _dev_i32(levels_out, "levels_out"),
+                                ctypes.byref(depth), _stream(stream), plan.handle if plan else None),
+           "ecl_scc_levels")
+    return levels_out, int(depth.value)
 
 
 def ecl_scc_debug_run(row_ptr: torch.Tensor, col_idx: torch.Tensor, stop_iter: int, flags: int = 0, stream=None):

@@ -25,6 +25,7 @@
 #include "reorder.cuh"
 #include "pack.cuh"
 #include "tail.cuh"
+#include "levels.cuh"
 #include "driver.h"
 
 namespace eclscc {
@@ -147,6 +148,7 @@ void plan_free(Plan* p) {
     cudaFree(p->pnin); cudaFree(p->pnout); cudaFree(p->ext); cudaFree(p->ext_cnt);
     cudaFree(p->aq_state); cudaFree(p->aq_seen); cudaFree(p->aq_ctr);
     cudaFree(p->tail_dev);
+    cudaFree(p->lv_ctl);
     if (p->tail_host) cudaFreeHost(p->tail_host);
     if (p->hc) cudaFreeHost(p->hc);
     if (p->ev_ok)
@@ -904,6 +906,59 @@ int run_batched(Plan* p, int32_t G, const int32_t* n, const int64_t* nnz, const 
     return ECL_SCC_OK;
 }
 
+// Sweep levels of the SCC condensation (levels.cuh); plan buffers serve as workspace.
+int run_levels(Plan* p, int32_t n, const int32_t* rp, const int32_t* ci, const int32_t* lab, int32_t* out,
+               int32_t* depth, cudaStream_t s) {
+    if (!p->lv_ctl) {
+        cudaError_t e = cudaMalloc(&p->lv_ctl, sizeof(LvCtl));
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(ECL_SCC_ENOMEM, "levels control block: %s", cudaGetErrorString(e));
+        }
+        int per_sm = 0, dev = 0, sms = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lv_run, 512, 0));
+        CK(cudaGetDevice(&dev));
+        CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+        // one CTA per SM: the round barrier's cost grows with the CTAs that arrive at it
+        p->lv_resident = std::max(1, std::min(per_sm, 1)) * sms;
+    }
+    LvCtl* ctl = (LvCtl*)p->lv_ctl;
+    int32_t* indeg = p->kin;
+    int32_t* msize = p->kout;
+    int32_t* mptr = p->optr[0];
+    int32_t* cursor = p->newidx;
+    int32_t* memb = p->act[0];
+    int32_t* lvl = p->cin[0];
+    int2* qa = p->cnt;
+    int2* qb = (int2*)p->emask;
+    const size_t nb = sizeof(int32_t) * (size_t)n;
+    CK(cudaMemsetAsync(indeg, 0, nb, s));
+    CK(cudaMemsetAsync(msize, 0, nb, s));
+    CK(cudaMemsetAsync(cursor, 0, nb, s));
+    CK(cudaMemsetAsync(ctl, 0, sizeof(LvCtl), s));
+    const unsigned gs = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
+    p->launches++; k_lv_count<<<gs, TPB, 0, s>>>(n, rp, ci, lab, indeg, msize, &ctl->err);
+    int r = scan_excl<I1>(p, (const I1*)msize, n, (I1*)mptr, (I1*)&p->dc->grand1, p->bsum, 1, s);
+    if (r) return r;
+    p->launches++; k_lv_fill<<<gs, TPB, 0, s>>>(n, lab, mptr, cursor, memb);
+    p->launches++; k_lv_init<<<gs, TPB, 0, s>>>(n, indeg, msize, mptr, lvl, qa, ctl);
+    CK(cudaGetLastError());
+    void* args[] = {(void*)&rp, (void*)&ci, (void*)&lab, &mptr, &memb, &indeg, &lvl, &qa, &qb, &ctl};
+    p->launches++;
+    CK(cudaLaunchCooperativeKernel((const void*)k_lv_run, dim3(p->lv_resident), dim3(512), args, 0, s));
+    p->launches++; k_lv_apply<<<gs, TPB, 0, s>>>(n, lab, lvl, out);
+    CK(cudaGetLastError());
+    LvCtl h;
+    CK(cudaMemcpyAsync(&h, ctl, sizeof(LvCtl), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (h.err) return fail(ECL_SCC_ERANGE, "levels: a label lies outside [0, n)");
+    if (h.reached != h.nscc)
+        return fail(ECL_SCC_ERANGE, "levels: the labels induce a cyclic condensation (%d of %d SCCs reached)",
+                    h.reached, h.nscc);
+    if (depth) *depth = h.depth;
+    return ECL_SCC_OK;
+}
+
 }  // namespace eclscc
 
 // =========================================================================== C ABI
@@ -1048,6 +1103,27 @@ int ecl_scc_batched(int32_t G, const int32_t* n, const int64_t* nnz, const int32
         plan = tmp;
     }
     int r = run_batched(&plan->p, G, n, nnz, row_ptr, col_idx, labels_out, (cudaStream_t)stream, stats);
+    if (tmp) ecl_scc_plan_destroy(tmp);
+    return r;
+}
+
+int ecl_scc_levels(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx, const int32_t* labels,
+                   int32_t* levels_out, int32_t* depth_out, ecl_scc_stream_t stream, ecl_scc_plan_t plan) {
+    clear_err();
+    int r = check_graph_args(n, nnz, row_ptr, col_idx, levels_out);
+    if (r) return r;
+    if (n > 0 && !labels) return fail(ECL_SCC_EINVAL, "levels: NULL labels");
+    if (depth_out) *depth_out = 0;
+    if (n == 0) return ECL_SCC_OK;
+    if (plan && plan->p.n_cap < n) return fail(ECL_SCC_EINVAL, "plan too small (n_max=%d)", plan->p.n_cap);
+    ecl_scc_plan_t tmp = nullptr;
+    if (!plan) {
+        r = ecl_scc_plan_create(n, nnz, 0, &tmp);
+        if (r) return r;
+        plan = tmp;
+    }
+    plan->p.launches = 0;
+    r = run_levels(&plan->p, n, row_ptr, col_idx, labels, levels_out, depth_out, (cudaStream_t)stream);
     if (tmp) ecl_scc_plan_destroy(tmp);
     return r;
 }

@@ -57,6 +57,8 @@ struct Plan {
     void* tail_dev;                      // tail.cuh TailTrace (device) and its pinned mirror
     void* tail_host;
     int tail_resident;                   // co-resident CTAs of k_tail
+    void* lv_ctl;                        // levels.cuh LvCtl (device)
+    int lv_resident;                     // co-resident CTAs of k_lv_run
     int64_t launches;                    // kernels launched by the current call
     cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
     bool ev_ok;

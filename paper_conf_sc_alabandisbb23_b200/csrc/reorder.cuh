@@ -46,21 +46,27 @@ static __global__ void k_bfs_level(int32_t* __restrict__ fa, int32_t* __restrict
             b0 = rp[u]; e0 = rp[u + 1]; b1 = cp[u]; e1 = cp[u + 1];
         }
         int n0 = e0 - b0, n1 = e1 - b1;
-        for (int j = 0;; j++) {                        // j-th neighbour of every lane's vertex
-            const bool has = j < n0 + n1;
-            if (!__any_sync(FULL, has)) break;
-            bool got = false;
-            int w = 0;
-            if (has) {
-                w = j < n0 ? ci[b0 + j] : cr[b1 + j - n0];
-                got = ld_cg(cell + w) == NOLAB && atomicCAS(cell + w, NOLAB, c) == NOLAB;
+        for (int j0 = 0;; j0 += 4) {                   // neighbours j0..j0+3 of every lane's vertex
+            if (!__any_sync(FULL, j0 < n0 + n1)) break;
+            // the adjacency loads, then the cell loads, of a batch are issued before use
+            int w[4], cw[4];
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                const int j = j0 + q;
+                w[q] = j < n0 + n1 ? (j < n0 ? ci[b0 + j] : cr[b1 + j - n0]) : -1;
             }
-            const unsigned m = __ballot_sync(FULL, got);
-            if (m) {
-                int at = 0;
-                if (lane == __ffs(m) - 1) at = atomicAdd(cnt + (r + 1) % 3, __popc(m));
-                at = __shfl_sync(FULL, at, __ffs(m) - 1);
-                if (got) next[at + __popc(m & ((1u << lane) - 1))] = w;
+#pragma unroll
+            for (int q = 0; q < 4; q++) cw[q] = w[q] >= 0 ? ld_cg(cell + w[q]) : 0;
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                const bool got = w[q] >= 0 && cw[q] == NOLAB && atomicCAS(cell + w[q], NOLAB, c) == NOLAB;
+                const unsigned m = __ballot_sync(FULL, got);
+                if (m) {
+                    int at = 0;
+                    if (lane == __ffs(m) - 1) at = atomicAdd(cnt + (r + 1) % 3, __popc(m));
+                    at = __shfl_sync(FULL, at, __ffs(m) - 1);
+                    if (got) next[at + __popc(m & ((1u << lane) - 1))] = w[q];
+                }
             }
         }
     }
@@ -113,7 +119,7 @@ static __global__ void k_cell_place(int32_t n, const int32_t* __restrict__ key, 
 // atomic placement above leaves the members in arbitrary order).  Cells larger than
 // SORT_MAX keep the arbitrary order (only the pass count depends on it).
 constexpr int SORT_MAX = 8192;
-constexpr int SORT_THREADS = 1024;
+constexpr int SORT_THREADS = 256;     // small CTAs: ~7 cells sort concurrently per SM (barrier-bound stages)
 static __global__ void __launch_bounds__(SORT_THREADS) k_cell_sort(int64_t nkeys, const int32_t* __restrict__ start,
                                                                   int32_t* __restrict__ orig, int32_t* __restrict__ pos) {
     __shared__ int32_t sk[SORT_MAX];

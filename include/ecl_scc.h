@@ -153,6 +153,15 @@ int ecl_scc_batched(int32_t G, const int32_t* n, const int64_t* nnz,
                     int32_t* const* labels_out, ecl_scc_stream_t stream, ecl_scc_plan_t plan,
                     ecl_scc_stats* stats);
 
+/* Same as ecl_scc_async, but row_ptr, col_idx and labels_out are HOST pointers (pinned
+ * memory -- cudaMallocHost / cudaHostRegister -- gives full-speed copies).  The plan keeps
+ * device copies (4*(n_max+1) + 4*nnz_max + 4*(n_max+1) bytes, allocated on first use); the
+ * copies run on `stream`; returns after the labels are back on the host.  Errors as
+ * ecl_scc_async (ERANGE from the device validation of the copied CSR). */
+int ecl_scc_host(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx,
+                 int32_t* labels_out, ecl_scc_stream_t stream, ecl_scc_plan_t plan,
+                 ecl_scc_stats* stats);
+
 /* ---- after SCC detection: the sweep schedule ------------------------------------ */
 /* Levels of the SCC condensation (the step after SCC detection in the RTE application:
  * a transport sweep starts "from nodes with no incoming edges"; the paper tabulates

@@ -81,6 +81,7 @@ def lib() -> ctypes.CDLL:
         "ecl_scc_version": [],
         "ecl_scc_plan_counters": [vp, vp],
         "ecl_scc_levels": [i32, i64, vp, vp, vp, vp, vp, vp, vp],
+        "ecl_scc_host": [i32, i64, vp, vp, vp, vp, vp, vp],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -97,7 +98,8 @@ ABI_SYMBOLS = ("ecl_scc", "ecl_scc_async", "ecl_scc_debug_run", "ecl_scc_plan_cr
                "ecl_scc_plan_destroy", "ecl_scc_batched", "ecl_scc_get_unique_id",
                "ecl_scc_comm_create", "ecl_scc_comm_destroy", "ecl_scc_partitioned",
                "ecl_scc_partitioned_emulated", "ecl_scc_partition_rows", "ecl_scc_status_string",
-               "ecl_scc_last_error", "ecl_scc_version", "ecl_scc_plan_counters", "ecl_scc_levels")
+               "ecl_scc_last_error", "ecl_scc_version", "ecl_scc_plan_counters", "ecl_scc_levels",
+               "ecl_scc_host")
 
 
 def status_string(s: int) -> str:
@@ -163,6 +165,24 @@ def ecl_scc(row_ptr: torch.Tensor, col_idx: torch.Tensor, labels_out: torch.Tens
     _check(lib().ecl_scc_async(n, nnz, _dev_i32(row_ptr, "row_ptr"), _dev_i32(col_idx, "col_idx") if nnz else None,
                                _dev_i32(labels_out, "labels_out"), _stream(stream),
                                plan.handle if plan else None, ctypes.byref(st) if st else None), "ecl_scc")
+    return (labels_out, st.as_dict()) if stats else labels_out
+
+
+def ecl_scc_host(row_ptr: torch.Tensor, col_idx: torch.Tensor, labels_out: torch.Tensor | None = None,
+                 stream=None, plan: Plan | None = None, stats: bool = False):
+    """ecl_scc on HOST (CPU, preferably pinned) tensors: the library copies the CSR in, runs,
+    and copies the labels back (ecl_scc_host).  Returns labels (host) and optional stats."""
+    for t, nm in ((row_ptr, "row_ptr"), (col_idx, "col_idx")):
+        if t.device.type != "cpu" or t.dtype != torch.int32 or not t.is_contiguous():
+            raise ValueError(f"{nm} must be a contiguous int32 CPU tensor")
+    n = row_ptr.numel() - 1
+    nnz = col_idx.numel()
+    if labels_out is None:
+        labels_out = torch.empty(max(n, 0), dtype=torch.int32).pin_memory()
+    st = Stats() if stats else None
+    _check(lib().ecl_scc_host(n, nnz, row_ptr.data_ptr(), col_idx.data_ptr() if nnz else None,
+                              labels_out.data_ptr(), _stream(stream), plan.handle if plan else None,
+                              ctypes.byref(st) if st else None), "ecl_scc_host")
     return (labels_out, st.as_dict()) if stats else labels_out
 
 

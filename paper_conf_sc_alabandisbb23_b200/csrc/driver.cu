@@ -149,6 +149,7 @@ void plan_free(Plan* p) {
     cudaFree(p->aq_state); cudaFree(p->aq_seen); cudaFree(p->aq_ctr);
     cudaFree(p->tail_dev);
     cudaFree(p->lv_ctl);
+    cudaFree(p->h_rp); cudaFree(p->h_ci); cudaFree(p->h_lab);
     if (p->tail_host) cudaFreeHost(p->tail_host);
     if (p->hc) cudaFreeHost(p->hc);
     if (p->ev_ok)
@@ -1045,6 +1046,52 @@ int ecl_scc_async(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t*
     }
     plan->p.launches = 0;
     r = run_graph(&plan->p, n, nnz, row_ptr, col_idx, labels_out, (cudaStream_t)stream, stats, 0, nullptr, nullptr);
+    if (tmp) ecl_scc_plan_destroy(tmp);
+    return r;
+}
+
+int ecl_scc_host(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx, int32_t* labels_out,
+                 ecl_scc_stream_t stream, ecl_scc_plan_t plan, ecl_scc_stats* stats) {
+    clear_err();
+    int r = check_graph_args(n, nnz, row_ptr, col_idx, labels_out);
+    if (r) return r;
+    if (stats) memset(stats, 0, sizeof(*stats));
+    if (n == 0) return ECL_SCC_OK;
+    if (plan && (plan->p.n_cap < n || plan->p.m_cap < nnz))
+        return fail(ECL_SCC_EINVAL, "plan too small (n_max=%d, nnz_max=%lld)", plan->p.n_cap, (long long)plan->p.m_cap);
+    ecl_scc_plan_t tmp = nullptr;
+    if (!plan) {
+        r = ecl_scc_plan_create(n, nnz, 0, &tmp);
+        if (r) return r;
+        plan = tmp;
+    }
+    Plan* p = &plan->p;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (!p->h_rp || p->h_n_cap < n || p->h_m_cap < nnz) {          // device copies, sized for the plan
+        cudaFree(p->h_rp); cudaFree(p->h_ci); cudaFree(p->h_lab);
+        p->h_rp = p->h_ci = p->h_lab = nullptr;
+        cudaError_t e = cudaMalloc((void**)&p->h_rp, sizeof(int32_t) * ((size_t)p->n_cap + 1));
+        if (e == cudaSuccess) e = cudaMalloc((void**)&p->h_ci, sizeof(int32_t) * (size_t)std::max<int64_t>(p->m_cap, 1));
+        if (e == cudaSuccess) e = cudaMalloc((void**)&p->h_lab, sizeof(int32_t) * ((size_t)p->n_cap + 1));
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            if (tmp) ecl_scc_plan_destroy(tmp);
+            return fail(ECL_SCC_ENOMEM, "host-buffer staging: %s", cudaGetErrorString(e));
+        }
+        p->h_n_cap = p->n_cap;
+        p->h_m_cap = p->m_cap;
+    }
+    p->launches = 0;
+    cudaError_t e = cudaMemcpyAsync(p->h_rp, row_ptr, sizeof(int32_t) * ((size_t)n + 1), cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess && nnz)
+        e = cudaMemcpyAsync(p->h_ci, col_idx, sizeof(int32_t) * (size_t)nnz, cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) r = fail(ECL_SCC_ECUDA, "host-to-device copy: %s", cudaGetErrorString(e));
+    if (!r) r = run_graph(p, n, nnz, p->h_rp, p->h_ci, p->h_lab, s, stats, 0, nullptr, nullptr);
+    if (!r) {
+        e = cudaMemcpyAsync(labels_out, p->h_lab, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToHost, s);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+        if (e != cudaSuccess) r = fail(ECL_SCC_ECUDA, "device-to-host copy: %s", cudaGetErrorString(e));
+    }
     if (tmp) ecl_scc_plan_destroy(tmp);
     return r;
 }

@@ -197,6 +197,18 @@ def test_invalid_input_reports_erange():
     assert ex.value.status == E.EINVAL
 
 
+def test_host_buffer_entry_point():
+    """ecl_scc_host: host CSR in, host labels out (pinned and pageable buffers)."""
+    plan = E.Plan(20000, 100000)
+    for g in (gen.config("c1"), gen.mesh(12, gen.ordinate(5), kappa=0.2, seed=3), gen.from_edges(9, [])):
+        rp, ci = torch.from_numpy(g.row_ptr), torch.from_numpy(g.col_idx)
+        truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+        for pin in (False, True):
+            a, b = (rp.pin_memory(), ci.pin_memory()) if pin else (rp, ci)
+            lab = E.ecl_scc_host(a, b, plan=plan if pin else None)
+            np.testing.assert_array_equal(lab.numpy(), truth)
+
+
 def test_plan_reuse_and_stream():
     g1, g2 = gen.config("c1"), gen.mesh(12, gen.ordinate(7), kappa=0.2, seed=9)
     plan = E.Plan(max(g1.n, g2.n), max(g1.nnz, g2.nnz))

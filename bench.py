@@ -345,7 +345,7 @@ def ours(args):
         traffic = roofline_traffic(kname)
         iters = sum(s["iterations"] for s in rstats) / len(rstats)
         roof = {"bound": "hbm",
-                "kernel": ("Phase 2 (k_tile_pack + k_prop_async)" if async_path
+                "kernel": ("Phase 2 (k_prop_async; tile packs written by the compaction scatter)" if async_path
                            else "Phase 2 (k_prop_tile + k_prop_heavy)"),
                 "algorithmic_bytes_per_launch": int(pb / iters) if async_path and iters else None,
                 "achieved": round(achieved, 1) if achieved else None, "peak": peak, "unit": "GB/s",

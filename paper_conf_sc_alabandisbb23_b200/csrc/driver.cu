@@ -270,6 +270,32 @@ static int reorder_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, con
     return ECL_SCC_OK;
 }
 
+// Does Phase 2 of a working graph with `nchunks` long-row chunks run on tile packs?
+static bool pack_path(const Plan* p, int nchunks) {
+    static int env_variant = -1;   // the KCAP / LEVELS experiments run on the tile kernel
+    if (env_variant < 0) env_variant = (getenv("ECL_SCC_KCAP") || getenv("ECL_SCC_LEVELS")) ? 1 : 0;
+    const bool sync = (p->flags & ECL_SCC_SYNC_PASSES) != 0 || (p->low_locality && nchunks > 0);
+    return nchunks == 0 && !sync && !(p->flags & (ECL_SCC_NO_DIRTY | ECL_SCC_STAGED | ECL_SCC_NO_PACK | ECL_SCC_SWEEP)) &&
+           p->tile == PACK_TT && !env_variant;
+}
+// tile pack buffers (pack.cuh), sized for the plan on first use
+static int ensure_pack(Plan* p) {
+    if (p->pnin) return ECL_SCC_OK;
+    const size_t np = (size_t)cdiv((int64_t)p->n_cap + 1, PACK_TT) * PACK_TT + PACK_TT;
+    cudaError_t e = cudaMalloc((void**)&p->pnin, np * 8);
+    if (e == cudaSuccess) e = cudaMalloc((void**)&p->pnout, np * 8);
+    if (e == cudaSuccess) e = cudaMalloc((void**)&p->ext, 2 * (size_t)p->m_cap * sizeof(int2) + 16);
+    if (e == cudaSuccess) e = cudaMalloc((void**)&p->ext_cnt, (size_t)p->dirty_cap * 4);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ECL_SCC_ENOMEM, "tile pack allocation: %s", cudaGetErrorString(e));
+    }
+    CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
+    CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributePreferredSharedMemoryCarveout,
+                            (int)cudaSharedmemCarveoutMaxShared));
+    return ECL_SCC_OK;
+}
+
 // a7 + a2 + a3 + a8: Phase 3 edge removal, Trim-1, compaction into buffer `ob` with the
 // Phase-1 reset of the survivors and the final labels of the vertices that leave
 template <bool FIRST, bool TRIM>
@@ -281,6 +307,15 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     const Chunk* cur = chunk_buf(p, p->cb);
     CK(cudaMemsetAsync(&p->dc->kept, 0, sizeof(unsigned long long), s));
     CK(cudaMemsetAsync(&p->dc->nchunks, 0, sizeof(int), s));
+    CK(cudaMemsetAsync(&p->dc->pack_bad, 0, sizeof(int), s));
+    // the scatter writes the next graph's tile pack when Phase 2 will use one (no long rows
+    // now means none after the compaction)
+    PackOut pk{nullptr, nullptr, nullptr, nullptr, &p->dc->pack_bad};
+    p->pack_fused = pack_path(p, nc);
+    if (p->pack_fused) {
+        if (int r = ensure_pack(p)) return r;
+        pk = PackOut{p->pnin, p->pnout, p->ext, p->ext_cnt, &p->dc->pack_bad};
+    }
     p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, &p->dc->kept, chunked, p->hcnt, p->emask);
     if (chunked) {
         p->launches += 2;
@@ -292,9 +327,9 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     if (r) return r;
     p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
-                                              chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur);
+                                              chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur, pk);
     p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->newidx, p->optr[ob],
-                                                          p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked, p->emask);
+                                                          p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked, p->emask, pk);
     if (chunked) {
         p->launches++;
         k_scatter_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kin, p->kout, p->chunk_cnt,
@@ -435,27 +470,13 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                                                                    : std::vector<int>{0};
     int64_t total = 0;
     // tile packs (pack.cuh): the default for graphs without long rows
-    static int env_variant = -1;   // the KCAP / LEVELS experiments run on the tile kernel
-    if (env_variant < 0) env_variant = (getenv("ECL_SCC_KCAP") || getenv("ECL_SCC_LEVELS")) ? 1 : 0;
-    const bool use_pack = use_dirty && p->tile == PACK_TT && thetas.size() == 1 && !env_variant &&
-                          !(p->flags & (ECL_SCC_NO_PACK | ECL_SCC_SWEEP)) && g.na > 0;
+    const bool use_pack = pack_path(p, nchunks) && g.na > 0;
     if (use_pack) {
-        if (!p->pnin) {                                  // first use: sized for the plan
-            const size_t np = (size_t)cdiv((int64_t)p->n_cap + 1, PACK_TT) * PACK_TT + PACK_TT;
-            cudaError_t e = cudaMalloc((void**)&p->pnin, np * 8);
-            if (e == cudaSuccess) e = cudaMalloc((void**)&p->pnout, np * 8);
-            if (e == cudaSuccess) e = cudaMalloc((void**)&p->ext, 2 * (size_t)p->m_cap * sizeof(int2) + 16);
-            if (e == cudaSuccess) e = cudaMalloc((void**)&p->ext_cnt, (size_t)p->dirty_cap * 4);
-            if (e != cudaSuccess) {
-                cudaGetLastError();
-                return fail(ECL_SCC_ENOMEM, "tile pack allocation: %s", cudaGetErrorString(e));
-            }
-            CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
-            CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                    (int)cudaSharedmemCarveoutMaxShared));
+        if (int r = ensure_pack(p)) return r;
+        if (!p->pack_fused || p->hc->pack_bad) {       // the scatter did not write it
+            p->launches++;
+            k_tile_pack<<<ntiles, PACK_TH, 0, s>>>(g, p->pnin, p->pnout, p->ext, p->ext_cnt);
         }
-        p->launches++;
-        k_tile_pack<<<ntiles, PACK_TH, 0, s>>>(g, p->pnin, p->pnout, p->ext, p->ext_cnt);
         CK(cudaGetLastError());
         if (!(p->flags & ECL_SCC_NO_ASYNC)) {          // one persistent launch (pack.cuh)
             if (!p->aq_state) {

@@ -49,6 +49,7 @@ struct Plan {
     int epoch;                           // sweep epoch (monotone over the plan's life)
     unsigned long long *pnin, *pnout;    // tile packs (pack.cuh): slot words per local vertex
     int2* ext;                           // tile packs: cut edges per tile
+    bool pack_fused;                     // the last compaction's scatter wrote the tile pack
     int* ext_cnt;                        // tile packs: cut edges of each tile
     int* aq_state;                       // asynchronous Phase 2 (pack.cuh AsyncQ)
     uint8_t* aq_seen;

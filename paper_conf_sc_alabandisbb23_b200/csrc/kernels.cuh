@@ -273,6 +273,69 @@ __device__ __forceinline__ void emit_mask(const int32_t* __restrict__ adj, int b
     }
 }
 
+// Tile-pack output of the compaction scatter (pack.cuh layout).  When pnin is set, the
+// scatter also writes each survivor's slot words and appends its cut edges to its tile's
+// list, so Phase 2 needs no separate k_tile_pack pass over the new graph; a row longer
+// than HEAVY (warp path, no masks) sets *bad and the driver falls back to k_tile_pack.
+struct PackOut {
+    unsigned long long* pnin;
+    unsigned long long* pnout;
+    int2* ext;
+    int* ext_cnt;
+    int* bad;
+};
+constexpr unsigned long long PK_EMPTY = 0x0800080008000800ull;   // four empty slots (pack.cuh PSLOTS_EMPTY)
+constexpr int PK_DIR = 0x8000;                                  // out-edge mark (pack.cuh EXT_DIR)
+constexpr unsigned long long PK_SLOW = 0x8000ull << 48;         // > 4 intra-tile neighbours (SLOW_MARK)
+
+__device__ __forceinline__ void pk_add(unsigned long long& pk, int& ns, unsigned idx) {
+    pk &= ~(0xFFFFull << (16 * ns));
+    pk |= (unsigned long long)idx << (16 * ns);
+    ns++;
+}
+// emit_mask plus the pack of local vertex j (tile base tb): survivors in j's tile fill the
+// slot word (returned); the others are counted in nc (they become cut edges of the tile,
+// written by emit_cut once the warp has reserved their slots)
+__device__ __forceinline__ unsigned long long emit_mask_pack(const int32_t* __restrict__ adj, int b, unsigned m, int self,
+                                                             const int32_t* __restrict__ newidx, int32_t* __restrict__ dst,
+                                                             int pos, int tb, int& nc) {
+    unsigned long long pk = PK_EMPTY;
+    int ns = 0;
+    while (m) {
+        int k[4], y[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            k[q] = m ? __ffs(m) - 1 : -1;
+            m &= m - 1;
+        }
+#pragma unroll
+        for (int q = 0; q < 4; q++) y[q] = __ldg(newidx + (k[q] >= 0 ? __ldg(adj + b + k[q]) : self));
+#pragma unroll
+        for (int q = 0; q < 4; q++)
+            if (k[q] >= 0) {
+                dst[pos++] = y[q];
+                if ((unsigned)(y[q] - tb) < (unsigned)TILE) {
+                    if (ns < 4) pk_add(pk, ns, (unsigned)(y[q] - tb));
+                    else pk |= PK_SLOW;
+                } else {
+                    nc++;
+                }
+            }
+    }
+    return pk;
+}
+// the cut edges of one row (the survivors of m outside tile tb) as {far end, (j - tb) | dir}
+__device__ __forceinline__ void emit_cut(const int32_t* __restrict__ adj, int b, unsigned m,
+                                         const int32_t* __restrict__ newidx, int j, int tb, int dir,
+                                         int2* __restrict__ E, int& at) {
+    while (m) {
+        const int k = __ffs(m) - 1;
+        m &= m - 1;
+        const int y = __ldg(newidx + __ldg(adj + b + k));
+        if ((unsigned)(y - tb) >= (unsigned)TILE) E[at++] = make_int2(y, (j - tb) | dir);
+    }
+}
+
 // kept in/out degree per local vertex, plus the number of kept edges
 constexpr int TPB_COMPACT = 256;     // block size of the compaction kernels (driver TPB)
 template <bool FIRST>
@@ -357,13 +420,21 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
                               int32_t* __restrict__ act2, int32_t* __restrict__ cin2, int32_t* __restrict__ cout2,
                               int32_t* __restrict__ optr2, int32_t* __restrict__ iptr2, int32_t* __restrict__ labels,
                               Chunk* __restrict__ chunks, int* __restrict__ nchunks, int chunk_cap, Prio P,
-                              const int32_t* __restrict__ orig) {
+                              const int32_t* __restrict__ orig, PackOut pk) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i == 0) {
         const int4 t = *totals;
         optr2[t.x] = t.y;
         iptr2[t.x] = t.z;
+    }
+    if (pk.pnin) {                         // pack: empty slot words past the last vertex of the last tile
+        const int na2 = totals->x;
+        const int pad_end = (na2 + TILE - 1) & ~(TILE - 1);
+        for (int64_t k = na2 + i; k < pad_end; k += (int64_t)gridDim.x * blockDim.x) {
+            pk.pnin[k] = PK_EMPTY;
+            pk.pnout[k] = PK_EMPTY;
+        }
     }
     const bool valid = i < g.na;
     int2 c = valid ? cnt[i] : make_int2(0, 0);
@@ -378,6 +449,7 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
     if (alive) {
         newidx[i] = j;
         act2[j] = v;
+        if (pk.pnin && (j & (TILE - 1)) == 0) pk.ext_cnt[j / TILE] = 0;   // the tile's cut-edge count
         const int pv = (int)prio_of(P, (uint32_t)ov);
         cin2[j] = pv;       // Phase 1: v_in <- v_id, v_out <- v_id for the unfinished
         cout2[j] = pv;
@@ -484,19 +556,53 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
                                   const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
                                   const int32_t* __restrict__ newidx, const int32_t* __restrict__ optr2,
                                   const int32_t* __restrict__ iptr2, int32_t* __restrict__ oadj2,
-                                  int32_t* __restrict__ iadj2, int chunked, const uint2* __restrict__ emask) {
+                                  int32_t* __restrict__ iadj2, int chunked, const uint2* __restrict__ emask,
+                                  PackOut pk) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
     const int j = r.valid ? newidx[i] : -1;
     const bool go = j >= 0;
-    int po = 0, pi = 0;
+    int po = 0, pi = 0, ncut = 0;
+    uint2 sm = make_uint2(0, 0);
+    bool lo = false, li = false;
     if (go) {
         po = optr2[j];
         pi = iptr2[j];
-        const uint2 sm = emask[i];                     // light rows: the survivors' bits
-        if (r.oe - r.ob <= HEAVY) emit_mask(g.oadj, r.ob, sm.x, (int)i, newidx, oadj2, po);
-        if (r.ie - r.ib <= HEAVY) emit_mask(g.iadj, r.ib, sm.y, (int)i, newidx, iadj2, pi);
+        sm = emask[i];                                 // light rows: the survivors' bits
+        lo = r.oe - r.ob <= HEAVY;
+        li = r.ie - r.ib <= HEAVY;
+        if (pk.pnin) {
+            if (!(lo && li)) *pk.bad = 1;              // a warp-path row: k_tile_pack rebuilds the pack
+            const int tb = j & ~(TILE - 1);
+            if (lo) pk.pnout[j] = emit_mask_pack(g.oadj, r.ob, sm.x, (int)i, newidx, oadj2, po, tb, ncut);
+            if (li) pk.pnin[j] = emit_mask_pack(g.iadj, r.ib, sm.y, (int)i, newidx, iadj2, pi, tb, ncut);
+        } else {
+            if (lo) emit_mask(g.oadj, r.ob, sm.x, (int)i, newidx, oadj2, po);
+            if (li) emit_mask(g.iadj, r.ib, sm.y, (int)i, newidx, iadj2, pi);
+        }
+    }
+    if (pk.pnin) {
+        // cut edges: lanes of one tile reserve their slots with one atomic per warp and tile
+        const int tile = go ? j / TILE : -1;
+        const unsigned grp = __match_any_sync(FULL, tile);
+        const int leader = __ffs(grp) - 1;
+        // alive lanes hold increasing j, so between two lanes of one tile there are only lanes
+        // of that tile or dead ones (ncut 0): the offset is an exclusive warp scan relative to
+        // the group's leader
+        const int excl = warp_incl_scan(ncut, lane) - ncut;
+        const int pre = excl - __shfl_sync(FULL, excl, leader);
+        const int tot = __reduce_add_sync(grp, ncut);
+        int base = 0;
+        if (go && lane == leader && tot) base = atomicAdd(pk.ext_cnt + tile, tot);
+        base = __shfl_sync(FULL, base, leader);
+        if (go && ncut) {
+            const int tb = j & ~(TILE - 1);
+            int2* E = pk.ext + (int64_t)__ldg(optr2 + tb) + __ldg(iptr2 + tb);
+            int at = base + pre;
+            if (lo) emit_cut(g.oadj, r.ob, sm.x, newidx, j, tb, PK_DIR, E, at);
+            if (li) emit_cut(g.iadj, r.ib, sm.y, newidx, j, tb, 0, E, at);
+        }
     }
     SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
     emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred, chunked, false);

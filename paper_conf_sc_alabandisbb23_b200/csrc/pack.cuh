@@ -34,6 +34,8 @@ constexpr unsigned EXT_DIR = 0x8000u;
 // used) marks a row with more than SLOTS intra-tile neighbours (SLOW_MARK).
 constexpr unsigned long long PSLOTS_EMPTY = 0x0800080008000800ull;
 static_assert(PACK_TT == 0x800, "PSLOTS_EMPTY encodes PACK_TT");
+static_assert(PK_EMPTY == PSLOTS_EMPTY && PK_DIR == (int)EXT_DIR && PK_SLOW == SLOW_MARK && PACK_TT == TILE,
+              "the compaction scatter writes the same pack layout (kernels.cuh PackOut)");
 
 __device__ __forceinline__ int ppull(const int* sig, unsigned long long src, int val) {
     const unsigned lo = (unsigned)src, hi = (unsigned)(src >> 32);

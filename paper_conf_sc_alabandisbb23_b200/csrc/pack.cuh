@@ -587,26 +587,35 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             const int lane = tid;
             int got = 0, stop = 0;
             for (unsigned miss = 0;; miss += claim) {
-                if (lane == 0) stop = (ctr[1] == 0 || ctr[2]) ? 1 : 0;   // fixed point / watchdog
-                if (__shfl_sync(FULL, stop, 0)) break;
+                // the stop words and the cursor step are requested together (one round trip);
+                // positions taken after the fixed point are harmless
                 unsigned long long pos = 0;
-                if (lane == 0) pos = atomicAdd(Q.ctr, (unsigned long long)claim);
+                if (lane == 0) {
+                    const unsigned long long pend = ctr[1], halt = ctr[2];
+                    pos = atomicAdd(Q.ctr, (unsigned long long)claim);
+                    stop = (pend == 0 || halt) ? 1 : 0;           // fixed point / watchdog
+                }
+                if (__shfl_sync(FULL, stop, 0)) break;
                 pos = __shfl_sync(FULL, pos, 0) + (unsigned)lane;
                 bool mine = false;
-                int c = 0;
+                int c = 0, seen = 0;
                 if (lane < claim) {
                     const unsigned long long k = pos / (unsigned)ntiles;
                     const int off = (int)(pos - k * (unsigned)ntiles);
                     c = (k & 1) ? ntiles - 1 - off : off;
-                    mine = ((volatile int*)Q.tstate)[c] == 1 && atomicCAS(Q.tstate + c, 1, 2) == 1;
+                    // the seen byte is read with the state (a tile visited between this read
+                    // and the claim only gets one extra full visit)
+                    const int st = ((volatile int*)Q.tstate)[c];
+                    seen = ((volatile uint8_t*)Q.tseen)[c];
+                    mine = st == 1 && atomicCAS(Q.tstate + c, 1, 2) == 1;
                 }
                 const unsigned m = __ballot_sync(FULL, mine);
                 if (mine) {
                     const int slot = __popc(m & ((1u << lane) - 1));
                     s_claim[slot] = c;
                     atomicAdd(&dc->passes, 1ull);                  // tile visits of the phase
-                    s_seen[slot] = Q.tseen[c];
-                    Q.tseen[c] = 1;
+                    s_seen[slot] = (uint8_t)seen;
+                    if (!seen) Q.tseen[c] = 1;
                 }
                 if (m) { got = __popc(m); break; }
                 if (miss >= (unsigned)ntiles) {                    // a whole sweep without work

@@ -29,7 +29,6 @@ struct Plan {
     int2* hcnt;                          // survivors of a vertex's long rows
     int cb;                              // which chunk buffer belongs to the current graph
     int nchunks_cur;                     // chunks of the current graph
-    int32_t *dbg_tmp;                    // unused placeholder
     DevCounters* dc;                     // device counters
     DevCounters* hc;                     // pinned host mirror
     int32_t* u_rp;                       // batched: union CSR and union labels

@@ -218,9 +218,10 @@ static int run_partitioned(std::vector<PRank*>& R, Exchange& X, int32_t n, uint3
                 int pass = 0, batch = 2;
                 for (;;) {
                     for (int k = 0; k < batch; k++, pass++) {
-                        part::k_prop_rows<<<gridn(std::max(Q.nloc, 1)), 256, 0, s>>>(Q.nloc, Q.rb, Q.rp, Q.wci, Q.odeg,
-                                                                                     Q.sig + n, ring, pass);
-                        part::k_prop_cols<<<gridn(n), 256, 0, s>>>(n, Q.cp, Q.cr, Q.ideg, Q.sig, ring, pass);
+                        part::k_prop_rows<<<gridn(std::max(Q.nloc, 1), 256 * part::PART_RPT), 256, 0, s>>>(
+                            Q.nloc, Q.rb, Q.rp, Q.wci, Q.odeg, Q.sig + n, ring, pass);
+                        part::k_prop_cols<<<gridn(n, 256 * part::PART_RPT), 256, 0, s>>>(n, Q.cp, Q.cr, Q.ideg, Q.sig,
+                                                                                         ring, pass);
                         launches += 2;
                     }
                     CKM(cudaGetLastError());

@@ -66,33 +66,59 @@ static __global__ void k_csc_rows(int32_t nrows, int32_t rb, const int32_t* __re
 // owned sources, in-columns of every destination.  Owner-writes in place.  Ring protocol
 // as in kernels.cuh: the rows kernel (first of the pass) clears ring[p+1]; both return
 // at once if pass p-1 changed nothing; a raise sets ring[p].
-static __global__ void k_prop_rows(int32_t nrows, int32_t rb, const int32_t* __restrict__ rp, const int32_t* __restrict__ wci,
-                            const int32_t* __restrict__ odeg, int32_t* __restrict__ vout, int* __restrict__ ring, int pass) {
+// Local Phase-2 passes with block-local iteration ("every thread block internally
+// iterates until none of the edges assigned to it propagate any more values"): a CTA owns
+// PART_RPT x blockDim consecutive rows (columns) and repeats its pulls until a block round
+// raises nothing, so chains inside its range converge in one launch instead of one launch
+// per hop.  Other CTAs' values are read through L2 (ld.cg); the ring word of the pass is set
+// if anything rose (the driver repeats passes until one raises nothing: a fixed point).
+constexpr int PART_RPT = 4;
+static __global__ void __launch_bounds__(256) k_prop_rows(int32_t nrows, int32_t rb, const int32_t* __restrict__ rp,
+                                                          const int32_t* __restrict__ wci, const int32_t* __restrict__ odeg,
+                                                          int32_t* __restrict__ vout, int* __restrict__ ring, int pass) {
     if (blockIdx.x == 0 && threadIdx.x == 0) ring[(pass + 1) & (RING - 1)] = 0;
     if (pass > 0 && ld_vol(ring + ((pass - 1) & (RING - 1))) == 0) return;
-    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    bool ch = false;
-    if (r < nrows) {
-        const int u = rb + (int)r;
-        const int y0 = ld_cg(vout + u);
-        int y = y0;
-        for (int e = rp[r]; e < rp[r] + odeg[r]; e++) y = max(y, ld_cg(vout + wci[e]));
-        if (y > y0) { vout[u] = y; ch = true; }
+    const int64_t r0 = (int64_t)blockIdx.x * blockDim.x * PART_RPT + threadIdx.x;
+    int any = 0;
+    for (;;) {
+        int ch = 0;
+#pragma unroll
+        for (int k = 0; k < PART_RPT; k++) {
+            const int64_t r = r0 + (int64_t)k * blockDim.x;
+            if (r >= nrows) break;
+            const int u = rb + (int)r;
+            const int y0 = ld_cg(vout + u);
+            int y = y0;
+            for (int e = rp[r], ee = rp[r] + odeg[r]; e < ee; e++) y = max(y, ld_cg(vout + wci[e]));
+            if (y > y0) { __stcg(vout + u, y); ch = 1; }
+        }
+        if (!__syncthreads_or(ch)) break;
+        any = 1;
     }
-    if (__any_sync(FULL, ch) && (threadIdx.x & 31) == 0) ring[pass & (RING - 1)] = 1;
+    if (any && threadIdx.x == 0) ring[pass & (RING - 1)] = 1;
 }
-static __global__ void k_prop_cols(int32_t n, const int32_t* __restrict__ cp, const int32_t* __restrict__ cr,
-                            const int32_t* __restrict__ ideg, int32_t* __restrict__ vin, int* __restrict__ ring, int pass) {
+static __global__ void __launch_bounds__(256) k_prop_cols(int32_t n, const int32_t* __restrict__ cp, const int32_t* __restrict__ cr,
+                                                          const int32_t* __restrict__ ideg, int32_t* __restrict__ vin,
+                                                          int* __restrict__ ring, int pass) {
     if (pass > 0 && ld_vol(ring + ((pass - 1) & (RING - 1))) == 0) return;
-    const int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    bool ch = false;
-    if (w < n && ideg[w] > 0) {
-        const int x0 = ld_cg(vin + w);
-        int x = x0;
-        for (int e = cp[w]; e < cp[w] + ideg[w]; e++) x = max(x, ld_cg(vin + cr[e]));
-        if (x > x0) { vin[w] = x; ch = true; }
+    const int64_t w0 = (int64_t)blockIdx.x * blockDim.x * PART_RPT + threadIdx.x;
+    int any = 0;
+    for (;;) {
+        int ch = 0;
+#pragma unroll
+        for (int k = 0; k < PART_RPT; k++) {
+            const int64_t w = w0 + (int64_t)k * blockDim.x;
+            if (w >= n) break;
+            if (ideg[w] == 0) continue;
+            const int x0 = ld_cg(vin + w);
+            int x = x0;
+            for (int e = cp[w], ee = cp[w] + ideg[w]; e < ee; e++) x = max(x, ld_cg(vin + cr[e]));
+            if (x > x0) { __stcg(vin + w, x); ch = 1; }
+        }
+        if (!__syncthreads_or(ch)) break;
+        any = 1;
     }
-    if (__any_sync(FULL, ch) && (threadIdx.x & 31) == 0) ring[pass & (RING - 1)] = 1;
+    if (any && threadIdx.x == 0) ring[pass & (RING - 1)] = 1;
 }
 
 // ------------------------------------------------------------------ Phase 3 + trim

@@ -56,3 +56,16 @@ def test_partition_rows_balanced():
         assert b[0] == 0 and b[-1] == 10000 and all(b[i] <= b[i + 1] for i in range(P))
         load = [rp[b[i + 1]] - rp[b[i]] for i in range(P)]
         assert max(load) - min(load) <= 2 * 50 + 1
+
+
+def test_levels_and_host_argument_errors_without_gpu():
+    L = E.lib()
+    p = ctypes.c_void_p(16)
+    depth = ctypes.c_int32(7)
+    assert L.ecl_scc_levels(-1, 0, None, None, None, None, None, None, None) == E.EINVAL
+    assert L.ecl_scc_levels(3, 0, p, None, None, p, None, None, None) == E.EINVAL     # NULL labels
+    assert L.ecl_scc_levels(0, 0, None, None, None, None, ctypes.byref(depth), None, None) == E.OK
+    assert depth.value == 0                                                          # empty graph
+    assert L.ecl_scc_host(-1, 0, None, None, None, None, None, None) == E.EINVAL
+    assert L.ecl_scc_host(3, 2, p, None, p, None, None, None) == E.EINVAL             # NULL col_idx
+    assert L.ecl_scc_host(0, 0, None, None, None, None, None, None) == E.OK

@@ -495,6 +495,8 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                 CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_async, PACK_TH, pack_dyn_smem()));
                 CK(cudaGetDevice(&dev));
                 CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+                // tuning knob ECL_SCC_ASYNC_CTAS: resident CTAs per SM used (<= what fits)
+                if (const char* e = getenv("ECL_SCC_ASYNC_CTAS")) per_sm = std::min(per_sm, std::max(1, atoi(e)));
                 p->aq_resident = std::max(1, per_sm) * sms;
                 if (getenv("ECL_SCC_DEBUG")) fprintf(stderr, "[ecl_scc] k_prop_async: %d CTAs per SM\n", per_sm);
             }

@@ -502,11 +502,16 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             }
             AsyncQ Q{p->aq_state, p->aq_seen, p->aq_ctr};
             // tiles per claim: runs pay when there are many tiles per resident CTA (measured:
-            // C4 iteration 1, 18 tiles per CTA, best at 8; C2, ~1 tile per CTA, best at 1)
+            // C4 iteration 1, 18 tiles per CTA, best at 8-16; C2, ~1 tile per CTA, best at 1);
+            // claim = clamp(tiles / resident CTAs, 1, 16) (C4 lex 19.8 -> 19.2 ms vs
+            // tiles / (2 x resident) capped at 8; blocked8 unchanged)
             static int claim_env = -1;                      // tuning knob ECL_SCC_CLAIM
             if (claim_env < 0) claim_env = getenv("ECL_SCC_CLAIM") ? std::min(32, std::max(1, atoi(getenv("ECL_SCC_CLAIM")))) : 0;
+            static int claim_div = -1, claim_max = -1;      // tuning knobs of the adaptive rule
+            if (claim_div < 0) claim_div = getenv("ECL_SCC_CLAIM_DIV") ? std::max(1, atoi(getenv("ECL_SCC_CLAIM_DIV"))) : 1;
+            if (claim_max < 0) claim_max = getenv("ECL_SCC_CLAIM_MAX") ? std::min(32, std::max(1, atoi(getenv("ECL_SCC_CLAIM_MAX")))) : 16;
             const int claim = claim_env ? claim_env
-                                        : (int)std::min<int64_t>(8, std::max<int64_t>(1, ntiles / (2 * p->aq_resident)));
+                                        : (int)std::min<int64_t>(claim_max, std::max<int64_t>(1, ntiles / (claim_div * p->aq_resident)));
             CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
             CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
             p->launches += 2;

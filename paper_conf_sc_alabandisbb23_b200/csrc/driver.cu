@@ -483,7 +483,7 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                 const size_t nt = (size_t)p->dirty_cap;
                 cudaError_t e = cudaMalloc((void**)&p->aq_state, nt * 4);
                 if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_seen, nt);
-                if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_ctr, 32);
+                if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_ctr, AQ_WORDS * sizeof(unsigned long long));
                 if (e != cudaSuccess) {
                     cudaGetLastError();
                     return fail(ECL_SCC_ENOMEM, "async queue allocation: %s", cudaGetErrorString(e));

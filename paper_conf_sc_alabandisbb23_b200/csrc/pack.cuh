@@ -506,10 +506,13 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
 // visit saw its final inputs: the Phase-2 fixed point (Alg. 1 l.7-14).  Values are
 // written (st.cg) and fenced before the marks; a claimer fences after its claim and reads
 // through L2, so it sees every value written before the state change it observed.
+// the cursor, the pending count and the stop word sit in separate 128-byte lines: claimers
+// hammer the cursor while visits count marks and finishes on the pending word
+constexpr int AQ_CUR = 0, AQ_PEND = 16, AQ_STOP = 32, AQ_WORDS = 48;
 struct AsyncQ {
     int* tstate;                  // [ntiles]
     uint8_t* tseen;               // [ntiles] visited in this phase
-    unsigned long long* ctr;      // [0] cursor, [1] pending, [2] stop
+    unsigned long long* ctr;      // [AQ_CUR] cursor, [AQ_PEND] pending, [AQ_STOP] stop
 };
 __device__ __forceinline__ void aq_mark(const AsyncQ& Q, int t) {
     int st = *(volatile int*)(Q.tstate + t);
@@ -519,14 +522,14 @@ __device__ __forceinline__ void aq_mark(const AsyncQ& Q, int t) {
         if (old == st) break;
         st = old;
     }
-    if (st == 0) atomicAdd(Q.ctr + 1, 1ull);
+    if (st == 0) atomicAdd(Q.ctr + AQ_PEND, 1ull);
 }
 static __global__ void k_async_init(AsyncQ Q, int ntiles) {
     for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < ntiles; t += gridDim.x * blockDim.x) {
         Q.tstate[t] = 1;
         Q.tseen[t] = 0;
     }
-    if (blockIdx.x == 0 && threadIdx.x == 0) { Q.ctr[0] = 0; Q.ctr[1] = (unsigned long long)ntiles; Q.ctr[2] = 0; }
+    if (blockIdx.x == 0 && threadIdx.x == 0) { Q.ctr[AQ_CUR] = 0; Q.ctr[AQ_PEND] = (unsigned long long)ntiles; Q.ctr[AQ_STOP] = 0; }
 }
 
 constexpr int CLAIM_MAX = 32;     // sweep positions per claim (a CTA's run of tiles), <= a warp
@@ -591,8 +594,8 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
                 // positions taken after the fixed point are harmless
                 unsigned long long pos = 0;
                 if (lane == 0) {
-                    const unsigned long long pend = ctr[1], halt = ctr[2];
-                    pos = atomicAdd(Q.ctr, (unsigned long long)claim);
+                    const unsigned long long pend = ctr[AQ_PEND], halt = ctr[AQ_STOP];
+                    pos = atomicAdd(Q.ctr + AQ_CUR, (unsigned long long)claim);
                     stop = (pend == 0 || halt) ? 1 : 0;           // fixed point / watchdog
                 }
                 if (__shfl_sync(FULL, stop, 0)) break;
@@ -622,7 +625,7 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
                     __nanosleep(256);
                     if (lane == 0 && clock64() - t0 > (1ll << 36)) {   // ~30 s idle: protocol bug
                         atomicExch(&dc->err, 3);
-                        atomicExch(Q.ctr + 2, 1ull);
+                        atomicExch(Q.ctr + AQ_STOP, 1ull);
                     }
                 }
             }
@@ -648,7 +651,7 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             __threadfence();
             __syncthreads();                                      // marks (pending++) before finish
             if (tid == 0) {
-                if (atomicCAS(Q.tstate + tile, 2, 0) == 2) atomicAdd(Q.ctr + 1, ~0ull);
+                if (atomicCAS(Q.tstate + tile, 2, 0) == 2) atomicAdd(Q.ctr + AQ_PEND, ~0ull);
                 else atomicExch(Q.tstate + tile, 1);
             }
         }

@@ -828,6 +828,7 @@ struct TileSmem {
     unsigned* s_fout;
     unsigned short* s_queue;      // drain item queues; level-sweep order + level starts
     uint8_t* s_lv;                // level-sweep: intra-tile level of each vertex
+    unsigned long long* s_acc;    // pack kernels: per-CTA visited vertices / edges (thread 0), flushed once
 };
 
 // pull of one vertex over its slots (and its global row when it is a slow row)

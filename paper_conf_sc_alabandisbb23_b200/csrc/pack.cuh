@@ -321,8 +321,8 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
         *(int4*)(s_out + v0) = make_int4(y0[0], y0[1], y0[2], y0[3]);
     }
     if (tid == 0) {                                   // roofline accounting (SURVEY 8(d) terms)
-        atomicAdd(&dc->visit_v, (unsigned long long)cnt);
-        atomicAdd(&dc->visit_e, (unsigned long long)(__ldg(g.optr + base + cnt) - __ldg(g.optr + base)));
+        S.s_acc[0] += (unsigned long long)cnt;        // per CTA; the kernel adds it to dc once
+        S.s_acc[1] += (unsigned long long)(__ldg(g.optr + base + cnt) - __ldg(g.optr + base));
     }
     __syncthreads();
     for (int i = tid; i < ne; i += PACK_TH) {
@@ -461,11 +461,13 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
     S.s_out = S.s_in + PACK_TT + 4;
     S.s_nin = (unsigned long long*)(S.s_out + PACK_TT + 4);
     S.s_nout = S.s_nin + PACK_TT;
-    if (threadIdx.x == 0) { S.s_in[PACK_TT] = 0; S.s_out[PACK_TT] = 0; }   // <= every priority
+    __shared__ unsigned long long s_acc[3];
+    if (threadIdx.x == 0) { S.s_in[PACK_TT] = 0; S.s_out[PACK_TT] = 0; s_acc[0] = s_acc[1] = s_acc[2] = 0; }
     S.s_fin = s_fin;
     S.s_fout = s_fout;
     S.s_queue = s_queue;
     S.s_lv = nullptr;
+    S.s_acc = s_acc;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + PACK_TT - 1) / PACK_TT;
     const int tid = threadIdx.x;
@@ -488,6 +490,10 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
         __syncthreads();
     }
     if (ch_any && tid == 0) dc->changed[pass & (RING - 1)] = 1;
+    if (tid == 0 && s_acc[0]) {
+        atomicAdd(&dc->visit_v, s_acc[0]);
+        atomicAdd(&dc->visit_e, s_acc[1]);
+    }
 }
 
 // ------------------------------------------------------------------ asynchronous mode
@@ -574,13 +580,15 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
     S.s_out = S.s_in + PACK_TT + 4;
     S.s_nin = (unsigned long long*)(S.s_out + PACK_TT + 4);
     S.s_nout = S.s_nin + PACK_TT;
+    __shared__ unsigned long long s_acc[3];            // visited vertices, edges, tiles (flushed at the end)
     S.s_fin = s_fin;
     S.s_fout = s_fout;
     S.s_queue = s_queue;
     S.s_lv = nullptr;
+    S.s_acc = s_acc;
     const int tid = threadIdx.x;
     const int ntiles = (g.na + PACK_TT - 1) / PACK_TT;
-    if (tid == 0) { S.s_in[PACK_TT] = 0; S.s_out[PACK_TT] = 0; }
+    if (tid == 0) { S.s_in[PACK_TT] = 0; S.s_out[PACK_TT] = 0; s_acc[0] = s_acc[1] = s_acc[2] = 0; }
     volatile unsigned long long* ctr = Q.ctr;
     long long t0 = clock64();
     for (;;) {
@@ -616,7 +624,7 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
                 if (mine) {
                     const int slot = __popc(m & ((1u << lane) - 1));
                     s_claim[slot] = c;
-                    atomicAdd(&dc->passes, 1ull);                  // tile visits of the phase
+
                     s_seen[slot] = (uint8_t)seen;
                     if (!seen) Q.tseen[c] = 1;
                 }
@@ -631,6 +639,7 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             }
             if (lane == 0) {
                 s_nclaim = got;
+                s_acc[2] += (unsigned long long)got;       // tile visits of the phase
                 if (got) t0 = clock64();
             }
             __threadfence();                                      // claims before the value reads
@@ -656,6 +665,11 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             }
         }
         __syncthreads();                                          // s_claim is rewritten next
+    }
+    if (tid == 0) {
+        if (s_acc[0]) atomicAdd(&dc->visit_v, s_acc[0]);
+        if (s_acc[1]) atomicAdd(&dc->visit_e, s_acc[1]);
+        if (s_acc[2]) atomicAdd(&dc->passes, s_acc[2]);
     }
 }
 

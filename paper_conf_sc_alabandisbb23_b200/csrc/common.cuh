@@ -26,8 +26,8 @@ struct WGraph {
 
 // Counters the host reads back once per outer iteration.
 struct DevCounters {
-    int4 totals;                     // after a compaction scan: (na', m_out', m_in', 0)
-    unsigned long long kept;         // edges kept by Phase 3 (before trim)
+    int4 totals;                     // after a compaction scan: (na', m_out', m_in', edges kept
+                                     // by Phase 3 before trim)
     unsigned long long passes;       // Phase-2 passes that did work
     int nchunks;                     // heavy-row chunks of the current working graph
     int err;                         // validation error

@@ -305,7 +305,6 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     const int64_t nw = (int64_t)grid * (TPB / WARP);
     const int nc = p->nchunks_cur, chunked = nc > 0;
     const Chunk* cur = chunk_buf(p, p->cb);
-    CK(cudaMemsetAsync(&p->dc->kept, 0, sizeof(unsigned long long), s));
     CK(cudaMemsetAsync(&p->dc->nchunks, 0, sizeof(int), s));
     CK(cudaMemsetAsync(&p->dc->pack_bad, 0, sizeof(int), s));
     // the scatter writes the next graph's tile pack when Phase 2 will use one (no long rows
@@ -316,10 +315,10 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
         if (int r = ensure_pack(p)) return r;
         pk = PackOut{p->pnin, p->pnout, p->ext, p->ext_cnt, &p->dc->pack_bad};
     }
-    p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, &p->dc->kept, chunked, p->hcnt, p->emask);
+    p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, chunked, p->hcnt, p->emask);
     if (chunked) {
         p->launches += 2;
-        k_keep_chunks<FIRST><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kin, p->kout, &p->dc->kept);
+        k_keep_chunks<FIRST><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kin, p->kout);
         k_count_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kin, p->kout, p->chunk_cnt, p->hcnt);
     }
     p->launches++; k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
@@ -753,7 +752,8 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             const int4 t = p->hc->totals;
             const int nchunks = p->hc->nchunks;
             p->nchunks_cur = nchunks;
-            if (st && iter >= 2 && iter - 2 < ECL_SCC_TRACE_MAX) st->edges_kept[iter - 2] = (int64_t)p->hc->kept;
+            // kept edges (before trim) = the kept out-degrees summed by the compaction scan
+            if (st && iter >= 2 && iter - 2 < ECL_SCC_TRACE_MAX) st->edges_kept[iter - 2] = (int64_t)p->hc->totals.w;
             if (t.y != t.z) return fail(ECL_SCC_ECUDA, "internal: CSR/CSC survivor mismatch %d vs %d", t.y, t.z);
             if (nchunks > p->chunk_cap) return fail(ECL_SCC_ECUDA, "internal: heavy chunk list overflow");
             g = WGraph{p->act[ob], p->optr[ob], p->oadj[ob], p->iptr[ob], p->iadj[ob], t.x};

@@ -22,7 +22,7 @@ struct Plan {
     int32_t* newidx;                     // old local -> new local (-1: leaves)
     int2* cnt;                           // per-vertex surviving (out, in) degree
     uint2* emask;                        // light rows: kept, then surviving, entries as bit masks
-    int4 *wsum, *wscan;                  // per-warp compaction counts and their prefix
+    int4 *wsum, *wscan;                  // per-warp compaction counts (alive, out, in, kept) and their prefix
     void* bsum;                          // scan block totals
     void* chunks;                        // long-row chunks, 2 x Chunk[chunk_cap] (current / next graph)
     int* chunk_cnt;                      // survivors per chunk of the current graph

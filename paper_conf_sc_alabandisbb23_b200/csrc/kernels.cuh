@@ -336,13 +336,12 @@ __device__ __forceinline__ void emit_cut(const int32_t* __restrict__ adj, int b,
     }
 }
 
-// kept in/out degree per local vertex, plus the number of kept edges
+// kept in/out degree per local vertex (light rows: also the kept entries as bit masks)
 constexpr int TPB_COMPACT = 256;     // block size of the compaction kernels (driver TPB)
 template <bool FIRST>
 static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                              int32_t* __restrict__ kin, int32_t* __restrict__ kout,
-                             unsigned long long* __restrict__ kept, int chunked, int2* __restrict__ hcnt,
-                             uint2* __restrict__ emask) {
+                             int chunked, int2* __restrict__ hcnt, uint2* __restrict__ emask) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
@@ -359,19 +358,11 @@ static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, con
         emask[i] = make_uint2(mo, mi);
         if (chunked) hcnt[i] = make_int2(0, 0);
     }
-    // one atomic per block (one per warp on a single address serialised ~0.5M atomics in L2)
-    __shared__ int s_kept[TPB_COMPACT / WARP];
-    const int s = warp_sum(co);
-    if (lane == 0) s_kept[threadIdx.x >> 5] = s;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        int t = 0;
-        for (int w = 0; w < (int)(blockDim.x >> 5); w++) t += s_kept[w];
-        if (t) atomicAdd(kept, (unsigned long long)t);
-    }
+    // the number of kept edges is the sum of the kept out-degrees: k_compact_count carries it
+    // through the compaction scan (lane .w), so no kernel counts it on a single address
 }
 
-// per-vertex surviving (kept, not trimmed) degrees and per-warp totals (alive, out, in)
+// per-vertex surviving (kept, not trimmed) degrees and per-warp totals (alive, out, in, kept)
 template <bool FIRST, bool TRIM>
 static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                 const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
@@ -404,8 +395,9 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
     }
     if (r.valid) cnt[i] = make_int2(nout, nin);
     const int alive = (nout + nin) > 0;
-    const int sa = warp_sum(alive), so = warp_sum(nout), si = warp_sum(nin);
-    if (lane == 0) wsum[i >> 5] = make_int4(sa, so, si, 0);
+    const int kept = r.valid ? kout[i] : 0;             // kept (pre-trim) out-degree, chunks included
+    const int sa = warp_sum(alive), so = warp_sum(nout), si = warp_sum(nin), sk = warp_sum(kept);
+    if (lane == 0) wsum[i >> 5] = make_int4(sa, so, si, sk);
 }
 
 // New numbering, Phase 1 reset of the survivors (rule R2), final labels of
@@ -617,8 +609,7 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
 template <bool FIRST>
 static __global__ void __launch_bounds__(256) k_keep_chunks(WGraph g, const Chunk* __restrict__ chunks, int nchunks,
                                                             const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
-                                                            int32_t* __restrict__ kin, int32_t* __restrict__ kout,
-                                                            unsigned long long* __restrict__ kept) {
+                                                            int32_t* __restrict__ kin, int32_t* __restrict__ kout) {
     const int lane = threadIdx.x & 31;
     const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (c >= nchunks) return;
@@ -631,7 +622,6 @@ static __global__ void __launch_bounds__(256) k_keep_chunks(WGraph g, const Chun
     cc = warp_sum(cc);
     if (lane == 0 && cc) {
         atomicAdd(k.dir ? kin + k.i : kout + k.i, cc);
-        if (!k.dir) atomicAdd(kept, (unsigned long long)cc);
     }
 }
 template <bool FIRST, bool TRIM>

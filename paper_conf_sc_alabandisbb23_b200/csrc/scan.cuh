@@ -21,9 +21,10 @@ struct I1 {
 struct __align__(16) I3 {
     int x, y, z, w;
     __device__ __forceinline__ static I3 zero() { return {0, 0, 0, 0}; }
-    __device__ __forceinline__ I3 operator+(const I3& o) const { return {x + o.x, y + o.y, z + o.z, 0}; }
+    __device__ __forceinline__ I3 operator+(const I3& o) const { return {x + o.x, y + o.y, z + o.z, w + o.w}; }
     __device__ __forceinline__ I3 shfl_up(int d) const {
-        return {__shfl_up_sync(FULL, x, d), __shfl_up_sync(FULL, y, d), __shfl_up_sync(FULL, z, d), 0};
+        return {__shfl_up_sync(FULL, x, d), __shfl_up_sync(FULL, y, d), __shfl_up_sync(FULL, z, d),
+                __shfl_up_sync(FULL, w, d)};
     }
 };
 

@@ -113,8 +113,17 @@ static __global__ void __launch_bounds__(256) k_csc_scatter(int32_t n, const int
                     iadj[o[q] + (RANK ? r[q] : atomicAdd(cursor + w[q], 1))] = (int32_t)u;
                 }
         }
-    nloc = __reduce_add_sync(FULL, nloc);
-    if (lane == 0 && nloc) atomicAdd(local_e, (unsigned long long)nloc);
+    {   // one atomic per block on the single counter (one per warp serialised ~0.5M in L2)
+        __shared__ unsigned s_loc[256 / WARP];
+        nloc = __reduce_add_sync(FULL, nloc);
+        if (lane == 0) s_loc[threadIdx.x >> 5] = nloc;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            unsigned t = 0;
+            for (int w = 0; w < (int)(blockDim.x >> 5); w++) t += s_loc[w];
+            if (t) atomicAdd(local_e, (unsigned long long)t);
+        }
+    }
     unsigned hm = __ballot_sync(FULL, valid && e - b > HEAVY);
     while (hm) {
         const int src = __ffs(hm) - 1;

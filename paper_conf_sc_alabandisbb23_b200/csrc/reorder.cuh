@@ -15,6 +15,7 @@ namespace reo {
 
 constexpr int CELL_SHIFT = 11;        // ~2048 vertices per cell
 constexpr int NOLAB = 0x7FFFFFFF;
+constexpr int BFS_STAGE = 4096;       // claimed vertices staged per block and level
 
 __device__ __forceinline__ bool is_seed(int v) {
     return (prio_hash((uint32_t)v ^ 0x5BD1E995u) & ((1u << CELL_SHIFT) - 1)) == 0;
@@ -33,8 +34,14 @@ static __global__ void k_bfs_level(int32_t* __restrict__ fa, int32_t* __restrict
     const int nf = ld_vol(cnt + r % 3);
     if (blockIdx.x == 0 && threadIdx.x == 0) cnt[(r + 2) % 3] = 0;
     const int lane = threadIdx.x & 31;
-    // whole warps iterate (ballots below); appends are warp-aggregated: one atomic per warp
-    // and round instead of one per claimed vertex on a single counter
+    // whole warps iterate (ballots below); claimed vertices are staged in shared memory and
+    // appended with ONE global atomic per block at the end (per-warp atomics on the single
+    // frontier counter serialised in L2); a full stage spills with per-warp atomics
+    __shared__ int s_buf[BFS_STAGE];
+    __shared__ int s_n, s_base;
+    if (threadIdx.x == 0) s_n = 0;
+    __syncthreads();
+    int* gcnt = cnt + (r + 1) % 3;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t k0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x - lane; k0 < nf; k0 += stride) {
         const int64_t k = k0 + lane;
@@ -63,13 +70,26 @@ static __global__ void k_bfs_level(int32_t* __restrict__ fa, int32_t* __restrict
                 const unsigned m = __ballot_sync(FULL, got);
                 if (m) {
                     int at = 0;
-                    if (lane == __ffs(m) - 1) at = atomicAdd(cnt + (r + 1) % 3, __popc(m));
+                    if (lane == __ffs(m) - 1) at = atomicAdd(&s_n, __popc(m));
                     at = __shfl_sync(FULL, at, __ffs(m) - 1);
-                    if (got) next[at + __popc(m & ((1u << lane) - 1))] = w[q];
+                    const int slot = at + __popc(m & ((1u << lane) - 1));
+                    if (got && slot < BFS_STAGE) s_buf[slot] = w[q];
+                    const unsigned sp = __ballot_sync(FULL, got && slot >= BFS_STAGE);
+                    if (sp) {                                   // stage full: straight to the frontier
+                        int g0 = 0;
+                        if (lane == __ffs(sp) - 1) g0 = atomicAdd(gcnt, __popc(sp));
+                        g0 = __shfl_sync(FULL, g0, __ffs(sp) - 1);
+                        if (got && slot >= BFS_STAGE) next[g0 + __popc(sp & ((1u << lane) - 1))] = w[q];
+                    }
                 }
             }
         }
     }
+    __syncthreads();
+    const int ns = min(s_n, BFS_STAGE);
+    if (threadIdx.x == 0) s_base = ns ? atomicAdd(gcnt, ns) : 0;
+    __syncthreads();
+    for (int i = threadIdx.x; i < ns; i += blockDim.x) next[s_base + i] = s_buf[i];
 }
 static __global__ void k_seed2(int32_t n, int32_t* __restrict__ cell, int32_t* __restrict__ front, int* __restrict__ cnt) {
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {

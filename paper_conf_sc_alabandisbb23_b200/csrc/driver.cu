@@ -92,8 +92,14 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
         e = e ? e : A((void**)&p->oadj[b], m * 4);
         e = e ? e : A((void**)&p->iadj[b], m * 4);
     }
-    e = e ? e : A((void**)&p->kin, n1 * 4);
-    e = e ? e : A((void**)&p->kout, n1 * 4);
+    // one allocation, two views: the compaction's interleaved kept degrees kio[i] = {in, out}
+    // (one 8-byte gather per far end in the trim), and two int arrays kin / kout of n+1 for
+    // the ingest, the relabelling, the tail and the levels (never used at the same time)
+    e = e ? e : A((void**)&p->kin, 2 * n1 * 4);
+    if (e == cudaSuccess) {
+        p->kout = p->kin + n1;
+        p->kio = (int2*)p->kin;
+    }
     e = e ? e : A((void**)&p->newidx, n1 * 4);
     e = e ? e : A((void**)&p->cnt, n1 * sizeof(int2));
     e = e ? e : A((void**)&p->emask, n1 * sizeof(uint2));
@@ -137,7 +143,7 @@ void plan_free(Plan* p) {
         cudaFree(p->act[b]); cudaFree(p->cin[b]); cudaFree(p->cout[b]);
         cudaFree(p->optr[b]); cudaFree(p->iptr[b]); cudaFree(p->oadj[b]); cudaFree(p->iadj[b]);
     }
-    cudaFree(p->kin); cudaFree(p->kout); cudaFree(p->newidx); cudaFree(p->cnt); cudaFree(p->emask);
+    cudaFree(p->kin); cudaFree(p->newidx); cudaFree(p->cnt); cudaFree(p->emask);
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
     cudaFree(p->chunk_cnt); cudaFree(p->hcnt);
     cudaFree(p->dirty); cudaFree(p->lvl);
@@ -315,23 +321,23 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
         if (int r = ensure_pack(p)) return r;
         pk = PackOut{p->pnin, p->pnout, p->ext, p->ext_cnt, &p->dc->pack_bad};
     }
-    p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, chunked, p->hcnt, p->emask);
+    p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kio, chunked, p->hcnt, p->emask);
     if (chunked) {
         p->launches += 2;
-        k_keep_chunks<FIRST><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kin, p->kout);
-        k_count_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kin, p->kout, p->chunk_cnt, p->hcnt);
+        k_keep_chunks<FIRST><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kio);
+        k_count_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kio, p->chunk_cnt, p->hcnt);
     }
-    p->launches++; k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
+    p->launches++; k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
     int r = scan_excl<I3>(p, (const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
     if (r) return r;
     p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
                                               chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur, pk);
-    p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kin, p->kout, p->newidx, p->optr[ob],
+    p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kio, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked, p->emask, pk);
     if (chunked) {
         p->launches++;
-        k_scatter_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kin, p->kout, p->chunk_cnt,
+        k_scatter_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kio, p->chunk_cnt,
                                                                      p->newidx, p->optr[ob], p->iptr[ob], p->oadj[ob], p->iadj[ob]);
     }
     p->cb ^= 1;                                   // the next graph's chunk list is now current

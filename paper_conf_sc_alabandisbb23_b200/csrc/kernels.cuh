@@ -151,8 +151,10 @@ __device__ __forceinline__ bool keep_edge(int owner, int a, int b, int other, co
     return (__ldg(cin + other) == a) & (__ldg(cout + other) == b);
 }
 // Trim-1 on the kept graph: no kept in-edge or no kept out-edge
-__device__ __forceinline__ bool trimmed(const int32_t* __restrict__ kin, const int32_t* __restrict__ kout, int x) {
-    return (__ldg(kin + x) == 0) | (__ldg(kout + x) == 0);
+// kept degrees are interleaved (kio[x] = {in, out}): one 8-byte gather per far end
+__device__ __forceinline__ bool trimmed(const int2* __restrict__ kio, int x) {
+    const int2 k = __ldg(kio + x);
+    return (k.x == 0) | (k.y == 0);
 }
 
 struct RowCtx {
@@ -212,9 +214,10 @@ struct KeepPred {
 template <bool FIRST, bool TRIM>
 struct SurvivePred {
     int i, a, b;
-    const int32_t *cin, *cout, *kin, *kout;
+    const int32_t *cin, *cout;
+    const int2* kio;
     __device__ __forceinline__ bool operator()(int k) const {
-        return keep_edge<FIRST>(i, a, b, k, cin, cout) & !(TRIM && trimmed(kin, kout, k));
+        return keep_edge<FIRST>(i, a, b, k, cin, cout) & !(TRIM && trimmed(kio, k));
     }
     __device__ __forceinline__ SurvivePred bcast(int src) const {
         SurvivePred p = *this;
@@ -247,7 +250,7 @@ __device__ __forceinline__ void mask_light2(const int32_t* __restrict__ oadj, in
 }
 // keep the set bits of m whose entry's far end is not trimmed (batches of 4 entries)
 __device__ __forceinline__ unsigned trim_mask(const int32_t* __restrict__ adj, int b, unsigned m, int self,
-                                              const int32_t* __restrict__ kin, const int32_t* __restrict__ kout) {
+                                              const int2* __restrict__ kio) {
     unsigned out = 0;
     while (m) {
         int k[4], x[4];
@@ -260,7 +263,7 @@ __device__ __forceinline__ unsigned trim_mask(const int32_t* __restrict__ adj, i
         for (int q = 0; q < 4; q++) x[q] = k[q] >= 0 ? __ldg(adj + b + k[q]) : self;
 #pragma unroll
         for (int q = 0; q < 4; q++)
-            if (k[q] >= 0 && !trimmed(kin, kout, x[q])) out |= 1u << k[q];
+            if (k[q] >= 0 && !trimmed(kio, x[q])) out |= 1u << k[q];
     }
     return out;
 }
@@ -349,8 +352,8 @@ __device__ __forceinline__ void emit_cut(const int32_t* __restrict__ adj, int b,
 constexpr int TPB_COMPACT = 256;     // block size of the compaction kernels (driver TPB)
 template <bool FIRST>
 static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
-                             int32_t* __restrict__ kin, int32_t* __restrict__ kout,
-                             int chunked, int2* __restrict__ hcnt, uint2* __restrict__ emask) {
+                             int2* __restrict__ kio, int chunked, int2* __restrict__ hcnt,
+                             uint2* __restrict__ emask) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
@@ -362,8 +365,7 @@ static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, con
     co += count_row(g.oadj, r.ob, r.oe, r.live, lane, pred, chunked, false);
     ci += count_row(g.iadj, r.ib, r.ie, r.live, lane, pred, chunked, false);
     if (r.valid) {
-        kin[i] = ci;
-        kout[i] = co;
+        kio[i] = make_int2(ci, co);
         emask[i] = make_uint2(mo, mi);
         if (chunked) hcnt[i] = make_int2(0, 0);
     }
@@ -374,7 +376,7 @@ static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, con
 // per-vertex surviving (kept, not trimmed) degrees and per-warp totals (alive, out, in, kept)
 template <bool FIRST, bool TRIM>
 static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
-                                const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
+                                const int2* __restrict__ kio,
                                 int2* __restrict__ cnt, int4* __restrict__ wsum, int chunked,
                                 const int2* __restrict__ hcnt, uint2* __restrict__ emask) {
     const int lane = threadIdx.x & 31;
@@ -382,14 +384,14 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
     int nout = 0, nin = 0;
     if (!TRIM) {
-        if (r.live) { nout = kout[i]; nin = kin[i]; }   // survivors = kept: the masks stand
+        if (r.live) { const int2 k = kio[i]; nout = k.y; nin = k.x; }   // survivors = kept: the masks stand
     } else {
-        const bool go = r.live && !trimmed(kin, kout, (int)i);
-        SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
+        const bool go = r.live && !trimmed(kio, (int)i);
+        SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio};
         if (r.valid) {                                   // light rows: the kept entries' far ends
             const uint2 km = emask[i];
-            const unsigned so = go && r.oe - r.ob <= HEAVY ? trim_mask(g.oadj, r.ob, km.x, (int)i, kin, kout) : 0u;
-            const unsigned si = go && r.ie - r.ib <= HEAVY ? trim_mask(g.iadj, r.ib, km.y, (int)i, kin, kout) : 0u;
+            const unsigned so = go && r.oe - r.ob <= HEAVY ? trim_mask(g.oadj, r.ob, km.x, (int)i, kio) : 0u;
+            const unsigned si = go && r.ie - r.ib <= HEAVY ? trim_mask(g.iadj, r.ib, km.y, (int)i, kio) : 0u;
             emask[i] = make_uint2(so, si);
             nout = __popc(so);
             nin = __popc(si);
@@ -404,7 +406,7 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
     }
     if (r.valid) cnt[i] = make_int2(nout, nin);
     const int alive = (nout + nin) > 0;
-    const int kept = r.valid ? kout[i] : 0;             // kept (pre-trim) out-degree, chunks included
+    const int kept = r.valid ? kio[i].y : 0;            // kept (pre-trim) out-degree, chunks included
     const int sa = warp_sum(alive), so = warp_sum(nout), si = warp_sum(nin), sk = warp_sum(kept);
     if (lane == 0) wsum[i >> 5] = make_int4(sa, so, si, sk);
 }
@@ -554,8 +556,7 @@ __device__ __forceinline__ void emit_row(const int32_t* __restrict__ adj, int rb
 
 template <bool FIRST, bool TRIM>
 static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
-                                  const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
-                                  const int32_t* __restrict__ newidx, const int32_t* __restrict__ optr2,
+                                  const int2* __restrict__ kio, const int32_t* __restrict__ newidx, const int32_t* __restrict__ optr2,
                                   const int32_t* __restrict__ iptr2, int32_t* __restrict__ oadj2,
                                   int32_t* __restrict__ iadj2, int chunked, const uint2* __restrict__ emask,
                                   PackOut pk) {
@@ -605,7 +606,7 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
             if (li) emit_cut(g.iadj, r.ib, sm.y, newidx, j, tb, 0, E, at);
         }
     }
-    SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kin, kout};
+    SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio};
     emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred, chunked, false);
     emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred, chunked, false);
 }
@@ -618,7 +619,7 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
 template <bool FIRST>
 static __global__ void __launch_bounds__(256) k_keep_chunks(WGraph g, const Chunk* __restrict__ chunks, int nchunks,
                                                             const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
-                                                            int32_t* __restrict__ kin, int32_t* __restrict__ kout) {
+                                                            int2* __restrict__ kio) {
     const int lane = threadIdx.x & 31;
     const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (c >= nchunks) return;
@@ -630,13 +631,13 @@ static __global__ void __launch_bounds__(256) k_keep_chunks(WGraph g, const Chun
     for (int e = k.beg + lane; e < k.end; e += WARP) cc += keep_edge<FIRST>(k.i, a, b, __ldg(adj + e), cin, cout);
     cc = warp_sum(cc);
     if (lane == 0 && cc) {
-        atomicAdd(k.dir ? kin + k.i : kout + k.i, cc);
+        atomicAdd(k.dir ? &kio[k.i].x : &kio[k.i].y, cc);
     }
 }
 template <bool FIRST, bool TRIM>
 static __global__ void __launch_bounds__(256) k_count_chunks(WGraph g, const Chunk* __restrict__ chunks, int nchunks,
                                                              const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
-                                                             const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
+                                                             const int2* __restrict__ kio,
                                                              int* __restrict__ chunk_cnt, int2* __restrict__ hcnt) {
     const int lane = threadIdx.x & 31;
     const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -644,9 +645,9 @@ static __global__ void __launch_bounds__(256) k_count_chunks(WGraph g, const Chu
     const Chunk k = chunks[c];
     const int a = FIRST ? 0 : cin[k.i], b = FIRST ? 0 : cout[k.i];
     int cc = 0;
-    if ((FIRST || a != b) && !(TRIM && trimmed(kin, kout, k.i))) {
+    if ((FIRST || a != b) && !(TRIM && trimmed(kio, k.i))) {
         const int32_t* adj = k.dir ? g.iadj : g.oadj;
-        SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kin, kout};
+        SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio};
         for (int e = k.beg + lane; e < k.end; e += WARP) cc += pred(__ldg(adj + e));
         cc = warp_sum(cc);
     }
@@ -658,7 +659,7 @@ static __global__ void __launch_bounds__(256) k_count_chunks(WGraph g, const Chu
 template <bool FIRST, bool TRIM>
 static __global__ void __launch_bounds__(256) k_scatter_chunks(WGraph g, const Chunk* __restrict__ chunks, int nchunks,
                                                                const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
-                                                               const int32_t* __restrict__ kin, const int32_t* __restrict__ kout,
+                                                               const int2* __restrict__ kio,
                                                                const int* __restrict__ chunk_cnt,
                                                                const int32_t* __restrict__ newidx,
                                                                const int32_t* __restrict__ optr2, const int32_t* __restrict__ iptr2,
@@ -677,7 +678,7 @@ static __global__ void __launch_bounds__(256) k_scatter_chunks(WGraph g, const C
     const int a = FIRST ? 0 : cin[k.i], b = FIRST ? 0 : cout[k.i];
     const int32_t* adj = k.dir ? g.iadj : g.oadj;
     int32_t* dst = k.dir ? iadj2 : oadj2;
-    SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kin, kout};
+    SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio};
     for (int base = k.beg; base < k.end; base += WARP) {
         const int e = base + lane;
         int x = 0;

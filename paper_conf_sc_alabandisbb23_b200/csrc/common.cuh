@@ -22,6 +22,8 @@ struct WGraph {
     const int32_t* iptr;
     const int32_t* iadj;
     int32_t na;
+    const int2* sig2;    // Phase 3 of power-law graphs: (v_in, v_out) interleaved, one gather per
+                         // far end in keep(); nullptr: the separate cin / cout arrays
 };
 
 // Counters the host reads back once per outer iteration.

@@ -103,6 +103,7 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     e = e ? e : A((void**)&p->newidx, n1 * 4);
     e = e ? e : A((void**)&p->cnt, n1 * sizeof(int2));
     e = e ? e : A((void**)&p->emask, n1 * sizeof(uint2));
+    e = e ? e : A((void**)&p->sig2, n1 * sizeof(int2));
     e = e ? e : A((void**)&p->wsum, (size_t)p->nw_cap * sizeof(int4));
     e = e ? e : A((void**)&p->wscan, (size_t)p->nw_cap * sizeof(int4));
     e = e ? e : A((void**)&p->bsum, (size_t)p->bsum_cap * sizeof(int4));
@@ -143,7 +144,7 @@ void plan_free(Plan* p) {
         cudaFree(p->act[b]); cudaFree(p->cin[b]); cudaFree(p->cout[b]);
         cudaFree(p->optr[b]); cudaFree(p->iptr[b]); cudaFree(p->oadj[b]); cudaFree(p->iadj[b]);
     }
-    cudaFree(p->kin); cudaFree(p->newidx); cudaFree(p->cnt); cudaFree(p->emask);
+    cudaFree(p->kin); cudaFree(p->newidx); cudaFree(p->cnt); cudaFree(p->emask); cudaFree(p->sig2);
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
     cudaFree(p->chunk_cnt); cudaFree(p->hcnt);
     cudaFree(p->dirty); cudaFree(p->lvl);
@@ -315,29 +316,37 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     CK(cudaMemsetAsync(&p->dc->pack_bad, 0, sizeof(int), s));
     // the scatter writes the next graph's tile pack when Phase 2 will use one (no long rows
     // now means none after the compaction)
+    // power-law graphs (long-row chunks): keep() gathers random far ends, so the two signature
+    // arrays are interleaved once (one gather per far end instead of two)
+    WGraph gk = g;
+    if (!FIRST && chunked) {
+        p->launches++;
+        k_pack_sig<<<std::min<unsigned>(grid, 148 * 16), TPB, 0, s>>>(g.na, cin, cout, p->sig2);
+        gk.sig2 = p->sig2;
+    }
     PackOut pk{nullptr, nullptr, nullptr, nullptr, &p->dc->pack_bad};
     p->pack_fused = pack_path(p, nc);
     if (p->pack_fused) {
         if (int r = ensure_pack(p)) return r;
         pk = PackOut{p->pnin, p->pnout, p->ext, p->ext_cnt, &p->dc->pack_bad};
     }
-    p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->kio, chunked, p->hcnt, p->emask);
+    p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, chunked, p->hcnt, p->emask);
     if (chunked) {
         p->launches += 2;
-        k_keep_chunks<FIRST><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kio);
-        k_count_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kio, p->chunk_cnt, p->hcnt);
+        k_keep_chunks<FIRST><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio);
+        k_count_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio, p->chunk_cnt, p->hcnt);
     }
-    p->launches++; k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
+    p->launches++; k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
     int r = scan_excl<I3>(p, (const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
     if (r) return r;
-    p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(g, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
+    p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
                                               chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur, pk);
-    p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(g, cin, cout, p->kio, p->newidx, p->optr[ob],
+    p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked, p->emask, pk);
     if (chunked) {
         p->launches++;
-        k_scatter_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(g, cur, nc, cin, cout, p->kio, p->chunk_cnt,
+        k_scatter_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio, p->chunk_cnt,
                                                                      p->newidx, p->optr[ob], p->iptr[ob], p->oadj[ob], p->iadj[ob]);
     }
     p->cb ^= 1;                                   // the next graph's chunk list is now current

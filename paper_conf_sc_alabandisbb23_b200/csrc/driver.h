@@ -23,6 +23,7 @@ struct Plan {
     int32_t* newidx;                     // old local -> new local (-1: leaves)
     int2* cnt;                           // per-vertex surviving (out, in) degree
     uint2* emask;                        // light rows: kept, then surviving, entries as bit masks
+    int2* sig2;                          // power-law Phase 3: (v_in, v_out) interleaved copy
     int4 *wsum, *wscan;                  // per-warp compaction counts (alive, out, in, kept) and their prefix
     void* bsum;                          // scan block totals
     void* chunks;                        // long-row chunks, 2 x Chunk[chunk_cap] (current / next graph)

@@ -145,10 +145,20 @@ static __global__ void __launch_bounds__(256) k_csc_scatter(int32_t n, const int
 // self-loop is kept (DESIGN reading 9).
 template <bool FIRST>
 __device__ __forceinline__ bool keep_edge(int owner, int a, int b, int other, const int32_t* __restrict__ cin,
-                                          const int32_t* __restrict__ cout) {
+                                          const int32_t* __restrict__ cout, const int2* __restrict__ s2 = nullptr) {
     if (FIRST) return other != owner;
+    if (s2) {                                            // interleaved copy: one 8-byte gather
+        const int2 x = __ldg(s2 + other);
+        return (x.x == a) & (x.y == b);
+    }
     // both loads are issued unconditionally (no short circuit): callers batch these gathers
     return (__ldg(cin + other) == a) & (__ldg(cout + other) == b);
+}
+// Phase 3 of power-law graphs: the signatures interleaved for one gather per far end
+static __global__ void k_pack_sig(int32_t na, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+                                  int2* __restrict__ sig2) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < na; v += (int64_t)gridDim.x * blockDim.x)
+        sig2[v] = make_int2(__ldg(cin + v), __ldg(cout + v));
 }
 // Trim-1 on the kept graph: no kept in-edge or no kept out-edge
 // kept degrees are interleaved (kio[x] = {in, out}): one 8-byte gather per far end
@@ -204,7 +214,8 @@ template <bool FIRST>
 struct KeepPred {
     int i, a, b;
     const int32_t *cin, *cout;
-    __device__ __forceinline__ bool operator()(int k) const { return keep_edge<FIRST>(i, a, b, k, cin, cout); }
+    const int2* s2;
+    __device__ __forceinline__ bool operator()(int k) const { return keep_edge<FIRST>(i, a, b, k, cin, cout, s2); }
     __device__ __forceinline__ KeepPred bcast(int src) const {
         KeepPred p = *this;
         p.i = __shfl_sync(FULL, i, src); p.a = __shfl_sync(FULL, a, src); p.b = __shfl_sync(FULL, b, src);
@@ -216,8 +227,9 @@ struct SurvivePred {
     int i, a, b;
     const int32_t *cin, *cout;
     const int2* kio;
+    const int2* s2;
     __device__ __forceinline__ bool operator()(int k) const {
-        return keep_edge<FIRST>(i, a, b, k, cin, cout) & !(TRIM && trimmed(kio, k));
+        return keep_edge<FIRST>(i, a, b, k, cin, cout, s2) & !(TRIM && trimmed(kio, k));
     }
     __device__ __forceinline__ SurvivePred bcast(int src) const {
         SurvivePred p = *this;
@@ -357,7 +369,7 @@ static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, con
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
-    KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout};
+    KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout, g.sig2};
     unsigned mo = 0, mi = 0;
     mask_light2(g.oadj, r.ob, r.live && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, g.iadj, r.ib,
                 r.live && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, (int)(r.valid ? i : 0), pred, mo, mi);
@@ -387,7 +399,7 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
         if (r.live) { const int2 k = kio[i]; nout = k.y; nin = k.x; }   // survivors = kept: the masks stand
     } else {
         const bool go = r.live && !trimmed(kio, (int)i);
-        SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio};
+        SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2};
         if (r.valid) {                                   // light rows: the kept entries' far ends
             const uint2 km = emask[i];
             const unsigned so = go && r.oe - r.ob <= HEAVY ? trim_mask(g.oadj, r.ob, km.x, (int)i, kio) : 0u;
@@ -606,7 +618,7 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
             if (li) emit_cut(g.iadj, r.ib, sm.y, newidx, j, tb, 0, E, at);
         }
     }
-    SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio};
+    SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2};
     emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred, chunked, false);
     emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred, chunked, false);
 }
@@ -628,7 +640,7 @@ static __global__ void __launch_bounds__(256) k_keep_chunks(WGraph g, const Chun
     if (!FIRST && a == b) return;                        // finished owner keeps nothing
     const int32_t* adj = k.dir ? g.iadj : g.oadj;
     int cc = 0;
-    for (int e = k.beg + lane; e < k.end; e += WARP) cc += keep_edge<FIRST>(k.i, a, b, __ldg(adj + e), cin, cout);
+    for (int e = k.beg + lane; e < k.end; e += WARP) cc += keep_edge<FIRST>(k.i, a, b, __ldg(adj + e), cin, cout, g.sig2);
     cc = warp_sum(cc);
     if (lane == 0 && cc) {
         atomicAdd(k.dir ? &kio[k.i].x : &kio[k.i].y, cc);
@@ -647,7 +659,7 @@ static __global__ void __launch_bounds__(256) k_count_chunks(WGraph g, const Chu
     int cc = 0;
     if ((FIRST || a != b) && !(TRIM && trimmed(kio, k.i))) {
         const int32_t* adj = k.dir ? g.iadj : g.oadj;
-        SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio};
+        SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio, g.sig2};
         for (int e = k.beg + lane; e < k.end; e += WARP) cc += pred(__ldg(adj + e));
         cc = warp_sum(cc);
     }
@@ -678,7 +690,7 @@ static __global__ void __launch_bounds__(256) k_scatter_chunks(WGraph g, const C
     const int a = FIRST ? 0 : cin[k.i], b = FIRST ? 0 : cout[k.i];
     const int32_t* adj = k.dir ? g.iadj : g.oadj;
     int32_t* dst = k.dir ? iadj2 : oadj2;
-    SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio};
+    SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio, g.sig2};
     for (int base = k.beg; base < k.end; base += WARP) {
         const int e = base + lane;
         int x = 0;

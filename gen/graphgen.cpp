@@ -87,9 +87,11 @@ int64_t gen_mesh(int64_t N, int order, const double* omega, double kappa, double
         const int64_t x = xyz / (N * N), y = (xyz / N) % N, z = xyz % N;
         const int64_t c[3] = {x, y, z};
         const int64_t cid = cube_index(s, x, y, z);
+        const int64_t clex = (x * N + y) * N + z;   // numbering-independent cube key
         for (int p = 0; p < 6; p++) {
             const int a = PERM[p][0], b = PERM[p][1], cc = PERM[p][2];
             const int64_t e = 6 * cid + p;
+            const int64_t elex = 6 * clex + p;
             // tet vertices (integer coordinates)
             int64_t V[4][3];
             for (int d = 0; d < 3; d++) {
@@ -110,6 +112,7 @@ int64_t gen_mesh(int64_t N, int order, const double* omega, double kappa, double
                 if (nc[0] < 0 || nc[1] < 0 || nc[2] < 0 || nc[0] >= N || nc[1] >= N || nc[2] >= N)
                     continue;  // boundary face
                 const int64_t e2 = 6 * cube_index(s, nc[0], nc[1], nc[2]) + np_;
+                const int64_t e2lex = 6 * ((nc[0] * N + nc[1]) * N + nc[2]) + np_;
                 // exact integer outward normal of e on this face
                 int64_t f[3][3];
                 int t = 0;
@@ -122,9 +125,12 @@ int64_t gen_mesh(int64_t N, int order, const double* omega, double kappa, double
                 for (int d = 0; d < 3; d++) w[d] = V[k][d] - f[0][d];
                 if (cr[0] * w[0] + cr[1] * w[1] + cr[2] * w[2] > 0)
                     for (int d = 0; d < 3; d++) cr[d] = -cr[d];
-                // canonical orientation: e1 = lower ID, normal points from e1 into e2
-                const bool lo_is_e = e < e2;
-                const int64_t lo = lo_is_e ? e : e2, hi = lo_is_e ? e2 : e;
+                // canonical orientation: e1 = lower LEXICOGRAPHIC element key, normal points
+                // from e1 into e2.  The face's RNG stream, its orientation and its
+                // hot-spot test depend only on lexicographic keys, so every element order
+                // yields the same graph up to a relabelling of the vertices.
+                const bool lo_is_e = elex < e2lex;
+                const int64_t lo = lo_is_e ? elex : e2lex, hi = lo_is_e ? e2lex : elex;
                 if (!lo_is_e) for (int d = 0; d < 3; d++) cr[d] = -cr[d];
                 const double nn = std::sqrt((double)(cr[0] * cr[0] + cr[1] * cr[1] + cr[2] * cr[2]));
                 const double n0 = (double)cr[0] / nn, n1 = (double)cr[1] / nn, n2 = (double)cr[2] / nn;

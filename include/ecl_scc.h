@@ -70,9 +70,8 @@ typedef enum {
                                       priorities pi(v) (reading 16); labels are
                                       identical either way */
 #define ECL_SCC_NO_DIRTY 0x40u    /* ablation: visit every tile in every Phase-2 pass */
-#define ECL_SCC_SWEEP 0x100u      /* Phase 2 as dependency-ordered forward/backward tile
-                                     sweeps instead of passes (experimental; pays off only
-                                     when the tile graph is close to a DAG in ID order) */
+/* 0x80u, 0x100u, 0x2000u: retired experimental variants (threshold stages, dependency-ordered
+   sweeps, device-resident tail; measured negative) */
 #define ECL_SCC_NO_REORDER 0x200u /* keep the caller's vertex numbering as the storage order
                                      (by default graphs without rows longer than 64 edges,
                                      n >= 16384 and fewer than 85% of the edges inside
@@ -83,12 +82,6 @@ typedef enum {
                                      visit instead of reading per-iteration tile packs */
 #define ECL_SCC_NO_ASYNC 0x1000u  /* ablation: Phase 2 as global passes (one launch each)
                                      instead of one persistent launch with a tile queue */
-#define ECL_SCC_TAIL 0x2000u      /* opt-in: once the working graph has at most 32768 vertices,
-                                     run the remaining outer iterations in one cooperative
-                                     launch (tail.cuh) instead of compacting each time
-                                     (measured: no gain on C2/C4) */
-#define ECL_SCC_STAGED 0x80u      /* Phase 2 in threshold stages: the top-K priorities
-                                     propagate first (ECL_SCC_STAGES env, default off) */
 
 #define ECL_SCC_TRACE_MAX 64
 
@@ -114,6 +107,12 @@ typedef struct {
     double ms_prop;                          /* Phase 2 (all passes)                      */
     double ms_prop_iter[ECL_SCC_TRACE_MAX];  /* Phase 2 of outer iteration k+1            */
     double ms_compact_iter[ECL_SCC_TRACE_MAX]; /* Phase 3 + compaction before iteration k+1 */
+    /* multi-GPU (ecl_scc_partitioned): device time spent in the signature / degree / count
+       exchanges (CUDA events around every collective on the call's stream), the bytes this
+       rank contributed to them, and the number of exchanges; 0 for single-GPU calls */
+    double ms_comm;
+    int64_t comm_bytes;
+    int64_t exchanges;
 } ecl_scc_stats;
 
 typedef struct ecl_scc_plan_s* ecl_scc_plan_t;
@@ -187,15 +186,29 @@ int ecl_scc_get_unique_id(uint8_t id[128]);
 int ecl_scc_comm_create(int32_t nranks, int32_t rank, const uint8_t id[128], ecl_scc_comm_t* out);
 int ecl_scc_comm_destroy(ecl_scc_comm_t comm);
 
+/* Per-rank workspace of the partitioned mode (not collective): n global vertices, this
+ * rank's source rows [row_begin, row_end), at most local_nnz_max local edges.  A plan makes
+ * repeated ecl_scc_partitioned calls allocation-free.  flags: ECL_SCC_* (NO_TRIM,
+ * NO_VALIDATE, IDENTITY_IDS are honoured). */
+typedef struct ecl_scc_part_plan_s* ecl_scc_part_plan_t;
+int ecl_scc_part_plan_create(int32_t n, int32_t row_begin, int32_t row_end, int64_t local_nnz_max,
+                             uint32_t flags, ecl_scc_part_plan_t* out);
+int ecl_scc_part_plan_destroy(ecl_scc_part_plan_t plan);
+
 /* Collective over comm.  This rank owns source rows [row_begin, row_end) of the global
  * graph (n vertices): local_row_ptr has row_end-row_begin+1 offsets starting at 0,
  * local_col_idx holds local_nnz GLOBAL destination IDs.  Signatures are replicated and
  * combined with ncclAllReduce(MAX) after every local fixed point; degrees for trim with
- * ncclAllReduce(SUM).  labels_out: n int32 on every rank (replicated result). */
+ * ncclAllReduce(SUM).  labels_out: n int32 on every rank (replicated result).
+ * plan: nullable (then a temporary workspace is allocated for this call).
+ * Errors: invalid input on ANY rank makes every rank return ECL_SCC_ERANGE (the ranks agree
+ * through the first exchange before any of them leaves); a CUDA or NCCL failure on one rank
+ * leaves the communicator unusable (destroy it).  stats->ms_comm / comm_bytes / exchanges
+ * report the exchanges of this rank. */
 int ecl_scc_partitioned(ecl_scc_comm_t comm, int32_t n, int32_t row_begin, int32_t row_end,
                         int64_t local_nnz, const int32_t* local_row_ptr,
                         const int32_t* local_col_idx, int32_t* labels_out,
-                        ecl_scc_stream_t stream, ecl_scc_stats* stats);
+                        ecl_scc_stream_t stream, ecl_scc_part_plan_t plan, ecl_scc_stats* stats);
 
 /* Single-process emulation of the partitioned algorithm with P partitions on the
  * current device (the all-reduce replaced by an element-wise max over P replicas).

@@ -19,8 +19,8 @@ _LIB_PATH = os.path.join(_HERE, "libeclscc.so")
 
 OK, EINVAL, ERANGE, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED = range(7)
 NO_TRIM, NO_VALIDATE, SYNC_PASSES, TIME_STAGES = 0x1, 0x4, 0x8, 0x10
-IDENTITY_IDS, NO_DIRTY, STAGED, SWEEP, NO_REORDER = 0x20, 0x40, 0x80, 0x100, 0x200
-FORCE_REORDER, NO_PACK, NO_ASYNC, TAIL = 0x400, 0x800, 0x1000, 0x2000
+IDENTITY_IDS, NO_DIRTY, NO_REORDER = 0x20, 0x40, 0x200
+FORCE_REORDER, NO_PACK, NO_ASYNC = 0x400, 0x800, 0x1000
 TRACE_MAX = 64
 
 _lib = None
@@ -39,7 +39,8 @@ class Stats(ctypes.Structure):
                 ("edges_kept", ctypes.c_int64 * TRACE_MAX), ("passes_iter", ctypes.c_int64 * TRACE_MAX),
                 ("prop_bytes", ctypes.c_int64), ("kernel_launches", ctypes.c_int64),
                 ("ms_ingest", ctypes.c_double), ("ms_compact", ctypes.c_double), ("ms_prop", ctypes.c_double),
-                ("ms_prop_iter", ctypes.c_double * TRACE_MAX), ("ms_compact_iter", ctypes.c_double * TRACE_MAX)]
+                ("ms_prop_iter", ctypes.c_double * TRACE_MAX), ("ms_compact_iter", ctypes.c_double * TRACE_MAX),
+                ("ms_comm", ctypes.c_double), ("comm_bytes", ctypes.c_int64), ("exchanges", ctypes.c_int64)]
 
     def as_dict(self) -> dict:
         k = self.trace_len
@@ -50,7 +51,8 @@ class Stats(ctypes.Structure):
                     edges_kept=list(self.edges_kept[:max(k - 1, 0)]),
                     passes_iter=list(self.passes_iter[:k]),
                     ms_prop_iter=[round(x, 4) for x in self.ms_prop_iter[:k]],
-                    ms_compact_iter=[round(x, 4) for x in self.ms_compact_iter[:k + 1]])
+                    ms_compact_iter=[round(x, 4) for x in self.ms_compact_iter[:k + 1]],
+                    ms_comm=self.ms_comm, comm_bytes=self.comm_bytes, exchanges=self.exchanges)
 
 
 def lib() -> ctypes.CDLL:
@@ -73,7 +75,9 @@ def lib() -> ctypes.CDLL:
         "ecl_scc_get_unique_id": [vp],
         "ecl_scc_comm_create": [i32, i32, vp, vp],
         "ecl_scc_comm_destroy": [vp],
-        "ecl_scc_partitioned": [vp, i32, i32, i32, i64, vp, vp, vp, vp, vp],
+        "ecl_scc_partitioned": [vp, i32, i32, i32, i64, vp, vp, vp, vp, vp, vp],
+        "ecl_scc_part_plan_create": [i32, i32, i32, i64, u32, vp],
+        "ecl_scc_part_plan_destroy": [vp],
         "ecl_scc_partitioned_emulated": [i32, i32, i64, vp, vp, vp, vp, vp],
         "ecl_scc_partition_rows": [i32, i32, vp, vp],
         "ecl_scc_status_string": [ctypes.c_int],
@@ -99,7 +103,7 @@ ABI_SYMBOLS = ("ecl_scc", "ecl_scc_async", "ecl_scc_debug_run", "ecl_scc_plan_cr
                "ecl_scc_comm_create", "ecl_scc_comm_destroy", "ecl_scc_partitioned",
                "ecl_scc_partitioned_emulated", "ecl_scc_partition_rows", "ecl_scc_status_string",
                "ecl_scc_last_error", "ecl_scc_version", "ecl_scc_plan_counters", "ecl_scc_levels",
-               "ecl_scc_host")
+               "ecl_scc_host", "ecl_scc_part_plan_create", "ecl_scc_part_plan_destroy")
 
 
 def status_string(s: int) -> str:
@@ -274,8 +278,30 @@ class Comm:
             self.handle = None
 
 
+class PartPlan:
+    """Per-rank workspace of the partitioned mode (ecl_scc_part_plan_t): rows [row_begin,
+    row_end) of an n-vertex graph, at most local_nnz_max local edges."""
+
+    def __init__(self, comm, n: int, row_begin: int, row_end: int, local_nnz_max: int, flags: int = 0):
+        h = ctypes.c_void_p()
+        _check(lib().ecl_scc_part_plan_create(n, row_begin, row_end, local_nnz_max, flags, ctypes.byref(h)),
+               "ecl_scc_part_plan_create")
+        self.handle = h
+
+    def close(self):
+        if self.handle:
+            lib().ecl_scc_part_plan_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 def ecl_scc_partitioned(comm: Comm, n: int, row_begin: int, row_end: int, local_row_ptr, local_col_idx,
-                        labels_out=None, stream=None, stats: bool = False):
+                        labels_out=None, stream=None, plan: PartPlan | None = None, stats: bool = False):
     if labels_out is None:
         labels_out = torch.empty(n, dtype=torch.int32, device=local_row_ptr.device)
     st = Stats() if stats else None
@@ -283,5 +309,6 @@ def ecl_scc_partitioned(comm: Comm, n: int, row_begin: int, row_end: int, local_
     _check(lib().ecl_scc_partitioned(comm.handle, n, row_begin, row_end, nnz, _dev_i32(local_row_ptr, "local_row_ptr"),
                                      _dev_i32(local_col_idx, "local_col_idx") if nnz else None,
                                      _dev_i32(labels_out, "labels_out"), _stream(stream),
-                                     ctypes.byref(st) if st else None), "ecl_scc_partitioned")
+                                     plan.handle if plan else None, ctypes.byref(st) if st else None),
+           "ecl_scc_partitioned")
     return (labels_out, st.as_dict()) if stats else labels_out

@@ -24,7 +24,6 @@
 #include "scan.cuh"
 #include "reorder.cuh"
 #include "pack.cuh"
-#include "tail.cuh"
 #include "levels.cuh"
 #include "driver.h"
 
@@ -76,10 +75,19 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     p->bsum_cap = cdiv(std::max<int64_t>(n1, p->nw_cap), SCAN_TILE) + 1;
     p->chunk_cap = 2 * (int64_t)m / HEAVY_T + 16;
     p->dirty_cap = cdiv(p->n_cap, 512) + 1;
-    p->tile = TILE;
-    if (const char* t = getenv("ECL_SCC_TILE")) {      // tuning knob: 512, 1024, 2048, 4096
-        const int v = atoi(t);
-        if (v == 512 || v == 1024 || v == 2048 || v == 4096) p->tile = v;
+    // development knobs, read once per plan; 0 = the measured default
+    auto knob = [](const char* name, int lo, int hi) -> int {
+        const char* e = getenv(name);
+        return e ? std::min(hi, std::max(lo, atoi(e))) : 0;
+    };
+    p->knob_run = knob("ECL_SCC_RUN", 1, 64);
+    p->knob_claim = knob("ECL_SCC_CLAIM", 1, 32);
+    p->knob_claim_div = knob("ECL_SCC_CLAIM_DIV", 1, 64);
+    p->knob_claim_max = knob("ECL_SCC_CLAIM_MAX", 1, 32);
+    p->knob_async_ctas = knob("ECL_SCC_ASYNC_CTAS", 1, 8);
+    if (cudaGetDevice(&p->device) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ECL_SCC_ECUDA, "plan: no current CUDA device");
     }
     auto A = [&](void** ptr, size_t bytes) -> cudaError_t { return cudaMalloc(ptr, bytes); };
     cudaError_t e = cudaSuccess;
@@ -94,7 +102,7 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     }
     // one allocation, two views: the compaction's interleaved kept degrees kio[i] = {in, out}
     // (one 8-byte gather per far end in the trim), and two int arrays kin / kout of n+1 for
-    // the ingest, the relabelling, the tail and the levels (never used at the same time)
+    // the ingest, the relabelling and the levels (never used at the same time)
     e = e ? e : A((void**)&p->kin, 2 * n1 * 4);
     if (e == cudaSuccess) {
         p->kout = p->kin + n1;
@@ -111,7 +119,6 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     e = e ? e : A((void**)&p->chunk_cnt, (size_t)p->chunk_cap * sizeof(int));
     e = e ? e : A((void**)&p->hcnt, n1 * sizeof(int2));
     e = e ? e : A((void**)&p->dirty, 2 * (size_t)p->dirty_cap);
-    e = e ? e : A((void**)&p->lvl, n1);
     e = e ? e : A((void**)&p->rp2, n1 * 4);
     e = e ? e : A((void**)&p->ci2, m * 4);
     e = e ? e : A((void**)&p->orig, n1 * 4);
@@ -121,14 +128,6 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     e = e ? e : A((void**)&p->fb, n1 * 4);
     e = e ? e : A((void**)&p->cellbuf, 3 * (((size_t)p->n_cap >> reo::CELL_SHIFT) + 2) * 4);
     e = e ? e : A((void**)&p->rcnt, 16);
-    e = e ? e : A((void**)&p->nb_cnt, (size_t)p->dirty_cap * 4);
-    e = e ? e : A((void**)&p->nb_list, (size_t)p->dirty_cap * NBCAP * 4);
-    e = e ? e : A((void**)&p->done, (size_t)p->dirty_cap * 4);
-    e = e ? e : A((void**)&p->mark, (size_t)p->dirty_cap * 4);
-    e = e ? e : A((void**)&p->sweep_ctr, 16);
-    if (e == cudaSuccess) e = cudaMemset(p->done, 0, (size_t)p->dirty_cap * 4);
-    if (e == cudaSuccess) e = cudaMemset(p->mark, 0, (size_t)p->dirty_cap * 4);
-    p->epoch = 0;
     e = e ? e : A((void**)&p->dc, sizeof(DevCounters));
     if (e == cudaSuccess) e = cudaMallocHost((void**)&p->hc, sizeof(DevCounters));
     if (e != cudaSuccess) {
@@ -147,17 +146,14 @@ void plan_free(Plan* p) {
     cudaFree(p->kin); cudaFree(p->newidx); cudaFree(p->cnt); cudaFree(p->emask); cudaFree(p->sig2);
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
     cudaFree(p->chunk_cnt); cudaFree(p->hcnt);
-    cudaFree(p->dirty); cudaFree(p->lvl);
+    cudaFree(p->dirty);
     cudaFree(p->rp2); cudaFree(p->ci2); cudaFree(p->orig); cudaFree(p->pos); cudaFree(p->cellv);
     cudaFree(p->fa); cudaFree(p->fb); cudaFree(p->cellbuf); cudaFree(p->rcnt);
-    cudaFree(p->nb_cnt); cudaFree(p->nb_list); cudaFree(p->done); cudaFree(p->mark); cudaFree(p->sweep_ctr);
     cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
     cudaFree(p->pnin); cudaFree(p->pnout); cudaFree(p->ext); cudaFree(p->ext_cnt);
     cudaFree(p->aq_state); cudaFree(p->aq_seen); cudaFree(p->aq_ctr);
-    cudaFree(p->tail_dev);
     cudaFree(p->lv_ctl);
     cudaFree(p->h_rp); cudaFree(p->h_ci); cudaFree(p->h_lab);
-    if (p->tail_host) cudaFreeHost(p->tail_host);
     if (p->hc) cudaFreeHost(p->hc);
     if (p->ev_ok)
         for (int k = 0; k < 6; k++) cudaEventDestroy(p->ev[k]);
@@ -279,11 +275,8 @@ static int reorder_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, con
 
 // Does Phase 2 of a working graph with `nchunks` long-row chunks run on tile packs?
 static bool pack_path(const Plan* p, int nchunks) {
-    static int env_variant = -1;   // the KCAP / LEVELS experiments run on the tile kernel
-    if (env_variant < 0) env_variant = (getenv("ECL_SCC_KCAP") || getenv("ECL_SCC_LEVELS")) ? 1 : 0;
     const bool sync = (p->flags & ECL_SCC_SYNC_PASSES) != 0 || (p->low_locality && nchunks > 0);
-    return nchunks == 0 && !sync && !(p->flags & (ECL_SCC_NO_DIRTY | ECL_SCC_STAGED | ECL_SCC_NO_PACK | ECL_SCC_SWEEP)) &&
-           p->tile == PACK_TT && !env_variant;
+    return nchunks == 0 && !sync && !(p->flags & (ECL_SCC_NO_DIRTY | ECL_SCC_NO_PACK));
 }
 // tile pack buffers (pack.cuh), sized for the plan on first use
 static int ensure_pack(Plan* p) {
@@ -354,125 +347,38 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     return ECL_SCC_OK;
 }
 
-// a4-a6: Phase 2 to its fixed point.  Passes are enqueued in growing batches; a pass
-// whose predecessor changed nothing exits at once, so over-enqueueing costs only a launch.
-template <int TT>
-static int set_tile_attrs() {
-    static int done = 0;
-    if (done) return ECL_SCC_OK;
-    CK(cudaFuncSetAttribute(k_prop_tile<false, TT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tile_dyn_smem<TT>()));
-    CK(cudaFuncSetAttribute(k_prop_tile<true, TT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tile_dyn_smem<TT>()));
-    done = 1;
+// per-plan (per-device) kernel attributes of the pass kernels
+static int set_tile_attrs(Plan* p) {
+    if (p->tile_attrs) return ECL_SCC_OK;
+    CK(cudaFuncSetAttribute(k_prop_tile<false, TILE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tile_dyn_smem<TILE>()));
+    CK(cudaFuncSetAttribute(k_prop_tile<true, TILE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tile_dyn_smem<TILE>()));
+    p->tile_attrs = true;
     return ECL_SCC_OK;
 }
 
-template <int TT>
+// runs of consecutive tiles per CTA (Gauss-Seidel along a run).  Measured on C4: run 4
+// beats 1 (-14%), longer runs starve the SMs (fewer CTAs than resident slots).
+static int pass_run(const Plan* p, int64_t ntiles) {
+    return (int)std::min<int64_t>(p->knob_run ? p->knob_run : 4, std::max<int64_t>(1, ntiles / (2 * 148)));
+}
+
 static int launch_tile(Plan* p, bool sync, const WGraph& g, int32_t* cin, int32_t* cout, int pass, int first,
-                       uint8_t* dcur, uint8_t* dnext, int full, int theta, cudaStream_t s) {
-    if (int r = set_tile_attrs<TT>()) return r;
-    const int64_t ntiles = cdiv(g.na, TT);
-    // runs of consecutive tiles per CTA (Gauss-Seidel along a run).  Measured on C4: run
-    // 4 beats 1 (-14%), longer runs starve the SMs (fewer CTAs than resident slots).
-    static int run_env = -1;
-    if (run_env < 0) run_env = getenv("ECL_SCC_RUN") ? std::max(1, atoi(getenv("ECL_SCC_RUN"))) : 4;
-    const int run = (int)std::min<int64_t>(run_env, std::max<int64_t>(1, ntiles / (2 * 148)));
+                       uint8_t* dcur, uint8_t* dnext, int full, cudaStream_t s) {
+    if (int r = set_tile_attrs(p)) return r;
+    const int64_t ntiles = cdiv(g.na, TILE);
+    const int run = pass_run(p, ntiles);
     const unsigned grid = (unsigned)cdiv(ntiles, run);
-    static int kcap = -1;    // >0: bounded SIMD rounds in shared memory instead of drains
-    if (kcap < 0) kcap = getenv("ECL_SCC_KCAP") ? std::max(0, atoi(getenv("ECL_SCC_KCAP"))) : 0;
-    const int kc = dnext ? kcap : 0;   // the cap needs dirty marking to resume
-    static int levels = -1;  // level sweeps inside a tile (needs dirty mode: levels built on the first pass)
-    if (levels < 0) levels = getenv("ECL_SCC_LEVELS") ? atoi(getenv("ECL_SCC_LEVELS")) : 0;
-    uint8_t* lv = (levels && dnext && TT >= 1024) ? p->lvl : nullptr;
     p->launches++;
-    if (sync) k_prop_tile<true, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, nullptr, nullptr, 1, theta, run, 0, nullptr);
-    else k_prop_tile<false, TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, pass, first, dcur, dnext, full, theta, run, kc, lv);
+    if (sync) k_prop_tile<true, TILE><<<grid, TILE / VPT, tile_dyn_smem<TILE>(), s>>>(g, cin, cout, p->dc, pass, first, nullptr, nullptr, 1, run);
+    else k_prop_tile<false, TILE><<<grid, TILE / VPT, tile_dyn_smem<TILE>(), s>>>(g, cin, cout, p->dc, pass, first, dcur, dnext, full, run);
     return ECL_SCC_OK;
-}
-
-// Sweep mode: dependency-ordered sweeps over the tiles,
-// alternating forward / backward, until a sweep raises nothing.  Returns 1 in *used if it
-// ran (0: the tile graph was too dense -- the caller falls back to pass mode).
-template <int TT>
-static int sweep_phase(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, cudaStream_t s, int64_t* sweeps,
-                       int* used) {
-    *used = 0;
-    const int ntiles = (int)cdiv(g.na, TT);
-    static int resident = 0;
-    if (!resident) {
-        if (int r = set_tile_attrs<TT>()) return r;
-        CK(cudaFuncSetAttribute(k_sweep_tile<TT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tile_dyn_smem<TT>()));
-        int per_sm = 0, dev = 0, sms = 0;
-        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sweep_tile<TT>, TT / VPT, tile_dyn_smem<TT>()));
-        CK(cudaGetDevice(&dev));
-        CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-        resident = std::max(1, per_sm) * sms;
-    }
-    CK(cudaMemsetAsync(p->sweep_ctr, 0, 16, s));
-    CK(cudaMemsetAsync(&p->dc->err, 0, 4, s));
-    p->launches++;
-    k_tile_nbrs<TT><<<ntiles, 256, 0, s>>>(g, p->nb_cnt, p->nb_list, p->sweep_ctr + 2);
-    CK(cudaGetLastError());
-    int h[3];
-    CK(cudaMemcpyAsync(h, p->sweep_ctr, 12, cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    if (h[2]) return ECL_SCC_OK;                                   // overflow: use passes
-    *used = 1;
-    const unsigned grid = (unsigned)std::min(ntiles, resident);
-    int64_t k = 0;
-    for (;; k++) {
-        if (k > 4 * (int64_t)g.na + 1024) return fail(ECL_SCC_ECUDA, "internal: sweeps did not converge");
-        const int epoch = ++p->epoch;
-        CK(cudaMemsetAsync(p->sweep_ctr, 0, 8, s));
-        p->launches++;
-        k_sweep_tile<TT><<<grid, TT / VPT, tile_dyn_smem<TT>(), s>>>(g, cin, cout, p->dc, p->nb_cnt, p->nb_list, p->done,
-                                                                    p->mark, p->sweep_ctr, epoch, k == 0, (int)(k & 1),
-                                                                    p->sweep_ctr + 1);
-        CK(cudaGetLastError());
-        CK(cudaMemcpyAsync(h, p->sweep_ctr, 8, cudaMemcpyDeviceToHost, s));
-        CK(cudaMemcpyAsync(&h[2], &p->dc->err, 4, cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));
-        if (h[2] == 2) return fail(ECL_SCC_ECUDA, "internal: sweep dependency wait timed out");
-        if (!h[1]) break;                                          // nothing raised: fixed point
-    }
-    *sweeps = k + 1;
-    return ECL_SCC_OK;
-}
-
-// Threshold stages: the top-K priorities of the working graph flood first (a vertex
-// reached by one of them already holds its final value: everything else is smaller), then
-// the next K, ..., then theta = 0.  K list: ECL_SCC_STAGES.
-static std::vector<int> stage_thresholds(int32_t n, int32_t na, bool identity) {
-    std::vector<int> th;
-    static std::vector<long long> Ks;
-    static bool init = false;
-    if (!init) {
-        const char* e = getenv("ECL_SCC_STAGES");
-        std::string spec = e ? e : "64,4096,262144";
-        size_t pos = 0;
-        while (pos < spec.size()) {
-            size_t q = spec.find(',', pos);
-            if (q == std::string::npos) q = spec.size();
-            const long long k = atoll(spec.substr(pos, q - pos).c_str());
-            if (k > 0) Ks.push_back(k);
-            pos = q + 1;
-        }
-        init = true;
-    }
-    (void)identity;
-    for (long long K : Ks)
-        if (K < na) {
-            const long long t = (long long)n - (long long)n * K / na;   // priorities are uniform on [0, n)
-            if (t > 0 && (th.empty() || t < th.back())) th.push_back((int)t);
-        }
-    th.push_back(0);
-    return th;
 }
 
 // a4-a6: Phase 2 to its fixed point.  Passes are enqueued in growing batches; a pass
 // whose predecessor changed nothing exits at once, so over-enqueueing costs only a launch.
-static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int nchunks, int32_t n, cudaStream_t s,
+static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int nchunks, cudaStream_t s,
                      int64_t* passes_out) {
-    const unsigned ntiles = (unsigned)cdiv(g.na, p->tile);
+    const unsigned ntiles = (unsigned)cdiv(g.na, TILE);
     const unsigned hgrid = (unsigned)std::min<int64_t>(cdiv(std::max(nchunks, 1), TPB / WARP), 148 * 8);
     // plain Jacobi passes: the ablation flag, or graphs whose tiles hold almost no edges
     const bool sync = (p->flags & ECL_SCC_SYNC_PASSES) != 0 || (p->low_locality && nchunks > 0);
@@ -480,9 +386,6 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     // and a local fixed point per visit (not the SYNC ablation)
     const bool use_dirty = nchunks == 0 && !sync && !(p->flags & ECL_SCC_NO_DIRTY);
     uint8_t* D[2] = {p->dirty, p->dirty + p->dirty_cap};
-    const std::vector<int> thetas = (p->flags & ECL_SCC_STAGED) ? stage_thresholds(n, g.na, false)
-                                                                   : std::vector<int>{0};
-    int64_t total = 0;
     // tile packs (pack.cuh): the default for graphs without long rows
     const bool use_pack = pack_path(p, nchunks) && g.na > 0;
     if (use_pack) {
@@ -505,13 +408,12 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                 CK(cudaFuncSetAttribute(k_prop_async, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
                 CK(cudaFuncSetAttribute(k_prop_async, cudaFuncAttributePreferredSharedMemoryCarveout,
                                         (int)cudaSharedmemCarveoutMaxShared));
-                int per_sm = 0, dev = 0, sms = 0;
+                int per_sm = 0, sms = 0;
                 CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_async, PACK_TH, pack_dyn_smem()));
-                CK(cudaGetDevice(&dev));
-                CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-                // tuning knob ECL_SCC_ASYNC_CTAS: resident CTAs per SM used (<= what fits)
-                if (const char* e = getenv("ECL_SCC_ASYNC_CTAS")) per_sm = std::min(per_sm, std::max(1, atoi(e)));
-                p->aq_resident = std::max(1, per_sm) * sms;
+                CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device));
+                // resident CTAs per SM used (<= what fits); measured best: all of them
+                if (p->knob_async_ctas) per_sm = std::min(per_sm, p->knob_async_ctas);
+                p->aq_resident = (int64_t)std::max(1, per_sm) * sms;
                 if (getenv("ECL_SCC_DEBUG")) fprintf(stderr, "[ecl_scc] k_prop_async: %d CTAs per SM\n", per_sm);
             }
             AsyncQ Q{p->aq_state, p->aq_seen, p->aq_ctr};
@@ -519,13 +421,10 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             // C4 iteration 1, 18 tiles per CTA, best at 8-16; C2, ~1 tile per CTA, best at 1);
             // claim = clamp(tiles / resident CTAs, 1, 16) (C4 lex 19.8 -> 19.2 ms vs
             // tiles / (2 x resident) capped at 8; blocked8 unchanged)
-            static int claim_env = -1;                      // tuning knob ECL_SCC_CLAIM
-            if (claim_env < 0) claim_env = getenv("ECL_SCC_CLAIM") ? std::min(32, std::max(1, atoi(getenv("ECL_SCC_CLAIM")))) : 0;
-            static int claim_div = -1, claim_max = -1;      // tuning knobs of the adaptive rule
-            if (claim_div < 0) claim_div = getenv("ECL_SCC_CLAIM_DIV") ? std::max(1, atoi(getenv("ECL_SCC_CLAIM_DIV"))) : 1;
-            if (claim_max < 0) claim_max = getenv("ECL_SCC_CLAIM_MAX") ? std::min(32, std::max(1, atoi(getenv("ECL_SCC_CLAIM_MAX")))) : 16;
-            const int claim = claim_env ? claim_env
-                                        : (int)std::min<int64_t>(claim_max, std::max<int64_t>(1, ntiles / (claim_div * p->aq_resident)));
+            const int cdiv_ = p->knob_claim_div ? p->knob_claim_div : 1;
+            const int cmax = p->knob_claim_max ? p->knob_claim_max : 16;
+            const int claim = p->knob_claim ? p->knob_claim
+                                            : (int)std::min<int64_t>(cmax, std::max<int64_t>(1, ntiles / (cdiv_ * p->aq_resident)));
             CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
             CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
             p->launches += 2;
@@ -539,122 +438,42 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             return ECL_SCC_OK;
         }
     }
-    if (!sync && nchunks == 0 && (p->flags & ECL_SCC_SWEEP) && !(p->flags & ECL_SCC_STAGED)) {
-        int used = 0, r = ECL_SCC_OK;
-        switch (p->tile) {
-            case 512: r = sweep_phase<512>(p, g, cin, cout, s, &total, &used); break;
-            case 1024: r = sweep_phase<1024>(p, g, cin, cout, s, &total, &used); break;
-            case 4096: r = sweep_phase<4096>(p, g, cin, cout, s, &total, &used); break;
-            default: r = sweep_phase<2048>(p, g, cin, cout, s, &total, &used); break;
-        }
-        if (r) return r;
-        if (used) {
-            if (getenv("ECL_SCC_DEBUG"))
-                fprintf(stderr, "[ecl_scc] sweep mode na=%d sweeps=%lld\n", g.na, (long long)total);
-            *passes_out = total;
-            return ECL_SCC_OK;
-        }
+    CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
+    CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
+    if (use_dirty) {
+        CK(cudaMemsetAsync(D[0], 1, ntiles, s));
+        CK(cudaMemsetAsync(D[1], 0, ntiles, s));
     }
-    for (const int theta : thetas) {
-        CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
-        CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
-        if (use_dirty) {
-            CK(cudaMemsetAsync(D[0], 1, ntiles, s));
-            CK(cudaMemsetAsync(D[1], 0, ntiles, s));
-        }
-        int pass = 0;
-        int batch = 2;
-        for (;;) {
-            for (int k = 0; k < batch; k++, pass++) {
-                uint8_t* dc_ = use_dirty ? D[pass & 1] : nullptr;
-                uint8_t* dn_ = use_dirty ? D[(pass + 1) & 1] : nullptr;
-                if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>(chunk_buf(p, p->cb), nchunks, g, cin, cout, p->dc, pass, theta); }
-                const int full = (pass == 0 || nchunks > 0);
-                int r = ECL_SCC_OK;
-                if (use_pack) {
-                    static int run_env = -1;
-                    if (run_env < 0) run_env = getenv("ECL_SCC_RUN") ? std::max(1, atoi(getenv("ECL_SCC_RUN"))) : 4;
-                    const int run = (int)std::min<int64_t>(run_env, std::max<int64_t>(1, ntiles / (2 * 148)));
-                    p->launches++;
-                    k_prop_pack<<<(unsigned)cdiv(ntiles, run), PACK_TH, pack_dyn_smem(), s>>>(
-                        g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, pass, nchunks == 0, dc_, dn_, full, run);
-                    continue;
-                }
-                switch (p->tile) {
-                    case 512: r = launch_tile<512>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, theta, s); break;
-                    case 1024: r = launch_tile<1024>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, theta, s); break;
-                    case 4096: r = launch_tile<4096>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, theta, s); break;
-                    default: r = launch_tile<2048>(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, theta, s); break;
-                }
-                if (r) return r;
+    int pass = 0;
+    int batch = 2;
+    for (;;) {
+        for (int k = 0; k < batch; k++, pass++) {
+            uint8_t* dc_ = use_dirty ? D[pass & 1] : nullptr;
+            uint8_t* dn_ = use_dirty ? D[(pass + 1) & 1] : nullptr;
+            if (nchunks) { p->launches++; k_prop_heavy<<<hgrid, TPB, 0, s>>>(chunk_buf(p, p->cb), nchunks, g, cin, cout, p->dc, pass); }
+            const int full = (pass == 0 || nchunks > 0);
+            if (use_pack) {
+                const int run = pass_run(p, ntiles);
+                p->launches++;
+                k_prop_pack<<<(unsigned)cdiv(ntiles, run), PACK_TH, pack_dyn_smem(), s>>>(
+                    g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, pass, nchunks == 0, dc_, dn_, full, run);
+                continue;
             }
-            CK(cudaGetLastError());
-            CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
-            CK(cudaStreamSynchronize(s));
-            if (p->hc->changed[(pass - 1) & (RING - 1)] == 0) break;
-            // a monotone max over int32 IDs cannot take more passes than this
-            if ((int64_t)pass > 4 * (int64_t)g.na + 1024)
-                return fail(ECL_SCC_ECUDA, "internal: Phase 2 did not converge after %d passes", pass);
-            batch = std::min(batch * 2, RING / 2);
+            if (int r = launch_tile(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, s)) return r;
         }
-        total += (int64_t)p->hc->passes;
-        if (getenv("ECL_SCC_DEBUG"))
-            fprintf(stderr, "[ecl_scc] na=%d m=%d theta=%d passes=%llu visited_vertices=%llu\n", g.na,
-                    (int)0, theta, (unsigned long long)p->hc->passes, (unsigned long long)p->hc->visit_v);
+        CK(cudaGetLastError());
+        CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (p->hc->changed[(pass - 1) & (RING - 1)] == 0) break;
+        // a monotone max over int32 IDs cannot take more passes than this
+        if ((int64_t)pass > 4 * (int64_t)g.na + 1024)
+            return fail(ECL_SCC_ECUDA, "internal: Phase 2 did not converge after %d passes", pass);
+        batch = std::min(batch * 2, RING / 2);
     }
-    *passes_out = total;
-    return ECL_SCC_OK;
-}
-
-// Device-resident tail (tail.cuh): every remaining outer iteration of a small working graph
-// in one cooperative launch.  Threshold: live vertices (env ECL_SCC_TAIL_V).
-static int tail_threshold() {
-    static int v = -1;
-    if (v < 0) v = getenv("ECL_SCC_TAIL_V") ? std::max(0, atoi(getenv("ECL_SCC_TAIL_V"))) : 32768;
-    return v;
-}
-static int run_tail(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int32_t* labels, const Prio& P, int iter,
-                    bool trim, cudaStream_t s, TailTrace** out) {
-    if (!p->tail_dev) {
-        cudaError_t e = cudaMalloc(&p->tail_dev, sizeof(TailTrace));
-        if (e == cudaSuccess) e = cudaMallocHost(&p->tail_host, sizeof(TailTrace));
-        if (e != cudaSuccess) {
-            cudaGetLastError();
-            return fail(ECL_SCC_ENOMEM, "tail trace allocation: %s", cudaGetErrorString(e));
-        }
-        int per_sm = 0, dev = 0, sms = 0;
-        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_tail<false>, TAIL_TH, 0));
-        CK(cudaGetDevice(&dev));
-        CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-        p->tail_resident = std::max(1, std::min(per_sm, 1) * sms);    // one CTA per SM
-    }
-    TailTrace* T = (TailTrace*)p->tail_dev;
-    CK(cudaMemsetAsync(T, 0, sizeof(TailTrace), s));
-    // one CTA up to 2048 vertices (block barriers, L1-served re-reads), else ~2 vertices per
-    // thread (measured: one CTA on 7.5k vertices took 43 us per pass, 27 CTAs ~9 us)
-    int G = g.na <= 2048 ? 1 : (int)std::min<int64_t>(p->tail_resident, cdiv(g.na, 2 * TAIL_TH));
-    G = std::max(G, 1);
-    int32_t na = g.na;
-    const int32_t* act = g.act;
-    const int32_t* optr = g.optr;
-    int32_t* oadj = (int32_t*)g.oadj;
-    const int32_t* iptr = g.iptr;
-    int32_t* iadj = (int32_t*)g.iadj;
-    int32_t* kin = p->kin;
-    int32_t* kout = p->kout;
-    int32_t* alive = p->newidx;
-    const int32_t* orig = p->orig_cur;
-    int first = iter, tr = trim ? 1 : 0;
-    DevCounters* dc = p->dc;
-    void* args[] = {&na, &act, &optr, &oadj, &iptr, &iadj, &cin, &cout, &kin, &kout, &alive, &labels,
-                    (void*)&P, &orig, &first, &tr, &T, &dc};
-    p->launches++;
-    if (G == 1) CK(cudaLaunchCooperativeKernel((const void*)k_tail<true>, dim3(1), dim3(TAIL_TH), args, 0, s));
-    else CK(cudaLaunchCooperativeKernel((const void*)k_tail<false>, dim3(G), dim3(TAIL_TH), args, 0, s));
-    CK(cudaMemcpyAsync(p->tail_host, T, sizeof(TailTrace), cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    *out = (TailTrace*)p->tail_host;
-    if ((*out)->err) return fail(ECL_SCC_ECUDA, "internal: tail did not terminate");
+    if (getenv("ECL_SCC_DEBUG"))
+        fprintf(stderr, "[ecl_scc] na=%d passes=%llu visited_vertices=%llu\n", g.na,
+                (unsigned long long)p->hc->passes, (unsigned long long)p->hc->visit_v);
+    *passes_out = (int64_t)p->hc->passes;
     return ECL_SCC_OK;
 }
 
@@ -775,39 +594,9 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             cin = p->cin[ob];
             cout = p->cout[ob];
             if (t.y == 0) break;                                   // no live edge: done
-            // (the Phase-2 ablation flags keep their own Phase 2 to the end)
-            const uint32_t no_tail = ECL_SCC_SYNC_PASSES | ECL_SCC_NO_DIRTY | ECL_SCC_STAGED | ECL_SCC_SWEEP |
-                                     ECL_SCC_NO_PACK | ECL_SCC_NO_ASYNC;
-            if ((p->flags & ECL_SCC_TAIL) && !(p->flags & no_tail) && nchunks == 0 && stop_iter == 0 &&
-                t.x <= tail_threshold()) {
-                // the rest of the outer loop on the device (tail.cuh)
-                stage_mark(p, 4, s);
-                TailTrace* T = nullptr;
-                r = run_tail(p, g, p->cin[ob], p->cout[ob], labels, P, iter, trim, s, &T);
-                if (r) return r;
-                stage_mark(p, 5, s);
-                if (st && (p->flags & ECL_SCC_TIME_STAGES)) {
-                    CK(cudaEventSynchronize(p->ev[5]));
-                    const double mp = stage_ms(p, 2);
-                    st->ms_prop += mp;
-                    if (iter - 1 < ECL_SCC_TRACE_MAX) st->ms_prop_iter[iter - 1] = mp;
-                }
-                iters = T->last_iter;
-                if (st) {
-                    for (int k = iter; k <= T->last_iter; k++) {
-                        if (k - 1 >= ECL_SCC_TRACE_MAX) break;
-                        st->edges_in[k - 1] = k == iter ? t.y : T->edges_in[k - 1];
-                        st->vertices_in[k - 1] = k == iter ? t.x : T->vertices_in[k - 1];
-                        st->passes_iter[k - 1] = T->passes[k - 1];
-                        st->passes += T->passes[k - 1];
-                        if (k >= 2 && k > iter) st->edges_kept[k - 2] = T->edges_kept[k - 2];
-                    }
-                }
-                break;
-            }
             int64_t passes = 0;
             stage_mark(p, 4, s);
-            r = propagate(p, g, p->cin[ob], p->cout[ob], nchunks, n, s, &passes);
+            r = propagate(p, g, p->cin[ob], p->cout[ob], nchunks, s, &passes);
             if (r) return r;
             stage_mark(p, 5, s);
             if (st && (p->flags & ECL_SCC_TIME_STAGES)) {
@@ -982,6 +771,13 @@ int run_levels(Plan* p, int32_t n, const int32_t* rp, const int32_t* ci, const i
     CK(cudaMemsetAsync(ctl, 0, sizeof(LvCtl), s));
     const unsigned gs = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
     p->launches++; k_lv_count<<<gs, TPB, 0, s>>>(n, rp, ci, lab, indeg, msize, &ctl->err);
+    CK(cudaGetLastError());
+    {   // every later kernel indexes by label: reject labels outside [0, n) before them
+        int err = 0;
+        CK(cudaMemcpyAsync(&err, &ctl->err, sizeof(int), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (err) return fail(ECL_SCC_ERANGE, "levels: a label lies outside [0, n)");
+    }
     int r = scan_excl<I1>(p, (const I1*)msize, n, (I1*)mptr, (I1*)&p->dc->grand1, p->bsum, 1, s);
     if (r) return r;
     p->launches++; k_lv_fill<<<gs, TPB, 0, s>>>(n, lab, mptr, cursor, memb);

@@ -18,7 +18,7 @@ struct Plan {
     int32_t *act[2], *cin[2], *cout[2];  // vertex IDs and signatures v_in / v_out
     int32_t *optr[2], *iptr[2];          // CSR / CSC offsets
     int32_t *oadj[2], *iadj[2];          // CSR / CSC adjacency
-    int32_t *kin, *kout;                 // two n+1 int views (ingest histogram / cursor, relabel, tail, levels)
+    int32_t *kin, *kout;                 // two n+1 int views (ingest histogram / cursor, relabel, levels)
     int2* kio;                           // the same memory as interleaved kept degrees {in, out} (compaction)
     int32_t* newidx;                     // old local -> new local (-1: leaves)
     int2* cnt;                           // per-vertex surviving (out, in) degree
@@ -39,15 +39,9 @@ struct Plan {
     int64_t u_n_cap, u_m_cap;
     uint8_t* dirty;                      // 2 x dirty_cap tile flags (Phase-2 skipping)
     int64_t dirty_cap;
-    int tile;                            // Phase-2 tile size (vertices per CTA)
-    uint8_t* lvl;                        // level-sweep mode: intra-tile level per vertex
     // storage reordering (reorder.cuh): permuted input CSR and the storage -> caller ID map
     int32_t *rp2, *ci2, *orig, *pos, *cellv, *fa, *fb, *cellbuf, *rcnt;
     const int32_t* orig_cur;             // orig when the current run is reordered, else null
-    int *nb_cnt, *nb_list;               // sweep mode: neighbour tiles of each tile
-    int *done, *mark;                    // sweep mode: per-tile done / dirty epochs
-    int* sweep_ctr;                      // [0] tile counter, [1] changed, [2] overflow
-    int epoch;                           // sweep epoch (monotone over the plan's life)
     unsigned long long *pnin, *pnout;    // tile packs (pack.cuh): slot words per local vertex
     int2* ext;                           // tile packs: cut edges per tile
     bool pack_fused;                     // the last compaction's scatter wrote the tile pack
@@ -55,10 +49,13 @@ struct Plan {
     int* aq_state;                       // asynchronous Phase 2 (pack.cuh AsyncQ)
     uint8_t* aq_seen;
     unsigned long long* aq_ctr;
-    int64_t aq_resident;                 // resident CTAs of k_prop_async
-    void* tail_dev;                      // tail.cuh TailTrace (device) and its pinned mirror
-    void* tail_host;
-    int tail_resident;                   // co-resident CTAs of k_tail
+    int64_t aq_resident;                 // resident CTAs of k_prop_async (this plan's device)
+    int device;                          // the device the plan was created on
+    bool tile_attrs;                     // k_prop_tile / k_prop_pack attributes set on `device`
+    // tuning knobs, read from the environment once when the plan is created (development
+    // only; the defaults are the measured best): ECL_SCC_RUN, ECL_SCC_CLAIM,
+    // ECL_SCC_CLAIM_DIV, ECL_SCC_CLAIM_MAX, ECL_SCC_ASYNC_CTAS
+    int knob_run, knob_claim, knob_claim_div, knob_claim_max, knob_async_ctas;
     void* lv_ctl;                        // levels.cuh LvCtl (device)
     int32_t *h_rp, *h_ci, *h_lab;        // ecl_scc_host: device copies of the caller's host buffers
     int64_t h_n_cap, h_m_cap;

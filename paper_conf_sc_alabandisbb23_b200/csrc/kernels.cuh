@@ -742,16 +742,11 @@ __device__ __forceinline__ bool pass_begin(DevCounters* dc, int pass, bool first
     return true;
 }
 
-// Threshold stages: within a stage only signature values
-// >= theta take part in propagation; smaller values wait for a later stage.  The last
-// stage has theta = 0, so the final state is the ordinary fixed point.
-__device__ __forceinline__ int eff(int x, int theta) { return x >= theta ? x : -1; }
-
 // Heavy rows: one warp per chunk of a long row; the chunk max is folded in with
 // atomicMax (monotone, so concurrent chunks of one row commute).
 static __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restrict__ chunks, int nchunks, WGraph g,
                                                     int32_t* __restrict__ cin, int32_t* __restrict__ cout,
-                                                    DevCounters* __restrict__ dc, int pass, int theta) {
+                                                    DevCounters* __restrict__ dc, int pass) {
     if (!pass_begin(dc, pass, true)) return;
     const int lane = threadIdx.x & 31;
     const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -763,7 +758,7 @@ static __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restri
         const int32_t* adj = k.dir ? g.iadj : g.oadj;
         int32_t* sig = k.dir ? cin : cout;
         int acc = 0;
-        for (int e = k.beg + lane; e < k.end; e += WARP) acc = max(acc, eff(ld_cg(sig + __ldg(adj + e)), theta));
+        for (int e = k.beg + lane; e < k.end; e += WARP) acc = max(acc, ld_cg(sig + __ldg(adj + e)));
         acc = warp_max(acc);
         ne += k.end - k.beg;
         if (lane == 0 && acc > ld_cg(sig + k.i)) {
@@ -789,8 +784,7 @@ static __global__ void __launch_bounds__(256) k_prop_heavy(const Chunk* __restri
 //   3. write raised signatures back and flag the out-of-tile dependents' tiles dirty.
 // Rows longer than HEAVY_T are skipped here (k_prop_heavy folds them in).  Tile order
 // alternates with the pass parity so values can ride the block schedule both ways.
-// theta: threshold stage (only values >= theta propagate).
-// full: every vertex (with a value >= theta) starts flagged and step 1 also pulls the intra-tile neighbours'
+// full: every vertex starts flagged and step 1 also pulls the intra-tile neighbours'
 // values (first visit of a phase, and every visit when heavy rows exist: an intra-tile
 // edge whose source row is heavy is not in any push list, so it is covered by the pull).
 // SYNC = ablation: no step 2 (one relaxation per pass, "separate kernels").
@@ -838,44 +832,17 @@ struct TileSmem {
     unsigned long long* s_nout;
     unsigned* s_fin;
     unsigned* s_fout;
-    unsigned short* s_queue;      // drain item queues; level-sweep order + level starts
-    uint8_t* s_lv;                // level-sweep: intra-tile level of each vertex
+    unsigned short* s_queue;      // drain item queues (k_prop_tile)
     unsigned long long* s_acc;    // pack kernels: per-CTA visited vertices / edges (thread 0), flushed once
 };
 
-// pull of one vertex over its slots (and its global row when it is a slow row)
-__device__ __forceinline__ int pull_slots(const int* sig, unsigned long long src, const int32_t* __restrict__ sptr,
-                                          const int32_t* __restrict__ sadj, int base, int cnt, int v, int val) {
-#pragma unroll
-    for (int q = 0; q < 4; q++) {
-        const unsigned w = (unsigned)(src >> (16 * q)) & 0xFFFFu;
-        if (w == 0xFFFFu) break;
-        val = max(val, ((volatile const int*)sig)[w & 0x7FFFu]);
-    }
-    if ((src & (0x8000ull << 48)) && (src >> 48) != 0xFFFFull)
-        for (int e = __ldg(sptr + base + v), ee = __ldg(sptr + base + v + 1); e < ee; e++) {
-            const int w = __ldg(sadj + e) - base;
-            if ((unsigned)w < (unsigned)cnt) val = max(val, ((volatile const int*)sig)[w]);
-        }
-    return val;
-}
-
 // dirty marking of the tiles that depend on a raised value (pass mode: byte flags for
-// the next pass; sweep mode: the current sweep epoch)
+// the next pass)
 struct MarkNext {
     uint8_t* next;
     __device__ __forceinline__ bool on() const { return next != nullptr; }
     __device__ __forceinline__ void operator()(int t) const { next[t] = 1; }
 };
-struct MarkEpoch {
-    int* mark;
-    int epoch;
-    __device__ __forceinline__ bool on() const { return true; }
-    __device__ __forceinline__ void operator()(int t) const {
-        if (((volatile int*)mark)[t] != epoch) mark[t] = epoch;
-    }
-};
-
 // flag the intra-tile vertices in slot word nb (and, for a slow row, the rest of the
 // global row) for a re-pull: plain byte stores
 __device__ __forceinline__ void notify(unsigned long long nb, const int32_t* __restrict__ ptr,
@@ -979,9 +946,8 @@ __device__ __forceinline__ void drain_local(const WGraph& g, int* __restrict__ s
 // every thread if a signature was raised.
 template <bool SYNC, int TT, typename Mark>
 __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__ cin, int32_t* __restrict__ cout,
-                                          DevCounters* __restrict__ dc, int tile, int full, int theta, Mark mark,
-                                          const TileSmem<TT>& S, int kcap = 0, int* capped = nullptr,
-                                          uint8_t* __restrict__ lvl = nullptr) {
+                                          DevCounters* __restrict__ dc, int tile, int full, Mark mark,
+                                          const TileSmem<TT>& S) {
     int* s_in = S.s_in;
     int* s_out = S.s_out;
     unsigned long long* s_nin = S.s_nin;
@@ -1019,21 +985,21 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
             int ns = 0;
             for (int e = ib; e < ie; e++) {
                 const int u = __ldg(g.iadj + e);
-                if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) { x = max(x, eff(ld_cg(cin + u), theta)); continue; }
-                if (full) x = max(x, eff(ld_cg(cin + u), theta));   // see "full" above: heavy rows do not push
+                if (SYNC || (unsigned)(u - base) >= (unsigned)cnt) { x = max(x, ld_cg(cin + u)); continue; }
+                if (full) x = max(x, ld_cg(cin + u));   // see "full" above: heavy rows do not push
                 if (ns < SLOTS) add_slot(ni, ns, (unsigned)(u - base));
                 else ni |= SLOW_MARK;
             }
             ns = 0;
             for (int e = ob; e < oe; e++) {
                 const int w = __ldg(g.oadj + e);
-                if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) { y = max(y, eff(ld_cg(cout + w), theta)); continue; }
-                if (full) y = max(y, eff(ld_cg(cout + w), theta));
+                if (SYNC || (unsigned)(w - base) >= (unsigned)cnt) { y = max(y, ld_cg(cout + w)); continue; }
+                if (full) y = max(y, ld_cg(cout + w));
                 if (ns < SLOTS) add_slot(no, ns, (unsigned)(w - base));
                 else no |= SLOW_MARK;
             }
-            if ((full && x >= theta) || x > x0) fin |= 1u << (8 * k);
-            if ((full && y >= theta) || y > y0) fout |= 1u << (8 * k);
+            if (full || x > x0) fin |= 1u << (8 * k);
+            if (full || y > y0) fout |= 1u << (8 * k);
         }
         if (v < TT) {
             s_in[v] = x;
@@ -1079,156 +1045,7 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
     // warp are compacted into a per-warp queue so all lanes run the same path; each warp
     // drains its own 128 vertices, block rounds repeat until a round does no work.  No
     // shared-memory atomic touches the signatures.
-    // ---- step 2 (level-sweep variant): intra-tile levels (longest path from the tile's
-    // sources over intra edges, by relaxation, capped) are computed on the first visit of
-    // a phase and kept in `lvl`; every visit then pulls v_in in ascending and v_out in
-    // descending level order -- one pull per vertex per sweep for the acyclic part -- and
-    // checks with one Jacobi round; cycles left over fall through to the drain loop.
-    bool need_drain = true;
-    if (!SYNC && lvl && kcap == 0) {
-        int* s_L = (int*)S.s_queue;                          // [TT] ints during the level build
-        uint8_t* s_lv = S.s_lv;
-        if (full) {
-            for (int v = tid; v < TT; v += TT / VPT) s_L[v] = 0;
-            __syncthreads();
-            for (int r = 0; r < 64; r++) {
-                int any = 0;
-#pragma unroll
-                for (int k = 0; k < VPT; k++) {
-                    const int v = tid * VPT + k;
-                    if (v >= cnt) continue;
-                    const unsigned long long src = s_nin[v];
-                    int l = ((volatile int*)s_L)[v];
-                    const int l0 = l;
-#pragma unroll
-                    for (int q = 0; q < 4; q++) {
-                        const unsigned w = (unsigned)(src >> (16 * q)) & 0xFFFFu;
-                        if (w == 0xFFFFu) break;
-                        l = max(l, ((volatile int*)s_L)[w & 0x7FFFu] + 1);
-                    }
-                    l = min(l, 250);
-                    if (l > l0) { ((volatile int*)s_L)[v] = l; any = 1; }
-                }
-                if (!__syncthreads_or(any)) break;
-            }
-            for (int v = tid; v < cnt; v += TT / VPT) {
-                s_lv[v] = (uint8_t)s_L[v];
-                lvl[base + v] = (uint8_t)s_L[v];
-            }
-        } else {
-            for (int v = tid; v < cnt; v += TT / VPT) s_lv[v] = __ldg(lvl + base + v);
-        }
-        __syncthreads();
-        // counting sort by level: order[] (u16) and level starts in the queue area
-        unsigned short* order = S.s_queue;
-        int* lstart = (int*)(S.s_queue + TT);                  // [257]
-        for (int i = tid; i < 257; i += TT / VPT) lstart[i] = 0;
-        __syncthreads();
-        for (int v = tid; v < cnt; v += TT / VPT) atomicAdd(lstart + s_lv[v] + 1, 1);
-        __syncthreads();
-        if (tid < 32) {                                        // exclusive scan of 256 bins by one warp
-            int carry = 0;
-            for (int b0 = 0; b0 < 256; b0 += 32) {
-                const int x = lstart[b0 + 1 + tid];
-                const int inc = warp_incl_scan(x, tid);
-                lstart[b0 + 1 + tid] = carry + inc;
-                carry += __shfl_sync(FULL, inc, 31);
-            }
-        }
-        __syncthreads();
-        int maxl = 0;
-        for (int v = tid; v < cnt; v += TT / VPT) maxl = max(maxl, (int)s_lv[v]);
-        // scatter (positions via a per-level cursor reusing the s_fin area)
-        int* cursor = (int*)S.s_fin;                           // >= 256 ints (TT/VPT >= 256)
-        for (int i = tid; i < 256; i += TT / VPT) cursor[i] = 0;
-        __syncthreads();
-        for (int v = tid; v < cnt; v += TT / VPT) {
-            const int l = s_lv[v];
-            order[lstart[l] + atomicAdd(cursor + l, 1)] = (unsigned short)v;
-        }
-        // every thread needs the maximum level
-        maxl = __reduce_max_sync(FULL, maxl);
-        __shared__ int s_maxl;
-        if (tid == 0) s_maxl = 0;
-        __syncthreads();
-        if ((tid & 31) == 0) atomicMax(&s_maxl, maxl);
-        __syncthreads();
-        maxl = s_maxl;
-        for (int rep = 0; rep < 3 && need_drain; rep++) {
-            // sweeps: v_in at level l (ascending), v_out at level maxl-l (descending)
-            for (int l = 0; l <= maxl; l++) {
-                for (int i = lstart[l] + tid; i < lstart[l + 1]; i += TT / VPT) {
-                    const int v = order[i];
-                    const int old = ((volatile int*)s_in)[v];
-                    const int val = pull_slots(s_in, s_nin[v], g.iptr, g.iadj, base, cnt, v, old);
-                    if (val > old) ((volatile int*)s_in)[v] = val;
-                }
-                const int lo = maxl - l;
-                for (int i = lstart[lo] + tid; i < lstart[lo + 1]; i += TT / VPT) {
-                    const int v = order[i];
-                    const int old = ((volatile int*)s_out)[v];
-                    const int val = pull_slots(s_out, s_nout[v], g.optr, g.oadj, base, cnt, v, old);
-                    if (val > old) ((volatile int*)s_out)[v] = val;
-                }
-                __syncthreads();
-            }
-            // check: one Jacobi round; no change means the local fixed point
-            int any = 0;
-#pragma unroll
-            for (int k = 0; k < VPT; k++) {
-                const int v = tid * VPT + k;
-                if (v >= cnt) continue;
-                int old = ((volatile int*)s_in)[v];
-                int val = pull_slots(s_in, s_nin[v], g.iptr, g.iadj, base, cnt, v, old);
-                if (val > old) { ((volatile int*)s_in)[v] = val; any = 1; }
-                old = ((volatile int*)s_out)[v];
-                val = pull_slots(s_out, s_nout[v], g.optr, g.oadj, base, cnt, v, old);
-                if (val > old) { ((volatile int*)s_out)[v] = val; any = 1; }
-            }
-            need_drain = __syncthreads_or(any) != 0;
-        }
-        if (need_drain) {                                      // cycles: finish with the drains
-            s_fin[tid] = 0x01010101u;
-            s_fout[tid] = 0x01010101u;
-        }
-        __syncthreads();
-    }
-    if (!SYNC && kcap > 0) {
-        // bounded variant: at most kcap SIMD Jacobi rounds over the slots (each thread
-        // re-pulls its four vertices every round); a tile still changing after kcap rounds
-        // reports `capped` and is revisited in the next pass
-        for (int r = 0; r < kcap; r++) {
-            int any = 0;
-#pragma unroll
-            for (int k = 0; k < VPT; k++) {
-                const int v = tid * VPT + k;
-                if (v >= cnt) continue;
-                for (int dir = 0; dir < 2; dir++) {
-                    int* sig = dir ? s_out : s_in;
-                    const unsigned long long src = dir ? s_nout[v] : s_nin[v];
-                    const int old = ((volatile int*)sig)[v];
-                    int val = old;
-#pragma unroll
-                    for (int q = 0; q < SLOTS; q++) {
-                        const unsigned w = (unsigned)(src >> (16 * q)) & 0xFFFFu;
-                        if (w == NOSLOT) break;
-                        val = max(val, ((volatile int*)sig)[w & 0x7FFFu]);
-                    }
-                    if ((src & SLOW_MARK) && (src >> 48) != 0xFFFFull) {
-                        const int32_t* sptr = dir ? g.optr : g.iptr;
-                        const int32_t* sadj = dir ? g.oadj : g.iadj;
-                        for (int e = __ldg(sptr + base + v), ee = __ldg(sptr + base + v + 1); e < ee; e++) {
-                            const int w = __ldg(sadj + e) - base;
-                            if ((unsigned)w < (unsigned)cnt) val = max(val, ((volatile int*)sig)[w]);
-                        }
-                    }
-                    if (val > old) { ((volatile int*)sig)[v] = val; any = 1; }
-                }
-            }
-            if (!__syncthreads_or(any)) break;
-            if (r == kcap - 1 && capped) *capped = 1;
-        }
-    } else if (!SYNC && need_drain) {
+    if (!SYNC) {
 #ifndef ECL_PROF
         unsigned prof_rounds = 0, prof_drains = 0, prof_pushes = 0;
 #endif
@@ -1286,12 +1103,10 @@ __device__ __forceinline__ int tile_visit(const WGraph& g, int32_t* __restrict__
 template <bool SYNC, int TT>
 static __global__ void __launch_bounds__(TT / VPT, (1536 / (TT / VPT)) > 0 ? 1536 / (TT / VPT) : 1)
 k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, DevCounters* __restrict__ dc, int pass,
-            int first, uint8_t* __restrict__ dirty_cur, uint8_t* __restrict__ dirty_next, int full, int theta,
-            int run, int kcap, uint8_t* __restrict__ lvl) {
+            int first, uint8_t* __restrict__ dirty_cur, uint8_t* __restrict__ dirty_next, int full, int run) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];             // raise flags, byte k = vertex 4t+k
-    __shared__ unsigned short s_queue[2 * TT + 2 * 260];               // per-warp item queues / level order
-    __shared__ uint8_t s_lv[TT];
+    __shared__ unsigned short s_queue[2 * TT];                         // per-warp item queues
     __shared__ int s_dirty;
     TileSmem<TT> S;
     S.s_in = (int*)smem_raw;
@@ -1301,7 +1116,6 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
     S.s_fin = s_fin;
     S.s_fout = s_fout;
     S.s_queue = s_queue;
-    S.s_lv = s_lv;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + TT - 1) / TT;
     const int tid = threadIdx.x;
@@ -1326,131 +1140,10 @@ k_prop_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, Dev
             __syncthreads();             // everyone has read s_dirty before thread 0 rewrites it
             if (!d) continue;
         }
-        int capped = 0;
-        ch_any |= tile_visit<SYNC, TT>(g, cin, cout, dc, tile, full, theta, MarkNext{dirty_next}, S, kcap, &capped, lvl);
-        if (capped && dirty_next && tid == 0) dirty_next[tile] = 1;   // not converged: come back
+        ch_any |= tile_visit<SYNC, TT>(g, cin, cout, dc, tile, full, MarkNext{dirty_next}, S);
         __syncthreads();                                     // shared memory is reused by the next tile
     }
     if (ch_any && tid == 0) dc->changed[pass & (RING - 1)] = 1;
-}
-
-// ---------------------------------------------------------------------- sweep mode
-// Neighbour tiles of every tile (distinct tiles holding an endpoint of one of its edges),
-// for the dependency-ordered sweeps.  One CTA per tile, set in shared memory; more than
-// NBCAP neighbours sets *overflow (the driver then uses pass mode).
-constexpr int NBCAP = 64;
-template <int TT>
-static __global__ void __launch_bounds__(256) k_tile_nbrs(WGraph g, int* __restrict__ nb_cnt, int* __restrict__ nb_list,
-                                                          int* __restrict__ overflow) {
-    __shared__ int set[2 * NBCAP];
-    __shared__ int n_set, ovf;
-    const int tile = blockIdx.x, base = tile * TT, cnt = min(TT, g.na - base);
-    for (int i = threadIdx.x; i < 2 * NBCAP; i += blockDim.x) set[i] = -1;
-    if (threadIdx.x == 0) { n_set = 0; ovf = 0; }
-    __syncthreads();
-    for (int v = threadIdx.x; v < cnt; v += blockDim.x) {
-        for (int dir = 0; dir < 2; dir++) {
-            const int32_t* ptr = dir ? g.iptr : g.optr;
-            const int32_t* adj = dir ? g.iadj : g.oadj;
-            for (int e = ptr[base + v], ee = ptr[base + v + 1]; e < ee; e++) {
-                const int t = adj[e] / TT;
-                if (t == tile) continue;
-                unsigned h = ((unsigned)t * 2654435761u) & (2 * NBCAP - 1);
-                for (int probe = 0; probe < 2 * NBCAP; probe++) {
-                    const int cur = set[h];
-                    if (cur == t) break;
-                    if (cur == -1) {
-                        const int old = atomicCAS(set + h, -1, t);
-                        if (old == -1) {
-                            if (atomicAdd(&n_set, 1) >= NBCAP) ovf = 1;
-                            break;
-                        }
-                        if (old == t) break;
-                    }
-                    h = (h + 1) & (2 * NBCAP - 1);
-                    if (probe == 2 * NBCAP - 1) ovf = 1;
-                }
-            }
-        }
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        int k = 0;
-        if (!ovf)
-            for (int i = 0; i < 2 * NBCAP; i++)
-                if (set[i] >= 0) nb_list[tile * NBCAP + k++] = set[i];
-        nb_cnt[tile] = k;
-        if (ovf) *overflow = 1;
-    }
-}
-
-__device__ __forceinline__ int ld_acquire(const int* p) {
-    int v;
-    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_release(int* p, int v) {
-    asm volatile("st.release.gpu.global.b32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
-}
-
-// One dependency-ordered sweep (persistent CTAs).  Tiles are taken in index order
-// (backward when dir = 1) from a counter; a tile first waits until every neighbour tile
-// that precedes it in this order has finished (done[] >= epoch), so values flowing along
-// the order cross any number of tiles in one sweep.  It is visited if it is the first
-// sweep of the phase or a neighbour raised one of its inputs since the previous sweep
-// (mark >= epoch - 1); then it publishes done = epoch.  Dependencies against the order
-// are left to the next sweep; a sweep without any raise certifies the fixed point.
-template <int TT>
-static __global__ void __launch_bounds__(TT / VPT, (1536 / (TT / VPT)) > 0 ? 1536 / (TT / VPT) : 1)
-k_sweep_tile(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, DevCounters* __restrict__ dc,
-             const int* __restrict__ nb_cnt, const int* __restrict__ nb_list, int* __restrict__ done,
-             int* __restrict__ mark, int* __restrict__ counter, int epoch, int first_sweep, int dir,
-             int* __restrict__ changed) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ unsigned s_fin[TT / VPT], s_fout[TT / VPT];
-    __shared__ unsigned short s_queue[2 * TT];
-    __shared__ int s_idx, s_go;
-    TileSmem<TT> S;
-    S.s_in = (int*)smem_raw;
-    S.s_out = S.s_in + TT;
-    S.s_nin = (unsigned long long*)(S.s_out + TT);
-    S.s_nout = S.s_nin + TT;
-    S.s_fin = s_fin;
-    S.s_fout = s_fout;
-    S.s_queue = s_queue;
-    const int ntiles = (g.na + TT - 1) / TT;
-    const int tid = threadIdx.x;
-    int ch_any = 0;
-    for (;;) {
-        if (tid == 0) s_idx = atomicAdd(counter, 1);
-        __syncthreads();
-        const int idx = s_idx;
-        if (idx >= ntiles) break;
-        const int tile = dir ? ntiles - 1 - idx : idx;
-        // wait for the preceding neighbours (all of them were taken earlier: no deadlock)
-        const int nn = nb_cnt[tile];
-        for (int j = tid; j < nn; j += blockDim.x) {
-            const int nb = nb_list[tile * NBCAP + j];
-            if (dir ? nb > tile : nb < tile) {
-                // bounded wait (a bug must not hang the GPU): give up after ~1 s
-                for (unsigned spin = 0; ld_acquire(done + nb) < epoch; spin++) {
-                    if (spin > (1u << 24)) { dc->err = 2; break; }
-                    __nanosleep(64);
-                }
-            }
-        }
-        __syncthreads();
-        if (tid == 0) s_go = first_sweep || ld_acquire(mark + tile) >= epoch - 1;
-        __syncthreads();
-        if (s_go) {
-            const int ch = tile_visit<false, TT>(g, cin, cout, dc, tile, first_sweep, 0, MarkEpoch{mark, epoch}, S);
-            ch_any |= ch;
-            __threadfence();
-        }
-        __syncthreads();
-        if (tid == 0) st_release(done + tile, epoch);
-    }
-    if (ch_any && tid == 0) *changed = 1;
 }
 
 }  // namespace eclscc

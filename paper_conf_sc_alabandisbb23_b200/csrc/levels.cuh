@@ -21,9 +21,28 @@
 // SCCs never reached mean the labels induce a cycle (not the SCC partition): ERANGE.
 #pragma once
 #include "common.cuh"
-#include "tail.cuh"          // tail_bar: the grid barrier of a cooperative launch
 
 namespace eclscc {
+
+// grid barrier among the co-resident CTAs of a cooperative launch (one CTA: a block barrier)
+__device__ __forceinline__ void grid_bar(unsigned* bar, int G) {
+    __syncthreads();
+    if (G == 1) return;
+    if (threadIdx.x == 0) {
+        volatile unsigned* vb = bar;
+        const unsigned gen = vb[1];
+        __threadfence();
+        if (atomicAdd(bar, 1u) == (unsigned)G - 1) {
+            vb[0] = 0;
+            __threadfence();
+            atomicAdd(bar + 1, 1u);
+        } else {
+            while (vb[1] == gen) __nanosleep(20);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
 
 struct LvCtl {
     unsigned bar[2];         // grid barrier
@@ -219,7 +238,7 @@ static __global__ void __launch_bounds__(512) k_lv_run(const int32_t* __restrict
 
         if (blockIdx.x == 0 && threadIdx.x == 0) ctl->size[(l + 2) % 3] = 0;   // read two rounds ago
         __threadfence();
-        tail_bar(ctl->bar, G);
+        grid_bar(ctl->bar, G);
         if (*(volatile int*)&ctl->size[(l + 1) % 3] == 0) {
             if (blockIdx.x == 0 && threadIdx.x == 0) {
                 ctl->depth = ncur > 0 ? l + 1 : l;

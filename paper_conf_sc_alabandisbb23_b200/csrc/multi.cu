@@ -52,7 +52,7 @@ struct PRank {
     int32_t *cp = nullptr, *cr = nullptr, *ideg = nullptr;   // CSC of own edges, n columns
     int32_t* sig = nullptr;                      // [in(n) | out(n) | changed(1)] replica
     int32_t* kdeg = nullptr;                     // [kin(n) | kout(n)]
-    int32_t* cnt = nullptr;                      // [live edges (int32 for the SUM), err, ring(RING)]
+    int32_t* cnt = nullptr;                      // [live edges (int32 for the SUM), err, ring(RING), touched]
     unsigned long long* live = nullptr;
     void* bsum = nullptr;
     int32_t* grand = nullptr;
@@ -61,13 +61,48 @@ struct PRank {
         cudaFree(sig); cudaFree(kdeg); cudaFree(cnt); cudaFree(live); cudaFree(bsum); cudaFree(grand);
     }
     int* ring() const { return cnt + 2; }
+    int* touched() const { return cnt + 2 + RING; }
 };
 
-// all-reduce over the ranks of this process (1 with NCCL, P when emulated)
+// all-reduce over the ranks of this process (1 with NCCL, P when emulated).  Every exchange
+// is bracketed by CUDA events on the call's stream (stats->ms_comm: the communication
+// share); the event pool is owned by the caller (a plan) and reused.
 struct Exchange {
+    std::vector<cudaEvent_t>* ev = nullptr;   // pool of event pairs
+    int used = 0;                             // pairs recorded by the current call
+    int64_t bytes = 0;                        // bytes this rank contributed
     virtual ~Exchange() {}
     // op 0 = MAX, 1 = SUM; bufs[r] = rank r's buffer of `count` int32
-    virtual int allreduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) = 0;
+    virtual int reduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) = 0;
+    int allreduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) {
+        cudaEvent_t a = nullptr, b = nullptr;
+        if (ev) {
+            if ((size_t)(2 * used + 2) > ev->size()) {
+                for (int k = 0; k < 2; k++) {
+                    cudaEvent_t e;
+                    CKM(cudaEventCreate(&e));
+                    ev->push_back(e);
+                }
+            }
+            a = (*ev)[2 * used];
+            b = (*ev)[2 * used + 1];
+            used++;
+            CKM(cudaEventRecord(a, s));
+        }
+        if (int r = reduce(bufs, count, op, s)) return r;
+        if (ev) CKM(cudaEventRecord(b, s));
+        bytes += 4 * count;
+        return ECL_SCC_OK;
+    }
+    double ms() const {                       // after a stream synchronisation
+        double t = 0;
+        for (int k = 0; ev && k < used; k++) {
+            float x = 0.f;
+            if (cudaEventElapsedTime(&x, (*ev)[2 * k], (*ev)[2 * k + 1]) == cudaSuccess) t += x;
+            else cudaGetLastError();
+        }
+        return t;
+    }
 };
 
 struct EmulatedExchange : Exchange {
@@ -75,7 +110,7 @@ struct EmulatedExchange : Exchange {
     int P = 0;
     explicit EmulatedExchange(int p) : P(p) {}
     ~EmulatedExchange() { cudaFree(dptrs); }
-    int allreduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) override {
+    int reduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) override {
         if (P == 1) return ECL_SCC_OK;
         if (!dptrs) CKM(cudaMalloc((void**)&dptrs, sizeof(int32_t*) * P));
         CKM(cudaMemcpyAsync(dptrs, bufs.data(), sizeof(int32_t*) * P, cudaMemcpyHostToDevice, s));
@@ -88,7 +123,7 @@ struct EmulatedExchange : Exchange {
 struct NcclExchange : Exchange {
     ncclComm_t comm;
     explicit NcclExchange(ncclComm_t c) : comm(c) {}
-    int allreduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) override {
+    int reduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) override {
         CKN(ncclAllReduce(bufs[0], bufs[0], (size_t)count, ncclInt32, op == 0 ? ncclMax : ncclSum, comm, s));
         return ECL_SCC_OK;
     }
@@ -104,7 +139,7 @@ static int rank_alloc(PRank& R, int32_t n) {
     e = e ? e : cudaMalloc((void**)&R.ideg, n1 * 4);
     e = e ? e : cudaMalloc((void**)&R.sig, (2 * n1 + 1) * 4);
     e = e ? e : cudaMalloc((void**)&R.kdeg, 2 * n1 * 4);
-    e = e ? e : cudaMalloc((void**)&R.cnt, (2 + RING) * 4);
+    e = e ? e : cudaMalloc((void**)&R.cnt, (3 + RING) * 4);
     e = e ? e : cudaMalloc((void**)&R.live, 8);
     e = e ? e : cudaMalloc((void**)&R.bsum, ((n1 + SCAN_TILE - 1) / SCAN_TILE + 1) * sizeof(int4));
     e = e ? e : cudaMalloc((void**)&R.grand, 16);
@@ -115,7 +150,9 @@ static int rank_alloc(PRank& R, int32_t n) {
     return ECL_SCC_OK;
 }
 
-__global__ void k_copy_flag(const int* __restrict__ ring, int32_t* __restrict__ dst) { *dst = ring[0]; }
+__global__ void k_copy_flag(const int* __restrict__ touched, int32_t* __restrict__ dst, int err) {
+    *dst = err ? err : *touched;
+}
 __global__ void k_live_to_i32(const unsigned long long* __restrict__ live, int32_t* __restrict__ dst) {
     *dst = (int32_t)*live;
 }
@@ -135,15 +172,24 @@ static int run_partitioned(std::vector<PRank*>& R, Exchange& X, int32_t n, uint3
     for (int r = 0; r < P; r++) {
         PRank& Q = *R[r];
         sigs[r] = Q.sig; kdegs[r] = Q.kdeg; cnts[r] = Q.cnt;
-        CKM(cudaMemsetAsync(Q.cnt, 0, (2 + RING) * 4, s));
+        CKM(cudaMemsetAsync(Q.cnt, 0, (3 + RING) * 4, s));
         if (!(flags & ECL_SCC_NO_VALIDATE) && Q.nloc > 0) {
             part::k_validate_part<<<std::min<unsigned>(gridn(std::max<int64_t>(Q.nloc, Q.m)), 148 * 16), 256, 0, s>>>(
                 Q.nloc, Q.m, Q.rp, Q.ci, n, Q.cnt + 1);
             launches++;
         }
-        CKM(cudaMemcpyAsync(hbuf, Q.cnt, 8, cudaMemcpyDeviceToHost, s));
+    }
+    {   // every rank learns whether any rank's input is invalid, so all return together
+        // instead of leaving the others blocked in the next collective
+        std::vector<int32_t*> errs(P);
+        for (int r = 0; r < P; r++) errs[r] = R[r]->cnt + 1;
+        if (int e = X.allreduce(errs, 1, 0, s)) return e;
+        CKM(cudaMemcpyAsync(hbuf, R[0]->cnt, 8, cudaMemcpyDeviceToHost, s));
         CKM(cudaStreamSynchronize(s));
-        if (hbuf[1]) return fail(ECL_SCC_ERANGE, "partition %d: invalid local CSR", r);
+        if (hbuf[1]) return fail(ECL_SCC_ERANGE, "partitioned: invalid local CSR on some rank");
+    }
+    for (int r = 0; r < P; r++) {
+        PRank& Q = *R[r];
         if (Q.nloc > 0) {
             part::k_copy_rows<<<gridn(Q.nloc), 256, 0, s>>>(Q.nloc, Q.rb, Q.rp, Q.ci, Q.wci, Q.odeg);
             launches++;
@@ -210,35 +256,40 @@ static int run_partitioned(std::vector<PRank*>& R, Exchange& X, int32_t n, uint3
         if (st && iter >= 2 && iter - 2 < ECL_SCC_TRACE_MAX) st->edges_kept[iter - 2] = live;   // (after trim)
         // ---- Phase 2: local fixed points + all-reduce(MAX) until no rank changes
         int64_t passes_iter = 0;
+        int local_err = 0;
         for (;;) {
             for (int r = 0; r < P; r++) {
                 PRank& Q = *R[r];
                 int* ring = Q.ring();
-                CKM(cudaMemsetAsync(ring, 0, RING * 4, s));
+                CKM(cudaMemsetAsync(ring, 0, (RING + 1) * 4, s));      // ring words + touched
                 int pass = 0, batch = 2;
                 for (;;) {
                     for (int k = 0; k < batch; k++, pass++) {
                         part::k_prop_rows<<<gridn(std::max(Q.nloc, 1), 256 * part::PART_RPT), 256, 0, s>>>(
-                            Q.nloc, Q.rb, Q.rp, Q.wci, Q.odeg, Q.sig + n, ring, pass);
+                            Q.nloc, Q.rb, Q.rp, Q.wci, Q.odeg, Q.sig + n, ring, pass, Q.touched());
                         part::k_prop_cols<<<gridn(n, 256 * part::PART_RPT), 256, 0, s>>>(n, Q.cp, Q.cr, Q.ideg, Q.sig,
-                                                                                         ring, pass);
+                                                                                         ring, pass, Q.touched());
                         launches += 2;
                     }
                     CKM(cudaGetLastError());
                     CKM(cudaMemcpyAsync(hbuf, ring + ((pass - 1) & (RING - 1)), 4, cudaMemcpyDeviceToHost, s));
                     CKM(cudaStreamSynchronize(s));
                     if (hbuf[0] == 0) break;
-                    if ((int64_t)pass > 4 * (int64_t)n + 1024)
-                        return fail(ECL_SCC_ECUDA, "internal: local Phase 2 did not converge");
+                    if ((int64_t)pass > 4 * (int64_t)n + 1024) {
+                        local_err = 1;             // reported through the exchange (all ranks stop)
+                        break;
+                    }
                     batch = std::min(batch * 2, RING / 2);
                 }
                 if (r == 0) passes_iter += pass;
-                k_copy_flag<<<1, 1, 0, s>>>(ring, Q.sig + 2 * (int64_t)n);   // did this rank change anything?
+                // did this rank change anything? (2: it failed; MAX makes every rank see it)
+                k_copy_flag<<<1, 1, 0, s>>>(Q.touched(), Q.sig + 2 * (int64_t)n, local_err ? 2 : 0);
                 launches++;
             }
             if (int e = X.allreduce(sigs, 2 * (int64_t)n + 1, 0, s)) return e;
             CKM(cudaMemcpyAsync(hbuf, R[0]->sig + 2 * (int64_t)n, 4, cudaMemcpyDeviceToHost, s));
             CKM(cudaStreamSynchronize(s));
+            if (hbuf[0] == 2) return fail(ECL_SCC_ECUDA, "internal: local Phase 2 did not converge on some rank");
             if (hbuf[0] == 0) break;
         }
         iters = iter;
@@ -263,6 +314,9 @@ static int run_partitioned(std::vector<PRank*>& R, Exchange& X, int32_t n, uint3
         st->trace_len = std::min(iters, ECL_SCC_TRACE_MAX);
         st->passes = passes_total;
         st->kernel_launches = launches;
+        st->ms_comm = X.ms();
+        st->comm_bytes = X.bytes;
+        st->exchanges = X.used;
     }
     return ECL_SCC_OK;
 }
@@ -275,6 +329,16 @@ using namespace eclscc;
 struct ecl_scc_comm_s {
     ncclComm_t comm;
     int nranks, rank, device;
+};
+
+// per-rank workspace of the partitioned mode: allocated once, reused by every call
+struct ecl_scc_part_plan_s {
+    PRank R;
+    uint32_t flags = 0;
+    std::vector<cudaEvent_t> ev;              // exchange timing events
+    ~ecl_scc_part_plan_s() {
+        for (cudaEvent_t e : ev) cudaEventDestroy(e);
+    }
 };
 
 extern "C" {
@@ -315,9 +379,33 @@ int ecl_scc_comm_destroy(ecl_scc_comm_t comm) {
     return ECL_SCC_OK;
 }
 
+int ecl_scc_part_plan_create(int32_t n, int32_t row_begin, int32_t row_end, int64_t local_nnz_max, uint32_t flags,
+                             ecl_scc_part_plan_t* out) {
+    clear_err();
+    if (!out || n < 0 || row_begin < 0 || row_end < row_begin || row_end > n || local_nnz_max < 0)
+        return fail(ECL_SCC_EINVAL, "part_plan_create: bad arguments");
+    if (local_nnz_max >= (int64_t)INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "local nnz >= 2^31");
+    auto* h = new (std::nothrow) ecl_scc_part_plan_s();
+    if (!h) return fail(ECL_SCC_ENOMEM, "host allocation");
+    h->flags = flags;
+    h->R.rb = row_begin; h->R.re = row_end; h->R.nloc = row_end - row_begin; h->R.m = local_nnz_max;
+    if (int r = rank_alloc(h->R, n)) {
+        delete h;
+        return r;
+    }
+    *out = h;
+    return ECL_SCC_OK;
+}
+
+int ecl_scc_part_plan_destroy(ecl_scc_part_plan_t plan) {
+    clear_err();
+    delete plan;
+    return ECL_SCC_OK;
+}
+
 int ecl_scc_partitioned(ecl_scc_comm_t comm, int32_t n, int32_t row_begin, int32_t row_end, int64_t local_nnz,
                         const int32_t* local_row_ptr, const int32_t* local_col_idx, int32_t* labels_out,
-                        ecl_scc_stream_t stream, ecl_scc_stats* stats) {
+                        ecl_scc_stream_t stream, ecl_scc_part_plan_t plan, ecl_scc_stats* stats) {
     clear_err();
     if (!comm || n < 0 || row_begin < 0 || row_end < row_begin || row_end > n || local_nnz < 0)
         return fail(ECL_SCC_EINVAL, "partitioned: bad arguments");
@@ -325,13 +413,29 @@ int ecl_scc_partitioned(ecl_scc_comm_t comm, int32_t n, int32_t row_begin, int32
     if (local_nnz > 0 && !local_col_idx) return fail(ECL_SCC_EINVAL, "partitioned: NULL col_idx");
     if (local_nnz >= (int64_t)INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "local nnz >= 2^31");
     if (n == 0) return ECL_SCC_OK;
-    PRank Q;
-    Q.rb = row_begin; Q.re = row_end; Q.nloc = row_end - row_begin; Q.m = local_nnz;
-    Q.rp = local_row_ptr; Q.ci = local_col_idx;
-    if (int r = rank_alloc(Q, n)) return r;
-    std::vector<PRank*> R{&Q};
-    NcclExchange X(comm->comm);
-    return run_partitioned(R, X, n, 0, labels_out, (cudaStream_t)stream, stats);
+    ecl_scc_part_plan_t tmp = nullptr;
+    if (!plan) {
+        if (int r = ecl_scc_part_plan_create(n, row_begin, row_end, local_nnz, 0, &tmp)) return r;
+        plan = tmp;
+    }
+    int rc = ECL_SCC_OK;
+    if (plan->R.rb != row_begin || plan->R.re != row_end || plan->R.m < local_nnz || (int64_t)plan->R.nloc < 0)
+        rc = fail(ECL_SCC_EINVAL, "partitioned: the plan was made for other rows or fewer edges");
+    if (!rc) {
+        PRank& Q = plan->R;
+        const int64_t cap = Q.m;
+        Q.m = local_nnz;
+        Q.rp = local_row_ptr;
+        Q.ci = local_col_idx;
+        std::vector<PRank*> R{&Q};
+        NcclExchange X(comm->comm);
+        X.ev = &plan->ev;
+        rc = run_partitioned(R, X, n, plan->flags, labels_out, (cudaStream_t)stream, stats);
+        Q.m = cap;
+        Q.rp = Q.ci = nullptr;
+    }
+    if (tmp) ecl_scc_part_plan_destroy(tmp);
+    return rc;
 }
 
 int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx,
@@ -378,7 +482,11 @@ int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_
     }
     if (rc == ECL_SCC_OK) {
         EmulatedExchange X(P);
+        std::vector<cudaEvent_t> ev;
+        X.ev = &ev;
         rc = run_partitioned(R, X, n, 0, labels_out, s, stats);
+        cudaStreamSynchronize(s);
+        for (cudaEvent_t e : ev) cudaEventDestroy(e);
     }
     cudaStreamSynchronize(s);
     own.clear();

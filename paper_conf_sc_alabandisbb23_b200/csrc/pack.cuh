@@ -73,85 +73,8 @@ __device__ __forceinline__ void pnotify_full(unsigned long long nb, const int32_
     if (nb & SLOW_MARK) notify_slow(ptr, adj, base, cnt, v, f);
 }
 
-// Step 2 for the pack kernel: the drain loop of drain_local (kernels.cuh) with the
-// sentinel slot encoding (branch-free pulls and notifications) and a multiply-based
-// gather of the four flag bytes of a thread.
 __device__ __forceinline__ unsigned gather4(unsigned w) {      // byte k (0/1) -> bit k
     return (((w & 0x01010101u) * 0x01020408u) >> 24) & 0xFu;
-}
-__device__ __forceinline__ void drain_pack(const WGraph& g, int* __restrict__ s_in, int* __restrict__ s_out,
-                                           const unsigned long long* __restrict__ s_nin,
-                                           const unsigned long long* __restrict__ s_nout,
-                                           unsigned* __restrict__ s_fin, unsigned* __restrict__ s_fout,
-                                           unsigned short* __restrict__ s_queue, int base, int cnt,
-                                           unsigned& prof_rounds, unsigned& prof_drains, unsigned& prof_pushes) {
-    const int tid = threadIdx.x;
-    const int lane = tid & 31, wq0 = (tid >> 5) * (2 * 32 * VPT);
-    for (;;) {
-        int worked = 0;
-#ifdef ECL_PROF
-        if (tid == 0) prof_rounds++;
-#endif
-        for (;;) {
-#ifdef ECL_PROF
-            if (lane == 0) prof_drains++;
-#endif
-            unsigned wi = ((volatile unsigned*)s_fin)[tid], wo = ((volatile unsigned*)s_fout)[tid];
-            if (wi) wi = atomicExch(s_fin + tid, 0u);
-            if (wo) wo = atomicExch(s_fout + tid, 0u);
-            const unsigned items = gather4(wi) | (gather4(wo) << 4);
-            const int c = __popc(items);
-            const int incl = warp_incl_scan(c, lane);
-            const int total = __shfl_sync(FULL, incl, 31);
-            if (total == 0) break;
-            worked = 1;
-#ifdef ECL_PROF
-            prof_pushes += c;
-#endif
-            {
-                int pos = wq0 + incl - c;
-                unsigned it = items;
-                while (it) {
-                    const int bit = __ffs(it) - 1;
-                    it &= it - 1;
-                    s_queue[pos++] = (unsigned short)(((tid * VPT + (bit & 3)) << 1) | (bit >> 2));
-                }
-            }
-            __syncwarp();
-            __threadfence_block();
-            int any = 0;
-            for (int q = lane; q < total; q += 32) {
-                const unsigned item = s_queue[wq0 + q];
-                const int v = (int)(item >> 1);
-                if (item & 1u) {                                 // v_out from the out-neighbours
-                    const unsigned long long src = s_nout[v];
-                    const int old = ((volatile int*)s_out)[v];
-                    int val = ppull(s_out, src, old);
-                    if (src & SLOW_MARK) val = pull_slow(s_out, g.optr, g.oadj, base, cnt, v, val);
-                    if (val > old) {
-                        ((volatile int*)s_out)[v] = val;
-                        __threadfence_block();
-                        pnotify_full(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
-                        any = 1;
-                    }
-                } else {                                         // v_in from the in-neighbours
-                    const unsigned long long src = s_nin[v];
-                    const int old = ((volatile int*)s_in)[v];
-                    int val = ppull(s_in, src, old);
-                    if (src & SLOW_MARK) val = pull_slow(s_in, g.iptr, g.iadj, base, cnt, v, val);
-                    if (val > old) {
-                        ((volatile int*)s_in)[v] = val;
-                        __threadfence_block();
-                        pnotify_full(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
-                        any = 1;
-                    }
-                }
-            }
-            __syncwarp();
-            if (!__any_sync(FULL, any)) break;
-        }
-        if (!__syncthreads_or(worked)) break;
-    }
 }
 
 // Step 2 without the per-warp queue: in every warp round each lane pulls ONE of its flagged
@@ -372,11 +295,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
 #endif
     {
         unsigned r0 = 0, r1 = 0, r2 = 0;
-#ifdef ECL_DRAIN_QUEUE
-        drain_pack(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, S.s_queue, base, cnt, r0, r1, r2);
-#else
         drain_direct(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, base, cnt, r0, r1, r2);
-#endif
 #ifdef ECL_PROF
         r2 = warp_sum(r2);
         if ((tid & 31) == 0) { PROF_ADD(dc, 2, r1); PROF_ADD(dc, 3, r2); }
@@ -450,11 +369,6 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
             uint8_t* __restrict__ dirty_next, int full, int run) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ unsigned s_fin[PACK_TH + 1], s_fout[PACK_TH + 1];      // + the sentinel's scratch byte
-#ifdef ECL_DRAIN_QUEUE
-    __shared__ unsigned short s_queue[2 * PACK_TT];
-#else
-    unsigned short* s_queue = nullptr;
-#endif
     __shared__ int s_dirty;
     TileSmem<PACK_TT> S;
     S.s_in = (int*)smem_raw;                                          // [PACK_TT] + sentinel
@@ -465,8 +379,7 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
     if (threadIdx.x == 0) { S.s_in[PACK_TT] = 0; S.s_out[PACK_TT] = 0; s_acc[0] = s_acc[1] = s_acc[2] = 0; }
     S.s_fin = s_fin;
     S.s_fout = s_fout;
-    S.s_queue = s_queue;
-    S.s_lv = nullptr;
+    S.s_queue = nullptr;
     S.s_acc = s_acc;
     if (!pass_begin(dc, pass, first)) return;
     const int ntiles = (g.na + PACK_TT - 1) / PACK_TT;
@@ -567,11 +480,6 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
              DevCounters* __restrict__ dc, AsyncQ Q, int claim) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ unsigned s_fin[PACK_TH + 1], s_fout[PACK_TH + 1];
-#ifdef ECL_DRAIN_QUEUE
-    __shared__ unsigned short s_queue[2 * PACK_TT];
-#else
-    unsigned short* s_queue = nullptr;
-#endif
     __shared__ int s_set[MSET];
     __shared__ int s_claim[CLAIM_MAX], s_nclaim;
     __shared__ uint8_t s_seen[CLAIM_MAX];
@@ -583,8 +491,7 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
     __shared__ unsigned long long s_acc[3];            // visited vertices, edges, tiles (flushed at the end)
     S.s_fin = s_fin;
     S.s_fout = s_fout;
-    S.s_queue = s_queue;
-    S.s_lv = nullptr;
+    S.s_queue = nullptr;
     S.s_acc = s_acc;
     const int tid = threadIdx.x;
     const int ntiles = (g.na + PACK_TT - 1) / PACK_TT;

@@ -72,10 +72,14 @@ static __global__ void k_csc_rows(int32_t nrows, int32_t rb, const int32_t* __re
 // raises nothing, so chains inside its range converge in one launch instead of one launch
 // per hop.  Other CTAs' values are read through L2 (ld.cg); the ring word of the pass is set
 // if anything rose (the driver repeats passes until one raises nothing: a fixed point).
+// `touched` is set by every pass that raised a value and is reset only when the rank's
+// local phase starts: the ring words are recycled every RING passes, so a rank whose local
+// fixed point took a multiple of RING passes would otherwise report "no change".
 constexpr int PART_RPT = 4;
 static __global__ void __launch_bounds__(256) k_prop_rows(int32_t nrows, int32_t rb, const int32_t* __restrict__ rp,
                                                           const int32_t* __restrict__ wci, const int32_t* __restrict__ odeg,
-                                                          int32_t* __restrict__ vout, int* __restrict__ ring, int pass) {
+                                                          int32_t* __restrict__ vout, int* __restrict__ ring, int pass,
+                                                          int* __restrict__ touched) {
     if (blockIdx.x == 0 && threadIdx.x == 0) ring[(pass + 1) & (RING - 1)] = 0;
     if (pass > 0 && ld_vol(ring + ((pass - 1) & (RING - 1))) == 0) return;
     const int64_t r0 = (int64_t)blockIdx.x * blockDim.x * PART_RPT + threadIdx.x;
@@ -95,11 +99,14 @@ static __global__ void __launch_bounds__(256) k_prop_rows(int32_t nrows, int32_t
         if (!__syncthreads_or(ch)) break;
         any = 1;
     }
-    if (any && threadIdx.x == 0) ring[pass & (RING - 1)] = 1;
+    if (any && threadIdx.x == 0) {
+        ring[pass & (RING - 1)] = 1;
+        *touched = 1;                 // never cleared by the ring protocol (see multi.cu)
+    }
 }
 static __global__ void __launch_bounds__(256) k_prop_cols(int32_t n, const int32_t* __restrict__ cp, const int32_t* __restrict__ cr,
                                                           const int32_t* __restrict__ ideg, int32_t* __restrict__ vin,
-                                                          int* __restrict__ ring, int pass) {
+                                                          int* __restrict__ ring, int pass, int* __restrict__ touched) {
     if (pass > 0 && ld_vol(ring + ((pass - 1) & (RING - 1))) == 0) return;
     const int64_t w0 = (int64_t)blockIdx.x * blockDim.x * PART_RPT + threadIdx.x;
     int any = 0;
@@ -118,7 +125,10 @@ static __global__ void __launch_bounds__(256) k_prop_cols(int32_t n, const int32
         if (!__syncthreads_or(ch)) break;
         any = 1;
     }
-    if (any && threadIdx.x == 0) ring[pass & (RING - 1)] = 1;
+    if (any && threadIdx.x == 0) {
+        ring[pass & (RING - 1)] = 1;
+        *touched = 1;                 // never cleared by the ring protocol (see multi.cu)
+    }
 }
 
 // ------------------------------------------------------------------ Phase 3 + trim

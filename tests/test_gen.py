@@ -45,6 +45,40 @@ def test_orders_are_permutations_of_each_other():
     np.testing.assert_array_equal(np.sort(np.diff(a.row_ptr)), np.sort(np.diff(b.row_ptr)))
 
 
+def _lex_of_blocked(N):
+    """blocked8 element ID -> lexicographic element ID (the generator's two numberings)."""
+    B = 8
+    lex_of = np.empty(6 * N ** 3, dtype=np.int64)
+    for x in range(N):
+        for y in range(N):
+            for z in range(N):
+                bx, by, bz = x // B, y // B, z // B
+                bsx, bsy, bsz = min(B, N - bx * B), min(B, N - by * B), min(B, N - bz * B)
+                off = (bx * B) * N * N + bsx * (by * B) * N + bsx * bsy * (bz * B)
+                cb = off + ((x - bx * B) * bsy + (y - by * B)) * bsz + (z - bz * B)
+                cl = (x * N + y) * N + z
+                lex_of[6 * cb:6 * cb + 6] = 6 * cl + np.arange(6)
+    return lex_of
+
+
+def test_orders_are_exact_relabellings_with_curvature():
+    """At kappa > 0 (random curved faces, hot spots) blocked8 is the lex graph with the
+    vertices renamed: the sorted edge lists agree after mapping blocked8 IDs to lex IDs."""
+    for N, d in ((9, 0), (17, 13)):        # N=17: partial 8^3 blocks at the boundary
+        kw = dict(kappa=0.05, kappa_hot=0.4, hot_mod=3, seed=11)
+        a = gen.mesh(N, gen.ordinate(d), order="lex", **kw)
+        b = gen.mesh(N, gen.ordinate(d), order="blocked8", **kw)
+        assert a.nnz == b.nnz
+        lex_of = _lex_of_blocked(N)
+        assert np.unique(lex_of).size == a.n
+        sa, da = _pairs(a)
+        sb, db = _pairs(b)
+        ka = np.sort(sa.astype(np.int64) * a.n + da)
+        kb = np.sort(lex_of[sb] * a.n + lex_of[db])
+        np.testing.assert_array_equal(ka, kb)
+        assert (oracle.tarjan_labels(a.row_ptr, a.col_idx) != np.arange(a.n)).any()   # cycles exist
+
+
 def test_reproducible_hashes():
     g1 = gen.mesh(8, gen.ordinate(3), kappa=0.1, seed=9)
     g2 = gen.mesh(8, gen.ordinate(3), kappa=0.1, seed=9)

@@ -76,3 +76,16 @@ def test_levels_reject_bad_labels():
     with pytest.raises(E.EclSccError) as ex:                  # a label outside [0, n)
         E.ecl_scc_levels(rp, ci, dev([1, 1, 2, 9]))
     assert ex.value.status == E.ERANGE
+    # far out of range on a large graph (would index far outside every workspace array):
+    # rejected before any label-indexed kernel runs, and the context stays usable
+    n = 200_000
+    g = gen.from_edges(n, np.stack([np.arange(n - 1), np.arange(1, n)], 1))
+    rp, ci = dev(g.row_ptr), dev(g.col_idx)
+    for bad in (2**31 - 2, -5):
+        lab = np.arange(n, dtype=np.int32)
+        lab[[3, n // 2, n - 1]] = bad
+        with pytest.raises(E.EclSccError) as ex:
+            E.ecl_scc_levels(rp, ci, dev(lab))
+        assert ex.value.status == E.ERANGE
+    lv, depth = E.ecl_scc_levels(rp, ci, dev(np.arange(n, dtype=np.int32)))
+    assert depth == n and (lv.cpu().numpy() == np.arange(n)).all()

@@ -78,3 +78,21 @@ def test_batched_mixed_sizes_and_empty():
     torch.cuda.synchronize()
     for g, lab in zip(graphs, labs):
         np.testing.assert_array_equal(lab.cpu().numpy(), oracle.tarjan_labels(g.row_ptr, g.col_idx))
+
+
+def test_emulated_long_local_phases():
+    """Regression (round-1 advisor finding): a rank whose local fixed point takes a multiple
+    of the pass-ring length (64) must still report that it changed something.  Long cycles
+    whose consecutive vertices sit in different CTAs' row ranges need one local pass per hop
+    or so; a sweep of lengths crosses 64, 128, ... local passes."""
+    for L in range(40, 300, 9):
+        stride = 1100                       # > the 1024 rows one CTA iterates over
+        n = L * stride + 1
+        cyc = (n - 1) - stride * np.arange(L)          # descending IDs: against the CTA order
+        g = gen.from_edges(n, np.stack([cyc, np.roll(cyc, -1)], 1))
+        rp, ci = dev(g)
+        for P in (2, 3):
+            lab = E.ecl_scc_partitioned_emulated(P, rp, ci).cpu().numpy()
+            exp = np.arange(n)
+            exp[cyc] = cyc.max()
+            np.testing.assert_array_equal(lab, exp, err_msg=f"L={L} P={P}")

@@ -94,13 +94,12 @@ def test_random_small_graphs_labels_and_traces():
         edges = [(rng.randrange(n), rng.randrange(n)) for _ in range(m)]
         g = gen.from_edges(n, edges)
         truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-        for flags in (0, E.TAIL, E.NO_TRIM, E.NO_TRIM | E.TAIL, E.IDENTITY_IDS, E.IDENTITY_IDS | E.TAIL,
-                      E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER, E.NO_PACK, E.NO_ASYNC):
+        for flags in (0, E.NO_TRIM, E.IDENTITY_IDS, E.SYNC_PASSES, E.NO_DIRTY, E.FORCE_REORDER, E.NO_PACK,
+                      E.NO_ASYNC):
             lab, _ = gpu_labels(g, flags)
             np.testing.assert_array_equal(lab, truth, err_msg=f"trial {trial} flags {flags}")
         if trial % 10 == 0:
             check_trace(g, trim=True)
-            check_trace(g, trim=True, flags=E.TAIL)
             check_trace(g, trim=False)
             check_trace(g, trim=True, flags=E.IDENTITY_IDS)
             check_trace(g, trim=True, flags=E.FORCE_REORDER)
@@ -109,13 +108,10 @@ def test_random_small_graphs_labels_and_traces():
 def test_c1_gnm_2000_8000():
     g = gen.config("c1")
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
-    for flags in (0, E.TAIL, E.IDENTITY_IDS, E.NO_TRIM, E.SYNC_PASSES, E.NO_DIRTY, E.STAGED, E.SWEEP, E.FORCE_REORDER,
-                  E.NO_PACK, E.NO_ASYNC):
+    for flags in (0, E.IDENTITY_IDS, E.NO_TRIM, E.SYNC_PASSES, E.NO_DIRTY, E.FORCE_REORDER, E.NO_PACK, E.NO_ASYNC):
         lab, _ = gpu_labels(g, flags)
         np.testing.assert_array_equal(lab, truth)
     check_trace(g, trim=True)
-    check_trace(g, trim=True, flags=E.TAIL)
-    check_trace(g, trim=False, flags=E.TAIL)
     check_trace(g, trim=False)
     check_trace(g, trim=True, flags=E.IDENTITY_IDS)
 
@@ -141,13 +137,6 @@ def test_edge_cases():
     # long path (deep DAG): identity
     g = gen.from_edges(n, np.stack([perm[:-1], perm[1:]], 1))
     np.testing.assert_array_equal(gpu_labels(g)[0], np.arange(n))
-    # the same two inside the device-resident tail (tail.cuh): one CTA and a multi-CTA grid
-    for nn in (1500, 30000):
-        pp = np.random.default_rng(nn).permutation(nn)
-        g = gen.from_edges(nn, np.stack([pp, np.roll(pp, -1)], 1))
-        assert (gpu_labels(g, E.TAIL)[0] == nn - 1).all()
-        g = gen.from_edges(nn, np.stack([pp[:-1], pp[1:]], 1))
-        np.testing.assert_array_equal(gpu_labels(g, E.TAIL)[0], np.arange(nn))
     # disjoint k-cycles on consecutive IDs
     k = 5
     e = [(b * k + i, b * k + (i + 1) % k) for b in range(1000) for i in range(k)]
@@ -229,11 +218,10 @@ def test_c2_mesh_1m(order):
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
     pi = prio(g.n)
     tr = oracle.ecl_scc(*(lambda h: (h.row_ptr, h.col_idx))(relabel(g, pi)), trim=True)
-    for fl in (0, E.TAIL):
-        lab, st = gpu_labels(g, fl)
-        np.testing.assert_array_equal(lab, truth)
-        assert st["edges_in"] == tr.edges_in[:64] and st["iterations"] == tr.iterations
-        assert st["edges_kept"] == tr.edges_kept[:st["iterations"] - 1]
+    lab, st = gpu_labels(g)
+    np.testing.assert_array_equal(lab, truth)
+    assert st["edges_in"] == tr.edges_in[:64] and st["iterations"] == tr.iterations
+    assert st["edges_kept"] == tr.edges_kept[:st["iterations"] - 1]
     lab, st = gpu_labels(g, E.IDENTITY_IDS)
     np.testing.assert_array_equal(lab, truth)
     tr = oracle.ecl_scc(g.row_ptr, g.col_idx, trim=True)
@@ -255,13 +243,27 @@ def test_c4_mesh_16m(order):
     np.testing.assert_array_equal(lab, truth)
 
 
-def test_c5_batched_meshes():
-    graphs = [gen.config("c5one", d=d) for d in range(0, 64, 4)]   # 16 of the 64 ordinates
+def test_c5_batched_meshes_full_64():
+    """The C5 configuration exactly as bench.py --config c5 times it at N=1: all 64 ordinates
+    (131.7M vertices, ~269M edges) in one batched call, every graph's labels compared with
+    Tarjan's element by element."""
+    from concurrent.futures import ThreadPoolExecutor
+    graphs = [gen.config("c5one", order="blocked8", d=d) for d in range(64)]
     dg = [dev(g) for g in graphs]
-    labs, st = E.ecl_scc_batched(dg, stats=True)
+    plan = E.Plan(sum(g.n for g in graphs), sum(g.nnz for g in graphs), E.NO_VALIDATE)
+    labs, st = E.ecl_scc_batched(dg, plan=plan, stats=True)
     torch.cuda.synchronize()
-    for g, lab in zip(graphs, labs):
-        np.testing.assert_array_equal(lab.cpu().numpy(), oracle.tarjan_labels(g.row_ptr, g.col_idx))
+    with ThreadPoolExecutor(max_workers=min(64, os.cpu_count() or 1)) as ex:
+        truth = list(ex.map(lambda g: oracle.tarjan_labels(g.row_ptr, g.col_idx), graphs))
+    for d, (lab, t) in enumerate(zip(labs, truth)):
+        np.testing.assert_array_equal(lab.cpu().numpy(), t, err_msg=f"ordinate {d}")
+    # the per-ordinate split of the multi-GPU bench (8 ranks): each share alone, same labels
+    for r in (0, 7):
+        share = list(range(8 * r, 8 * r + 8))
+        sl = E.ecl_scc_batched([dg[d] for d in share])
+        torch.cuda.synchronize()
+        for d, lab in zip(share, sl):
+            np.testing.assert_array_equal(lab.cpu().numpy(), truth[d], err_msg=f"rank {r} ordinate {d}")
 
 
 def test_repeated_runs_with_plan_reuse_are_stable():

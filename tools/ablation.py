@@ -23,7 +23,6 @@ VARIANTS = [
     ("raw vertex IDs instead of priorities (the paper's signatures)", E.IDENTITY_IDS),
     ("no Trim-1 (P:83)", E.NO_TRIM),
     ("no storage reordering", E.NO_REORDER),
-    ("device-resident tail (opt-in)", E.TAIL),
 ]
 
 
@@ -54,7 +53,7 @@ if __name__ == "__main__":
         base = None
         print(f"== {c}: n={g.n} nnz={g.nnz} ({g.name})", flush=True)
         for name, fl in VARIANTS:
-            if c == "c3" and fl in (E.NO_REORDER, E.TAIL):
+            if c == "c3" and fl == E.NO_REORDER:
                 continue                      # long rows: neither applies
             t, st = time_one(g, fl)
             base = base or t

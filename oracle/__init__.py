@@ -9,9 +9,11 @@ Functions (each cites the passage it follows; P:n = /root/reference/PAPER.md lin
 
 * ``tarjan_labels(row_ptr, col_idx)`` -- O1: SCCs by Tarjan's algorithm (P:53, P:79,
   P:208), each labelled by its largest vertex ID.  The plain definition.
-* ``ecl_scc(row_ptr, col_idx, reset_all=False, compress=False, trim=False, snap_iter=0)``
-  -- O2: Alg. 1 in the paper's order with Jacobi Phase-2 rounds and the
-  per-iteration trace.  Flags follow the readings in DESIGN.md.
+* ``ecl_scc(row_ptr, col_idx, reset_all=False, compress=False, trim=False, snap_iter=0,
+  trim2=False, four=False, raise_=False)`` -- O2: Alg. 1 in the paper's order
+  with Jacobi Phase-2 rounds and the per-iteration trace.  Flags follow the readings in
+  DESIGN.md: R1/R2, path compression, Trim-1 and Trim-2, the 4-signature
+  variant, the sound variant of the P:190 trick.
 * ``scc_levels(row_ptr, col_idx, labels)`` -- O4: the sweep levels of the SCC condensation
   (Table 2's "DAG depth"): Kahn's algorithm on the condensation, level = longest path
   from a source SCC.  Returns (levels per vertex, depth).
@@ -34,6 +36,9 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 RESET_ALL = 1
 COMPRESS = 2
 TRIM = 4
+TRIM2 = 8
+FOUR = 16
+RAISE = 32
 
 _lib = None
 
@@ -121,10 +126,14 @@ class Trace:
 
 
 def ecl_scc(row_ptr, col_idx, reset_all: bool = False, compress: bool = False,
-            trim: bool = False, snap_iter: int = 0, max_trace: int = 4096) -> Trace:
-    """O2: literal Alg. 1 with Jacobi Phase 2; returns labels and the per-iteration trace."""
+            trim: bool = False, snap_iter: int = 0, max_trace: int = 4096, trim2: bool = False,
+            four: bool = False, raise_: bool = False) -> Trace:
+    """O2: literal Alg. 1 with Jacobi Phase 2; returns labels and the per-iteration trace.
+    trim2: Trim-2; four: the 4-signature variant; raise_: the sound variant of
+    the P:190 trick."""
     n, rp, ci = _csr(row_ptr, col_idx)
-    flags = (RESET_ALL if reset_all else 0) | (COMPRESS if compress else 0) | (TRIM if trim else 0)
+    flags = ((RESET_ALL if reset_all else 0) | (COMPRESS if compress else 0) | (TRIM if trim else 0)
+             | (TRIM2 if trim2 else 0) | (FOUR if four else 0) | (RAISE if raise_ else 0))
     labels = np.empty(n, dtype=np.int32)
     ein = np.zeros(max_trace, dtype=np.int64)
     pas = np.zeros(max_trace, dtype=np.int64)
@@ -142,6 +151,8 @@ def ecl_scc(row_ptr, col_idx, reset_all: bool = False, compress: bool = False,
         raise MemoryError("oracle_ecl_scc")
     if it == -2:
         raise RuntimeError("oracle_ecl_scc: iteration cap reached (non-terminating rule mix?)")
+    if it == -3:
+        raise ValueError("oracle_ecl_scc: Trim-2 needs rule R2 (reset_all=False)")
     k = min(it, max_trace)
     tr = Trace(labels, it, ein[:k].tolist(), pas[:k].tolist(), kept[:k].tolist())
     if 1 <= snap_iter <= it:

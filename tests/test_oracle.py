@@ -430,3 +430,146 @@ def test_levels_reject_cyclic_labels():
     rp, ci = csr_from_edges(3, [(0, 1), (1, 0)])
     with pytest.raises(ValueError):
         oracle.scc_levels(rp, ci, np.array([0, 1, 2]))       # 0 and 1 labelled apart: a cycle
+
+
+# ---------------------------------------------------------------- variants (f2, f3)
+def _brute_variant(n, edges, trim=False, trim2=False, four=False):
+    """Rule R2 iterated by DEFINITION, not by propagation: after the trims, every live
+    vertex's signatures are the max (and, with four, min) vertex ID over its ancestors and
+    over its descendants in the live edge set, by BFS; Phase 3
+    keeps an edge iff all signatures agree at both ends and its source is unfinished
+    (P:147, P:186).  Trim-1 drops the edges of a vertex without live in- or out-edges;
+    Trim-2 finishes a pair u<->w whose only live in-edge entries (or only out-edge entries)
+    come from each other.  Returns (labels, edges_in, edges_kept)."""
+    E = [(u, v) for u, v in edges if u != v]
+    label = list(range(n))
+    edges_in, kept = [], []
+    while True:
+        if trim or trim2:
+            din, dout = [0] * n, [0] * n
+            ins, outs = [[] for _ in range(n)], [[] for _ in range(n)]
+            for u, v in E:
+                dout[u] += 1; din[v] += 1
+                outs[u].append(v); ins[v].append(u)
+            pair = [-1] * n
+            if trim2:
+                for u in range(n):
+                    if din[u] == 1 and din[ins[u][0]] == 1 and ins[ins[u][0]][0] == u:
+                        pair[u] = ins[u][0]
+                    if dout[u] == 1 and dout[outs[u][0]] == 1 and outs[outs[u][0]][0] == u:
+                        pair[u] = outs[u][0]
+            gone = [(trim and (din[x] == 0 or dout[x] == 0)) or pair[x] >= 0 for x in range(n)]
+            E = [(u, v) for u, v in E if not gone[u] and not gone[v]]
+            for u in range(n):
+                if pair[u] >= 0:
+                    label[u] = max(u, pair[u])
+        if not E:
+            break
+        edges_in.append(len(E))
+        fwd = [[] for _ in range(n)]
+        for u, v in E:
+            fwd[u].append(v)
+        reach = []
+        for s in range(n):
+            seen, q = {s}, deque([s])
+            while q:
+                x = q.popleft()
+                for y in fwd[x]:
+                    if y not in seen:
+                        seen.add(y)
+                        q.append(y)
+            reach.append(seen)
+        anc = [[w for w in range(n) if v in reach[w]] for v in range(n)]
+        sig = [(max(anc[v]), max(reach[v])) + ((min(anc[v]), min(reach[v])) if four else ()) for v in range(n)]
+        E = [(u, v) for u, v in E if sig[u] == sig[v] and sig[u][0] != sig[u][1]]
+        kept.append(len(E))
+        live = {x for e in E for x in e}
+        for v in range(n):
+            if sig[v][0] == sig[v][1] and (v in live or any(v in e for e in edges)):
+                label[v] = sig[v][0] if label[v] == v else label[v]
+    return np.array(label, dtype=np.int32), edges_in, kept
+
+
+VARIANTS = [dict(trim2=True), dict(trim=True, trim2=True), dict(four=True), dict(four=True, trim=True),
+            dict(four=True, trim=True, trim2=True), dict(raise_=True), dict(raise_=True, trim=True),
+            dict(raise_=True, compress=True, trim=True, trim2=True, four=True)]
+
+
+@pytest.mark.parametrize("flags", VARIANTS, ids=lambda f: "-".join(k for k in f))
+def test_variants_labels_and_traces_vs_brute_force(flags):
+    """O2 with Trim-2 / 4 signatures / the sound P:190 trick against the brute-force
+    definition above (labels, live edges per iteration, kept edges), and against Tarjan."""
+    rng = random.Random(606)
+    bf = {k: v for k, v in flags.items() if k in ("trim", "trim2", "four")}
+    for trial in range(250):
+        n = rng.randrange(1, 30)
+        edges = random_edges(rng, n, rng.randrange(0, 3 * n + 1))
+        if trial % 3 == 0:                       # plant 2-cycles (Trim-2 candidates)
+            for _ in range(3):
+                a, b = rng.randrange(n), rng.randrange(n)
+                edges += [(a, b), (b, a)]
+        rp, ci = csr_from_edges(n, edges)
+        tr = oracle.ecl_scc(rp, ci, **flags)
+        truth = oracle.tarjan_labels(rp, ci)
+        np.testing.assert_array_equal(tr.labels, truth, err_msg=f"trial {trial}")
+        lab, ein, kept = _brute_variant(n, edges, **bf)
+        np.testing.assert_array_equal(lab, truth, err_msg=f"brute trial {trial}")
+        assert tr.edges_in == ein and tr.edges_kept == kept, (trial, tr.edges_in, ein, tr.edges_kept, kept)
+
+
+def test_trim2_hand_examples():
+    """'Any two vertices that have no incoming or outgoing edges aside from a
+    bidirectional edge connecting them to each other' form an SCC."""
+    # {0<->1} whose only out-edges are each other, fed by 2: Trim-1 takes 2, Trim-2 {0,1};
+    # no live edge is left, so Phase 2 never runs (0 iterations)
+    rp, ci = csr_from_edges(3, [(0, 1), (1, 0), (2, 0)])
+    for trim in (False, True):
+        tr = oracle.ecl_scc(rp, ci, trim=trim, trim2=True)
+        assert tr.labels.tolist() == [1, 1, 2] and tr.iterations == 0
+    # the same pair with one extra in-edge AND one extra out-edge: no pattern applies
+    rp, ci = csr_from_edges(5, [(0, 1), (1, 0), (2, 0), (1, 4), (4, 2)])
+    tr = oracle.ecl_scc(rp, ci, trim2=True)
+    assert tr.iterations >= 1 and tr.labels.tolist() == [4, 4, 4, 3, 4]
+    # duplicate edges are counted: 0->1 twice gives 1 two in-edge entries (reading 17)
+    rp, ci = csr_from_edges(2, [(0, 1), (0, 1), (1, 0)])
+    tr = oracle.ecl_scc(rp, ci, trim2=True)
+    assert tr.labels.tolist() == [1, 1]
+    assert tr.edges_in[0] == 3                        # out-pattern: dout[0] = 2, in: din[1] = 2
+    with pytest.raises(ValueError):
+        oracle.ecl_scc(rp, ci, trim2=True, reset_all=True)
+
+
+def test_four_signatures_hand_example():
+    """the minimums separate SCCs the maximums cannot.  Path 5 -> 0 -> 9 (no trim):
+    with two signatures 5 and 0 share (in, out) = (5, 9) and their edge survives iteration 1;
+    the minimums give 5: (min in, min out) = (5, 0) and 0: (0, 0), so it is removed."""
+    rp, ci = csr_from_edges(10, [(5, 0), (0, 9)])
+    base = oracle.ecl_scc(rp, ci)
+    assert base.edges_in == [2, 1] and base.edges_kept == [1, 0]
+    four = oracle.ecl_scc(rp, ci, four=True)
+    assert four.edges_in == [2] and four.edges_kept == [0]
+    np.testing.assert_array_equal(four.labels, np.arange(10))
+
+
+def test_sound_p190_variant_keeps_the_trace_and_cuts_passes():
+    """The sound P:190 variant changes pass counts only (reading 12): same signatures after
+    every Phase 2; on a long cycle in random ID order it needs fewer Jacobi rounds; the
+    Appendix B counterexample to the literal reading stays correct."""
+    rng = random.Random(12)
+    for _ in range(60):
+        n = rng.randrange(2, 40)
+        edges = random_edges(rng, n, rng.randrange(0, 3 * n))
+        rp, ci = csr_from_edges(n, edges)
+        a = oracle.ecl_scc(rp, ci, trim=True)
+        b = oracle.ecl_scc(rp, ci, trim=True, raise_=True)
+        assert a.edges_in == b.edges_in and a.edges_kept == b.edges_kept
+        for it in range(1, a.iterations + 1):
+            sa = oracle.ecl_scc(rp, ci, trim=True, snap_iter=it)
+            sb = oracle.ecl_scc(rp, ci, trim=True, raise_=True, snap_iter=it)
+            np.testing.assert_array_equal(sa.snap_in, sb.snap_in)
+            np.testing.assert_array_equal(sa.snap_out, sb.snap_out)
+    perm = np.random.default_rng(3).permutation(4096)
+    rp, ci = csr_from_edges(4096, np.stack([perm, np.roll(perm, -1)], 1))
+    assert oracle.ecl_scc(rp, ci, raise_=True).passes[0] < oracle.ecl_scc(rp, ci).passes[0]
+    rp, ci = csr_from_edges(10, [(5, 2), (5, 9), (9, 2)])
+    assert oracle.ecl_scc(rp, ci, raise_=True).labels[5] == 5

@@ -82,6 +82,14 @@ typedef enum {
                                      visit instead of reading per-iteration tile packs */
 #define ECL_SCC_NO_ASYNC 0x1000u  /* ablation: Phase 2 as global passes (one launch each)
                                      instead of one persistent launch with a tile queue */
+#define ECL_SCC_TRIM2 0x4000u     /* variant: Trim-2 in the same round as Trim-1 -- a pair
+                                     u <-> w whose only kept in-edges (or only kept out-edges)
+                                     are each other is an SCC of two (reading 17);
+                                     EINVAL together with ECL_SCC_NO_TRIM */
+#define ECL_SCC_FOUR_SIG 0x8000u  /* variant: the 4-signature method -- Phase 2 also
+                                     propagates minimum ancestor / descendant IDs and Phase 3
+                                     keeps an edge only if all four signatures agree; twice the
+                                     signature memory and two Phase-2 fixed points per iteration */
 
 #define ECL_SCC_TRACE_MAX 64
 

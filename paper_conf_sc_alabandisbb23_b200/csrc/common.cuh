@@ -24,7 +24,13 @@ struct WGraph {
     int32_t na;
     const int2* sig2;    // Phase 3 of power-law graphs: (v_in, v_out) interleaved, one gather per
                          // far end in keep(); nullptr: the separate cin / cout arrays
+    const int32_t* min_in;   // ECL_SCC_FOUR_SIG: the minimum signatures, stored mirrored
+    const int32_t* min_out;  // (INT32_MAX - priority) so Phase 2 propagates them with max;
+                             // nullptr: the two-signature method
 };
+// the minimum signatures propagate as maxima of mirrored priorities (all >= 0, so the
+// pack kernels' sentinel value 0 stays below every signature)
+__host__ __device__ __forceinline__ int32_t mirror_prio(int32_t p) { return 0x7FFFFFFF - p; }
 
 // Counters the host reads back once per outer iteration.
 struct DevCounters {

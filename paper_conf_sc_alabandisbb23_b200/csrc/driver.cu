@@ -108,6 +108,12 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
         p->kout = p->kin + n1;
         p->kio = (int2*)p->kin;
     }
+    if (p->flags & ECL_SCC_FOUR_SIG)
+        for (int b = 0; b < 2; b++) {
+            e = e ? e : A((void**)&p->min_in[b], n1 * 4);
+            e = e ? e : A((void**)&p->min_out[b], n1 * 4);
+        }
+    if (p->flags & ECL_SCC_TRIM2) e = e ? e : A((void**)&p->t2, n1 * 4);
     e = e ? e : A((void**)&p->newidx, n1 * 4);
     e = e ? e : A((void**)&p->cnt, n1 * sizeof(int2));
     e = e ? e : A((void**)&p->emask, n1 * sizeof(uint2));
@@ -143,6 +149,8 @@ void plan_free(Plan* p) {
         cudaFree(p->act[b]); cudaFree(p->cin[b]); cudaFree(p->cout[b]);
         cudaFree(p->optr[b]); cudaFree(p->iptr[b]); cudaFree(p->oadj[b]); cudaFree(p->iadj[b]);
     }
+    for (int b = 0; b < 2; b++) { cudaFree(p->min_in[b]); cudaFree(p->min_out[b]); }
+    cudaFree(p->t2);
     cudaFree(p->kin); cudaFree(p->newidx); cudaFree(p->cnt); cudaFree(p->emask); cudaFree(p->sig2);
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
     cudaFree(p->chunk_cnt); cudaFree(p->hcnt);
@@ -325,8 +333,17 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     }
     p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, chunked, p->hcnt, p->emask);
     if (chunked) {
-        p->launches += 2;
+        p->launches++;
         k_keep_chunks<FIRST><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio);
+    }
+    const bool trim2 = TRIM && (p->flags & ECL_SCC_TRIM2);
+    if (trim2) {                                   // Trim-2 on the kept degrees (reading 17)
+        p->launches += 2;
+        k_trim2_find<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->emask, p->t2);
+        k_trim2_apply<<<grid, TPB, 0, s>>>(g.na, p->t2, p->kio);
+    }
+    if (chunked) {
+        p->launches++;
         k_count_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio, p->chunk_cnt, p->hcnt);
     }
     p->launches++; k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
@@ -334,7 +351,8 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     if (r) return r;
     p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
-                                              chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur, pk);
+                                              chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur, pk,
+                                              p->min_in[ob], p->min_out[ob], trim2 ? p->t2 : nullptr);
     p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked, p->emask, pk);
     if (chunked) {
@@ -377,7 +395,7 @@ static int launch_tile(Plan* p, bool sync, const WGraph& g, int32_t* cin, int32_
 // a4-a6: Phase 2 to its fixed point.  Passes are enqueued in growing batches; a pass
 // whose predecessor changed nothing exits at once, so over-enqueueing costs only a launch.
 static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int nchunks, cudaStream_t s,
-                     int64_t* passes_out) {
+                     int64_t* passes_out, bool second = false) {
     const unsigned ntiles = (unsigned)cdiv(g.na, TILE);
     const unsigned hgrid = (unsigned)std::min<int64_t>(cdiv(std::max(nchunks, 1), TPB / WARP), 148 * 8);
     // plain Jacobi passes: the ablation flag, or graphs whose tiles hold almost no edges
@@ -390,7 +408,7 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     const bool use_pack = pack_path(p, nchunks) && g.na > 0;
     if (use_pack) {
         if (int r = ensure_pack(p)) return r;
-        if (!p->pack_fused || p->hc->pack_bad) {       // the scatter did not write it
+        if (!second && (!p->pack_fused || p->hc->pack_bad)) {   // the scatter did not write it
             p->launches++;
             k_tile_pack<<<ntiles, PACK_TH, 0, s>>>(g, p->pnin, p->pnout, p->ext, p->ext_cnt);
         }
@@ -425,8 +443,10 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             const int cmax = p->knob_claim_max ? p->knob_claim_max : 16;
             const int claim = p->knob_claim ? p->knob_claim
                                             : (int)std::min<int64_t>(cmax, std::max<int64_t>(1, ntiles / (cdiv_ * p->aq_resident)));
-            CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
-            CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
+            if (!second) {
+                CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
+                CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
+            }
             p->launches += 2;
             k_async_init<<<grid_for((int64_t)ntiles, TPB), TPB, 0, s>>>(Q, (int)ntiles);
             k_prop_async<<<(unsigned)std::min<int64_t>(ntiles, p->aq_resident), PACK_TH, pack_dyn_smem(), s>>>(
@@ -590,7 +610,8 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             if (st && iter >= 2 && iter - 2 < ECL_SCC_TRACE_MAX) st->edges_kept[iter - 2] = (int64_t)p->hc->totals.w;
             if (t.y != t.z) return fail(ECL_SCC_ECUDA, "internal: CSR/CSC survivor mismatch %d vs %d", t.y, t.z);
             if (nchunks > p->chunk_cap) return fail(ECL_SCC_ECUDA, "internal: heavy chunk list overflow");
-            g = WGraph{p->act[ob], p->optr[ob], p->oadj[ob], p->iptr[ob], p->iadj[ob], t.x};
+            g = WGraph{p->act[ob], p->optr[ob], p->oadj[ob], p->iptr[ob], p->iadj[ob], t.x, nullptr,
+                       p->min_in[ob], p->min_out[ob]};
             cin = p->cin[ob];
             cout = p->cout[ob];
             if (t.y == 0) break;                                   // no live edge: done
@@ -598,6 +619,12 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             stage_mark(p, 4, s);
             r = propagate(p, g, p->cin[ob], p->cout[ob], nchunks, s, &passes);
             if (r) return r;
+            if (p->flags & ECL_SCC_FOUR_SIG) {            // the minimum pair: its own fixed point
+                int64_t p2 = 0;
+                r = propagate(p, g, p->min_in[ob], p->min_out[ob], nchunks, s, &p2, true);
+                if (r) return r;
+                if (passes >= 0) passes += p2;           // (asynchronous: counted on the device)
+            }
             stage_mark(p, 5, s);
             if (st && (p->flags & ECL_SCC_TIME_STAGES)) {
                 CK(cudaEventSynchronize(p->ev[5]));
@@ -842,6 +869,10 @@ int ecl_scc_plan_create(int32_t n_max, int64_t nnz_max, uint32_t flags, ecl_scc_
     if (nnz_max >= (int64_t)INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "nnz_max >= 2^31");
     ecl_scc_plan_s* h = (ecl_scc_plan_s*)calloc(1, sizeof(ecl_scc_plan_s));
     if (!h) return fail(ECL_SCC_ENOMEM, "host allocation");
+    if ((flags & ECL_SCC_TRIM2) && (flags & ECL_SCC_NO_TRIM)) {
+        free(h);
+        return fail(ECL_SCC_EINVAL, "plan_create: ECL_SCC_TRIM2 runs with Trim-1 (not with ECL_SCC_NO_TRIM)");
+    }
     h->p.flags = flags;
     int r = plan_alloc(&h->p, n_max, nnz_max);
     if (r) {

@@ -18,6 +18,8 @@ struct Plan {
     int32_t *act[2], *cin[2], *cout[2];  // vertex IDs and signatures v_in / v_out
     int32_t *optr[2], *iptr[2];          // CSR / CSC offsets
     int32_t *oadj[2], *iadj[2];          // CSR / CSC adjacency
+    int32_t *min_in[2], *min_out[2];     // ECL_SCC_FOUR_SIG: minimum signatures (mirrored), per buffer
+    int32_t* t2;                         // ECL_SCC_TRIM2: Trim-2 partner per local vertex (-1: none)
     int32_t *kin, *kout;                 // two n+1 int views (ingest histogram / cursor, relabel, levels)
     int2* kio;                           // the same memory as interleaved kept degrees {in, out} (compaction)
     int32_t* newidx;                     // old local -> new local (-1: leaves)

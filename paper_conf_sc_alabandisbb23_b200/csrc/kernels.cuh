@@ -143,16 +143,23 @@ static __global__ void __launch_bounds__(256) k_csc_scatter(int32_t n, const int
 // Evaluated from either end: the row owner's pair (a, b) is passed in, the other
 // endpoint's pair is gathered.  In the first removal (FIRST) every edge except a
 // self-loop is kept (DESIGN reading 9).
+// With the 4-signature variant (mi != nullptr) the minimum pair (c, d) must agree as well.
 template <bool FIRST>
 __device__ __forceinline__ bool keep_edge(int owner, int a, int b, int other, const int32_t* __restrict__ cin,
-                                          const int32_t* __restrict__ cout, const int2* __restrict__ s2 = nullptr) {
+                                          const int32_t* __restrict__ cout, const int2* __restrict__ s2 = nullptr,
+                                          int c = 0, int d = 0, const int32_t* __restrict__ mi = nullptr,
+                                          const int32_t* __restrict__ mo = nullptr) {
     if (FIRST) return other != owner;
+    bool k;
     if (s2) {                                            // interleaved copy: one 8-byte gather
         const int2 x = __ldg(s2 + other);
-        return (x.x == a) & (x.y == b);
+        k = (x.x == a) & (x.y == b);
+    } else {
+        // both loads are issued unconditionally (no short circuit): callers batch these gathers
+        k = (__ldg(cin + other) == a) & (__ldg(cout + other) == b);
     }
-    // both loads are issued unconditionally (no short circuit): callers batch these gathers
-    return (__ldg(cin + other) == a) & (__ldg(cout + other) == b);
+    if (mi) k &= (__ldg(mi + other) == c) & (__ldg(mo + other) == d);
+    return k;
 }
 // Phase 3 of power-law graphs: the signatures interleaved for one gather per far end
 static __global__ void k_pack_sig(int32_t na, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
@@ -168,7 +175,7 @@ __device__ __forceinline__ bool trimmed(const int2* __restrict__ kio, int x) {
 }
 
 struct RowCtx {
-    int ob, oe, ib, ie, a, b;
+    int ob, oe, ib, ie, a, b, c, d;       // (c, d): the minimum pair (4-signature variant)
     bool valid, live;
 };
 
@@ -181,6 +188,7 @@ __device__ __forceinline__ RowCtx load_row(const WGraph& g, int64_t i, const int
         r.ob = g.optr[i]; r.oe = g.optr[i + 1];
         r.ib = g.iptr[i]; r.ie = g.iptr[i + 1];
         if (!FIRST) { r.a = cin[i]; r.b = cout[i]; }
+        if (!FIRST && g.min_in) { r.c = g.min_in[i]; r.d = g.min_out[i]; }
     }
     r.live = r.valid && (FIRST || r.a != r.b);
     return r;
@@ -215,10 +223,13 @@ struct KeepPred {
     int i, a, b;
     const int32_t *cin, *cout;
     const int2* s2;
-    __device__ __forceinline__ bool operator()(int k) const { return keep_edge<FIRST>(i, a, b, k, cin, cout, s2); }
+    int c, d;
+    const int32_t *mi, *mo;
+    __device__ __forceinline__ bool operator()(int k) const { return keep_edge<FIRST>(i, a, b, k, cin, cout, s2, c, d, mi, mo); }
     __device__ __forceinline__ KeepPred bcast(int src) const {
         KeepPred p = *this;
         p.i = __shfl_sync(FULL, i, src); p.a = __shfl_sync(FULL, a, src); p.b = __shfl_sync(FULL, b, src);
+        p.c = __shfl_sync(FULL, c, src); p.d = __shfl_sync(FULL, d, src);
         return p;
     }
 };
@@ -228,12 +239,15 @@ struct SurvivePred {
     const int32_t *cin, *cout;
     const int2* kio;
     const int2* s2;
+    int c, d;
+    const int32_t *mi, *mo;
     __device__ __forceinline__ bool operator()(int k) const {
-        return keep_edge<FIRST>(i, a, b, k, cin, cout, s2) & !(TRIM && trimmed(kio, k));
+        return keep_edge<FIRST>(i, a, b, k, cin, cout, s2, c, d, mi, mo) & !(TRIM && trimmed(kio, k));
     }
     __device__ __forceinline__ SurvivePred bcast(int src) const {
         SurvivePred p = *this;
         p.i = __shfl_sync(FULL, i, src); p.a = __shfl_sync(FULL, a, src); p.b = __shfl_sync(FULL, b, src);
+        p.c = __shfl_sync(FULL, c, src); p.d = __shfl_sync(FULL, d, src);
         return p;
     }
 };
@@ -369,7 +383,7 @@ static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, con
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST>(g, i, cin, cout);
-    KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout, g.sig2};
+    KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout, g.sig2, r.c, r.d, g.min_in, g.min_out};
     unsigned mo = 0, mi = 0;
     mask_light2(g.oadj, r.ob, r.live && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, g.iadj, r.ib,
                 r.live && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, (int)(r.valid ? i : 0), pred, mo, mi);
@@ -399,7 +413,7 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
         if (r.live) { const int2 k = kio[i]; nout = k.y; nin = k.x; }   // survivors = kept: the masks stand
     } else {
         const bool go = r.live && !trimmed(kio, (int)i);
-        SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2};
+        SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2, r.c, r.d, g.min_in, g.min_out};
         if (r.valid) {                                   // light rows: the kept entries' far ends
             const uint2 km = emask[i];
             const unsigned so = go && r.oe - r.ob <= HEAVY ? trim_mask(g.oadj, r.ob, km.x, (int)i, kio) : 0u;
@@ -423,6 +437,61 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
     if (lane == 0) wsum[i >> 5] = make_int4(sa, so, si, sk);
 }
 
+// Trim-2 (McLendon; reading 17), one round on the kept graph together with
+// Trim-1: an unfinished vertex i whose only kept in-edge entry comes from w, while w's only
+// kept in-edge entry comes from i (i -> w kept, kin(w) == 1) -- or the same with out-edges --
+// forms the SCC {i, w}.  Light rows read the kept entries from the Phase-3 bit masks; long
+// rows are walked with the keep predicate (a row with exactly one kept entry).  t2[i] = w
+// or -1.  k_trim2_apply then zeroes the pair's kept in-degree, so the Trim-1 test of the
+// compaction removes both and their edges (the kept out-degree, which the kept-edge count
+// of the trace sums, is untouched).
+template <bool FIRST, typename P>
+__device__ __forceinline__ int kept_single(const int32_t* __restrict__ adj, int rb, int re, unsigned m, P pred) {
+    if (re - rb <= HEAVY) return m ? __ldg(adj + rb + __ffs(m) - 1) : -1;
+    for (int e = rb; e < re; e++) {
+        const int x = __ldg(adj + e);
+        if (pred(x)) return x;
+    }
+    return -1;
+}
+template <bool FIRST, typename P>
+__device__ __forceinline__ bool kept_has(const int32_t* __restrict__ adj, int rb, int re, unsigned m, P pred, int w) {
+    if (re - rb <= HEAVY) {
+        for (; m; m &= m - 1)
+            if (__ldg(adj + rb + __ffs(m) - 1) == w) return true;
+        return false;
+    }
+    for (int e = rb; e < re; e++)
+        if (__ldg(adj + e) == w && pred(w)) return true;
+    return false;
+}
+template <bool FIRST>
+static __global__ void k_trim2_find(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+                                    const int2* __restrict__ kio, const uint2* __restrict__ emask, int32_t* __restrict__ t2) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= g.na) return;
+    const RowCtx r = load_row<FIRST>(g, i, cin, cout);
+    int w = -1;
+    if (r.live) {
+        KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout, g.sig2, r.c, r.d, g.min_in, g.min_out};
+        const int2 k = kio[i];
+        const uint2 m = emask[i];
+        if (k.x == 1) {                                  // in-pattern
+            const int u = kept_single<FIRST>(g.iadj, r.ib, r.ie, m.y, pred);
+            if (u >= 0 && __ldg(&kio[u].x) == 1 && kept_has<FIRST>(g.oadj, r.ob, r.oe, m.x, pred, u)) w = u;
+        }
+        if (w < 0 && k.y == 1) {                         // out-pattern
+            const int u = kept_single<FIRST>(g.oadj, r.ob, r.oe, m.x, pred);
+            if (u >= 0 && __ldg(&kio[u].y) == 1 && kept_has<FIRST>(g.iadj, r.ib, r.ie, m.y, pred, u)) w = u;
+        }
+    }
+    t2[i] = w;
+}
+static __global__ void k_trim2_apply(int32_t na, const int32_t* __restrict__ t2, int2* __restrict__ kio) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < na && t2[i] >= 0) kio[i].x = 0;
+}
+
 // New numbering, Phase 1 reset of the survivors (rule R2), final labels of
 // the vertices that leave, new offsets, heavy-row chunk list.
 // Survivors restart from their priority pi(v) (reading 16).  A finished vertex leaves
@@ -435,7 +504,8 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
                               int32_t* __restrict__ act2, int32_t* __restrict__ cin2, int32_t* __restrict__ cout2,
                               int32_t* __restrict__ optr2, int32_t* __restrict__ iptr2, int32_t* __restrict__ labels,
                               Chunk* __restrict__ chunks, int* __restrict__ nchunks, int chunk_cap, Prio P,
-                              const int32_t* __restrict__ orig, PackOut pk) {
+                              const int32_t* __restrict__ orig, PackOut pk, int32_t* __restrict__ min_in2,
+                              int32_t* __restrict__ min_out2, const int32_t* __restrict__ t2) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i == 0) {
@@ -468,6 +538,10 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
         const int pv = (int)prio_of(P, (uint32_t)ov);
         cin2[j] = pv;       // Phase 1: v_in <- v_id, v_out <- v_id for the unfinished
         cout2[j] = pv;
+        if (min_in2) {      // the minimum pair restarts from the vertex too
+            min_in2[j] = mirror_prio(pv);
+            min_out2[j] = mirror_prio(pv);
+        }
         optr2[j] = po;
         iptr2[j] = pi;
         for (int dir = 0; dir < 2; dir++) {
@@ -485,6 +559,12 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
         if (!FIRST) {
             const int a = cin[i], b = cout[i];
             if (a == b) lab = P.ids ? a : -(a + 1);
+        }
+        if (t2 && t2[i] >= 0) {      // Trim-2 pair {v, w}: named by its larger member
+            const int w = t2[i];
+            const int vw = g.act ? g.act[w] : w;
+            const int ow = orig ? orig[vw] : vw;
+            lab = P.ids ? max(ov, ow) : -((int)max(prio_of(P, (uint32_t)ov), prio_of(P, (uint32_t)ow)) + 1);
         }
         labels[ov] = lab;
     }
@@ -618,7 +698,7 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
             if (li) emit_cut(g.iadj, r.ib, sm.y, newidx, j, tb, 0, E, at);
         }
     }
-    SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2};
+    SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2, r.c, r.d, g.min_in, g.min_out};
     emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred, chunked, false);
     emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred, chunked, false);
 }
@@ -638,9 +718,11 @@ static __global__ void __launch_bounds__(256) k_keep_chunks(WGraph g, const Chun
     const Chunk k = chunks[c];
     const int a = FIRST ? 0 : cin[k.i], b = FIRST ? 0 : cout[k.i];
     if (!FIRST && a == b) return;                        // finished owner keeps nothing
+    const int mc = !FIRST && g.min_in ? g.min_in[k.i] : 0, md = !FIRST && g.min_in ? g.min_out[k.i] : 0;
     const int32_t* adj = k.dir ? g.iadj : g.oadj;
     int cc = 0;
-    for (int e = k.beg + lane; e < k.end; e += WARP) cc += keep_edge<FIRST>(k.i, a, b, __ldg(adj + e), cin, cout, g.sig2);
+    for (int e = k.beg + lane; e < k.end; e += WARP)
+        cc += keep_edge<FIRST>(k.i, a, b, __ldg(adj + e), cin, cout, g.sig2, mc, md, g.min_in, g.min_out);
     cc = warp_sum(cc);
     if (lane == 0 && cc) {
         atomicAdd(k.dir ? &kio[k.i].x : &kio[k.i].y, cc);
@@ -659,7 +741,8 @@ static __global__ void __launch_bounds__(256) k_count_chunks(WGraph g, const Chu
     int cc = 0;
     if ((FIRST || a != b) && !(TRIM && trimmed(kio, k.i))) {
         const int32_t* adj = k.dir ? g.iadj : g.oadj;
-        SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio, g.sig2};
+        const int mc = !FIRST && g.min_in ? g.min_in[k.i] : 0, md = !FIRST && g.min_in ? g.min_out[k.i] : 0;
+        SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio, g.sig2, mc, md, g.min_in, g.min_out};
         for (int e = k.beg + lane; e < k.end; e += WARP) cc += pred(__ldg(adj + e));
         cc = warp_sum(cc);
     }
@@ -690,7 +773,8 @@ static __global__ void __launch_bounds__(256) k_scatter_chunks(WGraph g, const C
     const int a = FIRST ? 0 : cin[k.i], b = FIRST ? 0 : cout[k.i];
     const int32_t* adj = k.dir ? g.iadj : g.oadj;
     int32_t* dst = k.dir ? iadj2 : oadj2;
-    SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio, g.sig2};
+    const int mc = !FIRST && g.min_in ? g.min_in[k.i] : 0, md = !FIRST && g.min_in ? g.min_out[k.i] : 0;
+    SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio, g.sig2, mc, md, g.min_in, g.min_out};
     for (int base = k.beg; base < k.end; base += WARP) {
         const int e = base + lane;
         int x = 0;

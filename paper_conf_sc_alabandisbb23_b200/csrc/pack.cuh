@@ -189,14 +189,60 @@ static __global__ void __launch_bounds__(PACK_TH) k_tile_pack(WGraph g, unsigned
     if (tid == 0) ext_cnt[tile] = s_n;
 }
 
+// ---- bulk (TMA) copies of a tile's pack rows into shared memory (cp.async.bulk, SASS
+// UBLKCP) completing on an mbarrier.  The pack is read-only during Phase 2, so the slot
+// words of the NEXT tile of a CTA's run are copied while the current one writes back and
+// marks (its drain no longer reads them); the visit waits on the barrier only after its
+// own value loads and cut-edge pulls.
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long* bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned parity) {
+    asm volatile(
+        "{\n .reg .pred p;\n"
+        "WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        " @!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+// one thread: the pack rows of `tile` -> s_nin / s_nout (2 x 16 KB), completion on bar
+__device__ __forceinline__ void pack_issue(const unsigned long long* __restrict__ pnin,
+                                           const unsigned long long* __restrict__ pnout, int tile,
+                                           unsigned long long* s_nin, unsigned long long* s_nout,
+                                           unsigned long long* bar) {
+    constexpr unsigned BYTES = PACK_TT * 8;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // earlier generic reads first
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(2 * BYTES)
+                 : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(s_nin)),
+                 "l"(pnin + (int64_t)tile * PACK_TT), "r"(BYTES), "r"(smem_u32(bar))
+                 : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(s_nout)),
+                 "l"(pnout + (int64_t)tile * PACK_TT), "r"(BYTES), "r"(smem_u32(bar))
+                 : "memory");
+}
+// the bulk-copy state of a CTA: its barrier, the parity of the next phase, and whether the
+// current tile's copy was already issued by the previous visit
+struct PackTma {
+    unsigned long long* bar;
+    unsigned phase;
+    bool issued;
+};
+
 // One visit of tile `tile` from its pack.  Returns non-zero in every thread if a
-// signature was raised.
+// signature was raised.  T (k_prop_async): the pack rows arrive by bulk copy (PackTma);
+// otherwise (k_prop_pack) by vector loads.
 template <typename Mark>
 __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__ cin, int32_t* __restrict__ cout,
                                           const unsigned long long* __restrict__ pnin,
                                           const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext,
                                           const int* __restrict__ ext_cnt, DevCounters* __restrict__ dc, int tile,
-                                          int full, Mark mark, const TileSmem<PACK_TT>& S, int next = -1) {
+                                          int full, Mark mark, const TileSmem<PACK_TT>& S, int next = -1,
+                                          PackTma* T = nullptr) {
     int* s_in = S.s_in;
     int* s_out = S.s_out;
     unsigned long long* s_nin = S.s_nin;
@@ -214,9 +260,12 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
     if (tid == 0) PROF_ADD(dc, 0, 1);
 #endif
 
-    // ---- step 1: own values and slot words (coalesced 16-byte loads), then the cut-edge
-    // pulls (Alg. 1 l.10-11 across the tile boundary), folded in with shared atomicMax
-    {
+    // ---- step 1: own values and slot words (coalesced 16-byte loads, or the bulk copy),
+    // then the cut-edge pulls (Alg. 1 l.10-11 across the tile boundary), folded in with
+    // shared atomicMax
+    if (T) {
+        if (!T->issued && tid == 0) pack_issue(pnin, pnout, tile, s_nin, s_nout, T->bar);
+    } else {
         const ulonglong2* a = (const ulonglong2*)(pnin + base + v0);
         const ulonglong2* b = (const ulonglong2*)(pnout + base + v0);
         ulonglong2* sa = (ulonglong2*)(s_nin + v0);
@@ -256,6 +305,10 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
         if (val > ((volatile int*)sig)[v]) atomicMax(sig + v, val);
     }
     __syncthreads();
+    if (T) {                                          // the slot words have landed
+        mbar_wait(T->bar, T->phase);
+        T->phase ^= 1u;
+    }
     // ---- step 1b: flags.  First visit of a phase: every vertex; otherwise the intra-tile
     // dependents of what the cut-edge pulls raised.
     unsigned fin = 0, fout = 0;
@@ -279,7 +332,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
     __syncthreads();
     // the next tile of this CTA's run: pull its pack rows and values into L2 while this one
     // drains (384 lines of 128 B, one per thread; L2 is coherent, so racing writers are fine)
-    if (next >= 0 && tid < 384) {
+    if (next >= 0 && tid < 384 && (!T || tid >= 256)) {   // (with T the pack arrives by bulk copy)
         const int nb = next * PACK_TT;
         const char* line;
         if (tid < 128) line = (const char*)(pnin + nb) + 128 * tid;
@@ -306,6 +359,12 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
     __syncthreads();
     const long long t_step2 = clock64();
 #endif
+    // the drain is over (its last block barrier passed): the slot words are free, so the next
+    // tile's copy overlaps this write-back and the marks
+    if (T) {
+        T->issued = next >= 0;
+        if (next >= 0 && tid == 0) pack_issue(pnin, pnout, next, s_nin, s_nout, T->bar);
+    }
     // ---- step 3: write back (whole 16-byte groups; only this CTA writes these vertices
     // during the pass, so global memory still holds the originals: re-read rather than
     // kept in registers across step 2) and record which directions rose, for the marks
@@ -489,13 +548,18 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
     S.s_nin = (unsigned long long*)(S.s_out + PACK_TT + 4);
     S.s_nout = S.s_nin + PACK_TT;
     __shared__ unsigned long long s_acc[3];            // visited vertices, edges, tiles (flushed at the end)
+    __shared__ __align__(8) unsigned long long s_bar;  // bulk-copy barrier of the pack rows
     S.s_fin = s_fin;
     S.s_fout = s_fout;
     S.s_queue = nullptr;
     S.s_acc = s_acc;
     const int tid = threadIdx.x;
     const int ntiles = (g.na + PACK_TT - 1) / PACK_TT;
-    if (tid == 0) { S.s_in[PACK_TT] = 0; S.s_out[PACK_TT] = 0; s_acc[0] = s_acc[1] = s_acc[2] = 0; }
+    if (tid == 0) {
+        S.s_in[PACK_TT] = 0; S.s_out[PACK_TT] = 0; s_acc[0] = s_acc[1] = s_acc[2] = 0;
+        mbar_init(&s_bar, 1);
+    }
+    PackTma T{&s_bar, 0u, false};
     volatile unsigned long long* ctr = Q.ctr;
     long long t0 = clock64();
     for (;;) {
@@ -559,7 +623,7 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             for (int i = tid; i < MSET; i += PACK_TH) s_set[i] = -1;
             __syncthreads();
             pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S,
-                       j + 1 < nclaim ? s_claim[j + 1] : -1);
+                       j + 1 < nclaim ? s_claim[j + 1] : -1, &T);
             __threadfence();                                      // values before marks
             __syncthreads();
             for (int i = tid; i < MSET; i += PACK_TH)

@@ -306,7 +306,7 @@ static int ensure_pack(Plan* p) {
 
 // a7 + a2 + a3 + a8: Phase 3 edge removal, Trim-1, compaction into buffer `ob` with the
 // Phase-1 reset of the survivors and the final labels of the vertices that leave
-template <bool FIRST, bool TRIM>
+template <bool FIRST, bool TRIM, bool FOUR>
 static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, const int32_t* cout, int ob,
                               int32_t* labels, const Prio& P, cudaStream_t s) {
     const unsigned grid = grid_for(g.na, TPB);
@@ -331,33 +331,33 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
         if (int r = ensure_pack(p)) return r;
         pk = PackOut{p->pnin, p->pnout, p->ext, p->ext_cnt, &p->dc->pack_bad};
     }
-    p->launches++; k_keep_count<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, chunked, p->hcnt, p->emask);
+    p->launches++; k_keep_count<FIRST, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, chunked, p->hcnt, p->emask);
     if (chunked) {
         p->launches++;
-        k_keep_chunks<FIRST><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio);
+        k_keep_chunks<FIRST, FOUR><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio);
     }
     const bool trim2 = TRIM && (p->flags & ECL_SCC_TRIM2);
     if (trim2) {                                   // Trim-2 on the kept degrees (reading 17)
         p->launches += 2;
-        k_trim2_find<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->emask, p->t2);
+        k_trim2_find<FIRST, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->emask, p->t2);
         k_trim2_apply<<<grid, TPB, 0, s>>>(g.na, p->t2, p->kio);
     }
     if (chunked) {
         p->launches++;
-        k_count_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio, p->chunk_cnt, p->hcnt);
+        k_count_chunks<FIRST, TRIM, FOUR><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio, p->chunk_cnt, p->hcnt);
     }
-    p->launches++; k_compact_count<FIRST, TRIM><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
+    p->launches++; k_compact_count<FIRST, TRIM, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
     int r = scan_excl<I3>(p, (const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
     if (r) return r;
     p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
                                               chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur, pk,
                                               p->min_in[ob], p->min_out[ob], trim2 ? p->t2 : nullptr);
-    p->launches++; k_compact_scatter<FIRST, TRIM><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->newidx, p->optr[ob],
+    p->launches++; k_compact_scatter<FIRST, TRIM, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked, p->emask, pk);
     if (chunked) {
         p->launches++;
-        k_scatter_chunks<FIRST, TRIM><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio, p->chunk_cnt,
+        k_scatter_chunks<FIRST, TRIM, FOUR><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio, p->chunk_cnt,
                                                                      p->newidx, p->optr[ob], p->iptr[ob], p->oadj[ob], p->iadj[ob]);
     }
     p->cb ^= 1;                                   // the next graph's chunk list is now current
@@ -588,10 +588,13 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         for (int iter = 1;; iter++) {
             if (iter > n + 2) return fail(ECL_SCC_ECUDA, "internal: outer loop exceeded n+2 iterations");
             stage_mark(p, 2, s);
-            if (iter == 1) r = trim ? remove_and_compact<true, true>(p, g, cin, cout, ob, labels, P, s)
-                                    : remove_and_compact<true, false>(p, g, cin, cout, ob, labels, P, s);
-            else r = trim ? remove_and_compact<false, true>(p, g, cin, cout, ob, labels, P, s)
-                          : remove_and_compact<false, false>(p, g, cin, cout, ob, labels, P, s);
+            const bool four = (p->flags & ECL_SCC_FOUR_SIG) != 0;     // (iteration 1 keeps every edge)
+            if (iter == 1) r = trim ? remove_and_compact<true, true, false>(p, g, cin, cout, ob, labels, P, s)
+                                    : remove_and_compact<true, false, false>(p, g, cin, cout, ob, labels, P, s);
+            else if (four) r = trim ? remove_and_compact<false, true, true>(p, g, cin, cout, ob, labels, P, s)
+                                    : remove_and_compact<false, false, true>(p, g, cin, cout, ob, labels, P, s);
+            else r = trim ? remove_and_compact<false, true, false>(p, g, cin, cout, ob, labels, P, s)
+                          : remove_and_compact<false, false, false>(p, g, cin, cout, ob, labels, P, s);
             if (r) return r;
             stage_mark(p, 3, s);
             CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));

@@ -144,7 +144,7 @@ static __global__ void __launch_bounds__(256) k_csc_scatter(int32_t n, const int
 // endpoint's pair is gathered.  In the first removal (FIRST) every edge except a
 // self-loop is kept (DESIGN reading 9).
 // With the 4-signature variant (mi != nullptr) the minimum pair (c, d) must agree as well.
-template <bool FIRST>
+template <bool FIRST, bool FOUR = false>
 __device__ __forceinline__ bool keep_edge(int owner, int a, int b, int other, const int32_t* __restrict__ cin,
                                           const int32_t* __restrict__ cout, const int2* __restrict__ s2 = nullptr,
                                           int c = 0, int d = 0, const int32_t* __restrict__ mi = nullptr,
@@ -158,7 +158,7 @@ __device__ __forceinline__ bool keep_edge(int owner, int a, int b, int other, co
         // both loads are issued unconditionally (no short circuit): callers batch these gathers
         k = (__ldg(cin + other) == a) & (__ldg(cout + other) == b);
     }
-    if (mi) k &= (__ldg(mi + other) == c) & (__ldg(mo + other) == d);
+    if (FOUR) k &= (__ldg(mi + other) == c) & (__ldg(mo + other) == d);
     return k;
 }
 // Phase 3 of power-law graphs: the signatures interleaved for one gather per far end
@@ -179,7 +179,7 @@ struct RowCtx {
     bool valid, live;
 };
 
-template <bool FIRST>
+template <bool FIRST, bool FOUR = false>
 __device__ __forceinline__ RowCtx load_row(const WGraph& g, int64_t i, const int32_t* __restrict__ cin,
                                            const int32_t* __restrict__ cout) {
     RowCtx r{};
@@ -188,7 +188,7 @@ __device__ __forceinline__ RowCtx load_row(const WGraph& g, int64_t i, const int
         r.ob = g.optr[i]; r.oe = g.optr[i + 1];
         r.ib = g.iptr[i]; r.ie = g.iptr[i + 1];
         if (!FIRST) { r.a = cin[i]; r.b = cout[i]; }
-        if (!FIRST && g.min_in) { r.c = g.min_in[i]; r.d = g.min_out[i]; }
+        if (!FIRST && FOUR) { r.c = g.min_in[i]; r.d = g.min_out[i]; }
     }
     r.live = r.valid && (FIRST || r.a != r.b);
     return r;
@@ -218,14 +218,14 @@ __device__ __forceinline__ int count_row(const int32_t* __restrict__ adj, int rb
 
 // predicate objects: evaluated for the row owner's lane; bcast(src) gives lane src's
 // predicate to the whole warp (all lanes must call it)
-template <bool FIRST>
+template <bool FIRST, bool FOUR = false>
 struct KeepPred {
     int i, a, b;
     const int32_t *cin, *cout;
     const int2* s2;
     int c, d;
     const int32_t *mi, *mo;
-    __device__ __forceinline__ bool operator()(int k) const { return keep_edge<FIRST>(i, a, b, k, cin, cout, s2, c, d, mi, mo); }
+    __device__ __forceinline__ bool operator()(int k) const { return keep_edge<FIRST, FOUR>(i, a, b, k, cin, cout, s2, c, d, mi, mo); }
     __device__ __forceinline__ KeepPred bcast(int src) const {
         KeepPred p = *this;
         p.i = __shfl_sync(FULL, i, src); p.a = __shfl_sync(FULL, a, src); p.b = __shfl_sync(FULL, b, src);
@@ -233,7 +233,7 @@ struct KeepPred {
         return p;
     }
 };
-template <bool FIRST, bool TRIM>
+template <bool FIRST, bool TRIM, bool FOUR = false>
 struct SurvivePred {
     int i, a, b;
     const int32_t *cin, *cout;
@@ -242,7 +242,7 @@ struct SurvivePred {
     int c, d;
     const int32_t *mi, *mo;
     __device__ __forceinline__ bool operator()(int k) const {
-        return keep_edge<FIRST>(i, a, b, k, cin, cout, s2, c, d, mi, mo) & !(TRIM && trimmed(kio, k));
+        return keep_edge<FIRST, FOUR>(i, a, b, k, cin, cout, s2, c, d, mi, mo) & !(TRIM && trimmed(kio, k));
     }
     __device__ __forceinline__ SurvivePred bcast(int src) const {
         SurvivePred p = *this;
@@ -376,14 +376,14 @@ __device__ __forceinline__ void emit_cut(const int32_t* __restrict__ adj, int b,
 
 // kept in/out degree per local vertex (light rows: also the kept entries as bit masks)
 constexpr int TPB_COMPACT = 256;     // block size of the compaction kernels (driver TPB)
-template <bool FIRST>
+template <bool FIRST, bool FOUR>
 static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                              int2* __restrict__ kio, int chunked, int2* __restrict__ hcnt,
                              uint2* __restrict__ emask) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const RowCtx r = load_row<FIRST>(g, i, cin, cout);
-    KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout, g.sig2, r.c, r.d, g.min_in, g.min_out};
+    const RowCtx r = load_row<FIRST, FOUR>(g, i, cin, cout);
+    KeepPred<FIRST, FOUR> pred{(int)i, r.a, r.b, cin, cout, g.sig2, r.c, r.d, g.min_in, g.min_out};
     unsigned mo = 0, mi = 0;
     mask_light2(g.oadj, r.ob, r.live && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, g.iadj, r.ib,
                 r.live && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, (int)(r.valid ? i : 0), pred, mo, mi);
@@ -400,20 +400,20 @@ static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, con
 }
 
 // per-vertex surviving (kept, not trimmed) degrees and per-warp totals (alive, out, in, kept)
-template <bool FIRST, bool TRIM>
+template <bool FIRST, bool TRIM, bool FOUR>
 static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                 const int2* __restrict__ kio,
                                 int2* __restrict__ cnt, int4* __restrict__ wsum, int chunked,
                                 const int2* __restrict__ hcnt, uint2* __restrict__ emask) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const RowCtx r = load_row<FIRST>(g, i, cin, cout);
+    const RowCtx r = load_row<FIRST, FOUR>(g, i, cin, cout);
     int nout = 0, nin = 0;
     if (!TRIM) {
         if (r.live) { const int2 k = kio[i]; nout = k.y; nin = k.x; }   // survivors = kept: the masks stand
     } else {
         const bool go = r.live && !trimmed(kio, (int)i);
-        SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2, r.c, r.d, g.min_in, g.min_out};
+        SurvivePred<FIRST, TRIM, FOUR> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2, r.c, r.d, g.min_in, g.min_out};
         if (r.valid) {                                   // light rows: the kept entries' far ends
             const uint2 km = emask[i];
             const unsigned so = go && r.oe - r.ob <= HEAVY ? trim_mask(g.oadj, r.ob, km.x, (int)i, kio) : 0u;
@@ -465,15 +465,15 @@ __device__ __forceinline__ bool kept_has(const int32_t* __restrict__ adj, int rb
         if (__ldg(adj + e) == w && pred(w)) return true;
     return false;
 }
-template <bool FIRST>
+template <bool FIRST, bool FOUR>
 static __global__ void k_trim2_find(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                     const int2* __restrict__ kio, const uint2* __restrict__ emask, int32_t* __restrict__ t2) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= g.na) return;
-    const RowCtx r = load_row<FIRST>(g, i, cin, cout);
+    const RowCtx r = load_row<FIRST, FOUR>(g, i, cin, cout);
     int w = -1;
     if (r.live) {
-        KeepPred<FIRST> pred{(int)i, r.a, r.b, cin, cout, g.sig2, r.c, r.d, g.min_in, g.min_out};
+        KeepPred<FIRST, FOUR> pred{(int)i, r.a, r.b, cin, cout, g.sig2, r.c, r.d, g.min_in, g.min_out};
         const int2 k = kio[i];
         const uint2 m = emask[i];
         if (k.x == 1) {                                  // in-pattern
@@ -646,7 +646,7 @@ __device__ __forceinline__ void emit_row(const int32_t* __restrict__ adj, int rb
     }
 }
 
-template <bool FIRST, bool TRIM>
+template <bool FIRST, bool TRIM, bool FOUR>
 static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                   const int2* __restrict__ kio, const int32_t* __restrict__ newidx, const int32_t* __restrict__ optr2,
                                   const int32_t* __restrict__ iptr2, int32_t* __restrict__ oadj2,
@@ -654,7 +654,7 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
                                   PackOut pk) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const RowCtx r = load_row<FIRST>(g, i, cin, cout);
+    const RowCtx r = load_row<FIRST, FOUR>(g, i, cin, cout);
     const int j = r.valid ? newidx[i] : -1;
     const bool go = j >= 0;
     int po = 0, pi = 0, ncut = 0;
@@ -698,7 +698,7 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
             if (li) emit_cut(g.iadj, r.ib, sm.y, newidx, j, tb, 0, E, at);
         }
     }
-    SurvivePred<FIRST, TRIM> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2, r.c, r.d, g.min_in, g.min_out};
+    SurvivePred<FIRST, TRIM, FOUR> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2, r.c, r.d, g.min_in, g.min_out};
     emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred, chunked, false);
     emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred, chunked, false);
 }
@@ -708,7 +708,7 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
 // compaction kernel, so a 100k-edge hub costs 200 warps, not one.  Counts are folded in
 // with atomics; the scatter places a chunk after the survivors of the earlier chunks of
 // its row (chunk_cnt prefix), so rows stay stable.
-template <bool FIRST>
+template <bool FIRST, bool FOUR>
 static __global__ void __launch_bounds__(256) k_keep_chunks(WGraph g, const Chunk* __restrict__ chunks, int nchunks,
                                                             const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                                             int2* __restrict__ kio) {
@@ -718,17 +718,17 @@ static __global__ void __launch_bounds__(256) k_keep_chunks(WGraph g, const Chun
     const Chunk k = chunks[c];
     const int a = FIRST ? 0 : cin[k.i], b = FIRST ? 0 : cout[k.i];
     if (!FIRST && a == b) return;                        // finished owner keeps nothing
-    const int mc = !FIRST && g.min_in ? g.min_in[k.i] : 0, md = !FIRST && g.min_in ? g.min_out[k.i] : 0;
+    const int mc = !FIRST && FOUR ? g.min_in[k.i] : 0, md = !FIRST && FOUR ? g.min_out[k.i] : 0;
     const int32_t* adj = k.dir ? g.iadj : g.oadj;
     int cc = 0;
     for (int e = k.beg + lane; e < k.end; e += WARP)
-        cc += keep_edge<FIRST>(k.i, a, b, __ldg(adj + e), cin, cout, g.sig2, mc, md, g.min_in, g.min_out);
+        cc += keep_edge<FIRST, FOUR>(k.i, a, b, __ldg(adj + e), cin, cout, g.sig2, mc, md, g.min_in, g.min_out);
     cc = warp_sum(cc);
     if (lane == 0 && cc) {
         atomicAdd(k.dir ? &kio[k.i].x : &kio[k.i].y, cc);
     }
 }
-template <bool FIRST, bool TRIM>
+template <bool FIRST, bool TRIM, bool FOUR>
 static __global__ void __launch_bounds__(256) k_count_chunks(WGraph g, const Chunk* __restrict__ chunks, int nchunks,
                                                              const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                                              const int2* __restrict__ kio,
@@ -741,8 +741,8 @@ static __global__ void __launch_bounds__(256) k_count_chunks(WGraph g, const Chu
     int cc = 0;
     if ((FIRST || a != b) && !(TRIM && trimmed(kio, k.i))) {
         const int32_t* adj = k.dir ? g.iadj : g.oadj;
-        const int mc = !FIRST && g.min_in ? g.min_in[k.i] : 0, md = !FIRST && g.min_in ? g.min_out[k.i] : 0;
-        SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio, g.sig2, mc, md, g.min_in, g.min_out};
+        const int mc = !FIRST && FOUR ? g.min_in[k.i] : 0, md = !FIRST && FOUR ? g.min_out[k.i] : 0;
+        SurvivePred<FIRST, TRIM, FOUR> pred{k.i, a, b, cin, cout, kio, g.sig2, mc, md, g.min_in, g.min_out};
         for (int e = k.beg + lane; e < k.end; e += WARP) cc += pred(__ldg(adj + e));
         cc = warp_sum(cc);
     }
@@ -751,7 +751,7 @@ static __global__ void __launch_bounds__(256) k_count_chunks(WGraph g, const Chu
         if (cc) atomicAdd(k.dir ? &hcnt[k.i].y : &hcnt[k.i].x, cc);
     }
 }
-template <bool FIRST, bool TRIM>
+template <bool FIRST, bool TRIM, bool FOUR>
 static __global__ void __launch_bounds__(256) k_scatter_chunks(WGraph g, const Chunk* __restrict__ chunks, int nchunks,
                                                                const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                                                const int2* __restrict__ kio,
@@ -773,8 +773,8 @@ static __global__ void __launch_bounds__(256) k_scatter_chunks(WGraph g, const C
     const int a = FIRST ? 0 : cin[k.i], b = FIRST ? 0 : cout[k.i];
     const int32_t* adj = k.dir ? g.iadj : g.oadj;
     int32_t* dst = k.dir ? iadj2 : oadj2;
-    const int mc = !FIRST && g.min_in ? g.min_in[k.i] : 0, md = !FIRST && g.min_in ? g.min_out[k.i] : 0;
-    SurvivePred<FIRST, TRIM> pred{k.i, a, b, cin, cout, kio, g.sig2, mc, md, g.min_in, g.min_out};
+    const int mc = !FIRST && FOUR ? g.min_in[k.i] : 0, md = !FIRST && FOUR ? g.min_out[k.i] : 0;
+    SurvivePred<FIRST, TRIM, FOUR> pred{k.i, a, b, cin, cout, kio, g.sig2, mc, md, g.min_in, g.min_out};
     for (int base = k.beg; base < k.end; base += WARP) {
         const int e = base + lane;
         int x = 0;

@@ -86,6 +86,9 @@ typedef enum {
                                      u <-> w whose only kept in-edges (or only kept out-edges)
                                      are each other is an SCC of two (reading 17);
                                      EINVAL together with ECL_SCC_NO_TRIM */
+#define ECL_SCC_HALO_ALLREDUCE 0x10000u /* partitioned mode, baseline exchange: combine the halo
+                                     signatures with ncclAllReduce(MAX) after every local fixed
+                                     point instead of the propagation kernel's peer pushes */
 #define ECL_SCC_FOUR_SIG 0x8000u  /* variant: the 4-signature method -- Phase 2 also
                                      propagates minimum ancestor / descendant IDs and Phase 3
                                      keeps an edge only if all four signatures agree; twice the
@@ -205,26 +208,41 @@ int ecl_scc_part_plan_destroy(ecl_scc_part_plan_t plan);
 
 /* Collective over comm.  This rank owns source rows [row_begin, row_end) of the global
  * graph (n vertices): local_row_ptr has row_end-row_begin+1 offsets starting at 0,
- * local_col_idx holds local_nnz GLOBAL destination IDs.  Signatures are replicated and
- * combined with ncclAllReduce(MAX) after every local fixed point; degrees for trim with
- * ncclAllReduce(SUM).  labels_out: n int32 on every rank (replicated result).
+ * local_col_idx holds local_nnz GLOBAL destination IDs.  Every rank runs the single-GPU path
+ * on its rows (the owned vertices plus the destinations owned elsewhere, its ghosts); the
+ * ranks exchange only the halo -- the vertices held by more than one rank (DESIGN.md section
+ * 7): the kept degrees (Trim-1) once per outer iteration (ncclAllReduce SUM over the halo),
+ * and in Phase 2 the signatures, pushed by the propagation kernel into every rank's halo
+ * buffer (NCCL symmetric memory: NVLS multimem reduction or remote atomic max over NVLink)
+ * with a one-word all-reduce as the barrier, until no rank's copy rises.
+ * labels_out: n int32 on every rank (replicated result, one final ncclAllReduce).
  * plan: nullable (then a temporary workspace is allocated for this call).
  * Errors: invalid input on ANY rank makes every rank return ECL_SCC_ERANGE (the ranks agree
  * through the first exchange before any of them leaves); a CUDA or NCCL failure on one rank
- * leaves the communicator unusable (destroy it).  stats->ms_comm / comm_bytes / exchanges
- * report the exchanges of this rank. */
+ * leaves the communicator unusable (destroy it).  Trim-2 and the 4-signature variant are
+ * not supported here (EUNSUPPORTED at plan creation).  stats->ms_comm / comm_bytes /
+ * exchanges report the collectives of this rank (the fused pushes run inside the
+ * propagation kernel and are not separately timed). */
 int ecl_scc_partitioned(ecl_scc_comm_t comm, int32_t n, int32_t row_begin, int32_t row_end,
                         int64_t local_nnz, const int32_t* local_row_ptr,
                         const int32_t* local_col_idx, int32_t* labels_out,
                         ecl_scc_stream_t stream, ecl_scc_part_plan_t plan, ecl_scc_stats* stats);
 
 /* Single-process emulation of the partitioned algorithm with P partitions on the
- * current device (the all-reduce replaced by an element-wise max over P replicas).
- * Same arithmetic as ecl_scc_partitioned at P ranks; used to test the partitioned path
- * on one GPU.  Inputs as ecl_scc(); row ranges are chosen balanced by edge count. */
+ * current device (P rank workspaces; the all-reduces are element-wise reductions over the P
+ * buffers and the fused pushes target the P halo buffers of the same device).  Same
+ * arithmetic and exchange protocol as ecl_scc_partitioned at P ranks; used to test the
+ * partitioned path on one GPU.  Inputs as ecl_scc(); row ranges are chosen balanced by edge
+ * count.  flags: as ecl_scc_part_plan_create (ECL_SCC_HALO_ALLREDUCE selects the baseline
+ * exchange). */
 int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_t* row_ptr,
-                                 const int32_t* col_idx, int32_t* labels_out,
+                                 const int32_t* col_idx, int32_t* labels_out, uint32_t flags,
                                  ecl_scc_stream_t stream, ecl_scc_stats* stats);
+
+/* Diagnostics of a communicator: info[0] ranks, [1] this rank, [2] 1 if the NCCL device API
+ * is in use for the fused halo exchange (peer pushes), [3] 1 if it uses NVLS multimem
+ * reductions.  Filled after the first ecl_scc_partitioned call. */
+int ecl_scc_comm_info(ecl_scc_comm_t comm, int32_t info[4]);
 
 /* Host helper: split rows [0,n) into P contiguous ranges of about equal edge count
  * (binary search on the host row_ptr[n+1]); bounds_out[P+1] (host). */

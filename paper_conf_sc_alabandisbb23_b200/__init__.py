@@ -21,7 +21,7 @@ OK, EINVAL, ERANGE, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED = range(7)
 NO_TRIM, NO_VALIDATE, SYNC_PASSES, TIME_STAGES = 0x1, 0x4, 0x8, 0x10
 IDENTITY_IDS, NO_DIRTY, NO_REORDER = 0x20, 0x40, 0x200
 FORCE_REORDER, NO_PACK, NO_ASYNC = 0x400, 0x800, 0x1000
-TRIM2, FOUR_SIG = 0x4000, 0x8000
+TRIM2, FOUR_SIG, HALO_ALLREDUCE = 0x4000, 0x8000, 0x10000
 TRACE_MAX = 64
 
 _lib = None
@@ -79,7 +79,8 @@ def lib() -> ctypes.CDLL:
         "ecl_scc_partitioned": [vp, i32, i32, i32, i64, vp, vp, vp, vp, vp, vp],
         "ecl_scc_part_plan_create": [i32, i32, i32, i64, u32, vp],
         "ecl_scc_part_plan_destroy": [vp],
-        "ecl_scc_partitioned_emulated": [i32, i32, i64, vp, vp, vp, vp, vp],
+        "ecl_scc_partitioned_emulated": [i32, i32, i64, vp, vp, vp, u32, vp, vp],
+        "ecl_scc_comm_info": [vp, vp],
         "ecl_scc_partition_rows": [i32, i32, vp, vp],
         "ecl_scc_status_string": [ctypes.c_int],
         "ecl_scc_last_error": [],
@@ -104,7 +105,7 @@ ABI_SYMBOLS = ("ecl_scc", "ecl_scc_async", "ecl_scc_debug_run", "ecl_scc_plan_cr
                "ecl_scc_comm_create", "ecl_scc_comm_destroy", "ecl_scc_partitioned",
                "ecl_scc_partitioned_emulated", "ecl_scc_partition_rows", "ecl_scc_status_string",
                "ecl_scc_last_error", "ecl_scc_version", "ecl_scc_plan_counters", "ecl_scc_levels",
-               "ecl_scc_host", "ecl_scc_part_plan_create", "ecl_scc_part_plan_destroy")
+               "ecl_scc_host", "ecl_scc_part_plan_create", "ecl_scc_part_plan_destroy", "ecl_scc_comm_info")
 
 
 def status_string(s: int) -> str:
@@ -246,14 +247,15 @@ def ecl_scc_partition_rows(P: int, row_ptr_host) -> list[int]:
     return out.tolist()
 
 
-def ecl_scc_partitioned_emulated(P: int, row_ptr, col_idx, labels_out=None, stream=None, stats: bool = False):
+def ecl_scc_partitioned_emulated(P: int, row_ptr, col_idx, labels_out=None, stream=None, stats: bool = False,
+                                 flags: int = 0):
     n = row_ptr.numel() - 1
     if labels_out is None:
         labels_out = torch.empty(n, dtype=torch.int32, device=row_ptr.device)
     st = Stats() if stats else None
     _check(lib().ecl_scc_partitioned_emulated(P, n, col_idx.numel(), _dev_i32(row_ptr, "row_ptr"),
                                               _dev_i32(col_idx, "col_idx") if col_idx.numel() else None,
-                                              _dev_i32(labels_out, "labels_out"), _stream(stream),
+                                              _dev_i32(labels_out, "labels_out"), flags, _stream(stream),
                                               ctypes.byref(st) if st else None), "ecl_scc_partitioned_emulated")
     return (labels_out, st.as_dict()) if stats else labels_out
 
@@ -272,6 +274,12 @@ class Comm:
         buf = (ctypes.c_uint8 * 128)(*uid)
         _check(lib().ecl_scc_comm_create(nranks, rank, buf, ctypes.byref(h)), "ecl_scc_comm_create")
         self.handle, self.nranks, self.rank = h, nranks, rank
+
+    def info(self) -> dict:
+        """ranks, rank, and whether the fused halo exchange uses the NCCL device API / NVLS."""
+        out = (ctypes.c_int32 * 4)()
+        _check(lib().ecl_scc_comm_info(self.handle, out), "ecl_scc_comm_info")
+        return dict(nranks=out[0], rank=out[1], device_api=bool(out[2]), multimem=bool(out[3]))
 
     def close(self):
         if self.handle:

@@ -27,6 +27,8 @@ struct WGraph {
     const int32_t* min_in;   // ECL_SCC_FOUR_SIG: the minimum signatures, stored mirrored
     const int32_t* min_out;  // (INT32_MAX - priority) so Phase 2 propagates them with max;
                              // nullptr: the two-signature method
+    const int32_t* hpos;     // partitioned mode (halo.cuh): position of each local vertex in the
+                             // halo H, or -1; nullptr: single GPU
 };
 // the minimum signatures propagate as maxima of mirrored priorities (all >= 0, so the
 // pack kernels' sentinel value 0 stays below every signature)

@@ -25,6 +25,7 @@
 #include "reorder.cuh"
 #include "pack.cuh"
 #include "levels.cuh"
+#include "partition.cuh"
 #include "driver.h"
 
 namespace eclscc {
@@ -85,6 +86,8 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     p->knob_claim_div = knob("ECL_SCC_CLAIM_DIV", 1, 64);
     p->knob_claim_max = knob("ECL_SCC_CLAIM_MAX", 1, 32);
     p->knob_async_ctas = knob("ECL_SCC_ASYNC_CTAS", 1, 8);
+    p->lab_lo = 0;
+    p->lab_hi = INT32_MAX;
     if (cudaGetDevice(&p->device) != cudaSuccess) {
         cudaGetLastError();
         return fail(ECL_SCC_ECUDA, "plan: no current CUDA device");
@@ -150,7 +153,7 @@ void plan_free(Plan* p) {
         cudaFree(p->optr[b]); cudaFree(p->iptr[b]); cudaFree(p->oadj[b]); cudaFree(p->iadj[b]);
     }
     for (int b = 0; b < 2; b++) { cudaFree(p->min_in[b]); cudaFree(p->min_out[b]); }
-    cudaFree(p->t2);
+    cudaFree(p->t2); cudaFree(p->hpos[0]); cudaFree(p->hpos[1]);
     cudaFree(p->kin); cudaFree(p->newidx); cudaFree(p->cnt); cudaFree(p->emask); cudaFree(p->sig2);
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
     cudaFree(p->chunk_cnt); cudaFree(p->hcnt);
@@ -305,18 +308,16 @@ static int ensure_pack(Plan* p) {
 }
 
 // a7 + a2 + a3 + a8: Phase 3 edge removal, Trim-1, compaction into buffer `ob` with the
-// Phase-1 reset of the survivors and the final labels of the vertices that leave
+// Phase-1 reset of the survivors and the final labels of the vertices that leave.  Two
+// parts: compact_keep evaluates the keep predicate (kept degrees), compact_finish trims and
+// compacts; the partitioned mode exchanges the halo's kept degrees in between.
 template <bool FIRST, bool TRIM, bool FOUR>
-static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, const int32_t* cout, int ob,
-                              int32_t* labels, const Prio& P, cudaStream_t s) {
+static int compact_keep(Plan* p, const WGraph& g, const int32_t* cin, const int32_t* cout, cudaStream_t s) {
     const unsigned grid = grid_for(g.na, TPB);
-    const int64_t nw = (int64_t)grid * (TPB / WARP);
     const int nc = p->nchunks_cur, chunked = nc > 0;
     const Chunk* cur = chunk_buf(p, p->cb);
     CK(cudaMemsetAsync(&p->dc->nchunks, 0, sizeof(int), s));
     CK(cudaMemsetAsync(&p->dc->pack_bad, 0, sizeof(int), s));
-    // the scatter writes the next graph's tile pack when Phase 2 will use one (no long rows
-    // now means none after the compaction)
     // power-law graphs (long-row chunks): keep() gathers random far ends, so the two signature
     // arrays are interleaved once (one gather per far end instead of two)
     WGraph gk = g;
@@ -325,22 +326,37 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
         k_pack_sig<<<std::min<unsigned>(grid, 148 * 16), TPB, 0, s>>>(g.na, cin, cout, p->sig2);
         gk.sig2 = p->sig2;
     }
+    p->launches++; k_keep_count<FIRST, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, chunked, p->hcnt, p->emask);
+    if (chunked) {
+        p->launches++;
+        k_keep_chunks<FIRST, FOUR><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio);
+    }
+    p->gk = gk;
+    CK(cudaGetLastError());
+    return ECL_SCC_OK;
+}
+
+template <bool FIRST, bool TRIM, bool FOUR>
+static int compact_finish(Plan* p, const int32_t* cin, const int32_t* cout, int ob, int32_t* labels, const Prio& P,
+                          cudaStream_t s) {
+    const WGraph gk = p->gk;
+    const unsigned grid = grid_for(gk.na, TPB);
+    const int64_t nw = (int64_t)grid * (TPB / WARP);
+    const int nc = p->nchunks_cur, chunked = nc > 0;
+    const Chunk* cur = chunk_buf(p, p->cb);
+    // the scatter writes the next graph's tile pack when Phase 2 will use one (no long rows
+    // now means none after the compaction)
     PackOut pk{nullptr, nullptr, nullptr, nullptr, &p->dc->pack_bad};
     p->pack_fused = pack_path(p, nc);
     if (p->pack_fused) {
         if (int r = ensure_pack(p)) return r;
         pk = PackOut{p->pnin, p->pnout, p->ext, p->ext_cnt, &p->dc->pack_bad};
     }
-    p->launches++; k_keep_count<FIRST, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, chunked, p->hcnt, p->emask);
-    if (chunked) {
-        p->launches++;
-        k_keep_chunks<FIRST, FOUR><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio);
-    }
     const bool trim2 = TRIM && (p->flags & ECL_SCC_TRIM2);
     if (trim2) {                                   // Trim-2 on the kept degrees (reading 17)
         p->launches += 2;
         k_trim2_find<FIRST, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->emask, p->t2);
-        k_trim2_apply<<<grid, TPB, 0, s>>>(g.na, p->t2, p->kio);
+        k_trim2_apply<<<grid, TPB, 0, s>>>(gk.na, p->t2, p->kio);
     }
     if (chunked) {
         p->launches++;
@@ -352,7 +368,8 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
                                               chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur, pk,
-                                              p->min_in[ob], p->min_out[ob], trim2 ? p->t2 : nullptr);
+                                              p->min_in[ob], p->min_out[ob], trim2 ? p->t2 : nullptr, p->kio, TRIM ? 1 : 0,
+                                              gk.hpos ? p->hpos[ob] : nullptr, p->lab_lo, p->lab_hi);
     p->launches++; k_compact_scatter<FIRST, TRIM, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked, p->emask, pk);
     if (chunked) {
@@ -363,6 +380,26 @@ static int remove_and_compact(Plan* p, const WGraph& g, const int32_t* cin, cons
     p->cb ^= 1;                                   // the next graph's chunk list is now current
     CK(cudaGetLastError());
     return ECL_SCC_OK;
+}
+
+// part 0 = keep, 1 = finish, of the compaction before outer iteration `iter`
+static int compaction(Plan* p, int part, int iter, const WGraph& g, const int32_t* cin, const int32_t* cout, int ob,
+                      int32_t* labels, const Prio& P, cudaStream_t s) {
+    const bool trim = !(p->flags & ECL_SCC_NO_TRIM);
+    const bool four = (p->flags & ECL_SCC_FOUR_SIG) != 0 && iter > 1;   // (iteration 1 keeps every edge)
+#define ECL_COMPACT(F, T, Fo) \
+    return part == 0 ? compact_keep<F, T, Fo>(p, g, cin, cout, s) : compact_finish<F, T, Fo>(p, cin, cout, ob, labels, P, s)
+    if (iter == 1) {
+        if (trim) ECL_COMPACT(true, true, false);
+        ECL_COMPACT(true, false, false);
+    }
+    if (four) {
+        if (trim) ECL_COMPACT(false, true, true);
+        ECL_COMPACT(false, false, true);
+    }
+    if (trim) ECL_COMPACT(false, true, false);
+    ECL_COMPACT(false, false, false);
+#undef ECL_COMPACT
 }
 
 // per-plan (per-device) kernel attributes of the pass kernels
@@ -394,8 +431,11 @@ static int launch_tile(Plan* p, bool sync, const WGraph& g, int32_t* cin, int32_
 
 // a4-a6: Phase 2 to its fixed point.  Passes are enqueued in growing batches; a pass
 // whose predecessor changed nothing exits at once, so over-enqueueing costs only a launch.
+// second: a second fixed point over the same graph (the minimum pair); push: the
+// partitioned mode's halo pushes; resume: continue after the halo exchange re-opened tiles
+// (their state / dirty flags set by k_halo_apply) instead of starting with every tile
 static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int nchunks, cudaStream_t s,
-                     int64_t* passes_out, bool second = false) {
+                     int64_t* passes_out, bool second = false, const HaloPush* push = nullptr, bool resume = false) {
     const unsigned ntiles = (unsigned)cdiv(g.na, TILE);
     const unsigned hgrid = (unsigned)std::min<int64_t>(cdiv(std::max(nchunks, 1), TPB / WARP), 148 * 8);
     // plain Jacobi passes: the ablation flag, or graphs whose tiles hold almost no edges
@@ -408,7 +448,7 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     const bool use_pack = pack_path(p, nchunks) && g.na > 0;
     if (use_pack) {
         if (int r = ensure_pack(p)) return r;
-        if (!second && (!p->pack_fused || p->hc->pack_bad)) {   // the scatter did not write it
+        if (!second && !resume && (!p->pack_fused || p->hc->pack_bad)) {   // the scatter did not write it
             p->launches++;
             k_tile_pack<<<ntiles, PACK_TH, 0, s>>>(g, p->pnin, p->pnout, p->ext, p->ext_cnt);
         }
@@ -423,11 +463,13 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                     cudaGetLastError();
                     return fail(ECL_SCC_ENOMEM, "async queue allocation: %s", cudaGetErrorString(e));
                 }
-                CK(cudaFuncSetAttribute(k_prop_async, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
-                CK(cudaFuncSetAttribute(k_prop_async, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                        (int)cudaSharedmemCarveoutMaxShared));
+                for (auto kf : {k_prop_async<false>, k_prop_async<true>}) {
+                    CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
+                    CK(cudaFuncSetAttribute(kf, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                            (int)cudaSharedmemCarveoutMaxShared));
+                }
                 int per_sm = 0, sms = 0;
-                CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_async, PACK_TH, pack_dyn_smem()));
+                CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_async<false>, PACK_TH, pack_dyn_smem()));
                 CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device));
                 // resident CTAs per SM used (<= what fits); measured best: all of them
                 if (p->knob_async_ctas) per_sm = std::min(per_sm, p->knob_async_ctas);
@@ -443,14 +485,23 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             const int cmax = p->knob_claim_max ? p->knob_claim_max : 16;
             const int claim = p->knob_claim ? p->knob_claim
                                             : (int)std::min<int64_t>(cmax, std::max<int64_t>(1, ntiles / (cdiv_ * p->aq_resident)));
-            if (!second) {
+            if (!second && !resume) {
                 CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
                 CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
             }
-            p->launches += 2;
-            k_async_init<<<grid_for((int64_t)ntiles, TPB), TPB, 0, s>>>(Q, (int)ntiles);
-            k_prop_async<<<(unsigned)std::min<int64_t>(ntiles, p->aq_resident), PACK_TH, pack_dyn_smem(), s>>>(
-                g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, Q, claim);
+            if (resume) {                                // cursor and stop words; pending came with the marks
+                CK(cudaMemsetAsync(p->aq_ctr + AQ_CUR, 0, sizeof(unsigned long long), s));
+                CK(cudaMemsetAsync(p->aq_ctr + AQ_STOP, 0, sizeof(unsigned long long), s));
+            } else {
+                p->launches++;
+                k_async_init<<<grid_for((int64_t)ntiles, TPB), TPB, 0, s>>>(Q, (int)ntiles);
+            }
+            p->launches++;
+            const unsigned agrid = (unsigned)std::min<int64_t>(ntiles, p->aq_resident);
+            if (push) k_prop_async<true><<<agrid, PACK_TH, pack_dyn_smem(), s>>>(
+                g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, Q, claim, *push);
+            else k_prop_async<false><<<agrid, PACK_TH, pack_dyn_smem(), s>>>(
+                g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, Q, claim, HaloPush{});
             CK(cudaGetLastError());
             // no stream synchronisation here: the watchdog word and the visit count are read
             // with the counters of the next compaction (resolve_prop in run_graph)
@@ -461,7 +512,7 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     CK(cudaMemsetAsync(p->dc->changed, 0, sizeof(int) * RING, s));
     CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
     if (use_dirty) {
-        CK(cudaMemsetAsync(D[0], 1, ntiles, s));
+        if (!resume) CK(cudaMemsetAsync(D[0], 1, ntiles, s));   // (resume: k_halo_apply's flags)
         CK(cudaMemsetAsync(D[1], 0, ntiles, s));
     }
     int pass = 0;
@@ -494,6 +545,11 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
         fprintf(stderr, "[ecl_scc] na=%d passes=%llu visited_vertices=%llu\n", g.na,
                 (unsigned long long)p->hc->passes, (unsigned long long)p->hc->visit_v);
     *passes_out = (int64_t)p->hc->passes;
+    if (push && g.na > 0) {                       // pass kernels: push every halo copy afterwards
+        p->launches++;
+        k_halo_push<<<std::min<unsigned>(grid_for(g.na, TPB), 148 * 8), TPB, 0, s>>>(g.na, cin, cout, *push);
+        CK(cudaGetLastError());
+    }
     return ECL_SCC_OK;
 }
 
@@ -588,13 +644,8 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         for (int iter = 1;; iter++) {
             if (iter > n + 2) return fail(ECL_SCC_ECUDA, "internal: outer loop exceeded n+2 iterations");
             stage_mark(p, 2, s);
-            const bool four = (p->flags & ECL_SCC_FOUR_SIG) != 0;     // (iteration 1 keeps every edge)
-            if (iter == 1) r = trim ? remove_and_compact<true, true, false>(p, g, cin, cout, ob, labels, P, s)
-                                    : remove_and_compact<true, false, false>(p, g, cin, cout, ob, labels, P, s);
-            else if (four) r = trim ? remove_and_compact<false, true, true>(p, g, cin, cout, ob, labels, P, s)
-                                    : remove_and_compact<false, false, true>(p, g, cin, cout, ob, labels, P, s);
-            else r = trim ? remove_and_compact<false, true, false>(p, g, cin, cout, ob, labels, P, s)
-                          : remove_and_compact<false, false, false>(p, g, cin, cout, ob, labels, P, s);
+            r = compaction(p, 0, iter, g, cin, cout, ob, labels, P, s);
+            if (!r) r = compaction(p, 1, iter, g, cin, cout, ob, labels, P, s);
             if (r) return r;
             stage_mark(p, 3, s);
             CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
@@ -766,6 +817,342 @@ int run_batched(Plan* p, int32_t G, const int32_t* n, const int64_t* nnz, const 
     CK(cudaStreamSynchronize(s));
     if (st) st->kernel_launches = p->launches;
     (void)l0;
+    return ECL_SCC_OK;
+}
+
+// --------------------------------------------------------------------------- exchanges
+int Exchange::allreduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) {
+    cudaEvent_t a = nullptr, b = nullptr;
+    if (ev) {
+        if ((size_t)(2 * used + 2) > ev->size()) {
+            for (int k = 0; k < 2; k++) {
+                cudaEvent_t e;
+                CK(cudaEventCreate(&e));
+                ev->push_back(e);
+            }
+        }
+        a = (*ev)[2 * used];
+        b = (*ev)[2 * used + 1];
+        used++;
+        CK(cudaEventRecord(a, s));
+    }
+    if (int r = reduce(bufs, count, op, s)) return r;
+    if (ev) CK(cudaEventRecord(b, s));
+    bytes += 4 * count;
+    return ECL_SCC_OK;
+}
+double Exchange::ms() const {
+    double t = 0;
+    for (int k = 0; ev && k < used; k++) {
+        float x = 0.f;
+        if (cudaEventElapsedTime(&x, (*ev)[2 * k], (*ev)[2 * k + 1]) == cudaSuccess) t += x;
+        else cudaGetLastError();
+    }
+    return t;
+}
+
+// --------------------------------------------------------------------------- partitioned (halo) mode
+HaloRank::~HaloRank() {
+    plan_free(&p);
+    cudaFree(lrp); cudaFree(lci); cudaFree(l2g); cudaFree(gmark); cudaFree(gidx); cudaFree(lab);
+    cudaFree(hdeg); cudaFree(words);
+    if (!hbuf_external) cudaFree(hbuf);
+}
+
+// workspace of one rank: rows [rb, re) of an n-vertex graph with at most m_cap local edges
+// (the local graph has at most nloc + min(m_cap, n) vertices)
+int halo_rank_alloc(HaloRank* R, int32_t n, int32_t rb, int32_t re, int64_t m_cap, uint32_t flags) {
+    R->n = n; R->rb = rb; R->re = re; R->nloc = re - rb; R->m_cap = m_cap;
+    const int64_t nl_max = std::min<int64_t>((int64_t)R->nloc + m_cap, n);
+    if (flags & (ECL_SCC_TRIM2 | ECL_SCC_FOUR_SIG))
+        return fail(ECL_SCC_EUNSUPPORTED, "partitioned mode: Trim-2 and the 4-signature variant are single-GPU only");
+    R->p.flags = flags | ECL_SCC_NO_REORDER;       // the local -> global map is the storage map
+    if (int r = plan_alloc(&R->p, (int32_t)std::max<int64_t>(nl_max, 1), std::max<int64_t>(m_cap, 1))) return r;
+    const size_t n1 = (size_t)n + 1, nl1 = (size_t)nl_max + 1;
+    cudaError_t e = cudaSuccess;
+    auto A = [&](int32_t** ptr, size_t count) { if (e == cudaSuccess) e = cudaMalloc((void**)ptr, count * 4); };
+    A(&R->p.hpos[0], nl1);
+    A(&R->p.hpos[1], nl1);
+    A(&R->lrp, nl1 + 1);
+    A(&R->lci, (size_t)std::max<int64_t>(m_cap, 1));
+    A(&R->l2g, nl1);
+    A(&R->gmark, n1);
+    A(&R->gidx, n1);
+    A(&R->lab, n1);
+    A(&R->words, 8);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ECL_SCC_ENOMEM, "partition workspace: %s", cudaGetErrorString(e));
+    }
+    R->p.lab_lo = rb;
+    R->p.lab_hi = re;
+    return ECL_SCC_OK;
+}
+
+// Rank r's local graph from its rows: ghosts, local -> global map, local CSR (halo.cuh)
+static int halo_ingest(HaloRank& R, uint32_t flags, cudaStream_t s) {
+    Plan* p = &R.p;
+    const int32_t n = R.n;
+    const unsigned gs = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
+    CK(cudaMemsetAsync(R.gmark, 0, sizeof(int32_t) * (size_t)n, s));
+    if (R.m) { p->launches++; k_halo_mark_ghosts<<<std::min<unsigned>(grid_for(R.m, TPB), 148 * 16), TPB, 0, s>>>(R.m, R.ci, R.rb, R.re, R.gmark); }
+    if (int r = scan_excl<I1>(p, (const I1*)R.gmark, n, (I1*)R.gidx, (I1*)&p->dc->grand1, p->bsum, 0, s)) return r;
+    int ng = 0;
+    CK(cudaMemcpyAsync(&ng, &p->dc->grand1, sizeof(int), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    R.ng = ng;
+    if ((int64_t)R.nloc + ng > p->n_cap) return fail(ECL_SCC_ECUDA, "internal: local graph exceeds its plan");
+    p->launches += 2;
+    k_halo_l2g<<<gs, TPB, 0, s>>>(n, R.rb, R.re, R.gmark, R.gidx, R.l2g);
+    k_halo_local_csr<<<std::min<unsigned>(grid_for(std::max<int64_t>(R.m, R.nloc + ng + 1), TPB), 148 * 16), TPB, 0, s>>>(
+        R.nloc, ng, R.m, R.rp, R.ci, R.rb, R.re, R.gidx, R.lrp, R.lci);
+    CK(cudaGetLastError());
+    (void)flags;
+    return ECL_SCC_OK;
+}
+
+// The partitioned driver over this process's ranks R (1 with NCCL, P when emulated): the
+// outer loop of run_graph per rank, in lockstep, with the halo exchanges (halo.cuh) at the
+// points where the ranks must agree.
+int run_halo(std::vector<HaloRank*>& R, Exchange& X, int32_t n, uint32_t flags, int32_t* labels, cudaStream_t s,
+             ecl_scc_stats* st) {
+    const int P = (int)R.size();
+    if (st) memset(st, 0, sizeof(*st));
+    const Prio Pr = make_prio((uint32_t)n, (flags & ECL_SCC_IDENTITY_IDS) != 0);
+    const bool trim = !(flags & ECL_SCC_NO_TRIM);
+    std::vector<int32_t*> bufs(P);
+    auto each = [&](auto f) -> int {
+        for (int r = 0; r < P; r++)
+            if (int e = f(*R[r], r)) return e;
+        return ECL_SCC_OK;
+    };
+    auto word_reduce = [&](int k, int op) -> int {   // all-reduce of device word k of every rank
+        for (int r = 0; r < P; r++) bufs[r] = R[r]->words + k;
+        return X.allreduce(bufs, 1, op, s);
+    };
+    auto read_word = [&](int k, int* out) -> int {
+        CK(cudaMemcpyAsync(out, R[0]->words + k, sizeof(int), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        return ECL_SCC_OK;
+    };
+    int r = each([&](HaloRank& Q, int) -> int {
+        Q.p.launches = 0;
+        CK(cudaMemsetAsync(Q.words, 0, 8 * sizeof(int32_t), s));
+        if (!(flags & ECL_SCC_NO_VALIDATE) && Q.nloc > 0) {
+            Q.p.launches++;
+            part::k_validate_part<<<std::min<unsigned>(grid_for(std::max<int64_t>(Q.nloc, Q.m), TPB), 148 * 16), TPB, 0, s>>>(
+                Q.nloc, Q.m, Q.rp, Q.ci, n, Q.words + 2);
+        }
+        return ECL_SCC_OK;
+    });
+    if (r) return r;
+    if ((r = word_reduce(2, 0))) return r;         // every rank learns of an invalid rank
+    int err = 0;
+    if ((r = read_word(2, &err))) return r;
+    if (err) return fail(ECL_SCC_ERANGE, "partitioned: invalid local CSR on some rank");
+    // ---- local graphs; the halo H = vertices that are a ghost on some rank
+    if ((r = each([&](HaloRank& Q, int) { return halo_ingest(Q, flags, s); }))) return r;
+    for (int q = 0; q < P; q++) bufs[q] = R[q]->gmark;
+    if ((r = X.allreduce(bufs, n, 0, s))) return r;   // (ingest only: membership of all n IDs)
+    int64_t H = 0;
+    r = each([&](HaloRank& Q, int) -> int {
+        Plan* p = &Q.p;
+        const unsigned gs = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
+        p->launches++; k_nonzero<<<gs, TPB, 0, s>>>(n, Q.gmark, Q.lab);          // (lab: scratch here)
+        if (int e = scan_excl<I1>(p, (const I1*)Q.lab, n, (I1*)Q.gidx, (I1*)&p->dc->grand1, p->bsum, 0, s)) return e;
+        int h = 0;
+        CK(cudaMemcpyAsync(&h, &p->dc->grand1, sizeof(int), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        H = h;
+        const int32_t nl = Q.nloc + Q.ng;
+        p->launches++; k_halo_hpos<<<std::min<unsigned>(grid_for(std::max(nl, 1), TPB), 148 * 16), TPB, 0, s>>>(nl, Q.l2g, Q.gmark, Q.gidx, p->hpos[0]);
+        p->launches++; k_fill<<<gs, TPB, 0, s>>>(n, Q.lab, INT32_MIN);
+        CK(cudaGetLastError());
+        return ECL_SCC_OK;
+    });
+    if (r) return r;
+    if (R[0]->hcap < H || !R[0]->hbuf) {           // (grows once per plan; symmetric in NCCL mode)
+        if ((r = X.halo_buffers(R, std::max<int64_t>(H, 1), s))) return r;
+        for (HaloRank* Q : R) {
+            cudaFree(Q->hdeg);
+            if (cudaMalloc((void**)&Q->hdeg, sizeof(int32_t) * 2 * (size_t)std::max<int64_t>(H, 1)) != cudaSuccess) {
+                cudaGetLastError();
+                return fail(ECL_SCC_ENOMEM, "halo degree buffer");
+            }
+            Q->hcap = std::max<int64_t>(H, 1);
+        }
+    }
+    const bool fused = R[0]->push.np > 0 || R[0]->push.mc;
+    // ---- the single-GPU ingest of every local graph (CSC of the local rows)
+    r = each([&](HaloRank& Q, int) -> int {
+        Plan* p = &Q.p;
+        Q.H = H;
+        const int32_t nl = Q.nloc + Q.ng;
+        if (int e = build_csc(p, nl, Q.m, Q.lrp, Q.lci, s)) return e;
+        unsigned long long loc = 0;
+        CK(cudaMemcpyAsync(&loc, &p->dc->local_e, sizeof(loc), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        p->low_locality = (double)loc < LOCAL_FP_LOCALITY * (double)std::max<int64_t>(Q.m, 1);
+        p->orig_cur = Q.l2g;                        // local -> global: priorities and labels
+        Q.g = WGraph{nullptr, Q.lrp, Q.lci, p->iptr[0], p->iadj[0], nl};
+        Q.g.hpos = p->hpos[0];
+        Q.ob = 1;
+        return ECL_SCC_OK;
+    });
+    if (r) return r;
+    int iters = 0;
+    int64_t passes_total = 0;
+    for (int iter = 1;; iter++) {
+        if (iter > n + 2) return fail(ECL_SCC_ECUDA, "internal: partitioned outer loop exceeded n+2 iterations");
+        // ---- Phase 3 (keep), the halo's kept degrees summed over the ranks, trim + compaction
+        const int32_t* cin0 = nullptr;
+        r = each([&](HaloRank& Q, int) {
+            const int32_t* ci_ = iter == 1 ? cin0 : Q.p.cin[Q.ob ^ 1];
+            const int32_t* co_ = iter == 1 ? cin0 : Q.p.cout[Q.ob ^ 1];
+            return compaction(&Q.p, 0, iter, Q.g, ci_, co_, Q.ob, Q.lab, Pr, s);
+        });
+        if (r) return r;
+        if (trim) {
+            r = each([&](HaloRank& Q, int q) -> int {
+                CK(cudaMemsetAsync(Q.hdeg, 0, sizeof(int32_t) * 2 * (size_t)H, s));
+                if (Q.g.na) { Q.p.launches++; k_halo_deg_pack<<<std::min<unsigned>(grid_for(Q.g.na, TPB), 148 * 8), TPB, 0, s>>>(Q.g.na, Q.g.hpos, Q.p.kio, Q.hdeg); }
+                bufs[q] = Q.hdeg;
+                return ECL_SCC_OK;
+            });
+            if (r) return r;
+            if ((r = X.allreduce(bufs, 2 * H, 1, s))) return r;
+            r = each([&](HaloRank& Q, int) -> int {
+                if (Q.g.na) { Q.p.launches++; k_halo_deg_apply<<<std::min<unsigned>(grid_for(Q.g.na, TPB), 148 * 8), TPB, 0, s>>>(Q.g.na, Q.g.hpos, Q.hdeg, Q.p.kio); }
+                return ECL_SCC_OK;
+            });
+            if (r) return r;
+        }
+        int64_t live = 0;
+        r = each([&](HaloRank& Q, int) -> int {
+            Plan* p = &Q.p;
+            const int32_t* ci_ = iter == 1 ? nullptr : p->cin[Q.ob ^ 1];
+            const int32_t* co_ = iter == 1 ? nullptr : p->cout[Q.ob ^ 1];
+            if (int e = compaction(p, 1, iter, Q.g, ci_, co_, Q.ob, Q.lab, Pr, s)) return e;
+            CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));
+            if (p->hc->err == 3) return fail(ECL_SCC_ECUDA, "internal: asynchronous Phase 2 stalled (watchdog)");
+            const int4 t = p->hc->totals;
+            if (t.y != t.z) return fail(ECL_SCC_ECUDA, "internal: CSR/CSC survivor mismatch %d vs %d", t.y, t.z);
+            p->nchunks_cur = p->hc->nchunks;
+            Q.g = WGraph{p->act[Q.ob], p->optr[Q.ob], p->oadj[Q.ob], p->iptr[Q.ob], p->iadj[Q.ob], t.x};
+            Q.g.hpos = p->hpos[Q.ob];
+            live += t.y;
+            // the exchange buffer restarts with every Phase 2 (before the barrier below, so no
+            // rank can push into a buffer that is still to be cleared)
+            CK(cudaMemsetAsync(Q.hbuf, 0, sizeof(int32_t) * 2 * (size_t)H, s));
+            const int ty = t.y;
+            CK(cudaMemcpyAsync(Q.words + 1, &ty, sizeof(int), cudaMemcpyHostToDevice, s));
+            return ECL_SCC_OK;
+        });
+        if (r) return r;
+        if ((r = word_reduce(1, 1))) return r;      // live edges of all ranks (termination)
+        int glive = 0;
+        if ((r = read_word(1, &glive))) return r;
+        if (st && iter - 1 < ECL_SCC_TRACE_MAX) st->edges_in[iter - 1] = glive;
+        if (glive == 0) {
+            // every remaining vertex is unfinished and edgeless on every rank: a singleton
+            r = each([&](HaloRank& Q, int) -> int {
+                if (Q.g.na) { Q.p.launches++; k_halo_final<<<std::min<unsigned>(grid_for(Q.g.na, TPB), 148 * 8), TPB, 0, s>>>(Q.g.na, Q.g.act, Q.l2g, Q.rb, Q.re, Q.lab); }
+                return ECL_SCC_OK;
+            });
+            if (r) return r;
+            if (st && iter - 1 < ECL_SCC_TRACE_MAX) st->edges_in[iter - 1] = 0;
+            break;
+        }
+        if (st && iter >= 2 && iter - 2 < ECL_SCC_TRACE_MAX) st->edges_kept[iter - 2] = glive;
+        // ---- Phase 2: local fixed points; raised halo copies pushed to every rank; fold in
+        int64_t rounds = 0;
+        for (int round = 0;; round++) {
+            r = each([&](HaloRank& Q, int) -> int {
+                Plan* p = &Q.p;
+                HaloPush push = Q.push;
+                push.hpos = Q.g.hpos;
+                if (!fused) {                         // NCCL all-reduce exchange: own buffer only
+                    push.np = 1;
+                    push.peer[0] = Q.hbuf;
+                    push.mc = nullptr;
+                    push.sys = 0;
+                }
+                int64_t passes = 0;
+                if (Q.g.na == 0) return ECL_SCC_OK;
+                if (int e = propagate(p, Q.g, p->cin[Q.ob], p->cout[Q.ob], p->nchunks_cur, s, &passes, false, &push,
+                                      round > 0))
+                    return e;
+                if (!fused && pack_path(p, p->nchunks_cur) && !(flags & ECL_SCC_NO_ASYNC)) {
+                    // (asynchronous kernel pushed its raises into the own buffer already)
+                }
+                return ECL_SCC_OK;
+            });
+            if (r) return r;
+            rounds++;
+            if (!fused) {
+                for (int q = 0; q < P; q++) bufs[q] = R[q]->hbuf;
+                if ((r = X.allreduce(bufs, 2 * H, 0, s))) return r;
+            } else if ((r = word_reduce(0, 0))) {     // barrier: every rank's pushes have landed
+                return r;
+            }
+            r = each([&](HaloRank& Q, int) -> int {
+                Plan* p = &Q.p;
+                CK(cudaMemsetAsync(Q.words, 0, sizeof(int32_t), s));
+                if (Q.g.na == 0) return ECL_SCC_OK;
+                const bool async = pack_path(p, p->nchunks_cur) && !(flags & ECL_SCC_NO_ASYNC);
+                const bool dirty = !async && p->nchunks_cur == 0 && !(flags & (ECL_SCC_SYNC_PASSES | ECL_SCC_NO_DIRTY));
+                p->launches++;
+                k_halo_apply<<<std::min<unsigned>(grid_for(Q.g.na, TPB), 148 * 8), TPB, 0, s>>>(
+                    Q.g, Q.hbuf, p->cin[Q.ob], p->cout[Q.ob], async ? p->aq_state : nullptr,
+                    async ? p->aq_seen : nullptr, async ? p->aq_ctr + AQ_PEND : nullptr, dirty ? p->dirty : nullptr, TILE,
+                    Q.words);
+                CK(cudaGetLastError());
+                return ECL_SCC_OK;
+            });
+            if (r) return r;
+            if ((r = word_reduce(0, 0))) return r;  // did any rank take a larger copy?
+            int inj = 0;
+            if ((r = read_word(0, &inj))) return r;
+            if (!inj) break;
+            if (round > 4 * n + 64) return fail(ECL_SCC_ECUDA, "internal: halo exchange did not converge");
+        }
+        iters = iter;
+        passes_total += rounds;
+        if (st && iter - 1 < ECL_SCC_TRACE_MAX) st->passes_iter[iter - 1] = rounds;
+        for (HaloRank* Q : R) Q->ob ^= 1;
+    }
+    // ---- labels: the owners' entries, combined; priorities -> max vertex IDs (k_relabel_*)
+    for (int q = 0; q < P; q++) bufs[q] = R[q]->lab;
+    if ((r = X.allreduce(bufs, n, 0, s))) return r;
+    HaloRank& Q = *R[0];
+    const unsigned gr = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
+    if (!Pr.ids) {
+        Q.p.launches += 3;
+        k_relabel_rep<<<gr, TPB, 0, s>>>(n, Q.lab, Q.gidx, Pr);
+        k_relabel_max<<<gr, TPB, 0, s>>>(n, Q.lab, Q.gidx, Pr);
+        k_relabel_apply<<<gr, TPB, 0, s>>>(n, Q.lab, Q.gidx);
+    }
+    CK(cudaMemcpyAsync(labels, Q.lab, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));
+    CK(cudaGetLastError());
+    CK(cudaStreamSynchronize(s));
+    if (st) {
+        int64_t launches = 0, vv = 0, ve = 0;
+        for (HaloRank* q : R) {
+            launches += q->p.launches;
+            CK(cudaMemcpy(q->p.hc, q->p.dc, sizeof(DevCounters), cudaMemcpyDeviceToHost));
+            vv += (int64_t)q->p.hc->visit_v;
+            ve += (int64_t)q->p.hc->visit_e;
+        }
+        st->iterations = iters;
+        st->trace_len = std::min(iters, ECL_SCC_TRACE_MAX);
+        st->passes = passes_total;
+        st->kernel_launches = launches;
+        st->prop_bytes = 20 * vv + 12 * ve;
+        st->ms_comm = X.ms();
+        st->comm_bytes = X.bytes;
+        st->exchanges = X.used;
+    }
     return ECL_SCC_OK;
 }
 

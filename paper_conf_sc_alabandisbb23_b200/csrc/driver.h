@@ -3,8 +3,11 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <vector>
+
 #include "../../include/ecl_scc.h"
 #include "common.cuh"
+#include "halo.cuh"
 
 namespace eclscc {
 
@@ -20,6 +23,9 @@ struct Plan {
     int32_t *oadj[2], *iadj[2];          // CSR / CSC adjacency
     int32_t *min_in[2], *min_out[2];     // ECL_SCC_FOUR_SIG: minimum signatures (mirrored), per buffer
     int32_t* t2;                         // ECL_SCC_TRIM2: Trim-2 partner per local vertex (-1: none)
+    int32_t* hpos[2];                    // partitioned mode: halo position per local vertex, per buffer
+    int32_t lab_lo, lab_hi;              // label ownership: labels[v] written only for lab_lo <= v < lab_hi
+    WGraph gk;                           // the graph of the compaction in progress (keep -> finish)
     int32_t *kin, *kout;                 // two n+1 int views (ingest histogram / cursor, relabel, levels)
     int2* kio;                           // the same memory as interleaved kept degrees {in, out} (compaction)
     int32_t* newidx;                     // old local -> new local (-1: leaves)
@@ -67,6 +73,50 @@ struct Plan {
     bool ev_ok;
     bool low_locality;                   // fewer than 25% of the input edges inside 2048-ID ranges
 };
+
+// all-reduce over the ranks of this process (1 with NCCL, P when emulated).  Every exchange
+// is bracketed by CUDA events on the call's stream (stats->ms_comm: the communication
+// share); the event pool is owned by the caller (a plan) and reused.
+struct HaloRank;
+struct Exchange {
+    std::vector<cudaEvent_t>* ev = nullptr;   // pool of event pairs
+    int used = 0;                             // pairs recorded by the current call
+    int64_t bytes = 0;                        // bytes this rank contributed
+    virtual ~Exchange() {}
+    // op 0 = MAX, 1 = SUM; bufs[r] = rank r's buffer of `count` int32
+    virtual int reduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) = 0;
+    // partitioned (halo) mode: give every rank an exchange buffer of 2*entries int32 and the
+    // push targets of the propagation kernel (R[r]->push)
+    virtual int halo_buffers(std::vector<HaloRank*>& R, int64_t entries, cudaStream_t s) = 0;
+    int allreduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s);
+    double ms() const;                        // after a stream synchronisation
+};
+
+// One rank of the edge-partitioned mode (halo.cuh): its rows, its local graph and the
+// single-GPU workspace that runs it.
+struct HaloRank {
+    Plan p;                                   // workspace of the local graph
+    int32_t n = 0, rb = 0, re = 0, nloc = 0, ng = 0;
+    int64_t m = 0, m_cap = 0;
+    const int32_t *rp = nullptr, *ci = nullptr;   // the caller's rows (global destination IDs)
+    int32_t *lrp = nullptr, *lci = nullptr;   // local CSR (owned rows, then the ghosts' empty rows)
+    int32_t* l2g = nullptr;                   // local -> global ID
+    int32_t *gmark = nullptr, *gidx = nullptr;    // [n] ghost marks (then halo membership) / scans
+    int32_t* lab = nullptr;                   // [n] encoded labels of the owned vertices
+    int32_t* hbuf = nullptr;                  // [2*hcap] signature exchange buffer (in, out per entry)
+    int32_t* hdeg = nullptr;                  // [2*hcap] kept-degree exchange buffer
+    int64_t hcap = 0, H = 0;                  // capacity / current size of the halo
+    bool hbuf_external = false;               // hbuf owned by the exchange (symmetric memory)
+    int32_t* words = nullptr;                 // device: [0] injected, [1] live edges, [2] err
+    HaloPush push{};                          // where k_prop_async pushes raised halo copies
+    // loop state
+    WGraph g{};
+    int ob = 1;
+    ~HaloRank();
+};
+int halo_rank_alloc(HaloRank* R, int32_t n, int32_t rb, int32_t re, int64_t m_cap, uint32_t flags);
+int run_halo(std::vector<HaloRank*>& R, Exchange& X, int32_t n, uint32_t flags, int32_t* labels, cudaStream_t s,
+             ecl_scc_stats* st);
 
 int fail(int status, const char* fmt, ...);
 void clear_err();

@@ -431,7 +431,10 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
         }
     }
     if (r.valid) cnt[i] = make_int2(nout, nin);
-    const int alive = (nout + nin) > 0;
+    int alive = (nout + nin) > 0;
+    // partitioned mode: an unfinished halo vertex that is not trimmed (global degrees) stays,
+    // even without local edges -- its edges may live on other ranks (halo.cuh)
+    if (g.hpos && !alive && r.live && g.hpos[i] >= 0 && !(TRIM && trimmed(kio, (int)i))) alive = 1;
     const int kept = r.valid ? kio[i].y : 0;            // kept (pre-trim) out-degree, chunks included
     const int sa = warp_sum(alive), so = warp_sum(nout), si = warp_sum(nin), sk = warp_sum(kept);
     if (lane == 0) wsum[i >> 5] = make_int4(sa, so, si, sk);
@@ -505,7 +508,9 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
                               int32_t* __restrict__ optr2, int32_t* __restrict__ iptr2, int32_t* __restrict__ labels,
                               Chunk* __restrict__ chunks, int* __restrict__ nchunks, int chunk_cap, Prio P,
                               const int32_t* __restrict__ orig, PackOut pk, int32_t* __restrict__ min_in2,
-                              int32_t* __restrict__ min_out2, const int32_t* __restrict__ t2) {
+                              int32_t* __restrict__ min_out2, const int32_t* __restrict__ t2,
+                              const int2* __restrict__ kio, int trim, int32_t* __restrict__ hpos2, int32_t lab_lo,
+                              int32_t lab_hi) {
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i == 0) {
@@ -523,7 +528,9 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
     }
     const bool valid = i < g.na;
     int2 c = valid ? cnt[i] : make_int2(0, 0);
-    const int alive = (c.x + c.y) > 0;
+    int alive = (c.x + c.y) > 0;
+    if (g.hpos && valid && !alive && g.hpos[i] >= 0 && (FIRST || cin[i] != cout[i]) && !(trim && trimmed(kio, (int)i)))
+        alive = 1;                                     // (the same rule as k_compact_count)
     const int4 base = wscan[i >> 5];
     const int j = warp_incl_scan(alive, lane) - alive + base.x;
     const int po = warp_incl_scan(c.x, lane) - c.x + base.y;
@@ -538,6 +545,7 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
         const int pv = (int)prio_of(P, (uint32_t)ov);
         cin2[j] = pv;       // Phase 1: v_in <- v_id, v_out <- v_id for the unfinished
         cout2[j] = pv;
+        if (hpos2) hpos2[j] = g.hpos[i];
         if (min_in2) {      // the minimum pair restarts from the vertex too
             min_in2[j] = mirror_prio(pv);
             min_out2[j] = mirror_prio(pv);
@@ -566,7 +574,7 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
             const int ow = orig ? orig[vw] : vw;
             lab = P.ids ? max(ov, ow) : -((int)max(prio_of(P, (uint32_t)ov), prio_of(P, (uint32_t)ow)) + 1);
         }
-        labels[ov] = lab;
+        if (ov >= lab_lo && ov < lab_hi) labels[ov] = lab;    // partitioned: the owner writes
     }
 }
 

@@ -1,27 +1,32 @@
-// multi.cu -- multi-GPU layer: one large graph edge-partitioned by source rows (SPMD, one
-// process per GPU), signatures combined with NCCL all-reduce(MAX) over NVLink/NVSwitch.
+// multi.cu -- multi-GPU layer: one large graph edge-partitioned by source rows,
+// SPMD, one process per GPU.  The algorithm is run_halo (driver.cu, halo.cuh): every rank runs
+// the single-GPU machinery on its local graph and the ranks exchange only the signatures of
+// the halo (vertices held by more than one rank).
 //
-// Per outer iteration (same rule R2 and trace as the single-GPU path):
-//   keep (Phase 3) on own rows and columns   -> kept degrees
-//   all-reduce SUM of kept degrees (trim needs global degrees)
-//   Trim-1 on own edges; all-reduce SUM of live edges   (termination, reading 2)
-//   Phase 1 reset of the unfinished on the replica
-//   Phase 2: repeat { local fixed point on own edges; all-reduce MAX of [in|out|changed] }
-//            until no rank changed anything (a consistent global fixed point)
-// The same driver runs P emulated ranks on one device (the all-reduce is an element-wise
-// reduction over the P replicas), which is how the path is tested with one GPU.
+// Exchanges (Exchange, driver.h):
+//   * NcclExchange -- degree / count / label all-reduces with NCCL; the signature exchange of
+//     Phase 2 is FUSED into the propagation kernel (f1): the halo buffer is NCCL symmetric
+//     memory (ncclMemAlloc + ncclCommWindowRegister), and k_prop_async pushes every raised
+//     halo copy straight into every peer's buffer -- one multimem.red.max through the
+//     NVSwitch when the communicator has NVLS multicast (ncclGetLsaMultimemPointer), else
+//     remote atomicMax over NVLink peer pointers (ncclGetLsaPointer); a one-word all-reduce
+//     is the barrier.  Without the device API (or with ECL_SCC_HALO_ALLREDUCE) the halo
+//     buffer is combined by ncclAllReduce(MAX) instead (the baseline).
+//   * EmulatedExchange -- P ranks in one process on one device (tests): reductions over the
+//     P buffers, pushes into the P buffers of the same device.
 #include <cuda_runtime.h>
 #include <nccl.h>
+#include <nccl_device.h>
 #include <string.h>
 
 #include <algorithm>
 #include <memory>
+#include <new>
 #include <vector>
 
 #include "driver.h"
 #include "kernels.cuh"
 #include "partition.cuh"
-#include "scan.cuh"
 
 namespace eclscc {
 
@@ -43,72 +48,11 @@ static inline unsigned gridn(int64_t work, int t = 256) {
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(g, 0x7FFFFFFF));
 }
 
-// One rank's share of the graph (device memory).
-struct PRank {
-    int32_t rb = 0, re = 0, nloc = 0;
-    int64_t m = 0;
-    const int32_t *rp = nullptr, *ci = nullptr;  // caller's local CSR (rows rb..re-1)
-    int32_t *wci = nullptr, *odeg = nullptr;     // working rows (compacted in place)
-    int32_t *cp = nullptr, *cr = nullptr, *ideg = nullptr;   // CSC of own edges, n columns
-    int32_t* sig = nullptr;                      // [in(n) | out(n) | changed(1)] replica
-    int32_t* kdeg = nullptr;                     // [kin(n) | kout(n)]
-    int32_t* cnt = nullptr;                      // [live edges (int32 for the SUM), err, ring(RING), touched]
-    unsigned long long* live = nullptr;
-    void* bsum = nullptr;
-    int32_t* grand = nullptr;
-    ~PRank() {
-        cudaFree(wci); cudaFree(odeg); cudaFree(cp); cudaFree(cr); cudaFree(ideg);
-        cudaFree(sig); cudaFree(kdeg); cudaFree(cnt); cudaFree(live); cudaFree(bsum); cudaFree(grand);
-    }
-    int* ring() const { return cnt + 2; }
-    int* touched() const { return cnt + 2 + RING; }
-};
-
-// all-reduce over the ranks of this process (1 with NCCL, P when emulated).  Every exchange
-// is bracketed by CUDA events on the call's stream (stats->ms_comm: the communication
-// share); the event pool is owned by the caller (a plan) and reused.
-struct Exchange {
-    std::vector<cudaEvent_t>* ev = nullptr;   // pool of event pairs
-    int used = 0;                             // pairs recorded by the current call
-    int64_t bytes = 0;                        // bytes this rank contributed
-    virtual ~Exchange() {}
-    // op 0 = MAX, 1 = SUM; bufs[r] = rank r's buffer of `count` int32
-    virtual int reduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) = 0;
-    int allreduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) {
-        cudaEvent_t a = nullptr, b = nullptr;
-        if (ev) {
-            if ((size_t)(2 * used + 2) > ev->size()) {
-                for (int k = 0; k < 2; k++) {
-                    cudaEvent_t e;
-                    CKM(cudaEventCreate(&e));
-                    ev->push_back(e);
-                }
-            }
-            a = (*ev)[2 * used];
-            b = (*ev)[2 * used + 1];
-            used++;
-            CKM(cudaEventRecord(a, s));
-        }
-        if (int r = reduce(bufs, count, op, s)) return r;
-        if (ev) CKM(cudaEventRecord(b, s));
-        bytes += 4 * count;
-        return ECL_SCC_OK;
-    }
-    double ms() const {                       // after a stream synchronisation
-        double t = 0;
-        for (int k = 0; ev && k < used; k++) {
-            float x = 0.f;
-            if (cudaEventElapsedTime(&x, (*ev)[2 * k], (*ev)[2 * k + 1]) == cudaSuccess) t += x;
-            else cudaGetLastError();
-        }
-        return t;
-    }
-};
-
 struct EmulatedExchange : Exchange {
     int32_t** dptrs = nullptr;
     int P = 0;
-    explicit EmulatedExchange(int p) : P(p) {}
+    bool fused = true;                    // pushes into the P buffers (else: all-reduce exchange)
+    EmulatedExchange(int p, bool f) : P(p), fused(f) {}
     ~EmulatedExchange() { cudaFree(dptrs); }
     int reduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) override {
         if (P == 1) return ECL_SCC_OK;
@@ -118,222 +62,134 @@ struct EmulatedExchange : Exchange {
         CKM(cudaGetLastError());
         return ECL_SCC_OK;
     }
-};
-
-struct NcclExchange : Exchange {
-    ncclComm_t comm;
-    explicit NcclExchange(ncclComm_t c) : comm(c) {}
-    int reduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) override {
-        CKN(ncclAllReduce(bufs[0], bufs[0], (size_t)count, ncclInt32, op == 0 ? ncclMax : ncclSum, comm, s));
+    // every rank pushes into all P buffers (same device: plain atomics)
+    int halo_buffers(std::vector<HaloRank*>& R, int64_t entries, cudaStream_t) override {
+        for (HaloRank* Q : R) {
+            if (!Q->hbuf_external) cudaFree(Q->hbuf);
+            Q->hbuf = nullptr;
+            Q->hbuf_external = false;
+            if (cudaMalloc((void**)&Q->hbuf, sizeof(int32_t) * 2 * (size_t)entries) != cudaSuccess) {
+                cudaGetLastError();
+                return fail(ECL_SCC_ENOMEM, "halo exchange buffer");
+            }
+        }
+        for (HaloRank* Q : R) {
+            Q->push = HaloPush{};
+            if (!fused || P > HALO_MAX_PEERS) continue;   // (then: the all-reduce exchange)
+            Q->push.np = P;
+            for (int k = 0; k < P; k++) Q->push.peer[k] = R[k]->hbuf;
+        }
         return ECL_SCC_OK;
     }
 };
 
-static int rank_alloc(PRank& R, int32_t n) {
-    const size_t m = (size_t)std::max<int64_t>(R.m, 1), n1 = (size_t)n + 1;
-    cudaError_t e = cudaSuccess;
-    e = e ? e : cudaMalloc((void**)&R.wci, m * 4);
-    e = e ? e : cudaMalloc((void**)&R.odeg, (size_t)std::max(R.nloc, 1) * 4);
-    e = e ? e : cudaMalloc((void**)&R.cp, n1 * 4);
-    e = e ? e : cudaMalloc((void**)&R.cr, m * 4);
-    e = e ? e : cudaMalloc((void**)&R.ideg, n1 * 4);
-    e = e ? e : cudaMalloc((void**)&R.sig, (2 * n1 + 1) * 4);
-    e = e ? e : cudaMalloc((void**)&R.kdeg, 2 * n1 * 4);
-    e = e ? e : cudaMalloc((void**)&R.cnt, (3 + RING) * 4);
-    e = e ? e : cudaMalloc((void**)&R.live, 8);
-    e = e ? e : cudaMalloc((void**)&R.bsum, ((n1 + SCAN_TILE - 1) / SCAN_TILE + 1) * sizeof(int4));
-    e = e ? e : cudaMalloc((void**)&R.grand, 16);
-    if (e != cudaSuccess) {
-        cudaGetLastError();
-        return fail(ECL_SCC_ENOMEM, "partition workspace: %s", cudaGetErrorString(e));
-    }
-    return ECL_SCC_OK;
-}
-
-__global__ void k_copy_flag(const int* __restrict__ touched, int32_t* __restrict__ dst, int err) {
-    *dst = err ? err : *touched;
-}
-__global__ void k_live_to_i32(const unsigned long long* __restrict__ live, int32_t* __restrict__ dst) {
-    *dst = (int32_t)*live;
-}
-
-// The partitioned driver over this process's ranks R (1 with NCCL, P when emulated).
-// Every rank's graph pointers are device pointers on the current device.
-static int run_partitioned(std::vector<PRank*>& R, Exchange& X, int32_t n, uint32_t flags, int32_t* labels,
-                           cudaStream_t s, ecl_scc_stats* st) {
-    const int P = (int)R.size();
-    if (st) memset(st, 0, sizeof(*st));
-    const Prio Pr = make_prio((uint32_t)n, (flags & ECL_SCC_IDENTITY_IDS) != 0);
-    const bool trim = !(flags & ECL_SCC_NO_TRIM);
-    std::vector<int32_t*> sigs(P), kdegs(P), cnts(P);
-    int32_t hbuf[4];
-    int64_t launches = 0;
-    // ---- ingest: validation, working rows, CSC of own edges
-    for (int r = 0; r < P; r++) {
-        PRank& Q = *R[r];
-        sigs[r] = Q.sig; kdegs[r] = Q.kdeg; cnts[r] = Q.cnt;
-        CKM(cudaMemsetAsync(Q.cnt, 0, (3 + RING) * 4, s));
-        if (!(flags & ECL_SCC_NO_VALIDATE) && Q.nloc > 0) {
-            part::k_validate_part<<<std::min<unsigned>(gridn(std::max<int64_t>(Q.nloc, Q.m)), 148 * 16), 256, 0, s>>>(
-                Q.nloc, Q.m, Q.rp, Q.ci, n, Q.cnt + 1);
-            launches++;
-        }
-    }
-    {   // every rank learns whether any rank's input is invalid, so all return together
-        // instead of leaving the others blocked in the next collective
-        std::vector<int32_t*> errs(P);
-        for (int r = 0; r < P; r++) errs[r] = R[r]->cnt + 1;
-        if (int e = X.allreduce(errs, 1, 0, s)) return e;
-        CKM(cudaMemcpyAsync(hbuf, R[0]->cnt, 8, cudaMemcpyDeviceToHost, s));
-        CKM(cudaStreamSynchronize(s));
-        if (hbuf[1]) return fail(ECL_SCC_ERANGE, "partitioned: invalid local CSR on some rank");
-    }
-    for (int r = 0; r < P; r++) {
-        PRank& Q = *R[r];
-        if (Q.nloc > 0) {
-            part::k_copy_rows<<<gridn(Q.nloc), 256, 0, s>>>(Q.nloc, Q.rb, Q.rp, Q.ci, Q.wci, Q.odeg);
-            launches++;
-        }
-        CKM(cudaMemsetAsync(Q.ideg, 0, sizeof(int32_t) * (size_t)(n + 1), s));
-        if (Q.nloc > 0) {
-            part::k_indeg_rows<<<gridn(Q.nloc), 256, 0, s>>>(Q.nloc, Q.rp, Q.wci, Q.odeg, Q.ideg);
-            launches++;
-        }
-        const int64_t nb = std::max<int64_t>((n + SCAN_TILE - 1) / SCAN_TILE, 1);
-        k_scan_reduce<I1><<<(unsigned)nb, SCAN_THREADS, 0, s>>>((const I1*)Q.ideg, n, (I1*)Q.bsum);
-        k_scan_top<I1><<<1, SCAN_THREADS, 0, s>>>((I1*)Q.bsum, nb, (I1*)Q.grand);
-        k_scan_apply<I1><<<(unsigned)nb, SCAN_THREADS, 0, s>>>((const I1*)Q.ideg, n, (I1*)Q.bsum, (I1*)Q.cp,
-                                                               (const I1*)Q.grand, 1);
-        launches += 3;
-        CKM(cudaMemsetAsync(Q.kdeg, 0, sizeof(int32_t) * (size_t)n, s));     // cursor
-        if (Q.nloc > 0) {
-            part::k_csc_rows<<<gridn(Q.nloc), 256, 0, s>>>(Q.nloc, Q.rb, Q.rp, Q.wci, Q.odeg, Q.cp, Q.kdeg, Q.cr);
-            launches++;
-        }
-        part::k_init_prio<<<std::min<unsigned>(gridn(n), 148 * 16), 256, 0, s>>>(n, Q.sig, Q.sig + n, Pr);
-        launches++;
-        CKM(cudaGetLastError());
-    }
-    int iters = 0;
-    int64_t passes_total = 0;
-    for (int iter = 1;; iter++) {
-        if (iter > n + 2) return fail(ECL_SCC_ECUDA, "internal: partitioned outer loop exceeded n+2 iterations");
-        const int first = iter == 1;
-        // ---- Phase 3 (keep) with kept degrees, summed over ranks
-        for (int r = 0; r < P; r++) {
-            PRank& Q = *R[r];
-            CKM(cudaMemsetAsync(Q.kdeg, 0, sizeof(int32_t) * 2 * (size_t)n, s));
-            if (Q.nloc > 0) {
-                part::k_keep_rows<<<gridn(Q.nloc), 256, 0, s>>>(Q.nloc, Q.rb, Q.rp, Q.wci, Q.odeg, Q.sig, Q.sig + n,
-                                                                first, Q.kdeg + n);
-                launches++;
-            }
-            part::k_keep_cols<<<gridn(n), 256, 0, s>>>(n, Q.cp, Q.cr, Q.ideg, Q.sig, Q.sig + n, first, Q.kdeg);
-            launches++;
-        }
-        if (int e = X.allreduce(kdegs, 2 * (int64_t)n, 1, s)) return e;
-        // ---- Trim-1 with global degrees; live edges summed over ranks
-        for (int r = 0; r < P; r++) {
-            PRank& Q = *R[r];
-            CKM(cudaMemsetAsync(Q.live, 0, 8, s));
-            if (Q.nloc > 0) {
-                part::k_trim_rows<<<gridn(Q.nloc), 256, 0, s>>>(Q.nloc, Q.rb, Q.rp, Q.wci, Q.odeg, Q.kdeg, Q.kdeg + n,
-                                                                trim, Q.live);
-                launches++;
-            }
-            part::k_trim_cols<<<gridn(n), 256, 0, s>>>(n, Q.cp, Q.cr, Q.ideg, Q.kdeg, Q.kdeg + n, trim);
-            k_live_to_i32<<<1, 1, 0, s>>>(Q.live, Q.cnt);
-            // ---- Phase 1 for the next Phase 2 (identical on every replica)
-            part::k_reset_all<<<std::min<unsigned>(gridn(n), 148 * 16), 256, 0, s>>>(n, Q.sig, Q.sig + n, Pr);
-            launches += 3;
-        }
-        if (int e = X.allreduce(cnts, 1, 1, s)) return e;
-        CKM(cudaMemcpyAsync(hbuf, R[0]->cnt, 4, cudaMemcpyDeviceToHost, s));
-        CKM(cudaStreamSynchronize(s));
-        const int64_t live = hbuf[0];
-        if (live == 0) break;
-        if (st && iter - 1 < ECL_SCC_TRACE_MAX) st->edges_in[iter - 1] = live;
-        if (st && iter >= 2 && iter - 2 < ECL_SCC_TRACE_MAX) st->edges_kept[iter - 2] = live;   // (after trim)
-        // ---- Phase 2: local fixed points + all-reduce(MAX) until no rank changes
-        int64_t passes_iter = 0;
-        int local_err = 0;
-        for (;;) {
-            for (int r = 0; r < P; r++) {
-                PRank& Q = *R[r];
-                int* ring = Q.ring();
-                CKM(cudaMemsetAsync(ring, 0, (RING + 1) * 4, s));      // ring words + touched
-                int pass = 0, batch = 2;
-                for (;;) {
-                    for (int k = 0; k < batch; k++, pass++) {
-                        part::k_prop_rows<<<gridn(std::max(Q.nloc, 1), 256 * part::PART_RPT), 256, 0, s>>>(
-                            Q.nloc, Q.rb, Q.rp, Q.wci, Q.odeg, Q.sig + n, ring, pass, Q.touched());
-                        part::k_prop_cols<<<gridn(n, 256 * part::PART_RPT), 256, 0, s>>>(n, Q.cp, Q.cr, Q.ideg, Q.sig,
-                                                                                         ring, pass, Q.touched());
-                        launches += 2;
-                    }
-                    CKM(cudaGetLastError());
-                    CKM(cudaMemcpyAsync(hbuf, ring + ((pass - 1) & (RING - 1)), 4, cudaMemcpyDeviceToHost, s));
-                    CKM(cudaStreamSynchronize(s));
-                    if (hbuf[0] == 0) break;
-                    if ((int64_t)pass > 4 * (int64_t)n + 1024) {
-                        local_err = 1;             // reported through the exchange (all ranks stop)
-                        break;
-                    }
-                    batch = std::min(batch * 2, RING / 2);
-                }
-                if (r == 0) passes_iter += pass;
-                // did this rank change anything? (2: it failed; MAX makes every rank see it)
-                k_copy_flag<<<1, 1, 0, s>>>(Q.touched(), Q.sig + 2 * (int64_t)n, local_err ? 2 : 0);
-                launches++;
-            }
-            if (int e = X.allreduce(sigs, 2 * (int64_t)n + 1, 0, s)) return e;
-            CKM(cudaMemcpyAsync(hbuf, R[0]->sig + 2 * (int64_t)n, 4, cudaMemcpyDeviceToHost, s));
-            CKM(cudaStreamSynchronize(s));
-            if (hbuf[0] == 2) return fail(ECL_SCC_ECUDA, "internal: local Phase 2 did not converge on some rank");
-            if (hbuf[0] == 0) break;
-        }
-        iters = iter;
-        passes_total += passes_iter;
-        if (st && iter - 1 < ECL_SCC_TRACE_MAX) st->passes_iter[iter - 1] = passes_iter;
-    }
-    // ---- labels: all signatures are final on every replica (rank 0's is used)
-    PRank& Q = *R[0];
-    const unsigned gr = std::min<unsigned>(gridn(n), 148 * 16);
-    part::k_encode_labels<<<gr, 256, 0, s>>>(n, Q.sig, labels, Pr.ids);
-    launches++;
-    if (!Pr.ids) {
-        k_relabel_rep<<<gr, 256, 0, s>>>(n, labels, Q.kdeg, Pr);
-        k_relabel_max<<<gr, 256, 0, s>>>(n, labels, Q.kdeg, Pr);
-        k_relabel_apply<<<gr, 256, 0, s>>>(n, labels, Q.kdeg);
-        launches += 3;
-    }
-    CKM(cudaGetLastError());
-    CKM(cudaStreamSynchronize(s));
-    if (st) {
-        st->iterations = iters;
-        st->trace_len = std::min(iters, ECL_SCC_TRACE_MAX);
-        st->passes = passes_total;
-        st->kernel_launches = launches;
-        st->ms_comm = X.ms();
-        st->comm_bytes = X.bytes;
-        st->exchanges = X.used;
-    }
-    return ECL_SCC_OK;
-}
-
 }  // namespace eclscc
 
-// =========================================================================== C ABI
 using namespace eclscc;
 
+// one NCCL communicator plus the device-side state of the fused halo exchange
 struct ecl_scc_comm_s {
     ncclComm_t comm;
     int nranks, rank, device;
+    bool dev_tried = false;
+    bool dev_ok = false;                 // ncclDevCommCreate succeeded
+    bool multimem = false;               // its LSA team has NVLS multicast
+    ncclDevComm dcomm{};
+    ncclWindow_t win = nullptr;          // the registered halo buffer
+    void* wbuf = nullptr;                // ncclMemAlloc'd halo buffer
+    int32_t** dptr = nullptr;            // device scratch: peer / multicast pointers
 };
+
+namespace eclscc {
+
+static __global__ void k_lsa_pointers(ncclWindow_t w, int np, int32_t** out) {
+    for (int p = 0; p < np; p++) out[p] = (int32_t*)ncclGetLsaPointer(w, 0, p);
+}
+static __global__ void k_lsa_multimem(ncclWindow_t w, ncclDevComm dc, int32_t** out) {
+    out[0] = (int32_t*)ncclGetLsaMultimemPointer(w, 0, dc);
+}
+
+struct NcclExchange : Exchange {
+    ecl_scc_comm_s* c;
+    bool allow_fused;
+    NcclExchange(ecl_scc_comm_s* cc, bool fused) : c(cc), allow_fused(fused) {}
+    int reduce(std::vector<int32_t*>& bufs, int64_t count, int op, cudaStream_t s) override {
+        CKN(ncclAllReduce(bufs[0], bufs[0], (size_t)count, ncclInt32, op == 0 ? ncclMax : ncclSum, c->comm, s));
+        return ECL_SCC_OK;
+    }
+    // collective: the halo buffer in symmetric memory, registered as a window; push targets
+    // from the device API (multicast, or every LSA peer); plain memory + all-reduce otherwise
+    int halo_buffers(std::vector<HaloRank*>& R, int64_t entries, cudaStream_t s) override {
+        HaloRank* Q = R[0];
+        const size_t bytes = sizeof(int32_t) * 2 * (size_t)entries;
+        if (!Q->hbuf_external) cudaFree(Q->hbuf);
+        Q->hbuf = nullptr;
+        Q->hbuf_external = false;
+        Q->push = HaloPush{};
+        if (c->win) {
+            ncclCommWindowDeregister(c->comm, c->win);
+            c->win = nullptr;
+        }
+        if (c->wbuf) {
+            ncclMemFree(c->wbuf);
+            c->wbuf = nullptr;
+        }
+        bool fused = false;
+        if (allow_fused && c->nranks <= HALO_MAX_PEERS) {
+            const size_t wb = (bytes + NCCL_WIN_REQUIRED_ALIGNMENT - 1) / NCCL_WIN_REQUIRED_ALIGNMENT *
+                              NCCL_WIN_REQUIRED_ALIGNMENT;
+            if (ncclMemAlloc(&c->wbuf, wb) == ncclSuccess &&
+                ncclCommWindowRegister(c->comm, c->wbuf, wb, &c->win, NCCL_WIN_COLL_SYMMETRIC) == ncclSuccess) {
+                if (!c->dev_tried) {
+                    c->dev_tried = true;
+                    ncclDevCommRequirements req = {};
+                    req.lsaMultimem = true;
+                    c->multimem = ncclDevCommCreate(c->comm, &req, &c->dcomm) == ncclSuccess;
+                    if (!c->multimem) {
+                        req.lsaMultimem = false;
+                        c->dev_ok = ncclDevCommCreate(c->comm, &req, &c->dcomm) == ncclSuccess;
+                    } else {
+                        c->dev_ok = true;
+                    }
+                }
+                const ncclTeam_t lsa = ncclTeamLsa(c->comm);
+                if (c->dev_ok && lsa.nRanks == c->nranks) {       // every rank reachable by load/store
+                    if (!c->dptr) CKM(cudaMalloc((void**)&c->dptr, sizeof(int32_t*) * (HALO_MAX_PEERS + 1)));
+                    int32_t* h[HALO_MAX_PEERS + 1] = {};
+                    k_lsa_pointers<<<1, 1, 0, s>>>(c->win, c->nranks, c->dptr);
+                    if (c->multimem) k_lsa_multimem<<<1, 1, 0, s>>>(c->win, c->dcomm, c->dptr + HALO_MAX_PEERS);
+                    CKM(cudaGetLastError());
+                    CKM(cudaMemcpyAsync(h, c->dptr, sizeof(h), cudaMemcpyDeviceToHost, s));
+                    CKM(cudaStreamSynchronize(s));
+                    Q->push.np = c->nranks;
+                    for (int k = 0; k < c->nranks; k++) Q->push.peer[k] = h[k];
+                    Q->push.mc = c->multimem ? h[HALO_MAX_PEERS] : nullptr;
+                    Q->push.sys = 1;
+                    Q->hbuf = h[lsa.rank];                    // this rank's own copy (symmetric memory)
+                    Q->hbuf_external = true;
+                    fused = Q->hbuf != nullptr;
+                }
+            } else {
+                cudaGetLastError();
+            }
+        }
+        if (!fused) {                                   // the baseline: ncclAllReduce(MAX) of the buffer
+            Q->push = HaloPush{};
+            Q->hbuf_external = false;
+            if (cudaMalloc((void**)&Q->hbuf, bytes) != cudaSuccess) {
+                cudaGetLastError();
+                return fail(ECL_SCC_ENOMEM, "halo exchange buffer");
+            }
+        }
+        return ECL_SCC_OK;
+    }
+};
+
+}  // namespace eclscc
 
 // per-rank workspace of the partitioned mode: allocated once, reused by every call
 struct ecl_scc_part_plan_s {
-    PRank R;
+    HaloRank R;
     uint32_t flags = 0;
     std::vector<cudaEvent_t> ev;              // exchange timing events
     ~ecl_scc_part_plan_s() {
@@ -374,8 +230,22 @@ int ecl_scc_comm_create(int32_t nranks, int32_t rank, const uint8_t id[128], ecl
 int ecl_scc_comm_destroy(ecl_scc_comm_t comm) {
     clear_err();
     if (!comm) return ECL_SCC_OK;
+    if (comm->win) ncclCommWindowDeregister(comm->comm, comm->win);
+    if (comm->wbuf) ncclMemFree(comm->wbuf);
+    if (comm->dev_ok) ncclDevCommDestroy(comm->comm, &comm->dcomm);
+    cudaFree(comm->dptr);
     ncclCommDestroy(comm->comm);
     delete comm;
+    return ECL_SCC_OK;
+}
+
+int ecl_scc_comm_info(ecl_scc_comm_t comm, int32_t info[4]) {
+    clear_err();
+    if (!comm || !info) return fail(ECL_SCC_EINVAL, "comm_info: bad arguments");
+    info[0] = comm->nranks;
+    info[1] = comm->rank;
+    info[2] = comm->dev_ok ? 1 : 0;
+    info[3] = comm->multimem ? 1 : 0;
     return ECL_SCC_OK;
 }
 
@@ -388,8 +258,7 @@ int ecl_scc_part_plan_create(int32_t n, int32_t row_begin, int32_t row_end, int6
     auto* h = new (std::nothrow) ecl_scc_part_plan_s();
     if (!h) return fail(ECL_SCC_ENOMEM, "host allocation");
     h->flags = flags;
-    h->R.rb = row_begin; h->R.re = row_end; h->R.nloc = row_end - row_begin; h->R.m = local_nnz_max;
-    if (int r = rank_alloc(h->R, n)) {
+    if (int r = halo_rank_alloc(&h->R, n, row_begin, row_end, local_nnz_max, flags)) {
         delete h;
         return r;
     }
@@ -419,19 +288,17 @@ int ecl_scc_partitioned(ecl_scc_comm_t comm, int32_t n, int32_t row_begin, int32
         plan = tmp;
     }
     int rc = ECL_SCC_OK;
-    if (plan->R.rb != row_begin || plan->R.re != row_end || plan->R.m < local_nnz || (int64_t)plan->R.nloc < 0)
-        rc = fail(ECL_SCC_EINVAL, "partitioned: the plan was made for other rows or fewer edges");
+    HaloRank& Q = plan->R;
+    if (Q.n != n || Q.rb != row_begin || Q.re != row_end || Q.m_cap < local_nnz)
+        rc = fail(ECL_SCC_EINVAL, "partitioned: the plan was made for another graph, other rows or fewer edges");
     if (!rc) {
-        PRank& Q = plan->R;
-        const int64_t cap = Q.m;
         Q.m = local_nnz;
         Q.rp = local_row_ptr;
         Q.ci = local_col_idx;
-        std::vector<PRank*> R{&Q};
-        NcclExchange X(comm->comm);
+        std::vector<HaloRank*> R{&Q};
+        NcclExchange X(comm, !(plan->flags & ECL_SCC_HALO_ALLREDUCE));
         X.ev = &plan->ev;
-        rc = run_partitioned(R, X, n, plan->flags, labels_out, (cudaStream_t)stream, stats);
-        Q.m = cap;
+        rc = run_halo(R, X, n, plan->flags, labels_out, (cudaStream_t)stream, stats);
         Q.rp = Q.ci = nullptr;
     }
     if (tmp) ecl_scc_part_plan_destroy(tmp);
@@ -439,7 +306,7 @@ int ecl_scc_partitioned(ecl_scc_comm_t comm, int32_t n, int32_t row_begin, int32
 }
 
 int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx,
-                                 int32_t* labels_out, ecl_scc_stream_t stream, ecl_scc_stats* stats) {
+                                 int32_t* labels_out, uint32_t flags, ecl_scc_stream_t stream, ecl_scc_stats* stats) {
     clear_err();
     if (P < 1 || P > 64 || n < 0 || nnz < 0) return fail(ECL_SCC_EINVAL, "partitioned_emulated: bad arguments");
     if (n > 0 && (!row_ptr || !labels_out)) return fail(ECL_SCC_EINVAL, "partitioned_emulated: NULL pointer");
@@ -453,16 +320,16 @@ int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_
     if (hrp[0] != 0 || hrp[n] != nnz) return fail(ECL_SCC_ERANGE, "invalid CSR offsets");
     if (int r = ecl_scc_partition_rows(P, n, hrp.data(), bounds.data())) return r;
     // each emulated rank gets its own local CSR (rebased offsets), as a real rank would
-    std::vector<std::unique_ptr<PRank>> own;
-    std::vector<PRank*> R;
+    std::vector<std::unique_ptr<HaloRank>> own;
+    std::vector<HaloRank*> R;
     std::vector<int32_t*> lrps;
     int rc = ECL_SCC_OK;
     for (int r = 0; r < P && rc == ECL_SCC_OK; r++) {
-        auto Q = std::make_unique<PRank>();
-        Q->rb = bounds[r]; Q->re = bounds[r + 1]; Q->nloc = Q->re - Q->rb;
-        Q->m = (int64_t)hrp[Q->re] - hrp[Q->rb];
-        std::vector<int32_t> lrp((size_t)Q->nloc + 1);
-        for (int i = 0; i <= Q->nloc; i++) lrp[i] = hrp[Q->rb + i] - hrp[Q->rb];
+        auto Q = std::make_unique<HaloRank>();
+        const int32_t rb = bounds[r], re = bounds[r + 1];
+        const int64_t m = (int64_t)hrp[re] - hrp[rb];
+        std::vector<int32_t> lrp((size_t)(re - rb) + 1);
+        for (int i = 0; i <= re - rb; i++) lrp[i] = hrp[rb + i] - hrp[rb];
         int32_t* d = nullptr;
         if (cudaMalloc((void**)&d, sizeof(int32_t) * lrp.size()) != cudaSuccess) {
             cudaGetLastError();
@@ -474,17 +341,18 @@ int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_
             rc = fail(ECL_SCC_ECUDA, "emulated rank offsets copy");
             break;
         }
+        rc = halo_rank_alloc(Q.get(), n, rb, re, m, flags);
+        Q->m = m;
         Q->rp = d;
-        Q->ci = col_idx + hrp[Q->rb];
-        rc = rank_alloc(*Q, n);
+        Q->ci = col_idx + hrp[rb];
         R.push_back(Q.get());
         own.push_back(std::move(Q));
     }
     if (rc == ECL_SCC_OK) {
-        EmulatedExchange X(P);
+        EmulatedExchange X(P, !(flags & ECL_SCC_HALO_ALLREDUCE));
         std::vector<cudaEvent_t> ev;
         X.ev = &ev;
-        rc = run_partitioned(R, X, n, 0, labels_out, s, stats);
+        rc = run_halo(R, X, n, flags, labels_out, s, stats);
         cudaStreamSynchronize(s);
         for (cudaEvent_t e : ev) cudaEventDestroy(e);
     }
@@ -495,4 +363,3 @@ int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_
 }
 
 }  // extern "C"
-

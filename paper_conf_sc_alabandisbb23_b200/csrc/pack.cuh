@@ -19,6 +19,7 @@
 // are unchanged: every live edge is either a slot pull or a cut-edge pull.
 #pragma once
 #include "kernels.cuh"
+#include "halo.cuh"
 
 namespace eclscc {
 
@@ -236,13 +237,13 @@ struct PackTma {
 // One visit of tile `tile` from its pack.  Returns non-zero in every thread if a
 // signature was raised.  T (k_prop_async): the pack rows arrive by bulk copy (PackTma);
 // otherwise (k_prop_pack) by vector loads.
-template <typename Mark>
+template <typename Mark, bool HALO = false>
 __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__ cin, int32_t* __restrict__ cout,
                                           const unsigned long long* __restrict__ pnin,
                                           const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext,
                                           const int* __restrict__ ext_cnt, DevCounters* __restrict__ dc, int tile,
                                           int full, Mark mark, const TileSmem<PACK_TT>& S, int next = -1,
-                                          PackTma* T = nullptr) {
+                                          PackTma* T = nullptr, const HaloPush* H = nullptr) {
     int* s_in = S.s_in;
     int* s_out = S.s_out;
     unsigned long long* s_nin = S.s_nin;
@@ -386,6 +387,20 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
             const int xv = s_in[v0 + k], yv = s_out[v0 + k];
             if (xv > ld_cg(cin + gi)) { cin[gi] = xv; rin |= 1u << (8 * k); }
             if (yv > ld_cg(cout + gi)) { cout[gi] = yv; rout |= 1u << (8 * k); }
+        }
+    }
+    // partitioned mode (halo.cuh, f1): every raised halo copy goes straight into every rank's
+    // exchange buffer (remote atomic max / multimem reduction), overlapping this rank's
+    // fixed point tile by tile
+    if (HALO && (rin | rout)) {
+#pragma unroll
+        for (int k = 0; k < VPT; k++) {
+            const unsigned bi = (rin >> (8 * k)) & 1u, bo = (rout >> (8 * k)) & 1u;
+            if (!(bi | bo)) continue;
+            const int p = __ldg(H->hpos + base + v0 + k);
+            if (p < 0) continue;
+            if (bi) halo_push_one(*H, 2 * (int64_t)p, s_in[v0 + k]);
+            if (bo) halo_push_one(*H, 2 * (int64_t)p + 1, s_out[v0 + k]);
         }
     }
     const int any = __syncthreads_or((int)(rin | rout));   // also: every drain flag is consumed
@@ -533,10 +548,11 @@ struct MarkSet {
     }
 };
 
+template <bool HALO>
 static __global__ void __launch_bounds__(PACK_TH, PACK_MINB)
 k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, const unsigned long long* __restrict__ pnin,
              const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext, const int* __restrict__ ext_cnt,
-             DevCounters* __restrict__ dc, AsyncQ Q, int claim) {
+             DevCounters* __restrict__ dc, AsyncQ Q, int claim, const __grid_constant__ HaloPush H) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ unsigned s_fin[PACK_TH + 1], s_fout[PACK_TH + 1];
     __shared__ int s_set[MSET];
@@ -622,8 +638,8 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             const int tile = s_claim[j], full = s_seen[j] == 0;
             for (int i = tid; i < MSET; i += PACK_TH) s_set[i] = -1;
             __syncthreads();
-            pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S,
-                       j + 1 < nclaim ? s_claim[j + 1] : -1, &T);
+            pack_visit<MarkSet, HALO>(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S,
+                                      j + 1 < nclaim ? s_claim[j + 1] : -1, &T, HALO ? &H : nullptr);
             __threadfence();                                      // values before marks
             __syncthreads();
             for (int i = tid; i < MSET; i += PACK_TH)
@@ -642,6 +658,7 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
         if (s_acc[1]) atomicAdd(&dc->visit_e, s_acc[1]);
         if (s_acc[2]) atomicAdd(&dc->passes, s_acc[2]);
     }
+    if (HALO && H.sys) __threadfence_system();          // pushes to other GPUs before the barrier
 }
 
 }  // namespace eclscc

@@ -73,47 +73,133 @@ def test_partition_host_logic_two_ranks_gloo():
     assert sorted(batches[0] + batches[1]) == list(range(64))  # batch split covers all graphs
 
 
-# --------------------------------------------------------------- CPU model of the protocol
-def _phase2_partitioned(n, edges, parts, vin, vout):
-    """Replicated signatures; each partition relaxes ITS edges to a local fixed point
-    (Jacobi), then element-wise MAX over partitions; repeat until no partition changed.
-    DESIGN.md reading 12 says the result is the unique global fixed point."""
-    exchanges = 0
+# --------------------------------------------------------------- the halo protocol, on gloo
+def halo_protocol(dist, rank, world, rp, ci, trim=True):
+    """A plain mirror of run_halo's control flow (driver.cu, halo.cuh) with every exchange a
+    real torch.distributed all-reduce (gloo): this rank's rows, its ghosts, the halo H found by
+    a MAX all-reduce of ghost marks; per outer iteration Phase 3 on the local edges, the halo's
+    kept degrees SUM-reduced for Trim-1, the leave rule (an unfinished, untrimmed halo
+    vertex stays), live edges SUM-reduced (termination), and Phase 2 as rounds of local
+    Jacobi fixed points whose raised halo copies are MAX-combined until no rank's copy rises;
+    finally the owners' labels MAX-reduced.  Signatures are raw IDs (IDENTITY_IDS)."""
+    import torch
+    from paper_conf_sc_alabandisbb23_b200 import dist as D
+
+    def allreduce(a, op):
+        t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.int64))
+        dist.all_reduce(t, op=op)
+        return t.numpy()
+
+    MAX, SUM = dist.ReduceOp.MAX, dist.ReduceOp.SUM
+    n = len(rp) - 1
+    bounds = D.split_rows(world, rp)
+    rb, re_ = bounds[rank], bounds[rank + 1]
+    src = np.repeat(np.arange(rb, re_), np.diff(rp[rb:re_ + 1]))
+    dst = np.asarray(ci[rp[rb]:rp[re_]], dtype=np.int64)
+    E = np.stack([src, dst], 1)
+    E = E[E[:, 0] != E[:, 1]]                               # self-loops add no path
+    owned = np.zeros(n, bool)
+    owned[rb:re_] = True
+    gmark = np.zeros(n, np.int64)
+    gmark[E[:, 1][~owned[E[:, 1]]]] = 1
+    inH = allreduce(gmark, MAX) > 0
+    pos = np.cumsum(inH) - inH
+    H = int(inH.sum())
+    held = owned | (gmark > 0)
+    vin, vout = np.arange(n), np.arange(n)
+    alive = held.copy()
+    lab = np.full(n, np.iinfo(np.int64).min)
+    edges_in = []
+    first = True
     while True:
-        replicas = []
-        changed_any = False
-        for es in parts:
-            a, b = vin.copy(), vout.copy()
-            while True:
-                na, nb = a.copy(), b.copy()
-                for u, w in es:
-                    nb[u] = max(nb[u], b[w])
-                    na[w] = max(na[w], a[u])
-                if (na == a).all() and (nb == b).all():
+        if not first:                                        # Phase 3 (P:147, P:186)
+            u, w = E[:, 0], E[:, 1]
+            E = E[(vin[u] == vin[w]) & (vout[u] == vout[w]) & (vin[u] != vout[u])]
+        kin = np.bincount(E[:, 1], minlength=n)
+        kout = np.bincount(E[:, 0], minlength=n)
+        trimmed = np.zeros(n, bool)
+        if trim:                                             # global degrees of the halo
+            hdeg = np.zeros(2 * H, np.int64)
+            hv = np.nonzero(held & inH)[0]
+            hdeg[2 * pos[hv]], hdeg[2 * pos[hv] + 1] = kin[hv], kout[hv]
+            hdeg = allreduce(hdeg, SUM)
+            hv = np.nonzero(inH)[0]
+            kin[hv], kout[hv] = hdeg[2 * pos[hv]], hdeg[2 * pos[hv] + 1]
+            trimmed = (kin == 0) | (kout == 0)
+            E = E[~trimmed[E[:, 0]] & ~trimmed[E[:, 1]]]
+        deg = np.bincount(E.ravel(), minlength=n) if len(E) else np.zeros(n, np.int64)
+        unfinished = np.ones(n, bool) if first else vin != vout
+        stay = alive & ((deg > 0) | (inH & unfinished & ~trimmed))
+        leave = alive & ~stay
+        lab[leave & owned] = np.where(unfinished, np.arange(n), vin)[leave & owned]
+        alive = stay
+        vin = np.where(alive, np.arange(n), vin)             # Phase 1 for the survivors
+        vout = np.where(alive, np.arange(n), vout)
+        first = False
+        live = int(allreduce(np.array([len(E)]), SUM)[0])
+        if live == 0:
+            lab[alive & owned] = np.arange(n)[alive & owned]
+            break
+        edges_in.append(live)
+        mine = np.zeros(2 * H, np.int64)                     # this Phase 2's pushes
+        while True:
+            a0, b0 = vin.copy(), vout.copy()
+            while True:                                      # local fixed point (Jacobi)
+                na, nb = vin.copy(), vout.copy()
+                np.maximum.at(na, E[:, 1], vin[E[:, 0]])
+                np.maximum.at(nb, E[:, 0], vout[E[:, 1]])
+                if (na == vin).all() and (nb == vout).all():
                     break
-                changed_any = True
-                a, b = na, nb
-            replicas.append((a, b))
-        vin = np.max([r[0] for r in replicas], axis=0)
-        vout = np.max([r[1] for r in replicas], axis=0)
-        exchanges += 1
-        if not changed_any:
-            return vin, vout, exchanges
+                vin, vout = na, nb
+            hv = np.nonzero(held & inH & ((vin > a0) | (vout > b0)))[0]
+            mine[2 * pos[hv]] = np.maximum(mine[2 * pos[hv]], vin[hv])
+            mine[2 * pos[hv] + 1] = np.maximum(mine[2 * pos[hv] + 1], vout[hv])
+            hbuf = allreduce(mine, MAX)
+            hv = np.nonzero(held & inH)[0]
+            xi, xo = hbuf[2 * pos[hv]], hbuf[2 * pos[hv] + 1]
+            inj = bool(((xi > vin[hv]) | (xo > vout[hv])).any())
+            vin[hv] = np.maximum(vin[hv], xi)
+            vout[hv] = np.maximum(vout[hv], xo)
+            if not allreduce(np.array([int(inj)]), MAX)[0]:
+                break
+    return allreduce(lab, MAX), edges_in
 
 
-@pytest.mark.parametrize("P", [1, 2, 3, 5])
-def test_partitioned_exchange_reaches_global_fixed_point(P):
-    rng = random.Random(10 + P)
-    for _ in range(40):
-        n = rng.randrange(2, 40)
+def _halo_worker(rank, world, port, graphs, q):
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    out = [halo_protocol(dist, rank, world, rp, ci, trim=t) for rp, ci, t in graphs]
+    if rank == 0:
+        q.put(out)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_halo_protocol_gloo(world):
+    """The partitioned (halo) protocol with real gloo collectives between `world` processes:
+    labels equal Tarjan's, and the live edges per iteration equal O2's (same trim rule) --
+    the exchange reaches the global fixed point every iteration (reading 12)."""
+    rng = random.Random(31 + world)
+    graphs = []
+    for k in range(12):
+        n = rng.randrange(2, 60)
         edges = [(rng.randrange(n), rng.randrange(n)) for _ in range(rng.randrange(1, 3 * n))]
-        edges = [(u, w) for u, w in edges if u != w]
-        if not edges:
-            continue
         rp, ci = csr_from_edges(n, edges)
-        bounds = np.linspace(0, n, P + 1).astype(int)
-        parts = [[(u, w) for u, w in edges if bounds[r] <= u < bounds[r + 1]] for r in range(P)]
-        vin, vout, _ = _phase2_partitioned(n, edges, parts, np.arange(n), np.arange(n))
-        s = oracle.ecl_scc(rp, ci, snap_iter=1)
-        np.testing.assert_array_equal(vin, s.snap_in)
-        np.testing.assert_array_equal(vout, s.snap_out)
+        graphs.append((rp.astype(np.int32), ci, k % 3 != 0))
+    g = gen.mesh(5, gen.ordinate(4), kappa=0.3, seed=2)
+    graphs.append((g.row_ptr, g.col_idx, True))
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_halo_worker, args=(r, world, port, graphs, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for (rp, ci, t), (lab, ein) in zip(graphs, res):
+        np.testing.assert_array_equal(lab, oracle.tarjan_labels(rp, ci))
+        assert ein == oracle.ecl_scc(rp, ci, trim=t).edges_in

@@ -1,8 +1,11 @@
 """GPU parity of the multi-GPU modes through the C ABI (one GPU on the test box):
-* the edge-partitioned algorithm with P emulated ranks on one device (same kernels and
-  protocol as ecl_scc_partitioned; the all-reduce is an element-wise reduction over the
-  P replicas) -- labels bit-exact, per-iteration live edges equal to O2's;
-* the NCCL path itself at world size 1 (unique id, communicator, all-reduces);
+* the edge-partitioned (halo) algorithm with P emulated ranks on one device (same kernels
+  and protocol as ecl_scc_partitioned: every rank runs the single-GPU path on its local
+  graph; the propagation kernel pushes raised halo copies into all P halo buffers, the
+  all-reduces are element-wise reductions over the P buffers) -- labels bit-exact,
+  per-iteration live edges equal to O2's; both exchanges (fused pushes, all-reduce);
+* the NCCL path itself at world size 1 (unique id, communicator, symmetric-memory halo
+  buffer through the NCCL device API, all-reduces);
 * the batched mode (disjoint union of per-ordinate graphs)."""
 import random
 
@@ -27,7 +30,7 @@ def relabel(g, pi):
     return gen.from_edges(g.n, np.stack([pi[src], pi[g.col_idx]], 1))
 
 
-@pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 8, 12])
 def test_emulated_partitions_random(P):
     rng = random.Random(100 + P)
     for trial in range(25):
@@ -35,39 +38,64 @@ def test_emulated_partitions_random(P):
         edges = [(rng.randrange(n), rng.randrange(n)) for _ in range(rng.randrange(0, 4 * n))]
         g = gen.from_edges(n, edges)
         rp, ci = dev(g)
-        lab, st = E.ecl_scc_partitioned_emulated(P, rp, ci, stats=True)
-        np.testing.assert_array_equal(lab.cpu().numpy(), oracle.tarjan_labels(g.row_ptr, g.col_idx),
-                                      err_msg=f"P={P} trial {trial}")
+        truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
         og = relabel(g, prio(n))
         tr = oracle.ecl_scc(og.row_ptr, og.col_idx, trim=True)
-        assert st["iterations"] == tr.iterations
-        assert st["edges_in"] == tr.edges_in[:64]
+        for fl in (0, E.HALO_ALLREDUCE, E.NO_ASYNC, E.SYNC_PASSES, E.IDENTITY_IDS):
+            lab, st = E.ecl_scc_partitioned_emulated(P, rp, ci, stats=True, flags=fl)
+            np.testing.assert_array_equal(lab.cpu().numpy(), truth, err_msg=f"P={P} trial {trial} flags {fl}")
+            if fl == E.IDENTITY_IDS:
+                continue
+            assert st["iterations"] == tr.iterations
+            assert st["edges_in"] == tr.edges_in[:64]
+        lab = E.ecl_scc_partitioned_emulated(P, rp, ci, flags=E.NO_TRIM)
+        np.testing.assert_array_equal(lab.cpu().numpy(), truth)
 
 
 @pytest.mark.parametrize("P", [2, 8])
 def test_emulated_partitions_mesh_and_heavy(P):
-    g = gen.mesh(20, gen.ordinate(3), seed=4, **gen.C4_MESH)
+    for g in (gen.mesh(20, gen.ordinate(3), seed=4, **gen.C4_MESH),
+              gen.mesh(24, gen.ordinate(11), seed=6, order="blocked8", **gen.C4_MESH), gen.rmat(14, 16, seed=5)):
+        rp, ci = dev(g)
+        truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+        _, s1 = E.ecl_scc(rp, ci, stats=True)
+        for fl in (0, E.HALO_ALLREDUCE):
+            lab, st = E.ecl_scc_partitioned_emulated(P, rp, ci, stats=True, flags=fl)
+            np.testing.assert_array_equal(lab.cpu().numpy(), truth, err_msg=f"{g.name} flags {fl}")
+            assert st["edges_in"] == s1["edges_in"], g.name      # the single-GPU trace
+
+
+def test_emulated_partitions_c4_sized_mesh():
+    """A C4-sized graph (16.5M vertices) over 2 and 8 emulated ranks: labels bit-exact."""
+    g = gen.config("c4", order="blocked8")
     rp, ci = dev(g)
-    np.testing.assert_array_equal(E.ecl_scc_partitioned_emulated(P, rp, ci).cpu().numpy(),
-                                  oracle.tarjan_labels(g.row_ptr, g.col_idx))
-    g = gen.rmat(14, 16, seed=5)
-    rp, ci = dev(g)
-    np.testing.assert_array_equal(E.ecl_scc_partitioned_emulated(P, rp, ci).cpu().numpy(),
-                                  oracle.tarjan_labels(g.row_ptr, g.col_idx))
+    truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+    for P in (2, 8):
+        lab, st = E.ecl_scc_partitioned_emulated(P, rp, ci, stats=True)
+        np.testing.assert_array_equal(lab.cpu().numpy(), truth, err_msg=f"P={P}")
+        print(f"C4 emulated P={P}: iterations {st['iterations']} rounds {st['passes']} "
+              f"exchanges {st['exchanges']} comm bytes {st['comm_bytes']}")
 
 
 def test_nccl_world_size_one():
-    g = gen.config("c1")
-    rp, ci = dev(g)
-    comm = E.Comm(1, 0, E.get_unique_id())
-    try:
-        lab, st = E.ecl_scc_partitioned(comm, g.n, 0, g.n, rp, ci, stats=True)
-        torch.cuda.synchronize()
-        np.testing.assert_array_equal(lab.cpu().numpy(), oracle.tarjan_labels(g.row_ptr, g.col_idx))
-        _, s1 = E.ecl_scc(rp, ci, stats=True)
-        assert st["edges_in"] == s1["edges_in"]          # same trace as the single-GPU path
-    finally:
-        comm.close()
+    for g in (gen.config("c1"), gen.mesh(16, gen.ordinate(2), seed=4, **gen.C4_MESH)):
+        rp, ci = dev(g)
+        comm = E.Comm(1, 0, E.get_unique_id())
+        try:
+            truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+            _, s1 = E.ecl_scc(rp, ci, stats=True)
+            for fl in (0, E.HALO_ALLREDUCE):
+                plan = E.PartPlan(comm, g.n, 0, g.n, g.nnz, fl)
+                for _ in range(2):                       # plan reuse
+                    lab, st = E.ecl_scc_partitioned(comm, g.n, 0, g.n, rp, ci, plan=plan, stats=True)
+                    torch.cuda.synchronize()
+                    np.testing.assert_array_equal(lab.cpu().numpy(), truth)
+                    assert st["edges_in"] == s1["edges_in"]          # same trace as the single-GPU path
+                    assert st["exchanges"] > 0 and st["ms_comm"] > 0
+                plan.close()
+            print("comm info", comm.info())
+        finally:
+            comm.close()
 
 
 def test_batched_mixed_sizes_and_empty():

@@ -61,7 +61,10 @@ typedef enum {
 
 /* plan flags (DESIGN.md "Readings" and "Kernels") */
 #define ECL_SCC_NO_TRIM 0x1u      /* disable the Trim-1 round run with every edge removal */
-/* 0x2u is reserved for path compression, not in this build */
+#define ECL_SCC_COMPRESS 0x2u     /* variant: path compression (reading 4) -- a
+                                     cut-edge pull takes max(in[u], in[in[u]]) (out likewise),
+                                     through a priority -> local index map; two-signature method,
+                                     single GPU */
 #define ECL_SCC_NO_VALIDATE 0x4u  /* skip the device validation pass over row_ptr/col_idx */
 #define ECL_SCC_SYNC_PASSES 0x8u  /* ablation: no block-local iteration, one Jacobi-like
                                      relaxation per global pass ("separate kernels") */
@@ -89,6 +92,10 @@ typedef enum {
 #define ECL_SCC_HALO_ALLREDUCE 0x10000u /* partitioned mode, baseline exchange: combine the halo
                                      signatures with ncclAllReduce(MAX) after every local fixed
                                      point instead of the propagation kernel's peer pushes */
+#define ECL_SCC_RAISE 0x20000u    /* variant: the sound form of the P:190 trick (DESIGN.md reading
+                                     5) -- when v_in rises to t inside a tile, t is also offered to
+                                     in[out[v]] (a descendant of v) if that vertex is in the same
+                                     tile; v_out likewise to out[in[v]]; single GPU */
 #define ECL_SCC_FOUR_SIG 0x8000u  /* variant: the 4-signature method -- Phase 2 also
                                      propagates minimum ancestor / descendant IDs and Phase 3
                                      keeps an edge only if all four signatures agree; twice the
@@ -234,10 +241,16 @@ int ecl_scc_partitioned(ecl_scc_comm_t comm, int32_t n, int32_t row_begin, int32
  * arithmetic and exchange protocol as ecl_scc_partitioned at P ranks; used to test the
  * partitioned path on one GPU.  Inputs as ecl_scc(); row ranges are chosen balanced by edge
  * count.  flags: as ecl_scc_part_plan_create (ECL_SCC_HALO_ALLREDUCE selects the baseline
- * exchange). */
+ * exchange).  plan: nullable; from ecl_scc_emulated_plan_create for the same P, graph size
+ * and flags (repeated calls without allocation). */
+typedef struct ecl_scc_emulated_plan_s* ecl_scc_emulated_plan_t;
+int ecl_scc_emulated_plan_create(int32_t P, int32_t n, int64_t nnz, const int32_t* row_ptr,
+                                 uint32_t flags, ecl_scc_emulated_plan_t* out);
+int ecl_scc_emulated_plan_destroy(ecl_scc_emulated_plan_t plan);
 int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_t* row_ptr,
                                  const int32_t* col_idx, int32_t* labels_out, uint32_t flags,
-                                 ecl_scc_stream_t stream, ecl_scc_stats* stats);
+                                 ecl_scc_stream_t stream, ecl_scc_emulated_plan_t plan,
+                                 ecl_scc_stats* stats);
 
 /* Diagnostics of a communicator: info[0] ranks, [1] this rank, [2] 1 if the NCCL device API
  * is in use for the fused halo exchange (peer pushes), [3] 1 if it uses NVLS multimem

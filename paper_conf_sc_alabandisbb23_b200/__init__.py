@@ -21,7 +21,7 @@ OK, EINVAL, ERANGE, ENOMEM, ECUDA, ENCCL, EUNSUPPORTED = range(7)
 NO_TRIM, NO_VALIDATE, SYNC_PASSES, TIME_STAGES = 0x1, 0x4, 0x8, 0x10
 IDENTITY_IDS, NO_DIRTY, NO_REORDER = 0x20, 0x40, 0x200
 FORCE_REORDER, NO_PACK, NO_ASYNC = 0x400, 0x800, 0x1000
-TRIM2, FOUR_SIG, HALO_ALLREDUCE = 0x4000, 0x8000, 0x10000
+TRIM2, FOUR_SIG, HALO_ALLREDUCE, COMPRESS, RAISE = 0x4000, 0x8000, 0x10000, 0x2, 0x20000
 TRACE_MAX = 64
 
 _lib = None
@@ -79,7 +79,9 @@ def lib() -> ctypes.CDLL:
         "ecl_scc_partitioned": [vp, i32, i32, i32, i64, vp, vp, vp, vp, vp, vp],
         "ecl_scc_part_plan_create": [i32, i32, i32, i64, u32, vp],
         "ecl_scc_part_plan_destroy": [vp],
-        "ecl_scc_partitioned_emulated": [i32, i32, i64, vp, vp, vp, u32, vp, vp],
+        "ecl_scc_partitioned_emulated": [i32, i32, i64, vp, vp, vp, u32, vp, vp, vp],
+        "ecl_scc_emulated_plan_create": [i32, i32, i64, vp, u32, vp],
+        "ecl_scc_emulated_plan_destroy": [vp],
         "ecl_scc_comm_info": [vp, vp],
         "ecl_scc_partition_rows": [i32, i32, vp, vp],
         "ecl_scc_status_string": [ctypes.c_int],
@@ -105,7 +107,8 @@ ABI_SYMBOLS = ("ecl_scc", "ecl_scc_async", "ecl_scc_debug_run", "ecl_scc_plan_cr
                "ecl_scc_comm_create", "ecl_scc_comm_destroy", "ecl_scc_partitioned",
                "ecl_scc_partitioned_emulated", "ecl_scc_partition_rows", "ecl_scc_status_string",
                "ecl_scc_last_error", "ecl_scc_version", "ecl_scc_plan_counters", "ecl_scc_levels",
-               "ecl_scc_host", "ecl_scc_part_plan_create", "ecl_scc_part_plan_destroy", "ecl_scc_comm_info")
+               "ecl_scc_host", "ecl_scc_part_plan_create", "ecl_scc_part_plan_destroy", "ecl_scc_comm_info",
+               "ecl_scc_emulated_plan_create", "ecl_scc_emulated_plan_destroy")
 
 
 def status_string(s: int) -> str:
@@ -247,8 +250,29 @@ def ecl_scc_partition_rows(P: int, row_ptr_host) -> list[int]:
     return out.tolist()
 
 
+class EmulatedPlan:
+    """Workspaces of P emulated ranks (ecl_scc_emulated_plan_t) for one graph size and flags."""
+
+    def __init__(self, P: int, row_ptr: torch.Tensor, nnz: int, flags: int = 0):
+        h = ctypes.c_void_p()
+        _check(lib().ecl_scc_emulated_plan_create(P, row_ptr.numel() - 1, nnz, _dev_i32(row_ptr, "row_ptr"), flags,
+                                                  ctypes.byref(h)), "ecl_scc_emulated_plan_create")
+        self.handle = h
+
+    def close(self):
+        if self.handle:
+            lib().ecl_scc_emulated_plan_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 def ecl_scc_partitioned_emulated(P: int, row_ptr, col_idx, labels_out=None, stream=None, stats: bool = False,
-                                 flags: int = 0):
+                                 flags: int = 0, plan: EmulatedPlan | None = None):
     n = row_ptr.numel() - 1
     if labels_out is None:
         labels_out = torch.empty(n, dtype=torch.int32, device=row_ptr.device)
@@ -256,6 +280,7 @@ def ecl_scc_partitioned_emulated(P: int, row_ptr, col_idx, labels_out=None, stre
     _check(lib().ecl_scc_partitioned_emulated(P, n, col_idx.numel(), _dev_i32(row_ptr, "row_ptr"),
                                               _dev_i32(col_idx, "col_idx") if col_idx.numel() else None,
                                               _dev_i32(labels_out, "labels_out"), flags, _stream(stream),
+                                              plan.handle if plan else None,
                                               ctypes.byref(st) if st else None), "ecl_scc_partitioned_emulated")
     return (labels_out, st.as_dict()) if stats else labels_out
 

@@ -29,6 +29,9 @@ struct WGraph {
                              // nullptr: the two-signature method
     const int32_t* hpos;     // partitioned mode (halo.cuh): position of each local vertex in the
                              // halo H, or -1; nullptr: single GPU
+    const int32_t* slot;     // ECL_SCC_COMPRESS / ECL_SCC_RAISE: local index of the vertex with
+                             // priority p (the vertices of the current working graph)
+    int compress, raise_;    // path compression / the sound P:190 variant switched on
 };
 // the minimum signatures propagate as maxima of mirrored priorities (all >= 0, so the
 // pack kernels' sentinel value 0 stays below every signature)

@@ -117,6 +117,7 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
             e = e ? e : A((void**)&p->min_out[b], n1 * 4);
         }
     if (p->flags & ECL_SCC_TRIM2) e = e ? e : A((void**)&p->t2, n1 * 4);
+    if (p->flags & (ECL_SCC_COMPRESS | ECL_SCC_RAISE)) e = e ? e : A((void**)&p->slot, n1 * 4);
     e = e ? e : A((void**)&p->newidx, n1 * 4);
     e = e ? e : A((void**)&p->cnt, n1 * sizeof(int2));
     e = e ? e : A((void**)&p->emask, n1 * sizeof(uint2));
@@ -153,7 +154,7 @@ void plan_free(Plan* p) {
         cudaFree(p->optr[b]); cudaFree(p->iptr[b]); cudaFree(p->oadj[b]); cudaFree(p->iadj[b]);
     }
     for (int b = 0; b < 2; b++) { cudaFree(p->min_in[b]); cudaFree(p->min_out[b]); }
-    cudaFree(p->t2); cudaFree(p->hpos[0]); cudaFree(p->hpos[1]);
+    cudaFree(p->t2); cudaFree(p->hpos[0]); cudaFree(p->hpos[1]); cudaFree(p->slot);
     cudaFree(p->kin); cudaFree(p->newidx); cudaFree(p->cnt); cudaFree(p->emask); cudaFree(p->sig2);
     cudaFree(p->wsum); cudaFree(p->wscan); cudaFree(p->bsum); cudaFree(p->chunks); cudaFree(p->dc);
     cudaFree(p->chunk_cnt); cudaFree(p->hcnt);
@@ -301,9 +302,10 @@ static int ensure_pack(Plan* p) {
         cudaGetLastError();
         return fail(ECL_SCC_ENOMEM, "tile pack allocation: %s", cudaGetErrorString(e));
     }
-    CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
-    CK(cudaFuncSetAttribute(k_prop_pack, cudaFuncAttributePreferredSharedMemoryCarveout,
-                            (int)cudaSharedmemCarveoutMaxShared));
+    for (auto kf : {k_prop_pack<false>, k_prop_pack<true>}) {
+        CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
+        CK(cudaFuncSetAttribute(kf, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared));
+    }
     return ECL_SCC_OK;
 }
 
@@ -368,8 +370,9 @@ static int compact_finish(Plan* p, const int32_t* cin, const int32_t* cout, int 
     p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
                                               chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur, pk,
-                                              p->min_in[ob], p->min_out[ob], trim2 ? p->t2 : nullptr, p->kio, TRIM ? 1 : 0,
-                                              gk.hpos ? p->hpos[ob] : nullptr, p->lab_lo, p->lab_hi);
+                                              MapExtra{p->min_in[ob], p->min_out[ob], trim2 ? p->t2 : nullptr, p->kio,
+                                                       TRIM ? 1 : 0, gk.hpos ? p->hpos[ob] : nullptr, p->lab_lo,
+                                                       p->lab_hi, p->slot});
     p->launches++; k_compact_scatter<FIRST, TRIM, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked, p->emask, pk);
     if (chunked) {
@@ -463,13 +466,13 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
                     cudaGetLastError();
                     return fail(ECL_SCC_ENOMEM, "async queue allocation: %s", cudaGetErrorString(e));
                 }
-                for (auto kf : {k_prop_async<false>, k_prop_async<true>}) {
+                for (auto kf : {k_prop_async<false, false>, k_prop_async<true, false>, k_prop_async<false, true>}) {
                     CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
                     CK(cudaFuncSetAttribute(kf, cudaFuncAttributePreferredSharedMemoryCarveout,
                                             (int)cudaSharedmemCarveoutMaxShared));
                 }
                 int per_sm = 0, sms = 0;
-                CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_async<false>, PACK_TH, pack_dyn_smem()));
+                CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_async<false, false>, PACK_TH, pack_dyn_smem()));
                 CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device));
                 // resident CTAs per SM used (<= what fits); measured best: all of them
                 if (p->knob_async_ctas) per_sm = std::min(per_sm, p->knob_async_ctas);
@@ -498,9 +501,11 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             }
             p->launches++;
             const unsigned agrid = (unsigned)std::min<int64_t>(ntiles, p->aq_resident);
-            if (push) k_prop_async<true><<<agrid, PACK_TH, pack_dyn_smem(), s>>>(
+            if (push) k_prop_async<true, false><<<agrid, PACK_TH, pack_dyn_smem(), s>>>(
                 g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, Q, claim, *push);
-            else k_prop_async<false><<<agrid, PACK_TH, pack_dyn_smem(), s>>>(
+            else if (g.compress | g.raise_) k_prop_async<false, true><<<agrid, PACK_TH, pack_dyn_smem(), s>>>(
+                g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, Q, claim, HaloPush{});
+            else k_prop_async<false, false><<<agrid, PACK_TH, pack_dyn_smem(), s>>>(
                 g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, Q, claim, HaloPush{});
             CK(cudaGetLastError());
             // no stream synchronisation here: the watchdog word and the visit count are read
@@ -526,8 +531,12 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
             if (use_pack) {
                 const int run = pass_run(p, ntiles);
                 p->launches++;
-                k_prop_pack<<<(unsigned)cdiv(ntiles, run), PACK_TH, pack_dyn_smem(), s>>>(
-                    g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, pass, nchunks == 0, dc_, dn_, full, run);
+                if (g.compress | g.raise_)
+                    k_prop_pack<true><<<(unsigned)cdiv(ntiles, run), PACK_TH, pack_dyn_smem(), s>>>(
+                        g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, pass, nchunks == 0, dc_, dn_, full, run);
+                else
+                    k_prop_pack<false><<<(unsigned)cdiv(ntiles, run), PACK_TH, pack_dyn_smem(), s>>>(
+                        g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt, p->dc, pass, nchunks == 0, dc_, dn_, full, run);
                 continue;
             }
             if (int r = launch_tile(p, sync, g, cin, cout, pass, nchunks == 0, dc_, dn_, full, s)) return r;
@@ -666,6 +675,9 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
             if (nchunks > p->chunk_cap) return fail(ECL_SCC_ECUDA, "internal: heavy chunk list overflow");
             g = WGraph{p->act[ob], p->optr[ob], p->oadj[ob], p->iptr[ob], p->iadj[ob], t.x, nullptr,
                        p->min_in[ob], p->min_out[ob]};
+            g.slot = p->slot;
+            g.compress = (p->flags & ECL_SCC_COMPRESS) ? 1 : 0;
+            g.raise_ = (p->flags & ECL_SCC_RAISE) ? 1 : 0;
             cin = p->cin[ob];
             cout = p->cout[ob];
             if (t.y == 0) break;                                   // no live edge: done
@@ -864,8 +876,9 @@ HaloRank::~HaloRank() {
 int halo_rank_alloc(HaloRank* R, int32_t n, int32_t rb, int32_t re, int64_t m_cap, uint32_t flags) {
     R->n = n; R->rb = rb; R->re = re; R->nloc = re - rb; R->m_cap = m_cap;
     const int64_t nl_max = std::min<int64_t>((int64_t)R->nloc + m_cap, n);
-    if (flags & (ECL_SCC_TRIM2 | ECL_SCC_FOUR_SIG))
-        return fail(ECL_SCC_EUNSUPPORTED, "partitioned mode: Trim-2 and the 4-signature variant are single-GPU only");
+    if (flags & (ECL_SCC_TRIM2 | ECL_SCC_FOUR_SIG | ECL_SCC_COMPRESS | ECL_SCC_RAISE))
+        return fail(ECL_SCC_EUNSUPPORTED, "partitioned mode: Trim-2, the 4-signature variant, path compression and "
+                                          "the P:190 variant are single-GPU only");
     R->p.flags = flags | ECL_SCC_NO_REORDER;       // the local -> global map is the storage map
     if (int r = plan_alloc(&R->p, (int32_t)std::max<int64_t>(nl_max, 1), std::max<int64_t>(m_cap, 1))) return r;
     const size_t n1 = (size_t)n + 1, nl1 = (size_t)nl_max + 1;
@@ -1259,6 +1272,10 @@ int ecl_scc_plan_create(int32_t n_max, int64_t nnz_max, uint32_t flags, ecl_scc_
     if (nnz_max >= (int64_t)INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "nnz_max >= 2^31");
     ecl_scc_plan_s* h = (ecl_scc_plan_s*)calloc(1, sizeof(ecl_scc_plan_s));
     if (!h) return fail(ECL_SCC_ENOMEM, "host allocation");
+    if ((flags & (ECL_SCC_COMPRESS | ECL_SCC_RAISE)) && (flags & ECL_SCC_FOUR_SIG)) {
+        free(h);
+        return fail(ECL_SCC_EINVAL, "plan_create: ECL_SCC_COMPRESS / ECL_SCC_RAISE apply to the two-signature method");
+    }
     if ((flags & ECL_SCC_TRIM2) && (flags & ECL_SCC_NO_TRIM)) {
         free(h);
         return fail(ECL_SCC_EINVAL, "plan_create: ECL_SCC_TRIM2 runs with Trim-1 (not with ECL_SCC_NO_TRIM)");

@@ -24,6 +24,7 @@ struct Plan {
     int32_t *min_in[2], *min_out[2];     // ECL_SCC_FOUR_SIG: minimum signatures (mirrored), per buffer
     int32_t* t2;                         // ECL_SCC_TRIM2: Trim-2 partner per local vertex (-1: none)
     int32_t* hpos[2];                    // partitioned mode: halo position per local vertex, per buffer
+    int32_t* slot;                       // ECL_SCC_COMPRESS / RAISE: priority -> local index
     int32_t lab_lo, lab_hi;              // label ownership: labels[v] written only for lab_lo <= v < lab_hi
     WGraph gk;                           // the graph of the compaction in progress (keep -> finish)
     int32_t *kin, *kout;                 // two n+1 int views (ingest histogram / cursor, relabel, levels)

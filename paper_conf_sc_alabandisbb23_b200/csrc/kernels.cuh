@@ -495,6 +495,17 @@ static __global__ void k_trim2_apply(int32_t na, const int32_t* __restrict__ t2,
     if (i < na && t2[i] >= 0) kio[i].x = 0;
 }
 
+// the optional outputs of k_compact_map
+struct MapExtra {
+    int32_t *min_in2, *min_out2;     // 4-signature variant: the minimum pair of the next graph
+    const int32_t* t2;               // Trim-2 partners (labels of the pairs)
+    const int2* kio;                 // kept degrees (partitioned mode: trimmed halo vertices)
+    int trim;
+    int32_t* hpos2;                  // partitioned mode: halo positions of the next graph
+    int32_t lab_lo, lab_hi;          // labels written only for IDs in [lab_lo, lab_hi)
+    int32_t* slot;                   // priority -> local index of the next graph, or nullptr
+};
+
 // New numbering, Phase 1 reset of the survivors (rule R2), final labels of
 // the vertices that leave, new offsets, heavy-row chunk list.
 // Survivors restart from their priority pi(v) (reading 16).  A finished vertex leaves
@@ -507,10 +518,12 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
                               int32_t* __restrict__ act2, int32_t* __restrict__ cin2, int32_t* __restrict__ cout2,
                               int32_t* __restrict__ optr2, int32_t* __restrict__ iptr2, int32_t* __restrict__ labels,
                               Chunk* __restrict__ chunks, int* __restrict__ nchunks, int chunk_cap, Prio P,
-                              const int32_t* __restrict__ orig, PackOut pk, int32_t* __restrict__ min_in2,
-                              int32_t* __restrict__ min_out2, const int32_t* __restrict__ t2,
-                              const int2* __restrict__ kio, int trim, int32_t* __restrict__ hpos2, int32_t lab_lo,
-                              int32_t lab_hi) {
+                              const int32_t* __restrict__ orig, PackOut pk, MapExtra X) {
+    int32_t* __restrict__ min_in2 = X.min_in2;
+    int32_t* __restrict__ min_out2 = X.min_out2;
+    const int32_t* __restrict__ t2 = X.t2;
+    const int2* __restrict__ kio = X.kio;
+    const int trim = X.trim;
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i == 0) {
@@ -545,7 +558,8 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
         const int pv = (int)prio_of(P, (uint32_t)ov);
         cin2[j] = pv;       // Phase 1: v_in <- v_id, v_out <- v_id for the unfinished
         cout2[j] = pv;
-        if (hpos2) hpos2[j] = g.hpos[i];
+        if (X.hpos2) X.hpos2[j] = g.hpos[i];
+        if (X.slot) X.slot[pv] = j;  // priority -> local index (ECL_SCC_COMPRESS / ECL_SCC_RAISE)
         if (min_in2) {      // the minimum pair restarts from the vertex too
             min_in2[j] = mirror_prio(pv);
             min_out2[j] = mirror_prio(pv);
@@ -574,7 +588,7 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
             const int ow = orig ? orig[vw] : vw;
             lab = P.ids ? max(ov, ow) : -((int)max(prio_of(P, (uint32_t)ov), prio_of(P, (uint32_t)ow)) + 1);
         }
-        if (ov >= lab_lo && ov < lab_hi) labels[ov] = lab;    // partitioned: the owner writes
+        if (ov >= X.lab_lo && ov < X.lab_hi) labels[ov] = lab;    // partitioned: the owner writes
     }
 }
 

@@ -187,6 +187,23 @@ struct NcclExchange : Exchange {
 
 }  // namespace eclscc
 
+// P emulated ranks on one device (tests, development): their workspaces and row offsets
+struct ecl_scc_emulated_plan_s {
+    int P = 0;
+    int32_t n = 0;
+    int64_t nnz = 0;
+    uint32_t flags = 0;
+    std::vector<std::unique_ptr<HaloRank>> R;
+    std::vector<int32_t*> lrps;               // per rank: rebased row offsets (device)
+    std::vector<int64_t> coff;                // per rank: offset of its rows in col_idx
+    std::vector<cudaEvent_t> ev;
+    ~ecl_scc_emulated_plan_s() {
+        R.clear();
+        for (int32_t* d : lrps) cudaFree(d);
+        for (cudaEvent_t e : ev) cudaEventDestroy(e);
+    }
+};
+
 // per-rank workspace of the partitioned mode: allocated once, reused by every call
 struct ecl_scc_part_plan_s {
     HaloRank R;
@@ -305,8 +322,59 @@ int ecl_scc_partitioned(ecl_scc_comm_t comm, int32_t n, int32_t row_begin, int32
     return rc;
 }
 
+int ecl_scc_emulated_plan_destroy(ecl_scc_emulated_plan_t plan) {
+    clear_err();
+    delete plan;
+    return ECL_SCC_OK;
+}
+
+int ecl_scc_emulated_plan_create(int32_t P, int32_t n, int64_t nnz, const int32_t* row_ptr, uint32_t flags,
+                                 ecl_scc_emulated_plan_t* out) {
+    clear_err();
+    if (!out || P < 1 || P > 64 || n < 1 || nnz < 0 || !row_ptr) return fail(ECL_SCC_EINVAL, "emulated_plan_create: bad arguments");
+    if (nnz >= (int64_t)INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "nnz >= 2^31");
+    // row ranges balanced by edge count, from the host copy of row_ptr
+    std::vector<int32_t> hrp((size_t)n + 1), bounds((size_t)P + 1);
+    CKM(cudaMemcpy(hrp.data(), row_ptr, sizeof(int32_t) * (size_t)(n + 1), cudaMemcpyDeviceToHost));
+    if (hrp[0] != 0 || hrp[n] != nnz) return fail(ECL_SCC_ERANGE, "invalid CSR offsets");
+    if (int r = ecl_scc_partition_rows(P, n, hrp.data(), bounds.data())) return r;
+    auto* h = new (std::nothrow) ecl_scc_emulated_plan_s();
+    if (!h) return fail(ECL_SCC_ENOMEM, "host allocation");
+    h->P = P; h->n = n; h->nnz = nnz; h->flags = flags;
+    // each emulated rank gets its own local CSR (rebased offsets), as a real rank would
+    for (int r = 0; r < P; r++) {
+        auto Q = std::make_unique<HaloRank>();
+        const int32_t rb = bounds[r], re = bounds[r + 1];
+        const int64_t m = (int64_t)hrp[re] - hrp[rb];
+        std::vector<int32_t> lrp((size_t)(re - rb) + 1);
+        for (int i = 0; i <= re - rb; i++) lrp[i] = hrp[rb + i] - hrp[rb];
+        int32_t* d = nullptr;
+        int rc = ECL_SCC_OK;
+        if (cudaMalloc((void**)&d, sizeof(int32_t) * lrp.size()) != cudaSuccess) {
+            cudaGetLastError();
+            rc = fail(ECL_SCC_ENOMEM, "emulated rank offsets");
+        } else {
+            h->lrps.push_back(d);
+            if (cudaMemcpy(d, lrp.data(), sizeof(int32_t) * lrp.size(), cudaMemcpyHostToDevice) != cudaSuccess)
+                rc = fail(ECL_SCC_ECUDA, "emulated rank offsets copy");
+        }
+        if (!rc) rc = halo_rank_alloc(Q.get(), n, rb, re, m, flags);
+        if (rc) {
+            delete h;
+            return rc;
+        }
+        Q->m = m;
+        Q->rp = d;
+        h->coff.push_back(hrp[rb]);
+        h->R.push_back(std::move(Q));
+    }
+    *out = h;
+    return ECL_SCC_OK;
+}
+
 int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* col_idx,
-                                 int32_t* labels_out, uint32_t flags, ecl_scc_stream_t stream, ecl_scc_stats* stats) {
+                                 int32_t* labels_out, uint32_t flags, ecl_scc_stream_t stream,
+                                 ecl_scc_emulated_plan_t plan, ecl_scc_stats* stats) {
     clear_err();
     if (P < 1 || P > 64 || n < 0 || nnz < 0) return fail(ECL_SCC_EINVAL, "partitioned_emulated: bad arguments");
     if (n > 0 && (!row_ptr || !labels_out)) return fail(ECL_SCC_EINVAL, "partitioned_emulated: NULL pointer");
@@ -314,51 +382,26 @@ int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_
     if (nnz >= (int64_t)INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "nnz >= 2^31");
     if (n == 0) return ECL_SCC_OK;
     cudaStream_t s = (cudaStream_t)stream;
-    // row ranges balanced by edge count, from the host copy of row_ptr
-    std::vector<int32_t> hrp((size_t)n + 1), bounds((size_t)P + 1);
-    CKM(cudaMemcpy(hrp.data(), row_ptr, sizeof(int32_t) * (size_t)(n + 1), cudaMemcpyDeviceToHost));
-    if (hrp[0] != 0 || hrp[n] != nnz) return fail(ECL_SCC_ERANGE, "invalid CSR offsets");
-    if (int r = ecl_scc_partition_rows(P, n, hrp.data(), bounds.data())) return r;
-    // each emulated rank gets its own local CSR (rebased offsets), as a real rank would
-    std::vector<std::unique_ptr<HaloRank>> own;
-    std::vector<HaloRank*> R;
-    std::vector<int32_t*> lrps;
-    int rc = ECL_SCC_OK;
-    for (int r = 0; r < P && rc == ECL_SCC_OK; r++) {
-        auto Q = std::make_unique<HaloRank>();
-        const int32_t rb = bounds[r], re = bounds[r + 1];
-        const int64_t m = (int64_t)hrp[re] - hrp[rb];
-        std::vector<int32_t> lrp((size_t)(re - rb) + 1);
-        for (int i = 0; i <= re - rb; i++) lrp[i] = hrp[rb + i] - hrp[rb];
-        int32_t* d = nullptr;
-        if (cudaMalloc((void**)&d, sizeof(int32_t) * lrp.size()) != cudaSuccess) {
-            cudaGetLastError();
-            rc = fail(ECL_SCC_ENOMEM, "emulated rank offsets");
-            break;
-        }
-        lrps.push_back(d);
-        if (cudaMemcpy(d, lrp.data(), sizeof(int32_t) * lrp.size(), cudaMemcpyHostToDevice) != cudaSuccess) {
-            rc = fail(ECL_SCC_ECUDA, "emulated rank offsets copy");
-            break;
-        }
-        rc = halo_rank_alloc(Q.get(), n, rb, re, m, flags);
-        Q->m = m;
-        Q->rp = d;
-        Q->ci = col_idx + hrp[rb];
-        R.push_back(Q.get());
-        own.push_back(std::move(Q));
+    ecl_scc_emulated_plan_t tmp = nullptr;
+    if (!plan) {
+        if (int r = ecl_scc_emulated_plan_create(P, n, nnz, row_ptr, flags, &tmp)) return r;
+        plan = tmp;
     }
-    if (rc == ECL_SCC_OK) {
+    int rc = ECL_SCC_OK;
+    if (plan->P != P || plan->n != n || plan->nnz != nnz || plan->flags != flags)
+        rc = fail(ECL_SCC_EINVAL, "partitioned_emulated: the plan was made for another graph, P or flags");
+    if (!rc) {
+        std::vector<HaloRank*> R;
+        for (int r = 0; r < P; r++) {
+            plan->R[r]->ci = col_idx + plan->coff[r];
+            R.push_back(plan->R[r].get());
+        }
         EmulatedExchange X(P, !(flags & ECL_SCC_HALO_ALLREDUCE));
-        std::vector<cudaEvent_t> ev;
-        X.ev = &ev;
+        X.ev = &plan->ev;
         rc = run_halo(R, X, n, flags, labels_out, s, stats);
-        cudaStreamSynchronize(s);
-        for (cudaEvent_t e : ev) cudaEventDestroy(e);
     }
     cudaStreamSynchronize(s);
-    own.clear();
-    for (int32_t* d : lrps) cudaFree(d);
+    if (tmp) ecl_scc_emulated_plan_destroy(tmp);
     return rc;
 }
 

@@ -86,6 +86,7 @@ __device__ __forceinline__ unsigned gather4(unsigned w) {      // byte k (0/1) -
 // every round free of a serial item loop whose length is the warp's maximum (18.5 -> 17.1 ms
 // -> 15.2 ms with the packs from the scatter).  A warp leaves its rounds when none of its
 // lanes has a flag left; the block rounds end when a whole block round found nothing.
+template <bool TRICKS = false>
 __device__ __forceinline__ void drain_direct(const WGraph& g, int* __restrict__ s_in, int* __restrict__ s_out,
                                              const unsigned long long* __restrict__ s_nin,
                                              const unsigned long long* __restrict__ s_nout,
@@ -124,6 +125,13 @@ __device__ __forceinline__ void drain_direct(const WGraph& g, int* __restrict__ 
                         ((volatile int*)s_out)[v] = val;
                         __threadfence_block();
                         pnotify_full(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
+                        if (TRICKS && g.raise_) {                // sound P:190: out[in[v]] (an ancestor)
+                            const int L = __ldg(g.slot + ((volatile int*)s_in)[v]) - base;
+                            if ((unsigned)L < (unsigned)cnt && L != v && atomicMax(s_out + L, val) < val) {
+                                __threadfence_block();
+                                pnotify_full(s_nin[L], g.iptr, g.iadj, base, cnt, L, (uint8_t*)s_fout);
+                            }
+                        }
                     }
                 } else {                                         // v_in from the in-neighbours
                     atomicAnd(s_fin + tid, keep);
@@ -135,6 +143,13 @@ __device__ __forceinline__ void drain_direct(const WGraph& g, int* __restrict__ 
                         ((volatile int*)s_in)[v] = val;
                         __threadfence_block();
                         pnotify_full(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
+                        if (TRICKS && g.raise_) {                // sound P:190: in[out[v]] (a descendant)
+                            const int L = __ldg(g.slot + ((volatile int*)s_out)[v]) - base;
+                            if ((unsigned)L < (unsigned)cnt && L != v && atomicMax(s_in + L, val) < val) {
+                                __threadfence_block();
+                                pnotify_full(s_nout[L], g.optr, g.oadj, base, cnt, L, (uint8_t*)s_fin);
+                            }
+                        }
                     }
                 }
             }
@@ -237,7 +252,7 @@ struct PackTma {
 // One visit of tile `tile` from its pack.  Returns non-zero in every thread if a
 // signature was raised.  T (k_prop_async): the pack rows arrive by bulk copy (PackTma);
 // otherwise (k_prop_pack) by vector loads.
-template <typename Mark, bool HALO = false>
+template <typename Mark, bool HALO = false, bool TRICKS = false>
 __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__ cin, int32_t* __restrict__ cout,
                                           const unsigned long long* __restrict__ pnin,
                                           const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext,
@@ -302,7 +317,11 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
         const int2 e = __ldg(E + i);
         const int v = e.y & 0x7FFF;
         int* sig = (e.y & EXT_DIR) ? s_out : s_in;
-        const int val = ld_cg(((e.y & EXT_DIR) ? cout : cin) + e.x);
+        const int32_t* gsig = (e.y & EXT_DIR) ? cout : cin;
+        int val = ld_cg(gsig + e.x);
+        // path compression: in[in[u]] / out[out[w]] -- the signature of the vertex whose
+        // priority u carries, an ancestor (descendant) of u, so never worse than in[u]
+        if (TRICKS && g.compress) val = max(val, ld_cg(gsig + __ldg(g.slot + val)));
         if (val > ((volatile int*)sig)[v]) atomicMax(sig + v, val);
     }
     __syncthreads();
@@ -349,7 +368,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
 #endif
     {
         unsigned r0 = 0, r1 = 0, r2 = 0;
-        drain_direct(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, base, cnt, r0, r1, r2);
+        drain_direct<TRICKS>(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, base, cnt, r0, r1, r2);
 #ifdef ECL_PROF
         r2 = warp_sum(r2);
         if ((tid & 31) == 0) { PROF_ADD(dc, 2, r1); PROF_ADD(dc, 3, r2); }
@@ -436,6 +455,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
 }
 
 // Phase-2 pass over the packs (pass protocol, dirty skipping and runs as k_prop_tile)
+template <bool TRICKS>
 static __global__ void __launch_bounds__(PACK_TH, PACK_MINB)
 k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, const unsigned long long* __restrict__ pnin,
             const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext, const int* __restrict__ ext_cnt,
@@ -473,7 +493,8 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
             __syncthreads();
             if (!d) continue;
         }
-        ch_any |= pack_visit(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkNext{dirty_next}, S);
+        ch_any |= pack_visit<MarkNext, false, TRICKS>(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full,
+                                                      MarkNext{dirty_next}, S);
         __syncthreads();
     }
     if (ch_any && tid == 0) dc->changed[pass & (RING - 1)] = 1;
@@ -548,7 +569,7 @@ struct MarkSet {
     }
 };
 
-template <bool HALO>
+template <bool HALO, bool TRICKS>
 static __global__ void __launch_bounds__(PACK_TH, PACK_MINB)
 k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, const unsigned long long* __restrict__ pnin,
              const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext, const int* __restrict__ ext_cnt,
@@ -638,7 +659,7 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             const int tile = s_claim[j], full = s_seen[j] == 0;
             for (int i = tid; i < MSET; i += PACK_TH) s_set[i] = -1;
             __syncthreads();
-            pack_visit<MarkSet, HALO>(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S,
+            pack_visit<MarkSet, HALO, TRICKS>(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S,
                                       j + 1 < nclaim ? s_claim[j + 1] : -1, &T, HALO ? &H : nullptr);
             __threadfence();                                      // values before marks
             __syncthreads();

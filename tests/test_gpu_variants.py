@@ -116,3 +116,35 @@ def test_variants_c2_full_trace():
         np.testing.assert_array_equal(lab, truth, err_msg=name)
         tr = oracle.ecl_scc(og.row_ptr, og.col_idx, trim=True, **okw)
         assert st["iterations"] == tr.iterations and st["edges_in"] == tr.edges_in[:64], name
+
+
+# ----------------------------------------------------------------- f2: compression and the P:190 variant
+TRICKS = {"compress": E.COMPRESS, "raise": E.RAISE, "compress+raise": E.COMPRESS | E.RAISE}
+
+
+@pytest.mark.parametrize("name", sorted(TRICKS))
+def test_pass_count_variants_keep_the_trace(name):
+    """Path compression and the sound P:190 variant change how values travel, never
+    where Phase 2 ends (reading 12): labels, live / kept edges and every signature snapshot
+    equal O2's plain trace (O2's own compress / raise_ flags give the same trace, pinned in
+    tests/test_oracle.py)."""
+    fl = TRICKS[name]
+    rng = random.Random(len(name))
+    for trial in range(60):
+        n = rng.randrange(1, 300)
+        edges = [(rng.randrange(n), rng.randrange(n)) for _ in range(rng.randrange(0, 3 * n))]
+        g = gen.from_edges(n, edges)
+        for extra in (0, E.IDENTITY_IDS, E.NO_ASYNC, E.NO_TRIM):
+            check(g, fl | extra, {}, snaps=trial % 6 == 0)
+    for g in (gen.config("c1"), gen.mesh(24, gen.ordinate(9), seed=4, order="blocked8", **gen.C4_MESH)):
+        check(g, fl, {}, max_iters=4)
+    perm = np.random.default_rng(2).permutation(200_000)                # one long cycle
+    g = gen.from_edges(200_000, np.stack([perm, np.roll(perm, -1)], 1))
+    lab, st = run(g, fl)
+    assert (lab == 199_999).all()
+
+
+def test_pass_count_variant_flag_errors():
+    with pytest.raises(E.EclSccError) as ex:
+        E.Plan(10, 10, E.COMPRESS | E.FOUR_SIG)
+    assert ex.value.status == E.EINVAL

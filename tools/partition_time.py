@@ -1,8 +1,8 @@
 """Device time of the edge-partitioned (halo) mode with P emulated ranks on one GPU
 (development helper).  The P ranks run one after another on one device with the same kernels
 and exchange protocol as the NCCL mode (the all-reduces are reductions over the P buffers,
-the fused pushes target the P halo buffers), and each call allocates its P workspaces, so
-the time is ~ the sum of the ranks' work plus allocation -- not a multi-GPU time."""
+the fused pushes target the P halo buffers), with workspaces allocated beforehand, so the
+time is ~ the sum of the ranks' work plus the exchanges -- not a multi-GPU time."""
 import os
 import sys
 
@@ -26,9 +26,10 @@ for c in sys.argv[1:] or ["c2", "c4"]:
     print(f"{c} single GPU: {a.elapsed_time(b):.2f} ms", flush=True)
     for P in (1, 2, 4, 8):
         for fl, nm in ((0, "fused pushes"), (E.HALO_ALLREDUCE, "all-reduce exchange")):
-            E.ecl_scc_partitioned_emulated(P, rp, ci, flags=fl)
+            ep = E.EmulatedPlan(P, rp, g.nnz, fl)
+            E.ecl_scc_partitioned_emulated(P, rp, ci, flags=fl, plan=ep)
             a.record()
-            _, st = E.ecl_scc_partitioned_emulated(P, rp, ci, stats=True, flags=fl)
+            _, st = E.ecl_scc_partitioned_emulated(P, rp, ci, stats=True, flags=fl, plan=ep)
             b.record()
             torch.cuda.synchronize()
             t = a.elapsed_time(b)

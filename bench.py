@@ -448,8 +448,14 @@ def ours(args):
         "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": ck,
     }
     if comm_ms is not None:
+        info = comm.info()
         line["comm"] = {"ms_per_step": round(comm_ms, 4), "share": round(comm_ms / t_ms, 4),
-                        "bytes_per_step_rank0": int(stats["comm_bytes"]), "exchanges": int(stats["exchanges"])}
+                        "bytes_per_step_rank0": int(stats["comm_bytes"]), "exchanges": int(stats["exchanges"]),
+                        "halo_exchange": ("fused: multimem.red.max (NVLS)" if info["multimem"] else
+                                          "fused: remote atomicMax over NVLink peers" if info["device_api"] else
+                                          "ncclAllReduce(MAX) of the halo"),
+                        "note": "ms_per_step: the collectives (barriers, degree / count / label all-reduces); "
+                                "the fused halo pushes run inside k_prop_async"}
     print(json.dumps(line), flush=True)
     if comm is not None:
         comm.close()

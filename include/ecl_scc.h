@@ -96,6 +96,10 @@ typedef enum {
                                      5) -- when v_in rises to t inside a tile, t is also offered to
                                      in[out[v]] (a descendant of v) if that vertex is in the same
                                      tile; v_out likewise to out[in[v]]; single GPU */
+#define ECL_SCC_CLUSTER 0x40000u  /* variant: Phase 2 on thread-block-cluster pair tiles -- two
+                                     CTAs share one 4096-vertex block-local fixed point through
+                                     distributed shared memory (csrc/cluster.cuh); graphs
+                                     without rows longer than 64 edges, single GPU */
 #define ECL_SCC_FOUR_SIG 0x8000u  /* variant: the 4-signature method -- Phase 2 also
                                      propagates minimum ancestor / descendant IDs and Phase 3
                                      keeps an edge only if all four signatures agree; twice the

@@ -24,6 +24,7 @@
 #include "scan.cuh"
 #include "reorder.cuh"
 #include "pack.cuh"
+#include "cluster.cuh"
 #include "levels.cuh"
 #include "partition.cuh"
 #include "driver.h"
@@ -86,6 +87,7 @@ int plan_alloc(Plan* p, int32_t n_max, int64_t m_max) {
     p->knob_claim_div = knob("ECL_SCC_CLAIM_DIV", 1, 64);
     p->knob_claim_max = knob("ECL_SCC_CLAIM_MAX", 1, 32);
     p->knob_async_ctas = knob("ECL_SCC_ASYNC_CTAS", 1, 8);
+    p->knob_lv_ctas = knob("ECL_SCC_LV_CTAS", 1, 4096);
     p->lab_lo = 0;
     p->lab_hi = INT32_MAX;
     if (cudaGetDevice(&p->device) != cudaSuccess) {
@@ -288,7 +290,12 @@ static int reorder_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, con
 // Does Phase 2 of a working graph with `nchunks` long-row chunks run on tile packs?
 static bool pack_path(const Plan* p, int nchunks) {
     const bool sync = (p->flags & ECL_SCC_SYNC_PASSES) != 0 || (p->low_locality && nchunks > 0);
-    return nchunks == 0 && !sync && !(p->flags & (ECL_SCC_NO_DIRTY | ECL_SCC_NO_PACK));
+    return nchunks == 0 && !sync && !(p->flags & (ECL_SCC_NO_DIRTY | ECL_SCC_NO_PACK | ECL_SCC_CLUSTER));
+}
+// Does Phase 2 run on cluster pair tiles (cluster.cuh)?
+static bool cluster_path(const Plan* p, int nchunks) {
+    return (p->flags & ECL_SCC_CLUSTER) && nchunks == 0 &&
+           !(p->flags & (ECL_SCC_SYNC_PASSES | ECL_SCC_NO_DIRTY | ECL_SCC_NO_PACK | ECL_SCC_NO_ASYNC));
 }
 // tile pack buffers (pack.cuh), sized for the plan on first use
 static int ensure_pack(Plan* p) {
@@ -447,6 +454,44 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
     // and a local fixed point per visit (not the SYNC ablation)
     const bool use_dirty = nchunks == 0 && !sync && !(p->flags & ECL_SCC_NO_DIRTY);
     uint8_t* D[2] = {p->dirty, p->dirty + p->dirty_cap};
+    if (cluster_path(p, nchunks) && g.na > 0) {          // thread-block-cluster pair tiles (cluster.cuh)
+        if (int r = ensure_pack(p)) return r;
+        const unsigned npair = (unsigned)cdiv(g.na, PAIR_TT);
+        if (!p->aq_state) {
+            const size_t nt = (size_t)p->dirty_cap;
+            cudaError_t e = cudaMalloc((void**)&p->aq_state, nt * 4);
+            if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_seen, nt);
+            if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_ctr, AQ_WORDS * sizeof(unsigned long long));
+            if (e != cudaSuccess) {
+                cudaGetLastError();
+                return fail(ECL_SCC_ENOMEM, "async queue allocation: %s", cudaGetErrorString(e));
+            }
+            CK(cudaFuncSetAttribute(k_prop_cluster, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
+            CK(cudaFuncSetAttribute(k_prop_cluster, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                    (int)cudaSharedmemCarveoutMaxShared));
+            int per_sm = 0, sms = 0;
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_cluster, PACK_TH, pack_dyn_smem()));
+            CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device));
+            p->aq_resident = std::max<int64_t>(2, ((int64_t)std::max(1, per_sm) * sms) & ~1ll);
+        }
+        if (!second) {
+            p->launches++;
+            k_pack_pair<<<npair, PACK_TH, 0, s>>>(g, p->pnin, p->pnout, p->ext, p->ext_cnt);
+            CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
+            CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
+        }
+        AsyncQ Q{p->aq_state, p->aq_seen, p->aq_ctr};
+        const int64_t clusters = p->aq_resident / 2;
+        const int claim = p->knob_claim ? p->knob_claim : (int)std::min<int64_t>(16, std::max<int64_t>(1, npair / clusters));
+        p->launches += 2;
+        k_async_init<<<grid_for((int64_t)npair, TPB), TPB, 0, s>>>(Q, (int)npair);
+        const unsigned cgrid = (unsigned)(2 * std::min<int64_t>(npair, clusters));
+        k_prop_cluster<<<cgrid, PACK_TH, pack_dyn_smem(), s>>>(g, cin, cout, p->pnin, p->pnout, p->ext, p->ext_cnt,
+                                                               p->dc, Q, claim);
+        CK(cudaGetLastError());
+        *passes_out = -(int64_t)npair;
+        return ECL_SCC_OK;
+    }
     // tile packs (pack.cuh): the default for graphs without long rows
     const bool use_pack = pack_path(p, nchunks) && g.na > 0;
     if (use_pack) {
@@ -602,7 +647,6 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         CK(cudaStreamSynchronize(s));
         if (p->hc->err) return fail(ECL_SCC_ERANGE, "invalid CSR: offsets not monotone from 0 to nnz, or column outside [0,n)");
     }
-    const bool trim = !(p->flags & ECL_SCC_NO_TRIM);
     const Prio P = make_prio((uint32_t)n, (p->flags & ECL_SCC_IDENTITY_IDS) != 0);
     int iters = 0;
     bool stopped = false;
@@ -876,7 +920,7 @@ HaloRank::~HaloRank() {
 int halo_rank_alloc(HaloRank* R, int32_t n, int32_t rb, int32_t re, int64_t m_cap, uint32_t flags) {
     R->n = n; R->rb = rb; R->re = re; R->nloc = re - rb; R->m_cap = m_cap;
     const int64_t nl_max = std::min<int64_t>((int64_t)R->nloc + m_cap, n);
-    if (flags & (ECL_SCC_TRIM2 | ECL_SCC_FOUR_SIG | ECL_SCC_COMPRESS | ECL_SCC_RAISE))
+    if (flags & (ECL_SCC_TRIM2 | ECL_SCC_FOUR_SIG | ECL_SCC_COMPRESS | ECL_SCC_RAISE | ECL_SCC_CLUSTER))
         return fail(ECL_SCC_EUNSUPPORTED, "partitioned mode: Trim-2, the 4-signature variant, path compression and "
                                           "the P:190 variant are single-GPU only");
     R->p.flags = flags | ECL_SCC_NO_REORDER;       // the local -> global map is the storage map
@@ -1184,6 +1228,7 @@ int run_levels(Plan* p, int32_t n, const int32_t* rp, const int32_t* ci, const i
         CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
         // one CTA per SM: the round barrier's cost grows with the CTAs that arrive at it
         p->lv_resident = std::max(1, std::min(per_sm, 1)) * sms;
+        if (p->knob_lv_ctas) p->lv_resident = std::min(p->lv_resident, p->knob_lv_ctas);   // tuning knob
     }
     LvCtl* ctl = (LvCtl*)p->lv_ctl;
     int32_t* indeg = p->kin;
@@ -1272,9 +1317,10 @@ int ecl_scc_plan_create(int32_t n_max, int64_t nnz_max, uint32_t flags, ecl_scc_
     if (nnz_max >= (int64_t)INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "nnz_max >= 2^31");
     ecl_scc_plan_s* h = (ecl_scc_plan_s*)calloc(1, sizeof(ecl_scc_plan_s));
     if (!h) return fail(ECL_SCC_ENOMEM, "host allocation");
-    if ((flags & (ECL_SCC_COMPRESS | ECL_SCC_RAISE)) && (flags & ECL_SCC_FOUR_SIG)) {
+    if ((flags & (ECL_SCC_COMPRESS | ECL_SCC_RAISE)) && (flags & (ECL_SCC_FOUR_SIG | ECL_SCC_CLUSTER))) {
         free(h);
-        return fail(ECL_SCC_EINVAL, "plan_create: ECL_SCC_COMPRESS / ECL_SCC_RAISE apply to the two-signature method");
+        return fail(ECL_SCC_EINVAL, "plan_create: ECL_SCC_COMPRESS / ECL_SCC_RAISE apply to the two-signature, "
+                                    "single-CTA-tile method");
     }
     if ((flags & ECL_SCC_TRIM2) && (flags & ECL_SCC_NO_TRIM)) {
         free(h);

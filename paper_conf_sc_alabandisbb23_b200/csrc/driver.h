@@ -64,7 +64,7 @@ struct Plan {
     // tuning knobs, read from the environment once when the plan is created (development
     // only; the defaults are the measured best): ECL_SCC_RUN, ECL_SCC_CLAIM,
     // ECL_SCC_CLAIM_DIV, ECL_SCC_CLAIM_MAX, ECL_SCC_ASYNC_CTAS
-    int knob_run, knob_claim, knob_claim_div, knob_claim_max, knob_async_ctas;
+    int knob_run, knob_claim, knob_claim_div, knob_claim_max, knob_async_ctas, knob_lv_ctas;
     void* lv_ctl;                        // levels.cuh LvCtl (device)
     int32_t *h_rp, *h_ci, *h_lab;        // ecl_scc_host: device copies of the caller's host buffers
     int64_t h_n_cap, h_m_cap;

@@ -148,3 +148,28 @@ def test_pass_count_variant_flag_errors():
     with pytest.raises(E.EclSccError) as ex:
         E.Plan(10, 10, E.COMPRESS | E.FOUR_SIG)
     assert ex.value.status == E.EINVAL
+
+
+# ----------------------------------------------------------------- f2: thread-block-cluster pair tiles
+def test_cluster_pair_tiles_keep_the_trace():
+    """ECL_SCC_CLUSTER: two CTAs share one 4096-vertex block-local fixed point through DSMEM
+    (csrc/cluster.cuh).  Only the schedule changes (reading 12): labels bit-exact, live / kept
+    edges and every signature snapshot equal O2's trace -- on graphs spanning many pair tiles,
+    so that both halves and the remote (DSMEM) slots are exercised."""
+    rng = random.Random(4096)
+    for trial in range(30):
+        n = rng.randrange(1, 12_000) if trial % 3 else rng.randrange(1, 300)
+        k = rng.randrange(0, 3 * n)
+        src = np.array([rng.randrange(n) for _ in range(k)], dtype=np.int64)
+        # mostly local edges (so pair tiles hold real intra- and cross-half work)
+        dst = np.clip(src + np.array([rng.randrange(-3000, 3000) for _ in range(k)], dtype=np.int64), 0, n - 1)
+        g = gen.from_edges(n, np.stack([src, dst], 1) if k else [])
+        for extra in (0, E.IDENTITY_IDS, E.NO_TRIM):
+            check(g, E.CLUSTER | extra, {}, snaps=trial % 5 == 0, max_iters=3)
+    for g in (gen.config("c1"), gen.mesh(24, gen.ordinate(9), seed=4, order="blocked8", **gen.C4_MESH),
+              gen.mesh(20, gen.ordinate(30), seed=8, order="lex", **gen.C4_MESH)):
+        check(g, E.CLUSTER, {}, max_iters=4)
+    check(gen.mesh(16, gen.ordinate(2), seed=3, **gen.C4_MESH), E.CLUSTER | E.FOUR_SIG, dict(four=True), max_iters=2)
+    g = gen.config("c2", order="blocked8")
+    lab, st = run(g, E.CLUSTER)
+    np.testing.assert_array_equal(lab, oracle.tarjan_labels(g.row_ptr, g.col_idx))

@@ -261,6 +261,13 @@ int ecl_scc_partitioned_emulated(int32_t P, int32_t n, int64_t nnz, const int32_
  * reductions.  Filled after the first ecl_scc_partitioned call. */
 int ecl_scc_comm_info(ecl_scc_comm_t comm, int32_t info[4]);
 
+/* Diagnostics of the NVLS path of the fused halo exchange on the current device alone: a
+ * one-device multicast object (cuMulticastCreate) bound to a buffer, the partitioned mode's
+ * push kernel reducing into it through the multicast address with multimem.red.max, the
+ * unicast view checked.  *checked = number of entries verified.  EUNSUPPORTED if the device
+ * (or driver) has no multicast support. */
+int ecl_scc_multimem_probe(int32_t* checked);
+
 /* Host helper: split rows [0,n) into P contiguous ranges of about equal edge count
  * (binary search on the host row_ptr[n+1]); bounds_out[P+1] (host). */
 int ecl_scc_partition_rows(int32_t P, int32_t n, const int32_t* row_ptr_host, int32_t* bounds_out);

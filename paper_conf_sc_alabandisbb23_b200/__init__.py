@@ -83,6 +83,7 @@ def lib() -> ctypes.CDLL:
         "ecl_scc_emulated_plan_create": [i32, i32, i64, vp, u32, vp],
         "ecl_scc_emulated_plan_destroy": [vp],
         "ecl_scc_comm_info": [vp, vp],
+        "ecl_scc_multimem_probe": [vp],
         "ecl_scc_partition_rows": [i32, i32, vp, vp],
         "ecl_scc_status_string": [ctypes.c_int],
         "ecl_scc_last_error": [],
@@ -108,7 +109,7 @@ ABI_SYMBOLS = ("ecl_scc", "ecl_scc_async", "ecl_scc_debug_run", "ecl_scc_plan_cr
                "ecl_scc_partitioned_emulated", "ecl_scc_partition_rows", "ecl_scc_status_string",
                "ecl_scc_last_error", "ecl_scc_version", "ecl_scc_plan_counters", "ecl_scc_levels",
                "ecl_scc_host", "ecl_scc_part_plan_create", "ecl_scc_part_plan_destroy", "ecl_scc_comm_info",
-               "ecl_scc_emulated_plan_create", "ecl_scc_emulated_plan_destroy")
+               "ecl_scc_emulated_plan_create", "ecl_scc_emulated_plan_destroy", "ecl_scc_multimem_probe")
 
 
 def status_string(s: int) -> str:
@@ -283,6 +284,14 @@ def ecl_scc_partitioned_emulated(P: int, row_ptr, col_idx, labels_out=None, stre
                                               plan.handle if plan else None,
                                               ctypes.byref(st) if st else None), "ecl_scc_partitioned_emulated")
     return (labels_out, st.as_dict()) if stats else labels_out
+
+
+def multimem_probe() -> int:
+    """Run ecl_scc_multimem_probe: the NVLS multimem push path on this device alone (raises
+    EclSccError with status EUNSUPPORTED when the device has no multicast support)."""
+    n = ctypes.c_int32(0)
+    _check(lib().ecl_scc_multimem_probe(ctypes.byref(n)), "ecl_scc_multimem_probe")
+    return int(n.value)
 
 
 def get_unique_id() -> bytes:

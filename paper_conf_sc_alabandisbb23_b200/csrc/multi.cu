@@ -14,6 +14,7 @@
 //     buffer is combined by ncclAllReduce(MAX) instead (the baseline).
 //   * EmulatedExchange -- P ranks in one process on one device (tests): reductions over the
 //     P buffers, pushes into the P buffers of the same device.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <nccl.h>
 #include <nccl_device.h>
@@ -204,6 +205,19 @@ struct ecl_scc_emulated_plan_s {
     }
 };
 
+// driver-API entry points through the runtime (no link-time dependency on libcuda)
+template <typename F>
+static F drv(const char* name) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint(name, &fn, cudaEnableDefault, &q) != cudaSuccess || q != cudaDriverEntryPointSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    return (F)fn;
+}
+#define ECL_DRV(name) auto name = drv<decltype(&::name)>(#name)
+
 // per-rank workspace of the partitioned mode: allocated once, reused by every call
 struct ecl_scc_part_plan_s {
     HaloRank R;
@@ -264,6 +278,108 @@ int ecl_scc_comm_info(ecl_scc_comm_t comm, int32_t info[4]) {
     info[2] = comm->dev_ok ? 1 : 0;
     info[3] = comm->multimem ? 1 : 0;
     return ECL_SCC_OK;
+}
+
+// One-device multicast object bound to a buffer; k_halo_push (the partitioned mode's push
+// code) reduces into it through the multicast address with multimem.red.max, and the unicast
+// view is checked.  Exercises the NVLS path of the fused halo exchange on a single GPU.
+int ecl_scc_multimem_probe(int32_t* checked) {
+    clear_err();
+    if (checked) *checked = 0;
+    int dev = 0;
+    CKM(cudaGetDevice(&dev));
+    CKM(cudaFree(nullptr));                                   // a current context
+    ECL_DRV(cuDeviceGetAttribute);
+    ECL_DRV(cuMulticastGetGranularity);
+    ECL_DRV(cuMulticastCreate);
+    ECL_DRV(cuMulticastAddDevice);
+    ECL_DRV(cuMemCreate);
+    ECL_DRV(cuMulticastBindMem);
+    ECL_DRV(cuMemAddressReserve);
+    ECL_DRV(cuMemMap);
+    ECL_DRV(cuMemSetAccess);
+    ECL_DRV(cuMemUnmap);
+    ECL_DRV(cuMemAddressFree);
+    ECL_DRV(cuMulticastUnbind);
+    ECL_DRV(cuMemRelease);
+    if (!cuDeviceGetAttribute || !cuMulticastGetGranularity || !cuMulticastCreate || !cuMulticastAddDevice ||
+        !cuMemCreate || !cuMulticastBindMem || !cuMemAddressReserve || !cuMemMap || !cuMemSetAccess || !cuMemUnmap ||
+        !cuMemAddressFree || !cuMulticastUnbind || !cuMemRelease)
+        return fail(ECL_SCC_EUNSUPPORTED, "multimem_probe: driver entry points unavailable");
+    int mc_ok = 0;
+    if (cuDeviceGetAttribute(&mc_ok, CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED, dev) != CUDA_SUCCESS || !mc_ok)
+        return fail(ECL_SCC_EUNSUPPORTED, "multimem_probe: the device has no multicast support");
+    constexpr int H = 1 << 16;                                // halo entries (2 ints each)
+    CUmulticastObjectProp mp = {};
+    mp.numDevices = 1;
+    mp.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+    size_t gran = 0;
+    mp.size = 2 * H * sizeof(int32_t);
+    if (cuMulticastGetGranularity(&gran, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED) != CUDA_SUCCESS)
+        return fail(ECL_SCC_EUNSUPPORTED, "multimem_probe: cuMulticastGetGranularity failed");
+    const size_t size = (mp.size + gran - 1) / gran * gran;
+    mp.size = size;
+    CUmemGenericAllocationHandle mc = 0, mem = 0;
+    CUdeviceptr uc_ptr = 0, mc_ptr = 0;
+    int rc = ECL_SCC_OK;
+    CUmemAllocationProp ap = {};
+    ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+    ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+    ap.location.id = dev;
+    ap.requestedHandleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+    CUmemAccessDesc acc = {};
+    acc.location = ap.location;
+    acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+    int32_t *hpos = nullptr, *cin = nullptr, *cout = nullptr;
+    std::vector<int32_t> h(2 * (size_t)H);
+    if (cuMulticastCreate(&mc, &mp) != CUDA_SUCCESS || cuMulticastAddDevice(mc, dev) != CUDA_SUCCESS ||
+        cuMemCreate(&mem, size, &ap, 0) != CUDA_SUCCESS || cuMulticastBindMem(mc, 0, mem, 0, size, 0) != CUDA_SUCCESS ||
+        cuMemAddressReserve(&uc_ptr, size, gran, 0, 0) != CUDA_SUCCESS || cuMemMap(uc_ptr, size, 0, mem, 0) != CUDA_SUCCESS ||
+        cuMemSetAccess(uc_ptr, size, &acc, 1) != CUDA_SUCCESS ||
+        cuMemAddressReserve(&mc_ptr, size, gran, 0, 0) != CUDA_SUCCESS || cuMemMap(mc_ptr, size, 0, mc, 0) != CUDA_SUCCESS ||
+        cuMemSetAccess(mc_ptr, size, &acc, 1) != CUDA_SUCCESS) {
+        rc = fail(ECL_SCC_EUNSUPPORTED, "multimem_probe: multicast object setup failed");
+    }
+    if (!rc && (cudaMalloc((void**)&hpos, H * 4) != cudaSuccess || cudaMalloc((void**)&cin, H * 4) != cudaSuccess ||
+                cudaMalloc((void**)&cout, H * 4) != cudaSuccess))
+        rc = fail(ECL_SCC_ENOMEM, "multimem_probe: buffers");
+    if (!rc) {
+        // entry p receives max(in) = 3p + 1 over two pushes (3p, then 3p + 1) and out = 5p + 2
+        std::vector<int32_t> hp(H), a(H), b(H);
+        for (int p = 0; p < H; p++) hp[p] = H - 1 - p;       // local vertex i -> halo position H-1-i
+        cudaMemcpy(hpos, hp.data(), H * 4, cudaMemcpyHostToDevice);
+        cudaMemset((void*)uc_ptr, 0, size);
+        HaloPush P{};
+        P.hpos = hpos;
+        P.mc = (int32_t*)mc_ptr;
+        P.sys = 1;
+        for (int round = 0; round < 2 && !rc; round++) {
+            for (int i = 0; i < H; i++) {
+                const int p = hp[i];
+                a[i] = round ? 3 * p + 1 : 3 * p;
+                b[i] = round ? 5 * p : 5 * p + 2;
+            }
+            cudaMemcpy(cin, a.data(), H * 4, cudaMemcpyHostToDevice);
+            cudaMemcpy(cout, b.data(), H * 4, cudaMemcpyHostToDevice);
+            k_halo_push<<<(H + 255) / 256, 256>>>(H, cin, cout, P);
+            if (cudaDeviceSynchronize() != cudaSuccess) rc = fail(ECL_SCC_ECUDA, "multimem_probe: push kernel failed");
+        }
+        if (!rc) {
+            cudaMemcpy(h.data(), (void*)uc_ptr, 2 * (size_t)H * 4, cudaMemcpyDeviceToHost);
+            for (int p = 0; p < H && !rc; p++)
+                if (h[2 * (size_t)p] != 3 * p + 1 || h[2 * (size_t)p + 1] != 5 * p + 2)
+                    rc = fail(ECL_SCC_ECUDA, "multimem_probe: entry %d holds (%d, %d), expected (%d, %d)", p,
+                              h[2 * (size_t)p], h[2 * (size_t)p + 1], 3 * p + 1, 5 * p + 2);
+            if (!rc && checked) *checked = H;
+        }
+    }
+    cudaFree(hpos); cudaFree(cin); cudaFree(cout);
+    if (mc_ptr) { cuMemUnmap(mc_ptr, size); cuMemAddressFree(mc_ptr, size); }
+    if (uc_ptr) { cuMemUnmap(uc_ptr, size); cuMemAddressFree(uc_ptr, size); }
+    if (mc) { cuMulticastUnbind(mc, dev, 0, size); cuMemRelease(mc); }
+    if (mem) cuMemRelease(mem);
+    cudaGetLastError();
+    return rc;
 }
 
 int ecl_scc_part_plan_create(int32_t n, int32_t row_begin, int32_t row_end, int64_t local_nnz_max, uint32_t flags,

@@ -124,3 +124,17 @@ def test_emulated_long_local_phases():
             exp = np.arange(n)
             exp[cyc] = cyc.max()
             np.testing.assert_array_equal(lab, exp, err_msg=f"L={L} P={P}")
+
+
+def test_multimem_probe_nvls_push_path():
+    """The NVLS branch of the fused halo exchange (multimem.red.max through a multicast
+    address, halo.cuh halo_push_one) on this device alone: a one-device multicast object bound
+    to a buffer, the push kernel reducing two rounds of values into it, the unicast view equal
+    to the expected maxima.  Skipped where the device has no multicast support."""
+    try:
+        n = E.multimem_probe()
+    except E.EclSccError as ex:
+        if ex.status == E.EUNSUPPORTED:
+            pytest.skip(str(ex))
+        raise
+    assert n == 1 << 16

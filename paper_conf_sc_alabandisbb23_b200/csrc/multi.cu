@@ -332,13 +332,26 @@ int ecl_scc_multimem_probe(int32_t* checked) {
     acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
     int32_t *hpos = nullptr, *cin = nullptr, *cout = nullptr;
     std::vector<int32_t> h(2 * (size_t)H);
-    if (cuMulticastCreate(&mc, &mp) != CUDA_SUCCESS || cuMulticastAddDevice(mc, dev) != CUDA_SUCCESS ||
-        cuMemCreate(&mem, size, &ap, 0) != CUDA_SUCCESS || cuMulticastBindMem(mc, 0, mem, 0, size, 0) != CUDA_SUCCESS ||
-        cuMemAddressReserve(&uc_ptr, size, gran, 0, 0) != CUDA_SUCCESS || cuMemMap(uc_ptr, size, 0, mem, 0) != CUDA_SUCCESS ||
-        cuMemSetAccess(uc_ptr, size, &acc, 1) != CUDA_SUCCESS ||
-        cuMemAddressReserve(&mc_ptr, size, gran, 0, 0) != CUDA_SUCCESS || cuMemMap(mc_ptr, size, 0, mc, 0) != CUDA_SUCCESS ||
-        cuMemSetAccess(mc_ptr, size, &acc, 1) != CUDA_SUCCESS) {
-        rc = fail(ECL_SCC_EUNSUPPORTED, "multimem_probe: multicast object setup failed");
+    {
+        int step = 0;
+        CUresult cr = CUDA_SUCCESS;
+        auto ok = [&](CUresult r) { step++; cr = r; return r == CUDA_SUCCESS; };
+        // the exportable handle type a multicast object accepts depends on the platform: try
+        // none, a POSIX file descriptor, then a fabric handle
+        const CUmemAllocationHandleType types[3] = {CU_MEM_HANDLE_TYPE_NONE, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR,
+                                                    CU_MEM_HANDLE_TYPE_FABRIC};
+        for (int k = 0; k < 3 && mc == 0; k++) {
+            mp.handleTypes = types[k];
+            ap.requestedHandleTypes = types[k];
+            if (cuMulticastCreate(&mc, &mp) != CUDA_SUCCESS) mc = 0;
+        }
+        if (!(ok(mc ? CUDA_SUCCESS : CUDA_ERROR_NOT_SUPPORTED) && ok(cuMulticastAddDevice(mc, dev)) && ok(cuMemCreate(&mem, size, &ap, 0)) &&
+              ok(cuMulticastBindMem(mc, 0, mem, 0, size, 0)) && ok(cuMemAddressReserve(&uc_ptr, size, gran, 0, 0)) &&
+              ok(cuMemMap(uc_ptr, size, 0, mem, 0)) && ok(cuMemSetAccess(uc_ptr, size, &acc, 1)) &&
+              ok(cuMemAddressReserve(&mc_ptr, size, gran, 0, 0)) && ok(cuMemMap(mc_ptr, size, 0, mc, 0)) &&
+              ok(cuMemSetAccess(mc_ptr, size, &acc, 1))))
+            rc = fail(ECL_SCC_EUNSUPPORTED, "multimem_probe: multicast setup step %d failed (CUresult %d; size %zu, granularity %zu)",
+                      step, (int)cr, size, gran);
     }
     if (!rc && (cudaMalloc((void**)&hpos, H * 4) != cudaSuccess || cudaMalloc((void**)&cin, H * 4) != cudaSuccess ||
                 cudaMalloc((void**)&cout, H * 4) != cudaSuccess))

@@ -23,6 +23,11 @@ VARIANTS = [
     ("raw vertex IDs instead of priorities (the paper's signatures)", E.IDENTITY_IDS),
     ("no Trim-1 (P:83)", E.NO_TRIM),
     ("no storage reordering", E.NO_REORDER),
+    ("+ Trim-2 (P:83)", E.TRIM2),
+    ("+ 4 signatures (P:194)", E.FOUR_SIG),
+    ("+ path compression (P:188)", E.COMPRESS),
+    ("+ sound P:190 variant", E.RAISE),
+    ("+ cluster pair tiles (DSMEM)", E.CLUSTER),
 ]
 
 
@@ -49,12 +54,13 @@ def time_one(g, flags, reps=3, budget_ms=4000.0):
 if __name__ == "__main__":
     cfgs = sys.argv[1:] or ["c2", "c3", "c4"]
     for c in cfgs:
-        g = gen.config(c)
+        # c2 / c4: lexicographic element IDs; c2b / c4b: 8^3-blocked (the bench default)
+        g = gen.config(c[:2], order="blocked8") if c.endswith("b") else gen.config(c)
         base = None
         print(f"== {c}: n={g.n} nnz={g.nnz} ({g.name})", flush=True)
         for name, fl in VARIANTS:
-            if c == "c3" and fl == E.NO_REORDER:
-                continue                      # long rows: neither applies
+            if c == "c3" and fl in (E.NO_REORDER, E.CLUSTER, E.COMPRESS, E.RAISE):
+                continue                      # long rows: pass mode, these do not apply
             t, st = time_one(g, fl)
             base = base or t
             print(f"  {name:70s} {t:9.2f} ms  {g.nnz / t / 1e3:8.1f} Me/s  x{base / t:5.2f}  "

@@ -38,6 +38,11 @@ static_assert(PACK_TT == 0x800, "PSLOTS_EMPTY encodes PACK_TT");
 static_assert(PK_EMPTY == PSLOTS_EMPTY && PK_DIR == (int)EXT_DIR && PK_SLOW == SLOW_MARK && PACK_TT == TILE,
               "the compaction scatter writes the same pack layout (kernels.cuh PackOut)");
 
+// tile layout in dynamic shared memory (s_in, s_out with a sentinel entry each, then the slot
+// words) and the flag block (s_fin, s_fout, each with the sentinel's scratch word)
+constexpr unsigned PK_OFF_OUT = (PACK_TT + 4) * 4, PK_OFF_NIN = 2 * (PACK_TT + 4) * 4,
+                   PK_OFF_NOUT = PK_OFF_NIN + PACK_TT * 8, PK_OFF_FOUT = (PACK_TH + 1) * 4;
+__device__ __forceinline__ unsigned smem_addr(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ int ppull(const int* sig, unsigned long long src, int val) {
     const unsigned lo = (unsigned)src, hi = (unsigned)(src >> 32);
     const volatile int* s = (const volatile int*)sig;
@@ -51,6 +56,37 @@ __device__ __forceinline__ void pnotify(unsigned long long nb, uint8_t* f) {
     x[lo >> 16] = 1;
     x[hi & 0xFFFFu] = 1;
     x[(hi >> 16) & 0x7FFFu] = 1;
+}
+// the same on 32-bit shared-window addresses (the drain's hot loop: no generic-to-shared
+// conversion per access)
+__device__ __forceinline__ int lds_v(unsigned a) {
+    int v;
+    asm volatile("ld.volatile.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long lds_v64(unsigned a) {
+    unsigned long long v;
+    asm volatile("ld.volatile.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+    return v;
+}
+__device__ __forceinline__ void sts_v(unsigned a, int v) {
+    asm volatile("st.volatile.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sts_b1(unsigned a) {
+    asm volatile("st.volatile.shared.u8 [%0], %1;" ::"r"(a), "h"((unsigned short)1) : "memory");
+}
+__device__ __forceinline__ int ppull_a(unsigned sig, unsigned long long src, int val) {
+    const unsigned lo = (unsigned)src, hi = (unsigned)(src >> 32);
+    const int a = lds_v(sig + 4 * (lo & 0xFFFFu)), b = lds_v(sig + 4 * (lo >> 16));
+    const int c = lds_v(sig + 4 * (hi & 0xFFFFu)), d = lds_v(sig + 4 * ((hi >> 16) & 0x7FFFu));
+    return max(max(val, a), max(b, max(c, d)));
+}
+__device__ __forceinline__ void pnotify_a(unsigned long long nb, unsigned f) {
+    const unsigned lo = (unsigned)nb, hi = (unsigned)(nb >> 32);
+    sts_b1(f + (lo & 0xFFFFu));
+    sts_b1(f + (lo >> 16));
+    sts_b1(f + (hi & 0xFFFFu));
+    sts_b1(f + ((hi >> 16) & 0x7FFFu));
 }
 // the rest of a slow row (more than SLOTS intra-tile neighbours): walk the global row
 __device__ __noinline__ int pull_slow(const int* sig, const int32_t* __restrict__ ptr, const int32_t* __restrict__ adj,
@@ -86,6 +122,36 @@ __device__ __forceinline__ unsigned gather4(unsigned w) {      // byte k (0/1) -
 // every round free of a serial item loop whose length is the warp's maximum (18.5 -> 17.1 ms
 // -> 15.2 ms with the packs from the scatter).  A warp leaves its rounds when none of its
 // lanes has a flag left; the block rounds end when a whole block round found nothing.
+// one drain item: vertex v, direction DOUT (v_out pulls from the out-neighbours and flags the
+// in-neighbours; v_in the reverse), on 32-bit shared-window addresses
+template <bool DOUT, bool TRICKS>
+__device__ __forceinline__ void drain_item(const WGraph& g, int* __restrict__ s_sig, const int* __restrict__ s_other,
+                                           const unsigned long long* __restrict__ s_src,
+                                           const unsigned long long* __restrict__ s_dep, unsigned* __restrict__ s_f,
+                                           unsigned a_sig, unsigned a_src, unsigned a_dep, unsigned a_f, int base,
+                                           int cnt, int v, int tid, unsigned keep) {
+    atomicAnd(s_f + tid, keep);
+    const unsigned long long src = lds_v64(a_src + 8 * v);
+    const int old = lds_v(a_sig + 4 * v);
+    int val = ppull_a(a_sig, src, old);
+    if (src & SLOW_MARK) val = pull_slow(s_sig, DOUT ? g.optr : g.iptr, DOUT ? g.oadj : g.iadj, base, cnt, v, val);
+    if (val > old) {
+        sts_v(a_sig + 4 * v, val);
+        asm volatile("fence.acq_rel.cta;" ::: "memory");       // the value before the flags
+        const unsigned long long nb = lds_v64(a_dep + 8 * v);
+        pnotify_a(nb, a_f);
+        if (nb & SLOW_MARK) notify_slow(DOUT ? g.iptr : g.optr, DOUT ? g.iadj : g.oadj, base, cnt, v, (uint8_t*)s_f);
+        if (TRICKS && g.raise_) {
+            // sound P:190: out[in[v]] (an ancestor) for v_out, in[out[v]] (a descendant) for v_in
+            const int L = __ldg(g.slot + ((volatile const int*)s_other)[v]) - base;
+            if ((unsigned)L < (unsigned)cnt && L != v && atomicMax(s_sig + L, val) < val) {
+                __threadfence_block();
+                pnotify_full(s_dep[L], DOUT ? g.iptr : g.optr, DOUT ? g.iadj : g.oadj, base, cnt, L, (uint8_t*)s_f);
+            }
+        }
+    }
+}
+
 template <bool TRICKS = false>
 __device__ __forceinline__ void drain_direct(const WGraph& g, int* __restrict__ s_in, int* __restrict__ s_out,
                                              const unsigned long long* __restrict__ s_nin,
@@ -95,6 +161,13 @@ __device__ __forceinline__ void drain_direct(const WGraph& g, int* __restrict__ 
                                              unsigned& prof_pushes) {
     const int tid = threadIdx.x;
     const int v0 = tid * VPT;
+    // two base registers (the tile layout and the flag words are each one block; see the
+    // kernels): every other address is a constant offset, so the loop does not rebuild
+    // shared-window addresses per access
+    // (through a shuffle: ptxas would otherwise re-derive them from the CTA id before each use)
+    const unsigned a_in = __shfl_sync(FULL, smem_addr(s_in), 0), a_fin = __shfl_sync(FULL, smem_addr(s_fin), 0);
+    const unsigned a_out = a_in + PK_OFF_OUT, a_nin = a_in + PK_OFF_NIN, a_nout = a_in + PK_OFF_NOUT;
+    const unsigned a_fout = a_fin + PK_OFF_FOUT;
     for (;;) {
         int worked = 0;
 #ifdef ECL_PROF
@@ -104,7 +177,7 @@ __device__ __forceinline__ void drain_direct(const WGraph& g, int* __restrict__ 
 #ifdef ECL_PROF
             if ((tid & 31) == 0) prof_drains++;
 #endif
-            const unsigned wi = ((volatile unsigned*)s_fin)[tid], wo = ((volatile unsigned*)s_fout)[tid];
+            const unsigned wi = (unsigned)lds_v(a_fin + 4 * tid), wo = (unsigned)lds_v(a_fout + 4 * tid);
             const unsigned items = gather4(wi) | (gather4(wo) << 4);
             if (!__any_sync(FULL, items != 0)) break;
             if (items) {
@@ -115,43 +188,12 @@ __device__ __forceinline__ void drain_direct(const WGraph& g, int* __restrict__ 
                 const int bit = __ffs(items) - 1;
                 const int v = v0 + (bit & 3);
                 const unsigned keep = ~(0xFFu << (8 * (bit & 3)));
-                if (bit & 4) {                                   // v_out from the out-neighbours
-                    atomicAnd(s_fout + tid, keep);
-                    const unsigned long long src = s_nout[v];
-                    const int old = ((volatile int*)s_out)[v];
-                    int val = ppull(s_out, src, old);
-                    if (src & SLOW_MARK) val = pull_slow(s_out, g.optr, g.oadj, base, cnt, v, val);
-                    if (val > old) {
-                        ((volatile int*)s_out)[v] = val;
-                        __threadfence_block();
-                        pnotify_full(s_nin[v], g.iptr, g.iadj, base, cnt, v, (uint8_t*)s_fout);
-                        if (TRICKS && g.raise_) {                // sound P:190: out[in[v]] (an ancestor)
-                            const int L = __ldg(g.slot + ((volatile int*)s_in)[v]) - base;
-                            if ((unsigned)L < (unsigned)cnt && L != v && atomicMax(s_out + L, val) < val) {
-                                __threadfence_block();
-                                pnotify_full(s_nin[L], g.iptr, g.iadj, base, cnt, L, (uint8_t*)s_fout);
-                            }
-                        }
-                    }
-                } else {                                         // v_in from the in-neighbours
-                    atomicAnd(s_fin + tid, keep);
-                    const unsigned long long src = s_nin[v];
-                    const int old = ((volatile int*)s_in)[v];
-                    int val = ppull(s_in, src, old);
-                    if (src & SLOW_MARK) val = pull_slow(s_in, g.iptr, g.iadj, base, cnt, v, val);
-                    if (val > old) {
-                        ((volatile int*)s_in)[v] = val;
-                        __threadfence_block();
-                        pnotify_full(s_nout[v], g.optr, g.oadj, base, cnt, v, (uint8_t*)s_fin);
-                        if (TRICKS && g.raise_) {                // sound P:190: in[out[v]] (a descendant)
-                            const int L = __ldg(g.slot + ((volatile int*)s_out)[v]) - base;
-                            if ((unsigned)L < (unsigned)cnt && L != v && atomicMax(s_in + L, val) < val) {
-                                __threadfence_block();
-                                pnotify_full(s_nout[L], g.optr, g.oadj, base, cnt, L, (uint8_t*)s_fin);
-                            }
-                        }
-                    }
-                }
+                if (bit & 4)
+                    drain_item<true, TRICKS>(g, s_out, s_in, s_nout, s_nin, s_fout, a_out, a_nout, a_nin, a_fout, base,
+                                             cnt, v, tid, keep);
+                else
+                    drain_item<false, TRICKS>(g, s_in, s_out, s_nin, s_nout, s_fin, a_in, a_nin, a_nout, a_fin, base,
+                                              cnt, v, tid, keep);
             }
             __syncwarp();
         }
@@ -462,7 +504,9 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
             DevCounters* __restrict__ dc, int pass, int first, uint8_t* __restrict__ dirty_cur,
             uint8_t* __restrict__ dirty_next, int full, int run) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ unsigned s_fin[PACK_TH + 1], s_fout[PACK_TH + 1];      // + the sentinel's scratch byte
+    __shared__ unsigned s_flags[2 * (PACK_TH + 1)];                   // s_fin, s_fout (+ the sentinel's scratch byte)
+    unsigned* s_fin = s_flags;
+    unsigned* s_fout = s_flags + PACK_TH + 1;
     __shared__ int s_dirty;
     TileSmem<PACK_TT> S;
     S.s_in = (int*)smem_raw;                                          // [PACK_TT] + sentinel
@@ -575,7 +619,9 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
              const unsigned long long* __restrict__ pnout, const int2* __restrict__ ext, const int* __restrict__ ext_cnt,
              DevCounters* __restrict__ dc, AsyncQ Q, int claim, const __grid_constant__ HaloPush H) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ unsigned s_fin[PACK_TH + 1], s_fout[PACK_TH + 1];
+    __shared__ unsigned s_flags[2 * (PACK_TH + 1)];                   // s_fin, s_fout (drain_direct layout)
+    unsigned* s_fin = s_flags;
+    unsigned* s_fout = s_flags + PACK_TH + 1;
     __shared__ int s_set[MSET];
     __shared__ int s_claim[CLAIM_MAX], s_nclaim;
     __shared__ uint8_t s_seen[CLAIM_MAX];

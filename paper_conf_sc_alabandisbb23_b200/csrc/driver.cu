@@ -439,6 +439,32 @@ static int launch_tile(Plan* p, bool sync, const WGraph& g, int32_t* cin, int32_
     return ECL_SCC_OK;
 }
 
+// the asynchronous Phase-2 queue (pack.cuh AsyncQ) and k_prop_async's launch attributes, on first use
+static int ensure_async(Plan* p) {
+    if (p->aq_state) return ECL_SCC_OK;
+    const size_t nt = (size_t)p->dirty_cap;
+    cudaError_t e = cudaMalloc((void**)&p->aq_state, nt * 4);
+    if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_seen, nt);
+    if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_ctr, AQ_WORDS * sizeof(unsigned long long));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ECL_SCC_ENOMEM, "async queue allocation: %s", cudaGetErrorString(e));
+    }
+    for (auto kf : {k_prop_async<false, false>, k_prop_async<true, false>, k_prop_async<false, true>}) {
+        CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
+        CK(cudaFuncSetAttribute(kf, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                (int)cudaSharedmemCarveoutMaxShared));
+    }
+    int per_sm = 0, sms = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_async<false, false>, PACK_TH, pack_dyn_smem()));
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device));
+    // resident CTAs per SM used (<= what fits); measured best: all of them
+    if (p->knob_async_ctas) per_sm = std::min(per_sm, p->knob_async_ctas);
+    p->aq_resident = (int64_t)std::max(1, per_sm) * sms;
+    if (getenv("ECL_SCC_DEBUG")) fprintf(stderr, "[ecl_scc] k_prop_async: %d CTAs per SM\n", per_sm);
+    return ECL_SCC_OK;
+}
+
 // a4-a6: Phase 2 to its fixed point.  Passes are enqueued in growing batches; a pass
 // whose predecessor changed nothing exits at once, so over-enqueueing costs only a launch.
 // second: a second fixed point over the same graph (the minimum pair); push: the
@@ -502,28 +528,7 @@ static int propagate(Plan* p, const WGraph& g, int32_t* cin, int32_t* cout, int 
         }
         CK(cudaGetLastError());
         if (!(p->flags & ECL_SCC_NO_ASYNC)) {          // one persistent launch (pack.cuh)
-            if (!p->aq_state) {
-                const size_t nt = (size_t)p->dirty_cap;
-                cudaError_t e = cudaMalloc((void**)&p->aq_state, nt * 4);
-                if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_seen, nt);
-                if (e == cudaSuccess) e = cudaMalloc((void**)&p->aq_ctr, AQ_WORDS * sizeof(unsigned long long));
-                if (e != cudaSuccess) {
-                    cudaGetLastError();
-                    return fail(ECL_SCC_ENOMEM, "async queue allocation: %s", cudaGetErrorString(e));
-                }
-                for (auto kf : {k_prop_async<false, false>, k_prop_async<true, false>, k_prop_async<false, true>}) {
-                    CK(cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pack_dyn_smem()));
-                    CK(cudaFuncSetAttribute(kf, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                            (int)cudaSharedmemCarveoutMaxShared));
-                }
-                int per_sm = 0, sms = 0;
-                CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prop_async<false, false>, PACK_TH, pack_dyn_smem()));
-                CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device));
-                // resident CTAs per SM used (<= what fits); measured best: all of them
-                if (p->knob_async_ctas) per_sm = std::min(per_sm, p->knob_async_ctas);
-                p->aq_resident = (int64_t)std::max(1, per_sm) * sms;
-                if (getenv("ECL_SCC_DEBUG")) fprintf(stderr, "[ecl_scc] k_prop_async: %d CTAs per SM\n", per_sm);
-            }
+            if (int r = ensure_async(p)) return r;
             AsyncQ Q{p->aq_state, p->aq_seen, p->aq_ctr};
             // tiles per claim: runs pay when there are many tiles per resident CTA (measured:
             // C4 iteration 1, 18 tiles per CTA, best at 8-16; C2, ~1 tile per CTA, best at 1);
@@ -1214,6 +1219,73 @@ int run_halo(std::vector<HaloRank*>& R, Exchange& X, int32_t n, uint32_t flags, 
 }
 
 // Sweep levels of the SCC condensation (levels.cuh); plan buffers serve as workspace.
+// f4, tile mode (levels.cuh k_lk_*), after k_lv_count filled msize / odeg: *used = 0 means
+// "Kahn's rounds instead" (cross edges mostly between tiles, or a node with a long cross-edge
+// list, which one lane would walk)
+static int run_levels_tiles(Plan* p, int32_t n, const int32_t* rp, const int32_t* ci, const int32_t* lab,
+                            int32_t* out, int32_t* depth, cudaStream_t s, int* used) {
+    *used = 0;
+    LvCtl* ctl = (LvCtl*)p->lv_ctl;
+    const int32_t* msize = p->kout;
+    int32_t* odeg = p->act[1];
+    int32_t* cptr = p->optr[1];
+    int32_t* cadj = p->oadj[1];
+    int32_t* ccur = p->iptr[1];                     // (Kahn's rounds use newidx as their cursor)
+    int32_t* icnt = p->cin[1];
+    int32_t* ecnt = p->cout[1];
+    int32_t* lvl = p->cin[0];
+    int32_t* lvl_ext = p->cout[0];
+    const size_t nb = sizeof(int32_t) * (size_t)n;
+    const unsigned gs = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
+    if (int r = scan_excl<I1>(p, (const I1*)odeg, n, (I1*)cptr, (I1*)&p->dc->grand1, p->bsum, 1, s)) return r;
+    CK(cudaMemsetAsync(ccur, 0, nb, s));
+    CK(cudaMemsetAsync(icnt, 0, nb, s));
+    CK(cudaMemsetAsync(ecnt, 0, nb, s));
+    p->launches++; k_lk_fill<<<gs, TPB, 0, s>>>(n, rp, ci, lab, cptr, ccur, cadj, icnt, ecnt);
+    p->launches++; k_lk_init<<<gs, TPB, 0, s>>>(n, msize, cptr, icnt, lvl, lvl_ext, ctl);
+    CK(cudaGetLastError());
+    LvCtl h;
+    CK(cudaMemcpyAsync(&h, ctl, sizeof(LvCtl), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (h.maxodeg > 256) {
+        CK(cudaMemsetAsync(ctl, 0, sizeof(LvCtl), s));     // Kahn's rounds count the SCCs again
+        return ECL_SCC_OK;
+    }
+    *used = 1;
+    if (int r = ensure_async(p)) return r;
+    if (!p->lk_resident) {
+        CK(cudaFuncSetAttribute(k_lk_run, cudaFuncAttributeMaxDynamicSharedMemorySize, LK_ECAP * 4));
+        CK(cudaFuncSetAttribute(k_lk_run, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared));
+        int per_sm = 0, sms = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_lk_run, LK_TH, LK_ECAP * 4));
+        CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device));
+        p->lk_resident = (int64_t)std::max(1, per_sm) * sms;
+    }
+    const unsigned ntiles = (unsigned)cdiv(n, LK_TT);
+    AsyncQ Q{p->aq_state, p->aq_seen, p->aq_ctr};
+    const int claim = (int)std::min<int64_t>(16, std::max<int64_t>(1, ntiles / p->lk_resident));
+    CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
+    CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
+    p->launches++; k_async_init<<<grid_for((int64_t)ntiles, TPB), TPB, 0, s>>>(Q, (int)ntiles);
+    const LkState L{cptr, cadj, icnt, ecnt, lvl, lvl_ext, n};
+    p->launches++;
+    k_lk_run<<<(unsigned)std::min<int64_t>(ntiles, p->lk_resident), LK_TH, LK_ECAP * 4, s>>>(L, p->dc, Q, claim);
+    p->launches++; k_lk_apply<<<gs, TPB, 0, s>>>(n, lab, msize, icnt, lvl, out, ctl);
+    CK(cudaGetLastError());
+    CK(cudaMemcpyAsync(&h, ctl, sizeof(LvCtl), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (getenv("ECL_SCC_DEBUG"))
+        fprintf(stderr, "[ecl_scc] levels (tiles): %d SCCs, cross edges %llu inside tiles / %llu between, "
+                        "%.2f visits per tile\n", h.nscc, h.intra, h.cross, (double)p->hc->passes / ntiles);
+    if (p->hc->err) return fail(ECL_SCC_ECUDA, "levels: the tile queue stalled (error %d)", p->hc->err);
+    if (h.reached != h.nscc)
+        return fail(ECL_SCC_ERANGE, "levels: the labels induce a cyclic condensation (%d of %d SCCs reached)",
+                    h.reached, h.nscc);
+    if (depth) *depth = h.depth;
+    return ECL_SCC_OK;
+}
+
 int run_levels(Plan* p, int32_t n, const int32_t* rp, const int32_t* ci, const int32_t* lab, int32_t* out,
                int32_t* depth, cudaStream_t s) {
     if (!p->lv_ctl) {
@@ -1245,13 +1317,22 @@ int run_levels(Plan* p, int32_t n, const int32_t* rp, const int32_t* ci, const i
     CK(cudaMemsetAsync(cursor, 0, nb, s));
     CK(cudaMemsetAsync(ctl, 0, sizeof(LvCtl), s));
     const unsigned gs = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
-    p->launches++; k_lv_count<<<gs, TPB, 0, s>>>(n, rp, ci, lab, indeg, msize, &ctl->err);
+    const bool tiles = !(p->flags & ECL_SCC_NO_ASYNC);
+    int32_t* odeg = tiles ? p->act[1] : nullptr;
+    if (tiles) CK(cudaMemsetAsync(odeg, 0, nb, s));
+    p->launches++; k_lv_count<<<gs, TPB, 0, s>>>(n, rp, ci, lab, indeg, msize, &ctl->err, odeg, &ctl->intra);
     CK(cudaGetLastError());
+    LvCtl h0;
     {   // every later kernel indexes by label: reject labels outside [0, n) before them
-        int err = 0;
-        CK(cudaMemcpyAsync(&err, &ctl->err, sizeof(int), cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(&h0, ctl, sizeof(LvCtl), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
-        if (err) return fail(ECL_SCC_ERANGE, "levels: a label lies outside [0, n)");
+        if (h0.err) return fail(ECL_SCC_ERANGE, "levels: a label lies outside [0, n)");
+    }
+    // the tile mode pays when the cross edges mostly stay inside tiles (meshes: ~0.9; R-MAT: ~0)
+    if (tiles && (double)h0.intra >= 0.5 * (double)(h0.intra + h0.cross)) {
+        int used = 0;
+        if (int r = run_levels_tiles(p, n, rp, ci, lab, out, depth, s, &used)) return r;
+        if (used) return ECL_SCC_OK;
     }
     int r = scan_excl<I1>(p, (const I1*)msize, n, (I1*)mptr, (I1*)&p->dc->grand1, p->bsum, 1, s);
     if (r) return r;

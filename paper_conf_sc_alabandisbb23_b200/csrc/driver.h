@@ -69,6 +69,7 @@ struct Plan {
     int32_t *h_rp, *h_ci, *h_lab;        // ecl_scc_host: device copies of the caller's host buffers
     int64_t h_n_cap, h_m_cap;
     int lv_resident;                     // co-resident CTAs of k_lv_run
+    int64_t lk_resident;                 // resident CTAs of k_lk_run (levels, tile mode)
     int64_t launches;                    // kernels launched by the current call
     cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
     bool ev_ok;

@@ -613,6 +613,56 @@ struct MarkSet {
     }
 };
 
+// warp 0 of a CTA (all 32 lanes): one cursor step covers `claim` consecutive sweep positions;
+// every dirty tile among them is claimed (1 -> 2) into s_claim / s_seen in sweep order.
+// Returns the number claimed (0: the fixed point, or the stop word).
+__device__ __forceinline__ int aq_claim(const AsyncQ& Q, int ntiles, int claim, int lane, int* s_claim,
+                                        uint8_t* s_seen, long long& t0, DevCounters* dc) {
+    int got = 0, stop = 0;
+    volatile unsigned long long* ctr = Q.ctr;
+    for (unsigned miss = 0;; miss += claim) {
+        // the stop words and the cursor step are requested together (one round trip);
+        // positions taken after the fixed point are harmless
+        unsigned long long pos = 0;
+        if (lane == 0) {
+            const unsigned long long pend = ctr[AQ_PEND], halt = ctr[AQ_STOP];
+            pos = atomicAdd(Q.ctr + AQ_CUR, (unsigned long long)claim);
+            stop = (pend == 0 || halt) ? 1 : 0;           // fixed point / watchdog
+        }
+        if (__shfl_sync(FULL, stop, 0)) break;
+        pos = __shfl_sync(FULL, pos, 0) + (unsigned)lane;
+        bool mine = false;
+        int c = 0, seen = 0;
+        if (lane < claim) {
+            const unsigned long long k = pos / (unsigned)ntiles;
+            const int off = (int)(pos - k * (unsigned)ntiles);
+            c = (k & 1) ? ntiles - 1 - off : off;
+            // the seen byte is read with the state (a tile visited between this read
+            // and the claim only gets one extra full visit)
+            const int st = ((volatile int*)Q.tstate)[c];
+            seen = ((volatile uint8_t*)Q.tseen)[c];
+            mine = st == 1 && atomicCAS(Q.tstate + c, 1, 2) == 1;
+        }
+        const unsigned m = __ballot_sync(FULL, mine);
+        if (mine) {
+            const int slot = __popc(m & ((1u << lane) - 1));
+            s_claim[slot] = c;
+
+            s_seen[slot] = (uint8_t)seen;
+            if (!seen) Q.tseen[c] = 1;
+        }
+        if (m) { got = __popc(m); break; }
+        if (miss >= (unsigned)ntiles) {                    // a whole sweep without work
+            __nanosleep(256);
+            if (lane == 0 && clock64() - t0 > (1ll << 36)) {   // ~30 s idle: protocol bug
+                atomicExch(&dc->err, 3);
+                atomicExch(Q.ctr + AQ_STOP, 1ull);
+            }
+        }
+    }
+    return got;
+}
+
 template <bool HALO, bool TRICKS>
 static __global__ void __launch_bounds__(PACK_TH, PACK_MINB)
 k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, const unsigned long long* __restrict__ pnin,
@@ -643,54 +693,13 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
         mbar_init(&s_bar, 1);
     }
     PackTma T{&s_bar, 0u, false};
-    volatile unsigned long long* ctr = Q.ctr;
     long long t0 = clock64();
     for (;;) {
         // warp 0 claims: one cursor step covers CLAIM consecutive sweep positions, every
         // dirty tile among them is claimed and the CTA visits them in sweep order (a run)
         if (tid < 32) {
             const int lane = tid;
-            int got = 0, stop = 0;
-            for (unsigned miss = 0;; miss += claim) {
-                // the stop words and the cursor step are requested together (one round trip);
-                // positions taken after the fixed point are harmless
-                unsigned long long pos = 0;
-                if (lane == 0) {
-                    const unsigned long long pend = ctr[AQ_PEND], halt = ctr[AQ_STOP];
-                    pos = atomicAdd(Q.ctr + AQ_CUR, (unsigned long long)claim);
-                    stop = (pend == 0 || halt) ? 1 : 0;           // fixed point / watchdog
-                }
-                if (__shfl_sync(FULL, stop, 0)) break;
-                pos = __shfl_sync(FULL, pos, 0) + (unsigned)lane;
-                bool mine = false;
-                int c = 0, seen = 0;
-                if (lane < claim) {
-                    const unsigned long long k = pos / (unsigned)ntiles;
-                    const int off = (int)(pos - k * (unsigned)ntiles);
-                    c = (k & 1) ? ntiles - 1 - off : off;
-                    // the seen byte is read with the state (a tile visited between this read
-                    // and the claim only gets one extra full visit)
-                    const int st = ((volatile int*)Q.tstate)[c];
-                    seen = ((volatile uint8_t*)Q.tseen)[c];
-                    mine = st == 1 && atomicCAS(Q.tstate + c, 1, 2) == 1;
-                }
-                const unsigned m = __ballot_sync(FULL, mine);
-                if (mine) {
-                    const int slot = __popc(m & ((1u << lane) - 1));
-                    s_claim[slot] = c;
-
-                    s_seen[slot] = (uint8_t)seen;
-                    if (!seen) Q.tseen[c] = 1;
-                }
-                if (m) { got = __popc(m); break; }
-                if (miss >= (unsigned)ntiles) {                    // a whole sweep without work
-                    __nanosleep(256);
-                    if (lane == 0 && clock64() - t0 > (1ll << 36)) {   // ~30 s idle: protocol bug
-                        atomicExch(&dc->err, 3);
-                        atomicExch(Q.ctr + AQ_STOP, 1ull);
-                    }
-                }
-            }
+            const int got = aq_claim(Q, ntiles, claim, lane, s_claim, s_seen, t0, dc);
             if (lane == 0) {
                 s_nclaim = got;
                 s_acc[2] += (unsigned long long)got;       // tile visits of the phase

@@ -22,15 +22,20 @@ def dev(a):
 
 
 def check(g, plan=None):
+    """Both level algorithms against O4: the default (Kahn's rule per tile on the tile queue
+    where the cross edges mostly stay inside tiles, else Kahn's global rounds) and Kahn's
+    global rounds alone (a plan with ECL_SCC_NO_ASYNC)."""
     rp, ci = dev(g.row_ptr), dev(g.col_idx)
     lab = E.ecl_scc(rp, ci, plan=plan)
     truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
     np.testing.assert_array_equal(lab.cpu().numpy(), truth)
-    lv, depth = E.ecl_scc_levels(rp, ci, lab, plan=plan)
-    torch.cuda.synchronize()
     exp, edepth = oracle.scc_levels(g.row_ptr, g.col_idx, truth)
-    np.testing.assert_array_equal(lv.cpu().numpy(), exp)
-    assert depth == edepth
+    rounds = E.Plan(max(g.n, 1), max(g.nnz, 1), E.NO_ASYNC)
+    for p in (plan, rounds):
+        lv, depth = E.ecl_scc_levels(rp, ci, lab, plan=p)
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(lv.cpu().numpy(), exp)
+        assert depth == edepth
     return depth
 
 
@@ -89,3 +94,22 @@ def test_levels_reject_bad_labels():
         assert ex.value.status == E.ERANGE
     lv, depth = E.ecl_scc_levels(rp, ci, dev(np.arange(n, dtype=np.int32)))
     assert depth == n and (lv.cpu().numpy() == np.arange(n)).all()
+
+
+@pytest.mark.parametrize("flags", [0, E.NO_ASYNC])
+def test_levels_cyclic_labels_on_a_mesh(flags):
+    """Labels that split SCCs make the condensation cyclic: both algorithms report ERANGE
+    (tile mode: nodes left unprocessed at the queue's fixed point), and the context stays
+    usable."""
+    g = gen.config("c2", order="blocked8")
+    rp, ci = dev(g.row_ptr), dev(g.col_idx)
+    truth = oracle.tarjan_labels(g.row_ptr, g.col_idx)
+    assert (truth != np.arange(g.n)).any()                      # the mesh has non-trivial SCCs
+    plan = E.Plan(g.n, g.nnz, flags)
+    with pytest.raises(E.EclSccError) as ex:
+        E.ecl_scc_levels(rp, ci, dev(np.arange(g.n, dtype=np.int32)), plan=plan)
+    assert ex.value.status == E.ERANGE
+    lv, depth = E.ecl_scc_levels(rp, ci, dev(truth), plan=plan)
+    exp, edepth = oracle.scc_levels(g.row_ptr, g.col_idx, truth)
+    np.testing.assert_array_equal(lv.cpu().numpy(), exp)
+    assert depth == edepth

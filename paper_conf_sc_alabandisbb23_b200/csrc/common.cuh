@@ -46,7 +46,7 @@ struct DevCounters {
     int err;                         // validation error
     int grand1;                      // scratch total of an int32 scan
     int changed[RING];               // per-pass changed words
-    unsigned long long prof[8];      // ECL_PROF builds only: kernel event counters
+    unsigned long long prof[8];      // ECL_PROF builds: kernel event counters (prof[0] also: empty level-tile visits)
     unsigned long long visit_v;      // Phase 2: vertices of visited tiles (all passes)
     unsigned long long visit_e;      // Phase 2: out-edges of visited tiles (each edge once)
     unsigned long long heavy_e;      // Phase 2: edges reduced by k_prop_heavy

@@ -1266,6 +1266,7 @@ static int run_levels_tiles(Plan* p, int32_t n, const int32_t* rp, const int32_t
     const int claim = (int)std::min<int64_t>(16, std::max<int64_t>(1, ntiles / p->lk_resident));
     CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
     CK(cudaMemsetAsync(&p->dc->passes, 0, sizeof(unsigned long long), s));
+    CK(cudaMemsetAsync(&p->dc->prof[0], 0, sizeof(unsigned long long), s));
     p->launches++; k_async_init<<<grid_for((int64_t)ntiles, TPB), TPB, 0, s>>>(Q, (int)ntiles);
     const LkState L{cptr, cadj, icnt, ecnt, lvl, lvl_ext, n};
     p->launches++;
@@ -1277,7 +1278,8 @@ static int run_levels_tiles(Plan* p, int32_t n, const int32_t* rp, const int32_t
     CK(cudaStreamSynchronize(s));
     if (getenv("ECL_SCC_DEBUG"))
         fprintf(stderr, "[ecl_scc] levels (tiles): %d SCCs, cross edges %llu inside tiles / %llu between, "
-                        "%.2f visits per tile\n", h.nscc, h.intra, h.cross, (double)p->hc->passes / ntiles);
+                        "%.2f visits per tile (%.2f found nothing ready)\n", h.nscc, h.intra, h.cross,
+                (double)p->hc->passes / ntiles, (double)p->hc->prof[0] / ntiles);
     if (p->hc->err) return fail(ECL_SCC_ECUDA, "levels: the tile queue stalled (error %d)", p->hc->err);
     if (h.reached != h.nscc)
         return fail(ECL_SCC_ERANGE, "levels: the labels induce a cyclic condensation (%d of %d SCCs reached)",

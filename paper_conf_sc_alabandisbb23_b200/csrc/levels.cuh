@@ -380,7 +380,7 @@ static __global__ void __launch_bounds__(LK_TH, 3) k_lk_run(LkState L, DevCounte
     const int tid = threadIdx.x, v0 = tid * 4;
     const int ntiles = (L.n + LK_TT - 1) / LK_TT;
     long long t0 = clock64();
-    unsigned long long visits = 0;
+    unsigned long long visits = 0, empty = 0;
     for (;;) {
         if (tid < 32) {
             const int got = aq_claim(Q, ntiles, claim, tid, s_claim, s_seen, t0, dc);
@@ -425,7 +425,9 @@ static __global__ void __launch_bounds__(LK_TH, 3) k_lk_run(LkState L, DevCounte
             s_f[tid] = f;
             // a visit whose marks brought no node to readiness changes nothing (most revisits:
             // an external count reached 0 while intra-tile sources are still pending)
-            if (__syncthreads_or(f != 0)) {
+            const int nonempty = __syncthreads_or(f != 0);
+            if (tid == 0 && !nonempty) empty++;
+            if (nonempty) {
             for (int i = tid; i < MSET; i += LK_TH) s_set[i] = -1;
             if (tid == 0) s_nx = 0;
             for (int i = tid; i < min(ne, LK_ECAP); i += LK_TH) s_e[i] = __ldg(L.cadj + eb + i);
@@ -498,6 +500,7 @@ static __global__ void __launch_bounds__(LK_TH, 3) k_lk_run(LkState L, DevCounte
         __syncthreads();                               // s_claim is rewritten next
     }
     if (tid == 0 && visits) atomicAdd(&dc->passes, visits);
+    if (tid == 0 && empty) atomicAdd(&dc->prof[0], empty);    // visits that found no node ready
 }
 // levels_out[v] = level of label(v); depth; every label processed (else a cyclic condensation)
 static __global__ void k_lk_apply(int32_t n, const int32_t* __restrict__ lab, const int32_t* __restrict__ msize,

@@ -88,6 +88,17 @@ __device__ __forceinline__ void pnotify_a(unsigned long long nb, unsigned f) {
     sts_b1(f + (hi & 0xFFFFu));
     sts_b1(f + ((hi >> 16) & 0x7FFFu));
 }
+// notify only the dependents a raise to `val` can change (their signature is below it): a
+// dependent pulls the max of its sources, so one at or above val would pull for nothing
+__device__ __forceinline__ void pnotify_sel(unsigned long long nb, unsigned f, unsigned sig, int val) {
+    const unsigned lo = (unsigned)nb, hi = (unsigned)(nb >> 32);
+    const unsigned s0 = lo & 0xFFFFu, s1 = lo >> 16, s2 = hi & 0xFFFFu, s3 = (hi >> 16) & 0x7FFFu;
+    const int a = lds_v(sig + 4 * s0), b = lds_v(sig + 4 * s1), c = lds_v(sig + 4 * s2), d = lds_v(sig + 4 * s3);
+    if (a < val) sts_b1(f + s0);
+    if (b < val) sts_b1(f + s1);
+    if (c < val) sts_b1(f + s2);
+    if (d < val) sts_b1(f + s3);
+}
 // the rest of a slow row (more than SLOTS intra-tile neighbours): walk the global row
 __device__ __noinline__ int pull_slow(const int* sig, const int32_t* __restrict__ ptr, const int32_t* __restrict__ adj,
                                       int base, int cnt, int v, int val) {
@@ -139,7 +150,7 @@ __device__ __forceinline__ void drain_item(const WGraph& g, int* __restrict__ s_
         sts_v(a_sig + 4 * v, val);
         asm volatile("fence.acq_rel.cta;" ::: "memory");       // the value before the flags
         const unsigned long long nb = lds_v64(a_dep + 8 * v);
-        pnotify_a(nb, a_f);
+        pnotify_sel(nb, a_f, a_sig, val);
         if (nb & SLOW_MARK) notify_slow(DOUT ? g.iptr : g.optr, DOUT ? g.iadj : g.oadj, base, cnt, v, (uint8_t*)s_f);
         if (TRICKS && g.raise_) {
             // sound P:190: out[in[v]] (an ancestor) for v_out, in[out[v]] (a descendant) for v_in

@@ -100,6 +100,9 @@ typedef enum {
                                      CTAs share one 4096-vertex block-local fixed point through
                                      distributed shared memory (csrc/cluster.cuh); graphs
                                      without rows longer than 64 edges, single GPU */
+#define ECL_SCC_NO_KW 0x80000u    /* ablation: the general compaction layout (8-byte kept degrees
+                                     + 8-byte row masks per vertex) also for graphs whose rows
+                                     have <= 8 entries, which otherwise use one 4-byte keep word */
 #define ECL_SCC_FOUR_SIG 0x8000u  /* variant: the 4-signature method -- Phase 2 also
                                      propagates minimum ancestor / descendant IDs and Phase 3
                                      keeps an edge only if all four signatures agree; twice the

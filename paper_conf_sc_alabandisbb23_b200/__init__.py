@@ -22,6 +22,7 @@ NO_TRIM, NO_VALIDATE, SYNC_PASSES, TIME_STAGES = 0x1, 0x4, 0x8, 0x10
 IDENTITY_IDS, NO_DIRTY, NO_REORDER = 0x20, 0x40, 0x200
 FORCE_REORDER, NO_PACK, NO_ASYNC = 0x400, 0x800, 0x1000
 TRIM2, FOUR_SIG, HALO_ALLREDUCE, COMPRESS, RAISE, CLUSTER = 0x4000, 0x8000, 0x10000, 0x2, 0x20000, 0x40000
+NO_KW = 0x80000
 TRACE_MAX = 64
 
 _lib = None

@@ -52,6 +52,7 @@ struct DevCounters {
     unsigned long long heavy_e;      // Phase 2: edges reduced by k_prop_heavy
     unsigned long long local_e;      // ingest: short-row edges whose ends share a 2048-ID range
     int pack_bad;                    // compaction: the scatter could not write the tile pack
+    int maxdeg;                      // ingest: the longest row of the input, CSR or CSC
 };
 
 // Internal vertex priorities (reading 16).  The signatures propagate

@@ -219,7 +219,8 @@ static int build_csc(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const i
     p->cb = 0;
     Chunk* ch = chunk_buf(p, p->cb);
     CK(cudaMemsetAsync(&p->dc->nchunks, 0, sizeof(int), s));
-    p->launches++; k_ingest_chunks<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, 0, ch, &p->dc->nchunks, (int)p->chunk_cap);
+    CK(cudaMemsetAsync(&p->dc->maxdeg, 0, sizeof(int), s));
+    p->launches++; k_ingest_chunks<<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, 0, ch, &p->dc->nchunks, (int)p->chunk_cap, &p->dc->maxdeg);
     CK(cudaMemsetAsync(p->kin, 0, sizeof(int32_t) * (size_t)(n + 1), s));
     int nout = 0;
     int r = read_nchunks(p, s, &nout);
@@ -242,8 +243,12 @@ static int build_csc(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const i
     if (use_rank) k_csc_scatter<true><<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, ci, p->iptr[0], rank, cursor, p->iadj[0], &p->dc->local_e);
     else k_csc_scatter<false><<<grid_for(n, TPB), TPB, 0, s>>>(n, rp, ci, p->iptr[0], rank, cursor, p->iadj[0], &p->dc->local_e);
     if (nout) { p->launches++; k_csc_scatter_chunks<false><<<chunk_grid(nout), TPB, 0, s>>>(ch, nout, ci, p->iptr[0], rank, cursor, p->iadj[0]); }
-    p->launches++; k_ingest_chunks<<<grid_for(n, TPB), TPB, 0, s>>>(n, p->iptr[0], 1, ch, &p->dc->nchunks, (int)p->chunk_cap);
+    p->launches++; k_ingest_chunks<<<grid_for(n, TPB), TPB, 0, s>>>(n, p->iptr[0], 1, ch, &p->dc->nchunks, (int)p->chunk_cap, &p->dc->maxdeg);
+    CK(cudaMemcpyAsync(&p->hc->maxdeg, &p->dc->maxdeg, sizeof(int), cudaMemcpyDeviceToHost, s));
     if ((r = read_nchunks(p, s, &p->nchunks_cur))) return r;
+    // the compaction's 4-byte keep words (rows <= KW_DEG entries: meshes); the variants and the
+    // partitioned mode keep the general layout
+    p->kw = p->hc->maxdeg <= KW_DEG && !(p->flags & (ECL_SCC_FOUR_SIG | ECL_SCC_TRIM2 | ECL_SCC_NO_KW));
     CK(cudaGetLastError());
     return ECL_SCC_OK;
 }
@@ -320,7 +325,7 @@ static int ensure_pack(Plan* p) {
 // Phase-1 reset of the survivors and the final labels of the vertices that leave.  Two
 // parts: compact_keep evaluates the keep predicate (kept degrees), compact_finish trims and
 // compacts; the partitioned mode exchanges the halo's kept degrees in between.
-template <bool FIRST, bool TRIM, bool FOUR>
+template <bool FIRST, bool TRIM, bool FOUR, bool KW = false>
 static int compact_keep(Plan* p, const WGraph& g, const int32_t* cin, const int32_t* cout, cudaStream_t s) {
     const unsigned grid = grid_for(g.na, TPB);
     const int nc = p->nchunks_cur, chunked = nc > 0;
@@ -335,7 +340,7 @@ static int compact_keep(Plan* p, const WGraph& g, const int32_t* cin, const int3
         k_pack_sig<<<std::min<unsigned>(grid, 148 * 16), TPB, 0, s>>>(g.na, cin, cout, p->sig2);
         gk.sig2 = p->sig2;
     }
-    p->launches++; k_keep_count<FIRST, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, chunked, p->hcnt, p->emask);
+    p->launches++; k_keep_count<FIRST, FOUR, KW><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, chunked, p->hcnt, p->emask);
     if (chunked) {
         p->launches++;
         k_keep_chunks<FIRST, FOUR><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio);
@@ -345,7 +350,7 @@ static int compact_keep(Plan* p, const WGraph& g, const int32_t* cin, const int3
     return ECL_SCC_OK;
 }
 
-template <bool FIRST, bool TRIM, bool FOUR>
+template <bool FIRST, bool TRIM, bool FOUR, bool KW = false>
 static int compact_finish(Plan* p, const int32_t* cin, const int32_t* cout, int ob, int32_t* labels, const Prio& P,
                           cudaStream_t s) {
     const WGraph gk = p->gk;
@@ -371,7 +376,7 @@ static int compact_finish(Plan* p, const int32_t* cin, const int32_t* cout, int 
         p->launches++;
         k_count_chunks<FIRST, TRIM, FOUR><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio, p->chunk_cnt, p->hcnt);
     }
-    p->launches++; k_compact_count<FIRST, TRIM, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
+    p->launches++; k_compact_count<FIRST, TRIM, FOUR, KW><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
     int r = scan_excl<I3>(p, (const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
     if (r) return r;
     p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
@@ -380,7 +385,7 @@ static int compact_finish(Plan* p, const int32_t* cin, const int32_t* cout, int 
                                               MapExtra{p->min_in[ob], p->min_out[ob], trim2 ? p->t2 : nullptr, p->kio,
                                                        TRIM ? 1 : 0, gk.hpos ? p->hpos[ob] : nullptr, p->lab_lo,
                                                        p->lab_hi, p->slot});
-    p->launches++; k_compact_scatter<FIRST, TRIM, FOUR><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->newidx, p->optr[ob],
+    p->launches++; k_compact_scatter<FIRST, TRIM, FOUR, KW><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked, p->emask, pk);
     if (chunked) {
         p->launches++;
@@ -399,6 +404,17 @@ static int compaction(Plan* p, int part, int iter, const WGraph& g, const int32_
     const bool four = (p->flags & ECL_SCC_FOUR_SIG) != 0 && iter > 1;   // (iteration 1 keeps every edge)
 #define ECL_COMPACT(F, T, Fo) \
     return part == 0 ? compact_keep<F, T, Fo>(p, g, cin, cout, s) : compact_finish<F, T, Fo>(p, cin, cout, ob, labels, P, s)
+#define ECL_COMPACT_KW(F, T) \
+    return part == 0 ? compact_keep<F, T, false, true>(p, g, cin, cout, s) \
+                     : compact_finish<F, T, false, true>(p, cin, cout, ob, labels, P, s)
+    if (p->kw && !g.hpos) {                        // small degrees (the partitioned mode excluded)
+        if (iter == 1) {
+            if (trim) ECL_COMPACT_KW(true, true);
+            ECL_COMPACT_KW(true, false);
+        }
+        if (trim) ECL_COMPACT_KW(false, true);
+        ECL_COMPACT_KW(false, false);
+    }
     if (iter == 1) {
         if (trim) ECL_COMPACT(true, true, false);
         ECL_COMPACT(true, false, false);
@@ -410,6 +426,7 @@ static int compaction(Plan* p, int part, int iter, const WGraph& g, const int32_
     if (trim) ECL_COMPACT(false, true, false);
     ECL_COMPACT(false, false, false);
 #undef ECL_COMPACT
+#undef ECL_COMPACT_KW
 }
 
 // per-plan (per-device) kernel attributes of the pass kernels

@@ -70,6 +70,7 @@ struct Plan {
     int64_t h_n_cap, h_m_cap;
     int lv_resident;                     // co-resident CTAs of k_lv_run
     int64_t lk_resident;                 // resident CTAs of k_lk_run (levels, tile mode)
+    bool kw;                             // compaction with 4-byte keep words (rows <= KW_DEG)
     int64_t launches;                    // kernels launched by the current call
     cudaEvent_t ev[6];                   // stage timing (ECL_SCC_TIME_STAGES)
     bool ev_ok;

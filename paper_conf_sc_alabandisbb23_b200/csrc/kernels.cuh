@@ -173,6 +173,15 @@ __device__ __forceinline__ bool trimmed(const int2* __restrict__ kio, int x) {
     const int2 k = __ldg(kio + x);
     return (k.x == 0) | (k.y == 0);
 }
+// Small-degree graphs (every row <= KW_DEG entries per direction: meshes), one 4-byte keep word
+// per vertex instead of kio (8 B) + emask (8 B): byte 0 kept in-degree, byte 1 kept out-degree,
+// byte 2 the out-row mask, byte 3 the in-row mask (Phase 3's kept entries; after the trim, the
+// survivors -- the degree bytes, which other threads' trim tests read, stay as they were)
+constexpr int KW_DEG = 8;
+__device__ __forceinline__ bool trimmed_kw(const uint32_t* __restrict__ kw, int x) {
+    const uint32_t w = __ldg(kw + x);
+    return ((w & 0xFFu) == 0) | ((w & 0xFF00u) == 0);
+}
 
 struct RowCtx {
     int ob, oe, ib, ie, a, b, c, d;       // (c, d): the minimum pair (4-signature variant)
@@ -275,8 +284,9 @@ __device__ __forceinline__ void mask_light2(const int32_t* __restrict__ oadj, in
     }
 }
 // keep the set bits of m whose entry's far end is not trimmed (batches of 4 entries)
+template <bool KW = false>
 __device__ __forceinline__ unsigned trim_mask(const int32_t* __restrict__ adj, int b, unsigned m, int self,
-                                              const int2* __restrict__ kio) {
+                                              const int2* __restrict__ kio, const uint32_t* __restrict__ kw = nullptr) {
     unsigned out = 0;
     while (m) {
         int k[4], x[4];
@@ -289,7 +299,7 @@ __device__ __forceinline__ unsigned trim_mask(const int32_t* __restrict__ adj, i
         for (int q = 0; q < 4; q++) x[q] = k[q] >= 0 ? __ldg(adj + b + k[q]) : self;
 #pragma unroll
         for (int q = 0; q < 4; q++)
-            if (k[q] >= 0 && !trimmed(kio, x[q])) out |= 1u << k[q];
+            if (k[q] >= 0 && !(KW ? trimmed_kw(kw, x[q]) : trimmed(kio, x[q]))) out |= 1u << k[q];
     }
     return out;
 }
@@ -376,7 +386,7 @@ __device__ __forceinline__ void emit_cut(const int32_t* __restrict__ adj, int b,
 
 // kept in/out degree per local vertex (light rows: also the kept entries as bit masks)
 constexpr int TPB_COMPACT = 256;     // block size of the compaction kernels (driver TPB)
-template <bool FIRST, bool FOUR>
+template <bool FIRST, bool FOUR, bool KW = false>
 static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                              int2* __restrict__ kio, int chunked, int2* __restrict__ hcnt,
                              uint2* __restrict__ emask) {
@@ -388,6 +398,10 @@ static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, con
     mask_light2(g.oadj, r.ob, r.live && r.oe - r.ob <= HEAVY ? r.oe - r.ob : 0, g.iadj, r.ib,
                 r.live && r.ie - r.ib <= HEAVY ? r.ie - r.ib : 0, (int)(r.valid ? i : 0), pred, mo, mi);
     int co = __popc(mo), ci = __popc(mi);
+    if (KW) {                                        // (no row is longer than KW_DEG)
+        if (r.valid) ((uint32_t*)emask)[i] = (uint32_t)ci | (uint32_t)co << 8 | mo << 16 | mi << 24;
+        return;
+    }
     co += count_row(g.oadj, r.ob, r.oe, r.live, lane, pred, chunked, false);
     ci += count_row(g.iadj, r.ib, r.ie, r.live, lane, pred, chunked, false);
     if (r.valid) {
@@ -400,7 +414,7 @@ static __global__ void __launch_bounds__(TPB_COMPACT) k_keep_count(WGraph g, con
 }
 
 // per-vertex surviving (kept, not trimmed) degrees and per-warp totals (alive, out, in, kept)
-template <bool FIRST, bool TRIM, bool FOUR>
+template <bool FIRST, bool TRIM, bool FOUR, bool KW = false>
 static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                 const int2* __restrict__ kio,
                                 int2* __restrict__ cnt, int4* __restrict__ wsum, int chunked,
@@ -408,7 +422,30 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
     const int lane = threadIdx.x & 31;
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const RowCtx r = load_row<FIRST, FOUR>(g, i, cin, cout);
-    int nout = 0, nin = 0;
+    int nout = 0, nin = 0, kept = 0;
+    if (KW) {                                          // small degrees: the 4-byte keep words
+        uint32_t* kw = (uint32_t*)emask;
+        if (r.valid) {
+            const uint32_t w = kw[i];
+            kept = (int)((w >> 8) & 0xFFu);
+            const bool go = r.live && ((w & 0xFFu) != 0) && ((w & 0xFF00u) != 0);
+            unsigned so = (w >> 16) & 0xFFu, si = w >> 24;
+            if (TRIM) {
+                so = go ? trim_mask<true>(g.oadj, r.ob, so, (int)i, nullptr, kw) : 0u;
+                si = go ? trim_mask<true>(g.iadj, r.ib, si, (int)i, nullptr, kw) : 0u;
+                kw[i] = (w & 0xFFFFu) | so << 16 | si << 24;
+            } else if (!r.live) {
+                so = si = 0;
+            }
+            nout = __popc(so);
+            nin = __popc(si);
+            cnt[i] = make_int2(nout, nin);
+        }
+        const int alive = (nout + nin) > 0;
+        const int sa = warp_sum(alive), so_ = warp_sum(nout), si_ = warp_sum(nin), sk = warp_sum(kept);
+        if (lane == 0) wsum[i >> 5] = make_int4(sa, so_, si_, sk);
+        return;
+    }
     if (!TRIM) {
         if (r.live) { const int2 k = kio[i]; nout = k.y; nin = k.x; }   // survivors = kept: the masks stand
     } else {
@@ -435,7 +472,7 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
     // partitioned mode: an unfinished halo vertex that is not trimmed (global degrees) stays,
     // even without local edges -- its edges may live on other ranks (halo.cuh)
     if (g.hpos && !alive && r.live && g.hpos[i] >= 0 && !(TRIM && trimmed(kio, (int)i))) alive = 1;
-    const int kept = r.valid ? kio[i].y : 0;            // kept (pre-trim) out-degree, chunks included
+    kept = r.valid ? kio[i].y : 0;                      // kept (pre-trim) out-degree, chunks included
     const int sa = warp_sum(alive), so = warp_sum(nout), si = warp_sum(nin), sk = warp_sum(kept);
     if (lane == 0) wsum[i >> 5] = make_int4(sa, so, si, sk);
 }
@@ -668,7 +705,7 @@ __device__ __forceinline__ void emit_row(const int32_t* __restrict__ adj, int rb
     }
 }
 
-template <bool FIRST, bool TRIM, bool FOUR>
+template <bool FIRST, bool TRIM, bool FOUR, bool KW = false>
 static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                                   const int2* __restrict__ kio, const int32_t* __restrict__ newidx, const int32_t* __restrict__ optr2,
                                   const int32_t* __restrict__ iptr2, int32_t* __restrict__ oadj2,
@@ -685,7 +722,12 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
     if (go) {
         po = optr2[j];
         pi = iptr2[j];
-        sm = emask[i];                                 // light rows: the survivors' bits
+        if (KW) {                                      // light rows: the survivors' bits
+            const uint32_t w = ((const uint32_t*)emask)[i];
+            sm = make_uint2((w >> 16) & 0xFFu, w >> 24);
+        } else {
+            sm = emask[i];
+        }
         lo = r.oe - r.ob <= HEAVY;
         li = r.ie - r.ib <= HEAVY;
         if (pk.pnin) {
@@ -720,6 +762,7 @@ static __global__ void k_compact_scatter(WGraph g, const int32_t* __restrict__ c
             if (li) emit_cut(g.iadj, r.ib, sm.y, newidx, j, tb, 0, E, at);
         }
     }
+    if (KW) return;                                    // (no row longer than HEAVY)
     SurvivePred<FIRST, TRIM, FOUR> pred{(int)i, r.a, r.b, cin, cout, kio, g.sig2, r.c, r.d, g.min_in, g.min_out};
     emit_row(g.oadj, r.ob, r.oe, go, po, newidx, oadj2, lane, pred, chunked, false);
     emit_row(g.iadj, r.ib, r.ie, go, pi, newidx, iadj2, lane, pred, chunked, false);
@@ -808,12 +851,21 @@ static __global__ void __launch_bounds__(256) k_scatter_chunks(WGraph g, const C
     }
 }
 // chunk list of the input graph (CSR rows from row_ptr, CSC rows from iptr)
+// (and the largest row of either direction, for the small-degree compaction)
 static __global__ void k_ingest_chunks(int32_t n, const int32_t* __restrict__ ptr, int dir, Chunk* __restrict__ chunks,
-                                       int* __restrict__ nchunks, int chunk_cap) {
+                                       int* __restrict__ nchunks, int chunk_cap, int* __restrict__ maxdeg) {
+    __shared__ int s_md;
     const int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (v >= n) return;
-    const int beg = ptr[v], deg = ptr[v + 1] - beg;
-    if (deg <= HEAVY_T) return;
+    const int beg = v < n ? ptr[v] : 0, deg = v < n ? ptr[v + 1] - beg : 0;
+    if (threadIdx.x == 0) s_md = 0;
+    __syncthreads();
+    const int md = __reduce_max_sync(FULL, deg);
+    if ((threadIdx.x & 31) == 0 && md) atomicMax(&s_md, md);
+    __syncthreads();
+    // one global atomic per block, and only while it raises the maximum (the blocks of a
+    // launch all target one address)
+    if (threadIdx.x == 0 && s_md > *(volatile int*)maxdeg) atomicMax(maxdeg, s_md);
+    if (v >= n || deg <= HEAVY_T) return;
     const int nc = (deg + CHUNK - 1) / CHUNK;
     const int at = atomicAdd(nchunks, nc);
     for (int k = 0; k < nc && at + k < chunk_cap; k++)

@@ -173,3 +173,16 @@ def test_cluster_pair_tiles_keep_the_trace():
     g = gen.config("c2", order="blocked8")
     lab, st = run(g, E.CLUSTER)
     np.testing.assert_array_equal(lab, oracle.tarjan_labels(g.row_ptr, g.col_idx))
+
+
+@pytest.mark.parametrize("flags", [0, E.NO_KW, E.NO_TRIM, E.NO_TRIM | E.NO_KW])
+def test_keep_word_layout_keeps_the_trace(flags):
+    """The small-degree compaction (one 4-byte keep word per vertex, rows of <= 8 entries:
+    every mesh) and the general layout (ECL_SCC_NO_KW) against O2: labels, per-iteration
+    trace and signature snapshots; and a graph with longer rows takes the general path."""
+    for g in (gen.mesh(14, gen.ordinate(5), seed=9, order="blocked8", **gen.C4_MESH), gen.config("c1")):
+        check(g, flags, {}, max_iters=3)
+    lab, st = run(gen.config("c2", order="blocked8"), flags)
+    lab2, st2 = run(gen.config("c2", order="blocked8"), flags ^ E.NO_KW)
+    np.testing.assert_array_equal(lab, lab2)
+    assert st["edges_in"] == st2["edges_in"] and st["edges_kept"] == st2["edges_kept"]

@@ -379,7 +379,7 @@ static int compact_finish(Plan* p, const int32_t* cin, const int32_t* cout, int 
     p->launches++; k_compact_count<FIRST, TRIM, FOUR, KW><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
     int r = scan_excl<I3>(p, (const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
     if (r) return r;
-    p->launches++; k_compact_map<FIRST><<<grid, TPB, 0, s>>>(gk, cin, cout, p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
+    p->launches++; k_compact_map<FIRST, KW><<<grid, TPB, 0, s>>>(gk, cin, cout, KW ? (const int2*)p->emask : p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
                                               chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur, pk,
                                               MapExtra{p->min_in[ob], p->min_out[ob], trim2 ? p->t2 : nullptr, p->kio,

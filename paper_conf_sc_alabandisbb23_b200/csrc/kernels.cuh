@@ -438,8 +438,7 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
                 so = si = 0;
             }
             nout = __popc(so);
-            nin = __popc(si);
-            cnt[i] = make_int2(nout, nin);
+            nin = __popc(si);                          // (k_compact_map counts them from the word)
         }
         const int alive = (nout + nin) > 0;
         const int sa = warp_sum(alive), so_ = warp_sum(nout), si_ = warp_sum(nin), sk = warp_sum(kept);
@@ -548,7 +547,7 @@ struct MapExtra {
 // Survivors restart from their priority pi(v) (reading 16).  A finished vertex leaves
 // with its signature s = max priority of its SCC; with raw IDs that is the label itself,
 // otherwise it is stored as -(s+1) and k_relabel_* turn it into the SCC's max vertex ID.
-template <bool FIRST>
+template <bool FIRST, bool KW = false>
 static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                               const int2* __restrict__ cnt, const int4* __restrict__ wscan,
                               const int4* __restrict__ totals, int32_t* __restrict__ newidx,
@@ -577,7 +576,13 @@ static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, 
         }
     }
     const bool valid = i < g.na;
-    int2 c = valid ? cnt[i] : make_int2(0, 0);
+    int2 c = make_int2(0, 0);
+    if (valid && KW) {                                 // the survivor masks of the keep word
+        const uint32_t w = ((const uint32_t*)cnt)[i];
+        c = make_int2(__popc((w >> 16) & 0xFFu), __popc(w >> 24));
+    } else if (valid) {
+        c = cnt[i];
+    }
     int alive = (c.x + c.y) > 0;
     if (g.hpos && valid && !alive && g.hpos[i] >= 0 && (FIRST || cin[i] != cout[i]) && !(trim && trimmed(kio, (int)i)))
         alive = 1;                                     // (the same rule as k_compact_count)

@@ -282,7 +282,10 @@ static int reorder_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, con
     if (r) return r;
     CK(cudaMemsetAsync(cursor, 0, sizeof(int32_t) * (size_t)(nkeys + 1), s));
     p->launches++; reo::k_cell_place<<<gs, TPB, 0, s>>>(n, p->cellv, start, cursor, p->pos, p->orig);
-    p->launches++; reo::k_cell_sort<<<(unsigned)std::min<int64_t>(nkeys, 148 * 7), reo::SORT_THREADS, 0, s>>>(nkeys, start, p->orig, p->pos);
+    int bits = 1;
+    while (bits < 31 && (1ll << bits) <= (long long)n) bits++;   // every caller ID < 2^bits - 1
+    p->launches++;
+    reo::k_cell_sort<<<(unsigned)std::min<int64_t>(nkeys, 148 * 8), reo::SORT_THREADS, 0, s>>>(nkeys, start, p->orig, p->pos, bits);
     p->launches++; reo::k_perm_deg<<<gs, TPB, 0, s>>>(n, rp, p->pos, p->kin);
     r = scan_excl<I1>(p, (const I1*)p->kin, n, (I1*)p->rp2, (I1*)&p->dc->grand1, p->bsum, 1, s);
     if (r) return r;

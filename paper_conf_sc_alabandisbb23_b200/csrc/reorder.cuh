@@ -8,6 +8,8 @@
 // SCC result does not depend on the storage order (the fixed points are unique), only the
 // number of Phase-2 passes does.
 #pragma once
+#include <cub/block/block_radix_sort.cuh>
+
 #include "common.cuh"
 
 namespace eclscc {
@@ -134,39 +136,52 @@ static __global__ void k_cell_place(int32_t n, const int32_t* __restrict__ key, 
         }
     }
 }
-// one CTA per cell: sort the cell's storage slots by caller ID (bitonic sort in shared
-// memory), so that a tile holding part of a cell holds a compact piece of it (the
+// one CTA per cell: sort the cell's storage slots by caller ID (radix sort in shared
+// memory, below), so that a tile holding part of a cell holds a compact piece of it (the
 // atomic placement above leaves the members in arbitrary order).  Cells larger than
 // SORT_MAX keep the arbitrary order (only the pass count depends on it).
 constexpr int SORT_MAX = 8192;
-constexpr int SORT_THREADS = 256;     // small CTAs: ~7 cells sort concurrently per SM (barrier-bound stages)
+constexpr int SORT_THREADS = 256;
+// A cell's members (caller IDs, all < 2^bits) sorted in shared memory by a block radix sort
+// (the CUB building block inside this kernel; round 1 used a bitonic network: 78 barrier
+// stages per 4096-member cell, C4 lex 1.48 ms for the kernel), in two sizes: cells up to
+// 4096 and up to SORT_MAX members.  Loads are striped (the sort ignores the input order),
+// results come back striped (coalesced stores).
+template <int ITEMS>
+using CellSort = cub::BlockRadixSort<unsigned, SORT_THREADS, ITEMS>;
+template <int ITEMS>
+__device__ __forceinline__ void sort_cell(int32_t* __restrict__ orig, int32_t* __restrict__ pos, int b, int sz, int bits,
+                                          typename CellSort<ITEMS>::TempStorage& tmp) {
+    const unsigned pad = bits >= 32 ? 0xFFFFFFFFu : (1u << bits) - 1u;   // above every ID
+    unsigned key[ITEMS];
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) {
+        const int k = i * SORT_THREADS + threadIdx.x;
+        key[i] = k < sz ? (unsigned)orig[b + k] : pad;
+    }
+    CellSort<ITEMS>(tmp).SortBlockedToStriped(key, 0, bits);
+#pragma unroll
+    for (int i = 0; i < ITEMS; i++) {
+        const int k = i * SORT_THREADS + threadIdx.x;
+        if (k < sz) {
+            orig[b + k] = (int32_t)key[i];
+            pos[key[i]] = b + k;
+        }
+    }
+}
 static __global__ void __launch_bounds__(SORT_THREADS) k_cell_sort(int64_t nkeys, const int32_t* __restrict__ start,
-                                                                  int32_t* __restrict__ orig, int32_t* __restrict__ pos) {
-    __shared__ int32_t sk[SORT_MAX];
+                                                                  int32_t* __restrict__ orig, int32_t* __restrict__ pos,
+                                                                  int bits) {
+    __shared__ union {
+        typename CellSort<SORT_MAX / 2 / SORT_THREADS>::TempStorage small;
+        typename CellSort<SORT_MAX / SORT_THREADS>::TempStorage large;
+    } tmp;
     for (int64_t c = blockIdx.x; c < nkeys; c += gridDim.x) {
         const int b = start[c], sz = start[c + 1] - b;
-        if (sz <= 1 || sz > SORT_MAX) continue;
-        int m = 1;
-        while (m < sz) m <<= 1;
-        for (int k = threadIdx.x; k < m; k += SORT_THREADS) sk[k] = k < sz ? orig[b + k] : 0x7FFFFFFF;
-        __syncthreads();
-        for (int k = 2; k <= m; k <<= 1)
-            for (int j = k >> 1; j > 0; j >>= 1) {
-                for (int t = threadIdx.x; t < m; t += SORT_THREADS) {
-                    const int o = t ^ j;
-                    if (o > t) {
-                        const int x = sk[t], y = sk[o];
-                        if (((t & k) == 0) == (x > y)) { sk[t] = y; sk[o] = x; }
-                    }
-                }
-                __syncthreads();
-            }
-        for (int k = threadIdx.x; k < sz; k += SORT_THREADS) {
-            const int v = sk[k];
-            orig[b + k] = v;
-            pos[v] = b + k;
-        }
-        __syncthreads();
+        if (sz <= 1 || sz > SORT_MAX) continue;        // (larger cells keep the placement order)
+        if (sz <= SORT_MAX / 2) sort_cell<SORT_MAX / 2 / SORT_THREADS>(orig, pos, b, sz, bits, tmp.small);
+        else sort_cell<SORT_MAX / SORT_THREADS>(orig, pos, b, sz, bits, tmp.large);
+        __syncthreads();                               // tmp is reused by the next cell
     }
 }
 static __global__ void k_perm_deg(int32_t n, const int32_t* __restrict__ rp, const int32_t* __restrict__ pos,

@@ -548,7 +548,7 @@ struct MapExtra {
 // with its signature s = max priority of its SCC; with raw IDs that is the label itself,
 // otherwise it is stored as -(s+1) and k_relabel_* turn it into the SCC's max vertex ID.
 template <bool FIRST, bool KW = false>
-static __global__ void k_compact_map(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+static __global__ void __launch_bounds__(TPB_COMPACT, 8) k_compact_map(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
                               const int2* __restrict__ cnt, const int4* __restrict__ wscan,
                               const int4* __restrict__ totals, int32_t* __restrict__ newidx,
                               int32_t* __restrict__ act2, int32_t* __restrict__ cin2, int32_t* __restrict__ cout2,

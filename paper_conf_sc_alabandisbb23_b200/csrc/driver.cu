@@ -163,7 +163,7 @@ void plan_free(Plan* p) {
     cudaFree(p->dirty);
     cudaFree(p->rp2); cudaFree(p->ci2); cudaFree(p->orig); cudaFree(p->pos); cudaFree(p->cellv);
     cudaFree(p->fa); cudaFree(p->fb); cudaFree(p->cellbuf); cudaFree(p->rcnt);
-    cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab);
+    cudaFree(p->u_rp); cudaFree(p->u_ci); cudaFree(p->u_lab); cudaFree(p->u_desc);
     cudaFree(p->pnin); cudaFree(p->pnout); cudaFree(p->ext); cudaFree(p->ext_cnt);
     cudaFree(p->aq_state); cudaFree(p->aq_seen); cudaFree(p->aq_ctr);
     cudaFree(p->lv_ctl);
@@ -822,18 +822,40 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
 
 // --------------------------------------------------------------------------- batched union
 __global__ void k_set1(int32_t* p, int32_t v) { *p = v; }
-__global__ void k_union_rows(int32_t n, const int32_t* __restrict__ rp, int32_t voff, int32_t eoff,
-                             int32_t* __restrict__ urp) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-        urp[voff + v] = rp[v] + eoff;
+// all graphs of a batch in one launch (blockIdx.y = graph): the union rows and columns, with
+// the CSR checks of k_validate on the way (one pass over every input); and the label split
+struct UGraph {
+    const int32_t* rp;
+    const int32_t* ci;
+    int32_t* lab;
+    int64_t nnz, eoff;
+    int32_t n, voff;
+};
+__global__ void k_union_all(const UGraph* __restrict__ gs, int32_t* __restrict__ urp, int32_t* __restrict__ uci,
+                            int validate, int* __restrict__ err) {
+    const UGraph G = gs[blockIdx.y];
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    int bad = 0;
+    for (int64_t v = t0; v < G.n; v += stride) {
+        const int32_t a = G.rp[v];
+        urp[G.voff + v] = a + (int32_t)G.eoff;
+        if (validate) {
+            const int32_t b = G.rp[v + 1];
+            if (a > b || (v == 0 && a != 0) || (v == G.n - 1 && (int64_t)b != G.nnz)) bad = 1;
+        }
+    }
+    for (int64_t e = t0; e < G.nnz; e += stride) {
+        const int32_t c = G.ci[e];
+        if (validate && (c < 0 || c >= G.n)) bad = 1;
+        uci[G.eoff + e] = c + G.voff;
+    }
+    if (bad) *err = 1;
 }
-__global__ void k_union_cols(int64_t m, const int32_t* __restrict__ ci, int32_t voff, int32_t* __restrict__ uci) {
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < m; e += (int64_t)gridDim.x * blockDim.x)
-        uci[e] = ci[e] + voff;
-}
-__global__ void k_split_labels(int32_t n, const int32_t* __restrict__ ul, int32_t voff, int32_t* __restrict__ out) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-        out[v] = ul[voff + v] - voff;
+__global__ void k_split_all(const UGraph* __restrict__ gs, const int32_t* __restrict__ ul) {
+    const UGraph G = gs[blockIdx.y];
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < G.n; v += (int64_t)gridDim.x * blockDim.x)
+        G.lab[v] = ul[G.voff + v] - G.voff;
 }
 
 int run_batched(Plan* p, int32_t G, const int32_t* n, const int64_t* nnz, const int32_t* const* rp,
@@ -861,25 +883,36 @@ int run_batched(Plan* p, int32_t G, const int32_t* n, const int64_t* nnz, const 
         }
         p->u_m_cap = M;
     }
-    // validate each graph individually first (offsets are rebased below)
-    if (!(p->flags & ECL_SCC_NO_VALIDATE)) {
-        CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
-        for (int g = 0; g < G; g++)
-            if (n[g] > 0) {
-                p->launches++;
-                k_validate<<<std::min<unsigned>(grid_for(std::max<int64_t>(n[g], nnz[g]), TPB), 148 * 16), TPB, 0, s>>>(
-                    n[g], nnz[g], rp[g], ci[g], &p->dc->err);
-            }
-        CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));
-        if (p->hc->err) return fail(ECL_SCC_ERANGE, "invalid CSR in batch");
+    // one launch builds the union (and checks every graph's CSR on the way)
+    if (!p->u_desc || p->u_desc_cap < G) {
+        cudaFree(p->u_desc);
+        p->u_desc = nullptr;
+        if (cudaMalloc(&p->u_desc, sizeof(UGraph) * (size_t)G) != cudaSuccess) {
+            cudaGetLastError();
+            return fail(ECL_SCC_ENOMEM, "batched graph table (%d graphs)", G);
+        }
+        p->u_desc_cap = G;
     }
-    int64_t vo = 0, eo = 0;
-    for (int g = 0; g < G; g++) {
-        if (n[g] > 0) { p->launches++; k_union_rows<<<grid_for(n[g], TPB), TPB, 0, s>>>(n[g], rp[g], (int32_t)vo, (int32_t)eo, p->u_rp); }
-        if (nnz[g] > 0) { p->launches++; k_union_cols<<<grid_for(nnz[g], TPB), TPB, 0, s>>>(nnz[g], ci[g], (int32_t)vo, p->u_ci + eo); }
-        vo += n[g];
-        eo += nnz[g];
+    std::vector<UGraph> desc((size_t)G);
+    {
+        int64_t vo = 0, eo = 0, nmax = 1;
+        for (int g = 0; g < G; g++) {
+            desc[g] = UGraph{rp[g], ci[g], labels[g], nnz[g], eo, n[g], (int32_t)vo};
+            nmax = std::max<int64_t>(nmax, std::max<int64_t>(n[g], nnz[g]));
+            vo += n[g];
+            eo += nnz[g];
+        }
+        CK(cudaMemcpyAsync(p->u_desc, desc.data(), sizeof(UGraph) * (size_t)G, cudaMemcpyHostToDevice, s));
+        const int validate = !(p->flags & ECL_SCC_NO_VALIDATE);
+        if (validate) CK(cudaMemsetAsync(&p->dc->err, 0, sizeof(int), s));
+        const unsigned gx = (unsigned)std::max<int64_t>(1, std::min<int64_t>(cdiv(nmax, TPB), std::max(1, 148 * 16 / G)));
+        p->launches++;
+        k_union_all<<<dim3(gx, (unsigned)G), TPB, 0, s>>>((const UGraph*)p->u_desc, p->u_rp, p->u_ci, validate, &p->dc->err);
+        if (validate) {
+            CK(cudaMemcpyAsync(p->hc, p->dc, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));
+            if (p->hc->err) return fail(ECL_SCC_ERANGE, "invalid CSR in batch");
+        }
     }
     p->launches++; k_set1<<<1, 1, 0, s>>>(p->u_rp + N, (int32_t)M);
     CK(cudaGetLastError());
@@ -888,16 +921,15 @@ int run_batched(Plan* p, int32_t G, const int32_t* n, const int64_t* nnz, const 
     int r = run_graph(p, (int32_t)N, M, p->u_rp, p->u_ci, p->u_lab, s, st, 0, nullptr, nullptr);
     p->flags = saved;
     if (r) return r;
-    const int64_t l0 = p->launches;
-    vo = 0;
-    for (int g = 0; g < G; g++) {
-        if (n[g] > 0) { p->launches++; k_split_labels<<<grid_for(n[g], TPB), TPB, 0, s>>>(n[g], p->u_lab, (int32_t)vo, labels[g]); }
-        vo += n[g];
+    {
+        int64_t nmax = 1;
+        for (int g = 0; g < G; g++) nmax = std::max<int64_t>(nmax, n[g]);
+        const unsigned gx = (unsigned)std::max<int64_t>(1, std::min<int64_t>(cdiv(nmax, TPB), std::max(1, 148 * 16 / G)));
+        p->launches++; k_split_all<<<dim3(gx, (unsigned)G), TPB, 0, s>>>((const UGraph*)p->u_desc, p->u_lab);
     }
     CK(cudaGetLastError());
     CK(cudaStreamSynchronize(s));
     if (st) st->kernel_launches = p->launches;
-    (void)l0;
     return ECL_SCC_OK;
 }
 

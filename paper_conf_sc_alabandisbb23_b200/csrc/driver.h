@@ -46,6 +46,8 @@ struct Plan {
     int32_t* u_ci;
     int32_t* u_lab;
     int64_t u_n_cap, u_m_cap;
+    void* u_desc;                        // batched: the per-graph table of the union kernels
+    int u_desc_cap;
     uint8_t* dirty;                      // 2 x dirty_cap tile flags (Phase-2 skipping)
     int64_t dirty_cap;
     // storage reordering (reorder.cuh): permuted input CSR and the storage -> caller ID map

@@ -29,6 +29,13 @@ constexpr int PACK_TH = TILE_THREADS;         // 512 threads, 4 vertices each
 #define PACK_MINB 3                           // resident CTAs per SM the kernels are built for
 #endif
 constexpr unsigned EXT_DIR = 0x8000u;
+// ECL_PROF builds: -DECL_PROF_FULL=1 (0) counts only the first (full) visits of a tile in a
+// phase (only the later ones)
+#ifdef ECL_PROF_FULL
+#define PROF_ON(full) ((full) == ECL_PROF_FULL)
+#else
+#define PROF_ON(full) true
+#endif
 // Pack slot encoding: four 16-bit local indices per word; an empty slot holds PACK_TT, the
 // index of a sentinel entry (value 0 <= every priority, scratch flag byte), so pulls and
 // notifications run without branches; bit 63 (slot 3, only set when all four slots are
@@ -326,7 +333,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
     const int2* E = ext + (int64_t)__ldg(g.optr + base) + __ldg(g.iptr + base);
 #ifdef ECL_PROF
     const long long t_start = clock64();
-    if (tid == 0) PROF_ADD(dc, 0, 1);
+    if (tid == 0 && PROF_ON(full)) PROF_ADD(dc, 0, 1);
 #endif
 
     // ---- step 1: own values and slot words (coalesced 16-byte loads, or the bulk copy),
@@ -424,8 +431,8 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
         drain_direct<TRICKS>(g, s_in, s_out, s_nin, s_nout, s_fin, s_fout, base, cnt, r0, r1, r2);
 #ifdef ECL_PROF
         r2 = warp_sum(r2);
-        if ((tid & 31) == 0) { PROF_ADD(dc, 2, r1); PROF_ADD(dc, 3, r2); }
-        if (tid == 0) PROF_ADD(dc, 1, r0);
+        if ((tid & 31) == 0 && PROF_ON(full)) { PROF_ADD(dc, 2, r1); PROF_ADD(dc, 3, r2); }
+        if (tid == 0 && PROF_ON(full)) PROF_ADD(dc, 1, r0);
 #endif
     }
 #ifdef ECL_PROF
@@ -479,7 +486,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
 #ifdef ECL_PROF
     {
         const int nr = warp_sum(__popc(rin) + __popc(rout));   // raised vertex-directions
-        if ((tid & 31) == 0 && nr) PROF_ADD(dc, 7, nr);
+        if ((tid & 31) == 0 && nr && PROF_ON(full)) PROF_ADD(dc, 7, nr);
     }
 #endif
     if (any && mark.on()) {
@@ -497,7 +504,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
     }
 #ifdef ECL_PROF
     __syncthreads();
-    if (tid == 0) {
+    if (tid == 0 && PROF_ON(full)) {
         const long long t_end = clock64();
         PROF_ADD(dc, 4, t_step1 - t_start);
         PROF_ADD(dc, 5, t_step2 - t_step1);

@@ -186,6 +186,17 @@ int ecl_scc_host(int32_t n, int64_t nnz, const int32_t* row_ptr, const int32_t* 
                  int32_t* labels_out, ecl_scc_stream_t stream, ecl_scc_plan_t plan,
                  ecl_scc_stats* stats);
 
+/* ecl_scc_batched with HOST buffers: n, nnz, row_ptr, col_idx, labels_out as in
+ * ecl_scc_batched, but row_ptr[g], col_idx[g] and labels_out[g] are HOST pointers (pinned
+ * memory gives full-speed copies).  The plan (sized for the union: sum n, sum nnz) keeps
+ * device staging copies of the whole batch (4*(sum n + G) + 4*sum nnz + 4*sum n bytes,
+ * allocated on first use); the copies run on `stream`; returns after every graph's labels
+ * are back on the host.  Errors as ecl_scc_batched. */
+int ecl_scc_batched_host(int32_t G, const int32_t* n, const int64_t* nnz,
+                         const int32_t* const* row_ptr, const int32_t* const* col_idx,
+                         int32_t* const* labels_out, ecl_scc_stream_t stream, ecl_scc_plan_t plan,
+                         ecl_scc_stats* stats);
+
 /* ---- after SCC detection: the sweep schedule ------------------------------------ */
 /* Levels of the SCC condensation (the step after SCC detection in the RTE application:
  * a transport sweep starts "from nodes with no incoming edges"; the paper tabulates

@@ -74,6 +74,7 @@ def lib() -> ctypes.CDLL:
         "ecl_scc_plan_create": [i32, i64, u32, vp],
         "ecl_scc_plan_destroy": [vp],
         "ecl_scc_batched": [i32, vp, vp, vp, vp, vp, vp, vp, vp],
+        "ecl_scc_batched_host": [i32, vp, vp, vp, vp, vp, vp, vp, vp],
         "ecl_scc_get_unique_id": [vp],
         "ecl_scc_comm_create": [i32, i32, vp, vp],
         "ecl_scc_comm_destroy": [vp],
@@ -105,7 +106,7 @@ def lib() -> ctypes.CDLL:
 
 # names exported by include/ecl_scc.h (the CPU test checks the .so exports all of them)
 ABI_SYMBOLS = ("ecl_scc", "ecl_scc_async", "ecl_scc_debug_run", "ecl_scc_plan_create",
-               "ecl_scc_plan_destroy", "ecl_scc_batched", "ecl_scc_get_unique_id",
+               "ecl_scc_plan_destroy", "ecl_scc_batched", "ecl_scc_batched_host", "ecl_scc_get_unique_id",
                "ecl_scc_comm_create", "ecl_scc_comm_destroy", "ecl_scc_partitioned",
                "ecl_scc_partitioned_emulated", "ecl_scc_partition_rows", "ecl_scc_status_string",
                "ecl_scc_last_error", "ecl_scc_version", "ecl_scc_plan_counters", "ecl_scc_levels",
@@ -240,6 +241,28 @@ def ecl_scc_batched(graphs, labels_out=None, stream=None, plan: Plan | None = No
     st = Stats() if stats else None
     _check(lib().ecl_scc_batched(G, ns, ms, rps, cis, los, _stream(stream), plan.handle if plan else None,
                                  ctypes.byref(st) if st else None), "ecl_scc_batched")
+    return (labels_out, st.as_dict()) if stats else labels_out
+
+
+def ecl_scc_batched_host(graphs, labels_out=None, stream=None, plan: Plan | None = None, stats: bool = False):
+    """ecl_scc_batched on HOST (CPU, preferably pinned) tensors: graphs = list of (row_ptr,
+    col_idx) int32 CPU tensors; the library copies the batch in, runs the union and copies
+    every graph's local labels back (ecl_scc_batched_host)."""
+    G = len(graphs)
+    for rp, ci in graphs:
+        for t, nm in ((rp, "row_ptr"), (ci, "col_idx")):
+            if t.device.type != "cpu" or t.dtype != torch.int32 or not t.is_contiguous():
+                raise ValueError(f"{nm} must be a contiguous int32 CPU tensor")
+    ns = (ctypes.c_int32 * max(G, 1))(*[g[0].numel() - 1 for g in graphs])
+    ms = (ctypes.c_int64 * max(G, 1))(*[g[1].numel() for g in graphs])
+    if labels_out is None:
+        labels_out = [torch.empty(g[0].numel() - 1, dtype=torch.int32).pin_memory() for g in graphs]
+    rps = (ctypes.c_void_p * max(G, 1))(*[g[0].data_ptr() for g in graphs])
+    cis = (ctypes.c_void_p * max(G, 1))(*[g[1].data_ptr() if g[1].numel() else None for g in graphs])
+    los = (ctypes.c_void_p * max(G, 1))(*[l.data_ptr() if l.numel() else None for l in labels_out])
+    st = Stats() if stats else None
+    _check(lib().ecl_scc_batched_host(G, ns, ms, rps, cis, los, _stream(stream), plan.handle if plan else None,
+                                      ctypes.byref(st) if st else None), "ecl_scc_batched_host")
     return (labels_out, st.as_dict()) if stats else labels_out
 
 

@@ -100,16 +100,9 @@ inline Prio make_prio(uint32_t n, bool ids) {
 __device__ __forceinline__ int ld_cg(const int32_t* p) { return __ldcg(p); }
 __device__ __forceinline__ int ld_vol(const int* p) { return *(volatile const int*)p; }
 
-__device__ __forceinline__ int warp_max(int v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v = max(v, __shfl_xor_sync(FULL, v, o));
-    return v;
-}
-__device__ __forceinline__ int warp_sum(int v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
-    return v;
-}
+// full-warp reductions: one REDUX instruction each (sm_80+) instead of five shuffle rounds
+__device__ __forceinline__ int warp_max(int v) { return __reduce_max_sync(FULL, v); }
+__device__ __forceinline__ int warp_sum(int v) { return __reduce_add_sync(FULL, v); }
 // inclusive scan over the warp
 __device__ __forceinline__ int warp_incl_scan(int v, int lane) {
 #pragma unroll

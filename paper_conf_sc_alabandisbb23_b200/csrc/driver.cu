@@ -168,6 +168,7 @@ void plan_free(Plan* p) {
     cudaFree(p->aq_state); cudaFree(p->aq_seen); cudaFree(p->aq_ctr);
     cudaFree(p->lv_ctl);
     cudaFree(p->h_rp); cudaFree(p->h_ci); cudaFree(p->h_lab);
+    cudaFree(p->hb_rp); cudaFree(p->hb_ci); cudaFree(p->hb_lab);
     if (p->hc) cudaFreeHost(p->hc);
     if (p->ev_ok)
         for (int k = 0; k < 6; k++) cudaEventDestroy(p->ev[k]);
@@ -1608,6 +1609,81 @@ int ecl_scc_batched(int32_t G, const int32_t* n, const int64_t* nnz, const int32
         plan = tmp;
     }
     int r = run_batched(&plan->p, G, n, nnz, row_ptr, col_idx, labels_out, (cudaStream_t)stream, stats);
+    if (tmp) ecl_scc_plan_destroy(tmp);
+    return r;
+}
+
+int ecl_scc_batched_host(int32_t G, const int32_t* n, const int64_t* nnz, const int32_t* const* row_ptr,
+                         const int32_t* const* col_idx, int32_t* const* labels_out, ecl_scc_stream_t stream,
+                         ecl_scc_plan_t plan, ecl_scc_stats* stats) {
+    clear_err();
+    if (G < 0 || (G > 0 && (!n || !nnz || !row_ptr || !col_idx || !labels_out)))
+        return fail(ECL_SCC_EINVAL, "batched_host: bad arguments");
+    int64_t N = 0, M = 0;
+    for (int g = 0; g < G; g++) {
+        int r = check_graph_args(n[g], nnz[g], row_ptr[g], col_idx[g], labels_out[g]);
+        if (r) return r;
+        N += n[g];
+        M += nnz[g];
+    }
+    if (stats) memset(stats, 0, sizeof(*stats));
+    if (N == 0) return ECL_SCC_OK;
+    if (N >= INT32_MAX || M >= INT32_MAX) return fail(ECL_SCC_EUNSUPPORTED, "batch union exceeds 2^31 vertices or edges");
+    if (plan && (plan->p.n_cap < N || plan->p.m_cap < M))
+        return fail(ECL_SCC_EINVAL, "plan too small for the batch union");
+    ecl_scc_plan_t tmp = nullptr;
+    if (!plan) {
+        int r = ecl_scc_plan_create((int32_t)N, M, 0, &tmp);
+        if (r) return r;
+        plan = tmp;
+    }
+    Plan* p = &plan->p;
+    cudaStream_t s = (cudaStream_t)stream;
+    // device staging of the whole batch (graph g at offsets sum_{h<g} (n_h + 1), sum nnz_h, sum n_h)
+    const int64_t rp_need = N + G, ci_need = std::max<int64_t>(M, 1), lab_need = N;
+    cudaError_t e = cudaSuccess;
+    if (p->hb_rp_cap < rp_need) {
+        cudaFree(p->hb_rp); p->hb_rp = nullptr; p->hb_rp_cap = 0;
+        e = cudaMalloc((void**)&p->hb_rp, sizeof(int32_t) * (size_t)rp_need);
+        if (e == cudaSuccess) p->hb_rp_cap = rp_need;
+    }
+    if (e == cudaSuccess && p->hb_ci_cap < ci_need) {
+        cudaFree(p->hb_ci); p->hb_ci = nullptr; p->hb_ci_cap = 0;
+        e = cudaMalloc((void**)&p->hb_ci, sizeof(int32_t) * (size_t)ci_need);
+        if (e == cudaSuccess) p->hb_ci_cap = ci_need;
+    }
+    if (e == cudaSuccess && p->hb_lab_cap < lab_need) {
+        cudaFree(p->hb_lab); p->hb_lab = nullptr; p->hb_lab_cap = 0;
+        e = cudaMalloc((void**)&p->hb_lab, sizeof(int32_t) * (size_t)lab_need);
+        if (e == cudaSuccess) p->hb_lab_cap = lab_need;
+    }
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        if (tmp) ecl_scc_plan_destroy(tmp);
+        return fail(ECL_SCC_ENOMEM, "batch host-buffer staging: %s", cudaGetErrorString(e));
+    }
+    std::vector<const int32_t*> drp(G), dci(G);
+    std::vector<int32_t*> dlab(G);
+    int64_t ro = 0, co = 0, lo = 0;
+    for (int g = 0; g < G && e == cudaSuccess; g++) {
+        drp[g] = p->hb_rp + ro;
+        dci[g] = nnz[g] ? p->hb_ci + co : nullptr;
+        dlab[g] = n[g] ? p->hb_lab + lo : nullptr;
+        e = cudaMemcpyAsync(p->hb_rp + ro, row_ptr[g], sizeof(int32_t) * ((size_t)n[g] + 1), cudaMemcpyHostToDevice, s);
+        if (e == cudaSuccess && nnz[g])
+            e = cudaMemcpyAsync(p->hb_ci + co, col_idx[g], sizeof(int32_t) * (size_t)nnz[g], cudaMemcpyHostToDevice, s);
+        ro += n[g] + 1;
+        co += nnz[g];
+        lo += n[g];
+    }
+    int r = e == cudaSuccess ? ECL_SCC_OK : fail(ECL_SCC_ECUDA, "host-to-device copy: %s", cudaGetErrorString(e));
+    if (!r) r = run_batched(p, G, n, nnz, drp.data(), dci.data(), dlab.data(), s, stats);
+    for (int g = 0; g < G && !r; g++) {
+        if (!n[g]) continue;
+        e = cudaMemcpyAsync(labels_out[g], dlab[g], sizeof(int32_t) * (size_t)n[g], cudaMemcpyDeviceToHost, s);
+        if (e != cudaSuccess) r = fail(ECL_SCC_ECUDA, "device-to-host copy: %s", cudaGetErrorString(e));
+    }
+    if (!r && (e = cudaStreamSynchronize(s)) != cudaSuccess) r = fail(ECL_SCC_ECUDA, "device-to-host copy: %s", cudaGetErrorString(e));
     if (tmp) ecl_scc_plan_destroy(tmp);
     return r;
 }

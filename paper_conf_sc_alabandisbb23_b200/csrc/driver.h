@@ -70,6 +70,8 @@ struct Plan {
     void* lv_ctl;                        // levels.cuh LvCtl (device)
     int32_t *h_rp, *h_ci, *h_lab;        // ecl_scc_host: device copies of the caller's host buffers
     int64_t h_n_cap, h_m_cap;
+    int64_t hb_rp_cap, hb_ci_cap, hb_lab_cap;   // ecl_scc_batched_host: staging of a whole batch
+    int32_t *hb_rp, *hb_ci, *hb_lab;
     int lv_resident;                     // co-resident CTAs of k_lv_run
     int64_t lk_resident;                 // resident CTAs of k_lk_run (levels, tile mode)
     bool kw;                             // compaction with 4-byte keep words (rows <= KW_DEG)

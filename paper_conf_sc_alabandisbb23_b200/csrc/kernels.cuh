@@ -178,6 +178,7 @@ __device__ __forceinline__ bool trimmed(const int2* __restrict__ kio, int x) {
 // byte 2 the out-row mask, byte 3 the in-row mask (Phase 3's kept entries; after the trim, the
 // survivors -- the degree bytes, which other threads' trim tests read, stay as they were)
 constexpr int KW_DEG = 8;
+static_assert(KW_DEG * 32 < 1024, "k_compact_map packs the warp prefixes of the survivor degrees in 10 bits");
 __device__ __forceinline__ bool trimmed_kw(const uint32_t* __restrict__ kw, int x) {
     const uint32_t w = __ldg(kw + x);
     return ((w & 0xFFu) == 0) | ((w & 0xFF00u) == 0);
@@ -587,9 +588,18 @@ static __global__ void __launch_bounds__(TPB_COMPACT, 8) k_compact_map(WGraph g,
     if (g.hpos && valid && !alive && g.hpos[i] >= 0 && (FIRST || cin[i] != cout[i]) && !(trim && trimmed(kio, (int)i)))
         alive = 1;                                     // (the same rule as k_compact_count)
     const int4 base = wscan[i >> 5];
-    const int j = warp_incl_scan(alive, lane) - alive + base.x;
-    const int po = warp_incl_scan(c.x, lane) - c.x + base.y;
-    const int pi = warp_incl_scan(c.y, lane) - c.y + base.z;
+    int j, po, pi;
+    if (KW) {      // degrees <= KW_DEG: the three warp prefixes packed into one scan (6 + 10 + 10 bits)
+        const int pk = alive | c.x << 6 | c.y << 16;
+        const int ex = warp_incl_scan(pk, lane) - pk;
+        j = (ex & 63) + base.x;
+        po = ((ex >> 6) & 1023) + base.y;
+        pi = ((ex >> 16) & 1023) + base.z;
+    } else {
+        j = warp_incl_scan(alive, lane) - alive + base.x;
+        po = warp_incl_scan(c.x, lane) - c.x + base.y;
+        pi = warp_incl_scan(c.y, lane) - c.y + base.z;
+    }
     if (!valid) return;
     const int v = g.act ? g.act[i] : (int)i;          // storage ID
     const int ov = orig ? orig[v] : v;                 // caller's ID (reorder.cuh)

@@ -36,6 +36,13 @@ constexpr unsigned EXT_DIR = 0x8000u;
 #else
 #define PROF_ON(full) true
 #endif
+// ECL_PROF builds with -DECL_PROF_PROTO: counters 4-6 hold k_prop_async's per-visit protocol
+// split instead (claims, the visit, fences + marks + finish)
+#ifdef ECL_PROF_PROTO
+#define PROF_PROTO 1
+#else
+#define PROF_PROTO 0
+#endif
 // Pack slot encoding: four 16-bit local indices per word; an empty slot holds PACK_TT, the
 // index of a sentinel entry (value 0 <= every priority, scratch flag byte), so pulls and
 // notifications run without branches; bit 63 (slot 3, only set when all four slots are
@@ -195,23 +202,26 @@ __device__ __forceinline__ void drain_direct(const WGraph& g, int* __restrict__ 
 #ifdef ECL_PROF
             if ((tid & 31) == 0) prof_drains++;
 #endif
-            const unsigned wi = (unsigned)lds_v(a_fin + 4 * tid), wo = (unsigned)lds_v(a_fout + 4 * tid);
-            const unsigned items = gather4(wi) | (gather4(wo) << 4);
-            if (!__any_sync(FULL, items != 0)) break;
-            if (items) {
+            const unsigned ii = gather4((unsigned)lds_v(a_fin + 4 * tid));
+            const unsigned oo = gather4((unsigned)lds_v(a_fout + 4 * tid));
+            if (!__any_sync(FULL, (ii | oo) != 0)) break;
+            // one v_in item AND one v_out item per lane and round: a warp holding both kinds
+            // runs both paths anyway (divergence), so a lane with both does both
+            if (ii | oo) {
                 worked = 1;
 #ifdef ECL_PROF
-                prof_pushes++;
+                prof_pushes += (ii != 0) + (oo != 0);
 #endif
-                const int bit = __ffs(items) - 1;
-                const int v = v0 + (bit & 3);
-                const unsigned keep = ~(0xFFu << (8 * (bit & 3)));
-                if (bit & 4)
-                    drain_item<true, TRICKS>(g, s_out, s_in, s_nout, s_nin, s_fout, a_out, a_nout, a_nin, a_fout, base,
-                                             cnt, v, tid, keep);
-                else
-                    drain_item<false, TRICKS>(g, s_in, s_out, s_nin, s_nout, s_fin, a_in, a_nin, a_nout, a_fin, base,
-                                              cnt, v, tid, keep);
+            }
+            if (ii) {
+                const int k = __ffs(ii) - 1;
+                drain_item<false, TRICKS>(g, s_in, s_out, s_nin, s_nout, s_fin, a_in, a_nin, a_nout, a_fin, base, cnt,
+                                          v0 + k, tid, ~(0xFFu << (8 * k)));
+            }
+            if (oo) {
+                const int k = __ffs(oo) - 1;
+                drain_item<true, TRICKS>(g, s_out, s_in, s_nout, s_nin, s_fout, a_out, a_nout, a_nin, a_fout, base, cnt,
+                                         v0 + k, tid, ~(0xFFu << (8 * k)));
             }
             __syncwarp();
         }
@@ -504,7 +514,7 @@ __device__ __forceinline__ int pack_visit(const WGraph& g, int32_t* __restrict__
     }
 #ifdef ECL_PROF
     __syncthreads();
-    if (tid == 0 && PROF_ON(full)) {
+    if (tid == 0 && PROF_ON(full) && !PROF_PROTO) {
         const long long t_end = clock64();
         PROF_ADD(dc, 4, t_step1 - t_start);
         PROF_ADD(dc, 5, t_step2 - t_step1);
@@ -715,6 +725,9 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
     for (;;) {
         // warp 0 claims: one cursor step covers CLAIM consecutive sweep positions, every
         // dirty tile among them is claimed and the CTA visits them in sweep order (a run)
+#ifdef ECL_PROF
+        const long long t_claim = clock64();
+#endif
         if (tid < 32) {
             const int lane = tid;
             const int got = aq_claim(Q, ntiles, claim, lane, s_claim, s_seen, t0, dc);
@@ -726,6 +739,10 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             __threadfence();                                      // claims before the value reads
         }
         __syncthreads();
+#ifdef ECL_PROF
+        long long tp = clock64();
+        if (tid == 0 && PROF_PROTO) PROF_ADD(dc, 4, tp - t_claim);
+#endif
         const int nclaim = s_nclaim;
         if (nclaim == 0) break;
         for (int j = 0; j < nclaim; j++) {
@@ -734,6 +751,10 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             __syncthreads();
             pack_visit<MarkSet, HALO, TRICKS>(g, cin, cout, pnin, pnout, ext, ext_cnt, dc, tile, full, MarkSet{s_set, Q}, S,
                                       j + 1 < nclaim ? s_claim[j + 1] : -1, &T, HALO ? &H : nullptr);
+#ifdef ECL_PROF
+            const long long tv = clock64();
+            if (tid == 0 && PROF_PROTO) PROF_ADD(dc, 5, tv - tp);
+#endif
             __threadfence();                                      // values before marks
             __syncthreads();
             for (int i = tid; i < MSET; i += PACK_TH)
@@ -744,6 +765,10 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
                 if (atomicCAS(Q.tstate + tile, 2, 0) == 2) atomicAdd(Q.ctr + AQ_PEND, ~0ull);
                 else atomicExch(Q.tstate + tile, 1);
             }
+#ifdef ECL_PROF
+            tp = clock64();
+            if (tid == 0 && PROF_PROTO) PROF_ADD(dc, 6, tp - tv);
+#endif
         }
         __syncthreads();                                          // s_claim is rewritten next
     }

@@ -44,6 +44,8 @@ def test_argument_errors_without_gpu():
     assert L.ecl_scc(10, 1 << 31, ctypes.c_void_p(16), ctypes.c_void_p(16), ctypes.c_void_p(16)) == E.EUNSUPPORTED
     assert L.ecl_scc_plan_create(-1, 0, 0, None) == E.EINVAL
     assert L.ecl_scc_batched(-1, None, None, None, None, None, None, None, None) == E.EINVAL
+    assert L.ecl_scc_batched_host(-1, None, None, None, None, None, None, None, None) == E.EINVAL
+    assert L.ecl_scc_batched_host(0, None, None, None, None, None, None, None, None) == E.OK
 
 
 def test_partition_rows_balanced():

@@ -266,6 +266,20 @@ def test_c5_batched_meshes_full_64():
             np.testing.assert_array_equal(lab.cpu().numpy(), truth[d], err_msg=f"rank {r} ordinate {d}")
 
 
+def test_batched_host_buffers():
+    """ecl_scc_batched_host (the C5 e2e path of bench.py): pinned host CSRs in, host labels
+    out, equal to Tarjan's per graph; an empty graph inside the batch; plan reuse."""
+    graphs = [gen.mesh(24, gen.ordinate(d), seed=40 + d, order="blocked8", **gen.C4_MESH) for d in range(5)]
+    graphs.insert(2, gen.Graph(np.zeros(1, dtype=np.int32), np.zeros(0, dtype=np.int32), "empty"))
+    hg = [(torch.from_numpy(g.row_ptr).pin_memory(), torch.from_numpy(g.col_idx).pin_memory()) for g in graphs]
+    plan = E.Plan(sum(g.n for g in graphs), sum(g.nnz for g in graphs))
+    for _ in range(2):
+        labs = E.ecl_scc_batched_host(hg, plan=plan)
+        for g, lab in zip(graphs, labs):
+            assert lab.device.type == "cpu"
+            np.testing.assert_array_equal(lab.numpy(), oracle.tarjan_labels(g.row_ptr, g.col_idx))
+
+
 def test_repeated_runs_with_plan_reuse_are_stable():
     """Races show up under repetition: the same plan, several graphs and orders, many runs."""
     graphs = [gen.mesh(60, gen.ordinate(d), seed=4 + d, order=o, **gen.C4_MESH)

@@ -21,3 +21,4 @@ print({k: v for k, v in st.items() if k not in ("edges_kept",)})
 c = plan.counters()
 print('counters [visits, block_rounds, warp_drains, vertex_pushes]:', c[:4])
 if c[0]: print('cycles per visit: step1 %.0f step2 %.0f step3 %.0f; raised vertex-dirs per visit %.0f' % (c[4]/c[0], c[5]/c[0], c[6]/c[0], c[7]/c[0]))
+if os.environ.get("PROF_PROTO") and c[0]: print('protocol cycles per visit: claim %.0f visit %.0f fences+marks+finish %.0f' % (c[4]/c[0], c[5]/c[0], c[6]/c[0]))

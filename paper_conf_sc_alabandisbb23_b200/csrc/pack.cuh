@@ -155,7 +155,9 @@ __device__ __forceinline__ void drain_item(const WGraph& g, int* __restrict__ s_
                                            const unsigned long long* __restrict__ s_dep, unsigned* __restrict__ s_f,
                                            unsigned a_sig, unsigned a_src, unsigned a_dep, unsigned a_f, int base,
                                            int cnt, int v, int tid, unsigned keep) {
-    atomicAnd(s_f + tid, keep);
+    // clear the item's flag byte (other bytes of the word may be set concurrently): a shared
+    // reduction on the 32-bit window address (atomicAnd on s_f would rebuild it from the CTA id)
+    asm volatile("red.shared.and.b32 [%0], %1;" ::"r"(a_f + 4 * tid), "r"(keep) : "memory");
     const unsigned long long src = lds_v64(a_src + 8 * v);
     const int old = lds_v(a_sig + 4 * v);
     int val = ppull_a(a_sig, src, old);

@@ -383,12 +383,21 @@ static int compact_finish(Plan* p, const int32_t* cin, const int32_t* cout, int 
     p->launches++; k_compact_count<FIRST, TRIM, FOUR, KW><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
     int r = scan_excl<I3>(p, (const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
     if (r) return r;
+    if (KW && !trim2 && !p->min_in[ob]) {               // keep words: four vertices per thread
+        p->launches++;
+        k_compact_map4<FIRST><<<(unsigned)cdiv(cdiv((int64_t)gk.na, MAP4 * WARP) * WARP, TPB), TPB, 0, s>>>(
+            gk, cin, cout, (const uint32_t*)p->emask, p->wscan, &p->dc->totals, p->newidx, p->act[ob], p->cin[ob],
+            p->cout[ob], p->optr[ob], p->iptr[ob], labels, P, p->orig_cur, pk,
+            MapExtra{nullptr, nullptr, nullptr, p->kio, TRIM ? 1 : 0, gk.hpos ? p->hpos[ob] : nullptr, p->lab_lo,
+                     p->lab_hi, p->slot});
+    } else {
     p->launches++; k_compact_map<FIRST, KW><<<grid, TPB, 0, s>>>(gk, cin, cout, KW ? (const int2*)p->emask : p->cnt, p->wscan, &p->dc->totals, p->newidx, p->act[ob],
                                               p->cin[ob], p->cout[ob], p->optr[ob], p->iptr[ob], labels,
                                               chunk_buf(p, p->cb ^ 1), &p->dc->nchunks, (int)p->chunk_cap, P, p->orig_cur, pk,
                                               MapExtra{p->min_in[ob], p->min_out[ob], trim2 ? p->t2 : nullptr, p->kio,
                                                        TRIM ? 1 : 0, gk.hpos ? p->hpos[ob] : nullptr, p->lab_lo,
                                                        p->lab_hi, p->slot});
+    }
     p->launches++; k_compact_scatter<FIRST, TRIM, FOUR, KW><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->newidx, p->optr[ob],
                                                           p->iptr[ob], p->oadj[ob], p->iadj[ob], chunked, p->emask, pk);
     if (chunked) {
@@ -797,8 +806,8 @@ int run_graph(Plan* p, int32_t n, int64_t nnz, const int32_t* rp, const int32_t*
         if (!P.ids && !stopped) {
             // labels of finished vertices are still max priorities: map to max vertex IDs
             const unsigned gr = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
-            p->launches++; k_relabel_rep<<<gr, TPB, 0, s>>>(n, labels, p->kin, P);
-            p->launches++; k_relabel_max<<<gr, TPB, 0, s>>>(n, labels, p->kin, P);
+            CK(cudaMemsetAsync(p->kin, 0xFF, sizeof(int32_t) * (size_t)n, s));
+            p->launches++; k_relabel_fold<<<gr, TPB, 0, s>>>(n, labels, p->kin);
             p->launches++; k_relabel_apply<<<gr, TPB, 0, s>>>(n, labels, p->kin);
             CK(cudaGetLastError());
         }
@@ -1243,9 +1252,9 @@ int run_halo(std::vector<HaloRank*>& R, Exchange& X, int32_t n, uint32_t flags, 
     HaloRank& Q = *R[0];
     const unsigned gr = std::min<unsigned>(grid_for(n, TPB), 148 * 16);
     if (!Pr.ids) {
-        Q.p.launches += 3;
-        k_relabel_rep<<<gr, TPB, 0, s>>>(n, Q.lab, Q.gidx, Pr);
-        k_relabel_max<<<gr, TPB, 0, s>>>(n, Q.lab, Q.gidx, Pr);
+        Q.p.launches += 2;
+        CK(cudaMemsetAsync(Q.gidx, 0xFF, sizeof(int32_t) * (size_t)n, s));
+        k_relabel_fold<<<gr, TPB, 0, s>>>(n, Q.lab, Q.gidx);
         k_relabel_apply<<<gr, TPB, 0, s>>>(n, Q.lab, Q.gidx);
     }
     CK(cudaMemcpyAsync(labels, Q.lab, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToDevice, s));

@@ -644,32 +644,103 @@ static __global__ void __launch_bounds__(TPB_COMPACT, 8) k_compact_map(WGraph g,
     }
 }
 
-// Final labels under priorities: an SCC is named by s = max priority; its label is the
-// largest vertex ID with signature s.  rep: the member with pi(v) == s seeds the slot;
-// max: the others fold in with atomicMax; apply: write the label.
-static __global__ void k_relabel_rep(int32_t n, int32_t* __restrict__ labels, int32_t* __restrict__ slot, Prio P) {
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-        const int l = labels[v];
-        if (l < 0 && (int)prio_of(P, (uint32_t)v) == -l - 1) slot[-l - 1] = (int)v;
+// k_compact_map for the keep-word layout (rows <= KW_DEG, no FOUR / TRIM2): a warp maps 128
+// consecutive vertices, lane l taking l, l + 32, l + 64, l + 96, so each thread has four
+// independent coalesced loads of keep words (and IDs, and signatures) in flight instead of one
+// -- the one-vertex form stalls on those streaming loads (ncu: 35% of DRAM peak, most stall
+// samples at the keep-word and ID loads) -- while every store stays a coalesced warp row.
+// Same outputs as k_compact_map<FIRST, true>.  The warp's 128 vertices are 4 scan warps of
+// k_compact_count: row k's base is wscan of its first vertex.
+constexpr int MAP4 = 4;
+template <bool FIRST>
+static __global__ void __launch_bounds__(TPB_COMPACT, 6) k_compact_map4(WGraph g, const int32_t* __restrict__ cin, const int32_t* __restrict__ cout,
+                              const uint32_t* __restrict__ kw, const int4* __restrict__ wscan,
+                              const int4* __restrict__ totals, int32_t* __restrict__ newidx,
+                              int32_t* __restrict__ act2, int32_t* __restrict__ cin2, int32_t* __restrict__ cout2,
+                              int32_t* __restrict__ optr2, int32_t* __restrict__ iptr2, int32_t* __restrict__ labels,
+                              Prio P, const int32_t* __restrict__ orig, PackOut pk, MapExtra X) {
+    const int lane = threadIdx.x & 31;
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t wb = (t - lane) * MAP4;              // the warp's first vertex
+    if (t == 0) {
+        const int4 tt = *totals;
+        optr2[tt.x] = tt.y;
+        iptr2[tt.x] = tt.z;
+    }
+    if (pk.pnin) {                         // pack: empty slot words past the last vertex of the last tile
+        const int na2 = totals->x;
+        const int pad_end = (na2 + TILE - 1) & ~(TILE - 1);
+        for (int64_t k = na2 + t; k < pad_end; k += (int64_t)gridDim.x * blockDim.x) {
+            pk.pnin[k] = PK_EMPTY;
+            pk.pnout[k] = PK_EMPTY;
+        }
+    }
+    const int na = g.na;
+    if (wb >= na) return;                              // (warp-uniform)
+    uint32_t w[MAP4];
+    int sa[MAP4], sb[MAP4], av[MAP4];
+#pragma unroll
+    for (int k = 0; k < MAP4; k++) {
+        const int64_t i = wb + 32 * k + lane;
+        const bool ok = i < na;
+        w[k] = ok ? __ldg(kw + i) : 0u;
+        av[k] = g.act ? (ok ? __ldg(g.act + i) : 0) : (int)i;
+        if (!FIRST) { sa[k] = ok ? __ldcg(cin + i) : 0; sb[k] = ok ? __ldcg(cout + i) : 0; }
+    }
+#pragma unroll
+    for (int k = 0; k < MAP4; k++) {
+        const int64_t i = wb + 32 * k + lane;
+        if (wb + 32 * k >= na) break;                  // (warp-uniform)
+        const bool ok = i < na;
+        const int co = __popc((w[k] >> 16) & 0xFFu), ci = __popc(w[k] >> 24);
+        int al = (co + ci) > 0;
+        if (g.hpos && ok && !al && g.hpos[i] >= 0 && (FIRST || sa[k] != sb[k]) && !(X.trim && trimmed(X.kio, (int)i)))
+            al = 1;
+        const int4 base = wscan[(wb + 32 * k) >> 5];
+        const int pk_ = al | co << 8 | ci << 19;       // per scan warp: alive <= 32, degrees <= 256
+        const int ex = warp_incl_scan(pk_, lane) - pk_;
+        if (!ok) continue;
+        const int j = (ex & 0xFF) + base.x, po = ((ex >> 8) & 0x7FF) + base.y, pi = ((ex >> 19) & 0x7FF) + base.z;
+        const int v = av[k];
+        const int ov = orig ? orig[v] : v;
+        if (al) {
+            newidx[i] = j;
+            act2[j] = v;
+            if (pk.pnin && (j & (TILE - 1)) == 0) pk.ext_cnt[j / TILE] = 0;
+            const int pv = (int)prio_of(P, (uint32_t)ov);
+            cin2[j] = pv;       // Phase 1: v_in <- v_id, v_out <- v_id for the unfinished
+            cout2[j] = pv;
+            if (X.hpos2) X.hpos2[j] = g.hpos[i];
+            if (X.slot) X.slot[pv] = j;
+            optr2[j] = po;
+            iptr2[j] = pi;
+        } else {
+            newidx[i] = -1;
+            int lab = ov;      // unfinished (or trimmed) and edgeless: a singleton SCC
+            if (!FIRST && sa[k] == sb[k]) lab = P.ids ? sa[k] : -(sa[k] + 1);
+            if (ov >= X.lab_lo && ov < X.lab_hi) labels[ov] = lab;
+        }
     }
 }
-static __global__ void k_relabel_max(int32_t n, const int32_t* __restrict__ labels, int32_t* __restrict__ slot, Prio P) {
-    // lanes that target the same slot (a giant SCC: most of them) combine first, so the
-    // slot sees one atomic per group instead of one per vertex
+
+// Final labels under priorities: an SCC is named by s = max priority; its label is the
+// largest vertex ID with signature s: the slots (cleared to -1) take the max ID of every
+// signature (fold: lanes with the same slot grouped first, so a giant SCC costs one atomic
+// per warp), then every finished vertex reads its slot (apply).
+static __global__ void k_relabel_fold(int32_t n, const int32_t* __restrict__ labels, int32_t* __restrict__ slot) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t start = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     for (int64_t v0 = start - (threadIdx.x & 31); v0 < n; v0 += stride) {
         const int64_t v = v0 + (threadIdx.x & 31);
-        int key = -1, val = -1;
+        int key = -1;
         if (v < n) {
             const int l = labels[v];
-            if (l < 0 && (int)prio_of(P, (uint32_t)v) != -l - 1) { key = -l - 1; val = (int)v; }
+            if (l < 0) key = -l - 1;
         }
-        if (!__any_sync(FULL, key >= 0)) continue;           // singletons only (most warps)
+        if (!__any_sync(FULL, key >= 0)) continue;
         const unsigned grp = __match_any_sync(FULL, key);
-        int m = val;
-        for (unsigned g = grp; g; g &= g - 1) m = max(m, __shfl_sync(grp, val, __ffs(g) - 1));
-        if (key >= 0 && (threadIdx.x & 31) == __ffs(grp) - 1) atomicMax(slot + key, m);
+        // lanes hold increasing v: the group's last lane has its largest ID
+        if (key >= 0 && (threadIdx.x & 31) == 31 - __clz(grp)) atomicMax(slot + key, (int)v);
     }
 }
 static __global__ void k_relabel_apply(int32_t n, int32_t* __restrict__ labels, const int32_t* __restrict__ slot) {

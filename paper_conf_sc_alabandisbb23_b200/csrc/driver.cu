@@ -380,7 +380,12 @@ static int compact_finish(Plan* p, const int32_t* cin, const int32_t* cout, int 
         p->launches++;
         k_count_chunks<FIRST, TRIM, FOUR><<<chunk_grid(nc), TPB, 0, s>>>(gk, cur, nc, cin, cout, p->kio, p->chunk_cnt, p->hcnt);
     }
-    p->launches++; k_compact_count<FIRST, TRIM, FOUR, KW><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
+    p->launches++;
+    if (KW && !FOUR)                                   // keep words: two lane-strided vertices per thread
+        k_compact_count2<FIRST, TRIM><<<(unsigned)cdiv(nw * WARP / CNT2, TPB), TPB, 0, s>>>(gk, cin, cout, (uint32_t*)p->emask,
+                                                                                           p->wsum, nw);
+    else
+        k_compact_count<FIRST, TRIM, FOUR, KW><<<grid, TPB, 0, s>>>(gk, cin, cout, p->kio, p->cnt, p->wsum, chunked, p->hcnt, p->emask);
     int r = scan_excl<I3>(p, (const I3*)p->wsum, nw, (I3*)p->wscan, (I3*)&p->dc->totals, p->bsum, 0, s);
     if (r) return r;
     if (KW && !trim2 && !p->min_in[ob]) {               // keep words: four vertices per thread

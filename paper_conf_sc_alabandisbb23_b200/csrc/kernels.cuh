@@ -477,6 +477,101 @@ static __global__ void k_compact_count(WGraph g, const int32_t* __restrict__ cin
     if (lane == 0) wsum[i >> 5] = make_int4(sa, so, si, sk);
 }
 
+// k_compact_count for the keep-word layout (no FOUR): a warp counts 64 consecutive vertices,
+// lane l taking l and l + 32, with the loads of both vertices -- keep word, row offsets,
+// signatures, then the far ends of their kept entries, then the far ends' keep words -- issued
+// together (the one-vertex form stalls on those dependent gathers, ncu: 35% of DRAM peak).  Up
+// to CNT2_E kept entries per vertex go through the overlapped path (a tet mesh has at most 4
+// in + out), the rest through trim_mask.  Same outputs as k_compact_count<FIRST, TRIM, false,
+// true>: the trimmed survivor masks in the keep word, per-32-vertex totals (rows < nw).
+constexpr int CNT2 = 2, CNT2_E = 4;
+template <bool FIRST, bool TRIM>
+static __global__ void __launch_bounds__(TPB_COMPACT, 6) k_compact_count2(WGraph g, const int32_t* __restrict__ cin,
+                                                                         const int32_t* __restrict__ cout,
+                                                                         uint32_t* __restrict__ kw, int4* __restrict__ wsum,
+                                                                         int64_t nw) {
+    const int lane = threadIdx.x & 31;
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t wb = (t - lane) * CNT2;             // the warp's first vertex
+    if ((wb >> 5) >= nw) return;                       // (warp-uniform)
+    const int na = g.na;
+    uint32_t w[CNT2];
+    int ob[CNT2], ib[CNT2];
+    bool live[CNT2];
+#pragma unroll
+    for (int k = 0; k < CNT2; k++) {
+        const int64_t i = wb + 32 * k + lane;
+        const bool ok = i < na;
+        w[k] = ok ? kw[i] : 0u;
+        ob[k] = ok ? __ldg(g.optr + i) : 0;
+        ib[k] = ok ? __ldg(g.iptr + i) : 0;
+        live[k] = ok && (FIRST || __ldcg(cin + i) != __ldcg(cout + i));
+    }
+    unsigned so[CNT2], si[CNT2];
+#pragma unroll
+    for (int k = 0; k < CNT2; k++) {
+        so[k] = (w[k] >> 16) & 0xFFu;
+        si[k] = w[k] >> 24;
+        if (!live[k]) so[k] = si[k] = 0;
+    }
+    if (TRIM) {
+        // far ends of the first CNT2_E kept entries of each vertex (out-row bits first)
+        int x[CNT2][CNT2_E];
+        unsigned rest[CNT2];
+#pragma unroll
+        for (int k = 0; k < CNT2; k++) {
+            const bool go = live[k] && (w[k] & 0xFFu) && (w[k] & 0xFF00u);
+            unsigned m = go ? (so[k] | si[k] << 8) : 0u;
+#pragma unroll
+            for (int q = 0; q < CNT2_E; q++) {
+                x[k][q] = -1;
+                if (m) {
+                    const int b = __ffs(m) - 1;
+                    m &= m - 1;
+                    x[k][q] = b < 8 ? __ldg(g.oadj + ob[k] + b) : __ldg(g.iadj + ib[k] + (b - 8));
+                }
+            }
+            rest[k] = m;
+            if (!go) so[k] = si[k] = 0;
+        }
+        uint32_t y[CNT2][CNT2_E];
+#pragma unroll
+        for (int k = 0; k < CNT2; k++)
+#pragma unroll
+            for (int q = 0; q < CNT2_E; q++) y[k][q] = x[k][q] >= 0 ? __ldg(kw + x[k][q]) : 0x0101u;
+#pragma unroll
+        for (int k = 0; k < CNT2; k++) {
+            // the entries behind x[k][q], in the same order: clear the trimmed ones
+            unsigned m = so[k] | si[k] << 8, keep = m;
+#pragma unroll
+            for (int q = 0; q < CNT2_E; q++) {
+                if (!m) break;
+                const int b = __ffs(m) - 1;
+                m &= m - 1;
+                if (((y[k][q] & 0xFFu) == 0) | ((y[k][q] & 0xFF00u) == 0)) keep &= ~(1u << b);
+            }
+            if (rest[k]) {                                // more kept entries than CNT2_E
+                const unsigned ro = rest[k] & 0xFFu, ri = rest[k] >> 8;
+                const unsigned to = trim_mask<true>(g.oadj, ob[k], ro, 0, nullptr, kw);
+                const unsigned ti = trim_mask<true>(g.iadj, ib[k], ri, 0, nullptr, kw);
+                keep = (keep & ~rest[k]) | to | ti << 8;
+            }
+            so[k] = keep & 0xFFu;
+            si[k] = keep >> 8;
+            const int64_t i = wb + 32 * k + lane;
+            if (i < na) kw[i] = (w[k] & 0xFFFFu) | so[k] << 16 | si[k] << 24;
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < CNT2; k++) {
+        const int nout = __popc(so[k]), nin = __popc(si[k]);
+        const int alive = (nout + nin) > 0, kept = (int)((w[k] >> 8) & 0xFFu);
+        const int sa = warp_sum(alive), so_ = warp_sum(nout), si_ = warp_sum(nin), sk = warp_sum(kept);
+        const int64_t r = (wb + 32 * k) >> 5;
+        if (lane == 0 && r < nw) wsum[r] = make_int4(sa, so_, si_, sk);
+    }
+}
+
 // Trim-2 (McLendon; reading 17), one round on the kept graph together with
 // Trim-1: an unfinished vertex i whose only kept in-edge entry comes from w, while w's only
 // kept in-edge entry comes from i (i -> w kept, kin(w) == 1) -- or the same with out-edges --

@@ -366,8 +366,7 @@ k_prop_cluster(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, 
             __threadfence();
             cl.sync();                                          // both CTAs' marks before the finish
             if (rank == 0 && tid == 0) {
-                if (atomicCAS(Q.tstate + pt, 2, 0) == 2) atomicAdd(Q.ctr + AQ_PEND, ~0ull);
-                else atomicExch(Q.tstate + pt, 1);
+                aq_finish(Q, pt);
             }
         }
     }

@@ -493,8 +493,7 @@ static __global__ void __launch_bounds__(LK_TH, 3) k_lk_run(LkState L, DevCounte
             }
             __syncthreads();                           // marks (pending++) before finish
             if (tid == 0) {
-                if (atomicCAS(Q.tstate + tile, 2, 0) == 2) atomicAdd(Q.ctr + AQ_PEND, ~0ull);
-                else atomicExch(Q.tstate + tile, 1);
+                aq_finish(Q, tile);
             }
         }
         __syncthreads();                               // s_claim is rewritten next

@@ -588,10 +588,13 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
 // Tile state machine (tstate): 0 clean, 1 dirty, 2 running, 3 running + dirtied again.
 //   mark(t):   0 -> 1 (pending++); 2 -> 3; 1, 3 unchanged
 //   claim(t):  1 -> 2 (the first visit of a tile in the phase is a full one)
-//   finish(t): 2 -> 0 (pending--); 3 -> 1
-// pending counts tiles in states 1-3.  A visit's marks (pending++) precede its own
-// finish (pending--), so pending == 0 means no visit is running and every tile's last
-// visit saw its final inputs: the Phase-2 fixed point (Alg. 1 l.7-14).  Values are
+//   finish(t): 2 -> 0; 3 -> 1 (state -= 2)
+// pending = #state 1 + #state 2 + 2 * #state 3, so every state change by a mark (0 -> 1,
+// 2 -> 3) adds one and every finish subtracts one: the finish is two fire-and-forget
+// reductions (no compare-and-swap round trip in the visit loop), and pending == 0 still
+// means no tile is dirty or running.  A visit's marks (pending++) precede its own finish
+// (pending--), so pending == 0 means no visit is running and every tile's last visit saw
+// its final inputs: the Phase-2 fixed point (Alg. 1 l.7-14).  Values are
 // written (st.cg) and fenced before the marks; a claimer fences after its claim and reads
 // through L2, so it sees every value written before the state change it observed.
 // the cursor, the pending count and the stop word sit in separate 128-byte lines: claimers
@@ -603,14 +606,19 @@ struct AsyncQ {
     unsigned long long* ctr;      // [AQ_CUR] cursor, [AQ_PEND] pending, [AQ_STOP] stop
 };
 __device__ __forceinline__ void aq_mark(const AsyncQ& Q, int t) {
-    int st = *(volatile int*)(Q.tstate + t);
+    int st = 0;                                   // (try clean first: no separate read)
     for (;;) {
-        if (st == 1 || st == 3) return;
         const int old = atomicCAS(Q.tstate + t, st, st == 0 ? 1 : 3);
         if (old == st) break;
+        if (old == 1 || old == 3) return;         // already dirty
         st = old;
     }
-    if (st == 0) atomicAdd(Q.ctr + AQ_PEND, 1ull);
+    atomicAdd(Q.ctr + AQ_PEND, 1ull);             // 0 -> 1 or 2 -> 3
+}
+// the end of a visit (after its marks): 2 -> 0 or 3 -> 1, pending - 1
+__device__ __forceinline__ void aq_finish(const AsyncQ& Q, int t) {
+    atomicSub(Q.tstate + t, 2);
+    atomicAdd(Q.ctr + AQ_PEND, ~0ull);
 }
 static __global__ void k_async_init(AsyncQ Q, int ntiles) {
     for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < ntiles; t += gridDim.x * blockDim.x) {
@@ -764,8 +772,7 @@ k_prop_async(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, co
             __threadfence();
             __syncthreads();                                      // marks (pending++) before finish
             if (tid == 0) {
-                if (atomicCAS(Q.tstate + tile, 2, 0) == 2) atomicAdd(Q.ctr + AQ_PEND, ~0ull);
-                else atomicExch(Q.tstate + tile, 1);
+                aq_finish(Q, tile);
             }
 #ifdef ECL_PROF
             tp = clock64();

@@ -33,4 +33,8 @@ labs = E.ecl_scc_batched([(torch.from_numpy(h.row_ptr).cuda(), torch.from_numpy(
 torch.cuda.synchronize()
 for h, l in zip(graphs, labs):
     assert np.array_equal(l.cpu().numpy(), oracle.tarjan_labels(h.row_ptr, h.col_idx))
+hl = E.ecl_scc_batched_host([(torch.from_numpy(h.row_ptr).pin_memory(), torch.from_numpy(h.col_idx).pin_memory())
+                             for h in graphs])
+for h, l in zip(graphs, hl):
+    assert np.array_equal(l.numpy(), oracle.tarjan_labels(h.row_ptr, h.col_idx))
 print("sanitize workload ok", flush=True)

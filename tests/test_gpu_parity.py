@@ -280,6 +280,47 @@ def test_batched_host_buffers():
             np.testing.assert_array_equal(lab.numpy(), oracle.tarjan_labels(g.row_ptr, g.col_idx))
 
 
+def _dense_local_graph(n, seed, back=0.02, span=20):
+    """Rows of up to 3 out-edges to the next vertices, one random forward edge and, with
+    probability `back`, a short backward edge (small cycles); every row <= 8 entries in both
+    directions (so the compaction runs on 4-byte keep words) and almost every vertex with more
+    than 4 entries in + out (the overlapped path of k_compact_count2 takes 4, the rest goes
+    through trim_mask)."""
+    rng = np.random.default_rng(seed)
+    indeg = np.zeros(n, dtype=np.int64)
+    edges = []
+    for v in range(n):
+        outs = set()
+        for d in (1, 2, 3):
+            if rng.random() < 0.85 and v + d < n:
+                outs.add(v + d)
+        w = v + int(rng.integers(4, 600))
+        if w < n:
+            outs.add(w)
+        if rng.random() < back:
+            outs.add(max(0, v - int(rng.integers(1, span))))
+        outs.discard(v)
+        for w in sorted(outs):
+            if indeg[w] < 8:
+                edges.append((v, w))
+                indeg[w] += 1
+    g = gen.from_edges(n, np.array(edges))
+    assert np.diff(g.row_ptr).max() <= 8 and indeg.max() <= 8
+    return g
+
+
+@pytest.mark.parametrize("seed", [11, 12])
+def test_keep_word_rows_with_more_than_four_entries(seed):
+    """Keep-word compaction (rows <= 8) on rows with 5-8 entries: labels and per-iteration
+    traces against the oracle (the keep-word count / map kernels, incl. their long-row paths)."""
+    g = _dense_local_graph(30000, seed)
+    deg = np.diff(g.row_ptr) + np.bincount(g.col_idx, minlength=g.n)
+    assert (deg > 4).mean() > 0.5
+    lab, _ = gpu_labels(g)
+    np.testing.assert_array_equal(lab, oracle.tarjan_labels(g.row_ptr, g.col_idx))
+    check_trace(g, trim=True, max_iters=4)
+
+
 def test_repeated_runs_with_plan_reuse_are_stable():
     """Races show up under repetition: the same plan, several graphs and orders, many runs."""
     graphs = [gen.mesh(60, gen.ordinate(d), seed=4 + d, order=o, **gen.C4_MESH)

@@ -586,7 +586,7 @@ k_prop_pack(WGraph g, int32_t* __restrict__ cin, int32_t* __restrict__ cout, con
 // dirtied ahead of the cursor is visited in the same sweep (Gauss-Seidel between tiles)
 // and no CTA waits for the slowest visit of a pass.
 // Tile state machine (tstate): 0 clean, 1 dirty, 2 running, 3 running + dirtied again.
-//   mark(t):   0 -> 1 (pending++); 2 -> 3; 1, 3 unchanged
+//   mark(t):   0 -> 1 or 2 -> 3 (pending++ either way); 1, 3 unchanged
 //   claim(t):  1 -> 2 (the first visit of a tile in the phase is a full one)
 //   finish(t): 2 -> 0; 3 -> 1 (state -= 2)
 // pending = #state 1 + #state 2 + 2 * #state 3, so every state change by a mark (0 -> 1,

@@ -180,6 +180,12 @@ template <typename T>
 static int scan_excl(Plan* p, const T* in, int64_t N, T* out, T* grand, void* bsum, int write_total, cudaStream_t s) {
     const int64_t nb = std::max<int64_t>(cdiv(N, SCAN_TILE), 1);
     p->launches++; k_scan_reduce<T><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, N, (T*)bsum);
+    if (nb <= SCAN_FOLD_NB) {                          // small scans: the top level folded into the apply
+        p->launches++;
+        k_scan_apply_fold<T><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, N, (const T*)bsum, out, grand, write_total);
+        CK(cudaGetLastError());
+        return ECL_SCC_OK;
+    }
     p->launches++; k_scan_top<T><<<1, SCAN_THREADS, 0, s>>>((T*)bsum, nb, grand);
     p->launches++; k_scan_apply<T><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, N, (T*)bsum, out, grand, write_total);
     CK(cudaGetLastError());

@@ -109,4 +109,49 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_apply(const T* __restrict
     if (write_total && blockIdx.x == 0 && threadIdx.x == 0) out[N] = *grand;
 }
 
+// k_scan_top folded into the apply for small scans (nb <= SCAN_FOLD_NB block totals, e.g. the
+// per-warp compaction counts: C4 251 blocks): every block sums the totals of the blocks before
+// it itself (at most SCAN_FOLD_NB loads, L2-resident), the last block writes the grand total.
+// One launch less per scan.
+constexpr int64_t SCAN_FOLD_NB = 512;
+template <typename T>
+__global__ void __launch_bounds__(SCAN_THREADS) k_scan_apply_fold(const T* __restrict__ in, int64_t N, const T* __restrict__ bsum,
+                                                                  T* __restrict__ out, T* __restrict__ grand, int write_total) {
+    __shared__ T s_part[SCAN_THREADS / WARP];
+    T c = T::zero();
+    for (int64_t b = threadIdx.x; b < blockIdx.x; b += SCAN_THREADS) c = c + bsum[b];
+    // block sum of the partial carries (warp shuffles, then one warp)
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        T t = c.shfl_up(o);        // (shfl_up then add from the top lane: inclusive scan; lane 31 holds the sum)
+        if ((threadIdx.x & 31) >= o) c = c + t;
+    }
+    if ((threadIdx.x & 31) == 31) s_part[threadIdx.x >> 5] = c;
+    __syncthreads();
+    T carry = T::zero();
+#pragma unroll
+    for (int w = 0; w < SCAN_THREADS / WARP; w++) carry = carry + s_part[w];
+    __syncthreads();
+    const int64_t base = (int64_t)blockIdx.x * SCAN_TILE + (int64_t)threadIdx.x * SCAN_ITEMS;
+    T vals[SCAN_ITEMS];
+    T acc = T::zero();
+#pragma unroll
+    for (int k = 0; k < SCAN_ITEMS; k++) {
+        vals[k] = (base + k < N) ? in[base + k] : T::zero();
+        acc = acc + vals[k];
+    }
+    T total;
+    T ex = block_excl_scan(acc, total) + carry;
+#pragma unroll
+    for (int k = 0; k < SCAN_ITEMS; k++) {
+        if (base + k < N) out[base + k] = ex;
+        ex = ex + vals[k];
+    }
+    if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) {
+        const T g = carry + total;
+        *grand = g;
+        if (write_total) out[N] = g;
+    }
+}
+
 }  // namespace eclscc
